@@ -1,0 +1,233 @@
+/*
+ * aceso.h — C-ABI of the B200-native batched configuration evaluator for
+ * Aceso (Liu et al., "Aceso: Efficient Parallel DNN Training through Iterative
+ * Bottleneck Alleviation", EuroSys '24).
+ *
+ * Citations: "P:Lnn" = line nn of the paper text; "R#" = a reading of
+ * an ambiguous passage, listed in DESIGN.md §3 (the register of readings).
+ *
+ * The library evaluates the paper's performance model (§3.3) over
+ * very large batches of candidate parallel configurations (§3.1) and
+ * selects the best candidate (Heuristic-1 P:L155, "better" P:L138, Alg. 1/2
+ * `Estimate`/`GetBestOf` P:L521-593). Every step runs in the sm_100a kernels of
+ * libaceso.so; there is no host or CPU fallback.
+ *
+ * All profiled costs are integers: times in nanoseconds, sizes in bytes. All
+ * accumulation is exact unsigned 64-bit; results are bit-exact and
+ * independent of reduction order.
+ *
+ * Threading: a context may be used from several host threads, on any streams.
+ * aceso_last_error() is thread-local.
+ */
+#ifndef ACESO_H_
+#define ACESO_H_
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+/* ------------------------------------------------------------------------- */
+/* Status codes (return values).                                             */
+/* ------------------------------------------------------------------------- */
+#define ACESO_OK       0
+#define ACESO_EINVAL  (-1) /* bad argument (null pointer, bad size, bad flags) */
+#define ACESO_ERANGE  (-2) /* a profile value does not fit the packed width,
+                              keep > act, or a model-wide bound could overflow */
+#define ACESO_ECUDA   (-3) /* a CUDA runtime call failed (message in last_error) */
+#define ACESO_ENOMEM  (-4) /* device or host allocation failed */
+#define ACESO_ENODEV  (-5) /* no usable sm_100 device */
+
+/* ------------------------------------------------------------------------- */
+/* Profile: the op-cost database of §3.3.                           */
+/* ------------------------------------------------------------------------- */
+/* Field order of one profile record rec[type][tpl][b][*] (ns | bytes).       */
+enum {
+  ACESO_F_FWD_COMP = 0, /* forward compute time of one microbatch (ns)        */
+  ACESO_F_FWD_COMM = 1, /* forward tensor-parallel collective time (ns)       */
+  ACESO_F_BWD_COMP = 2, /* backward compute time (ns)                         */
+  ACESO_F_BWD_COMM = 3, /* backward tensor-parallel collective time (ns)      */
+  ACESO_F_ACT      = 4, /* activation bytes kept for backward (no recompute)  */
+  ACESO_F_KEEP     = 5, /* bytes kept when the op is recomputed (R3); <= act  */
+  ACESO_F_PEAK     = 6, /* transient bytes while the op runs (R4)     */
+  ACESO_F_RESHARD  = 7, /* re-partition cost when this op's tp/dp differs from
+                           the previous op of the same stage (R13)    */
+  ACESO_F_P2P_FWD  = 8, /* send of this op's output to the next stage (R5)    */
+  ACESO_F_P2P_BWD  = 9, /* send of this op's input grad to the previous stage */
+  ACESO_REC_FIELDS = 10
+};
+
+/* Host-side profile description. All pointers are host pointers owned by the
+ * caller; aceso_load_profile copies what it needs. Index conventions:
+ *   tpl = log2(tensor-parallel degree)   in [0, n_tp)
+ *   dpl = log2(data-parallel degree)     in [0, n_dp)
+ *   b   = log2(per-GPU microbatch size)  in [0, n_b), b = mbs_log2 - dpl (R8)
+ */
+typedef struct {
+  int32_t n_ops;            /* L: operators in model order, 1..16384          */
+  int32_t n_types;          /* T: distinct op types, 1..4096                  */
+  int32_t n_tp;             /* tp choices, 1..8                               */
+  int32_t n_dp;             /* dp choices, 1..8                               */
+  int32_t n_b;              /* per-GPU batch choices, 1..16                   */
+  int32_t n_devices;        /* G: simulated devices, 1..255                   */
+  const uint16_t *op_type;  /* [n_ops], each < n_types                        */
+  const int64_t *rec;       /* [n_types][n_tp][n_b][ACESO_REC_FIELDS]         */
+  const int64_t *wmem;      /* [n_types][n_tp][2]: param+grad bytes, optimizer bytes */
+  const int64_t *dps;       /* [n_types][n_tp][n_dp]: DP gradient all-reduce ns */
+  int64_t mem_capacity;     /* C: device memory in bytes (OOM iff Mem_i > C, R10) */
+  int64_t global_batch;     /* Bg: samples per iteration, 1..2^31             */
+} aceso_profile_desc;
+
+typedef struct aceso_ctx aceso_ctx; /* opaque; owned by the library */
+
+/* Validates and packs the profile, uploads it to `cuda_device` and returns a
+ * context. Synchronous. Range rules (ACESO_ERANGE on violation):
+ *  - every rec/wmem/dps value in [0, 2^32);  keep <= act;  peak + act - keep < 2^32;
+ *  - fwd_comp+fwd_comm+bwd_comp+bwd_comm + (fwd_comp+fwd_comm) < 2^32;
+ *  - model-wide: L * max-per-op cost * Bg < 2^62 for time and memory, so that
+ *    every iteration time and stage memory is < 2^62 (exact packed keys).
+ * Returns ACESO_OK and sets *out, or a negative status (see aceso_last_error). */
+int aceso_load_profile(const aceso_profile_desc *desc, int cuda_device, aceso_ctx **out);
+
+/* Releases the context and its device memory. Null is ignored. */
+void aceso_free(aceso_ctx *ctx);
+
+/* ------------------------------------------------------------------------- */
+/* Candidate encoding (configuration representation, §3.1).       */
+/* ------------------------------------------------------------------------- */
+/* One byte per operator:
+ *   bit 0     head : 1 = this op opens a new pipeline stage (stage = contiguous op range)
+ *   bits 1..3 tpl  : log2 tensor-parallel degree of this op
+ *   bit 4     rc   : 1 = recompute this op in backward
+ *   bits 5..7 dpl  : log2 data-parallel degree of this op
+ * One 64-bit header per candidate (little-endian bytes):
+ *   byte 0 mbs_log2 : log2 of the aggregated microbatch size (R8)
+ *   byte 1 p        : number of pipeline stages
+ *   bytes 2..7      : reserved, must be 0
+ */
+#define ACESO_CODE(head, tpl, dpl, rc) \
+  ((uint8_t)(((head) & 1) | (((tpl) & 7) << 1) | (((rc) & 1) << 4) | (((dpl) & 7) << 5)))
+#define ACESO_HDR(mbs_log2, p) ((uint64_t)((mbs_log2) & 0xff) | ((uint64_t)((p) & 0xff) << 8))
+
+/* Tiled device layout of the op codes: tiles of 32 candidates, chunks of 16 ops.
+ * Byte (c, j) of candidate c, op j lives at
+ *   ((c / 32) * nch + j / 16) * 512 + (c % 32) * 16 + (j % 16),   nch = ceil(L/16).
+ * Pad ops (j >= L) and the pad candidates of a ragged last tile are ignored.
+ * A warp's 16-byte loads of one chunk are 512 contiguous bytes. */
+#define ACESO_TILE_CANDS 32
+#define ACESO_CHUNK_OPS 16
+
+/* Bytes of a tiled buffer holding n candidates of n_ops ops. */
+size_t aceso_tiled_bytes(int64_t n, int32_t n_ops);
+
+/* Converts row-major codes [n][n_ops] (device) into the tiled layout (device),
+ * writing zero pad bytes. Asynchronous on `stream` (a cudaStream_t; 0 = legacy
+ * default stream). */
+int aceso_pack_rowmajor(const uint8_t *d_rowmajor, int64_t n, int32_t n_ops,
+                        uint8_t *d_tiled, void *stream);
+
+/* ------------------------------------------------------------------------- */
+/* Evaluation outputs.                                                        */
+/* ------------------------------------------------------------------------- */
+/* info word of one candidate */
+#define ACESO_INFO_BOTTLENECK(x) ((x) & 0xffu)        /* Heuristic-1 stage   */
+#define ACESO_INFO_P(x)          (((x) >> 8) & 0xffu) /* header p                    */
+#define ACESO_INFO_OOM           (1u << 16)           /* some stage has Mem_i > C    */
+#define ACESO_INFO_INVALID       (1u << 17)           /* not a configuration         */
+#define ACESO_INFO_REASONS(x)    ((x) >> 18)          /* mask of ACESO_R_* below     */
+
+/* Invalid-configuration reasons (bitmask; every violated rule is reported). */
+#define ACESO_R_HEAD0   (1u << 0) /* op 0 does not open a stage                         */
+#define ACESO_R_NSTAGE  (1u << 1) /* number of heads != p                               */
+#define ACESO_R_PRANGE  (1u << 2) /* p == 0 or p > G                                    */
+#define ACESO_R_GSTAGE  (1u << 3) /* tp*dp differs between two ops of one stage */
+#define ACESO_R_GSUM    (1u << 4) /* sum over stages of tp*dp != G (R9)                 */
+#define ACESO_R_DPMBS   (1u << 5) /* dp > mbs for some op (per-GPU batch < 1)   */
+#define ACESO_R_TABLE   (1u << 6) /* tpl >= n_tp, dpl >= n_dp or b >= n_b               */
+#define ACESO_R_MBS     (1u << 7) /* mbs > Bg or Bg % mbs != 0                          */
+#define ACESO_R_HDR     (1u << 8) /* reserved header bytes not zero                     */
+
+/* Device output arrays (SoA). Pointers are device pointers owned by the caller.
+ * Summary (ACESO_OUT_SUMMARY):
+ *   iter_ns[n]  iteration time  max_i T_i (Eq. 2, R1)          0 if invalid
+ *   max_mem[n]  max_i Mem_i (Eq. 1 + P:L232 + P:L234)          0 if invalid
+ *   info[n]     bottleneck | p<<8 | status | reasons<<18
+ * Full (ACESO_OUT_FULL), stage-major [p_max][n], written for valid candidates
+ * and stages i < p only (other entries untouched):
+ *   stage_T    T_i = sum_k S_k + (N-1) S_i + D_i
+ *   stage_mem  Mem_i = Wst_i + min(p-i, N) A_i + E_i
+ *   stage_comp N * sum_j (fwd_comp + bwd_comp + rc*fwd_comp)
+ *   stage_comm N * sum_j (fwd_comm + bwd_comm + rc*fwd_comm + rs_j) + N*p2p_i + D_i
+ */
+typedef struct {
+  uint64_t *iter_ns;
+  uint64_t *max_mem;
+  uint32_t *info;
+  uint64_t *stage_T;
+  uint64_t *stage_mem;
+  uint64_t *stage_comp;
+  uint64_t *stage_comm;
+  int32_t p_max; /* row count of the stage arrays; must be >= n_devices for FULL */
+} aceso_eval_out;
+
+#define ACESO_OUT_SUMMARY  1u /* write iter_ns, max_mem, info                   */
+#define ACESO_OUT_FULL     2u /* also write the per-stage arrays                 */
+#define ACESO_FUSED_SELECT 4u /* reduce the batch argmin into d_sel (fused K2)   */
+
+/* ------------------------------------------------------------------------- */
+/* Selection (Alg. 1 GetBestOf P:L543, Alg. 2 `perf < init_perf` P:L576).     */
+/* ------------------------------------------------------------------------- */
+/* Order: lexicographic on (class, cost, global index); class 0 = feasible
+ * (cost = iteration time), class 1 = out of memory (cost = max_i Mem_i, R12);
+ * invalid candidates are excluded. Result written to the first 32 bytes of the
+ * caller's select buffer:                                                   */
+typedef struct {
+  int64_t key;       /* packed key for an all-reduce MIN across ranks:
+                        class<<62 | min(cost, 2^(62-IB)-1)<<IB | index,
+                        IB = bit length of n_total; INT64_MAX if nothing valid */
+  uint64_t cls_cost; /* exact class<<62 | cost; UINT64_MAX if nothing valid    */
+  int64_t index;     /* exact global index of the winner; -1 if nothing valid  */
+  uint64_t reserved;
+} aceso_select_result;
+
+/* Size in bytes of the select buffer for a batch of n candidates (result +
+ * per-CTA partials + a completion counter). The buffer must be zero-filled once
+ * at allocation; every call leaves it reusable. One buffer per in-flight call. */
+size_t aceso_select_buf_bytes(const aceso_ctx *ctx, int64_t n);
+
+/* Evaluates candidates [0, n) of a batch whose first candidate has global index
+ * `global_offset` in a job of `n_total` candidates (sharding, §8e).
+ *   d_codes : tiled op codes (device)        d_hdr : [n] headers (device)
+ *   flags   : OR of ACESO_OUT_SUMMARY / ACESO_OUT_FULL / ACESO_FUSED_SELECT
+ *   out     : host struct of device pointers (may be null if no OUT_* flag)
+ *   d_sel   : select buffer (device), required with ACESO_FUSED_SELECT
+ *   stream  : cudaStream_t
+ * Asynchronous; no allocation, no host synchronisation. n == 0 is valid (the
+ * select result becomes "nothing valid"). */
+int aceso_eval(aceso_ctx *ctx, const uint8_t *d_codes, const uint64_t *d_hdr, int64_t n,
+               int64_t global_offset, int64_t n_total, uint32_t flags,
+               const aceso_eval_out *out, void *d_sel, void *stream);
+
+/* Argmin over an already written summary (iter_ns, max_mem, info) of n
+ * candidates; same order and result layout as the fused select. Async. */
+int aceso_select(aceso_ctx *ctx, const aceso_eval_out *out, int64_t n, int64_t global_offset,
+                 int64_t n_total, void *d_sel, void *stream);
+
+/* Decodes a packed key. *saturated = 1 when the cost field is clamped (the
+ * exact cls_cost must then be used). Returns ACESO_OK; for INT64_MAX sets
+ * *cls = -1, *index = -1. */
+int aceso_decode_key(int64_t key, int64_t n_total, int *cls, uint64_t *cost, int64_t *index,
+                     int *saturated);
+
+/* Message of the last failing call on this thread ("" if none). */
+const char *aceso_last_error(void);
+
+/* Library version string. */
+const char *aceso_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* ACESO_H_ */

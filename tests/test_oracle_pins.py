@@ -1,0 +1,368 @@
+"""Pins for the CPU oracle (no GPU): each test checks the oracle against something
+the paper or mathematics fixes, not against a retyped copy of its formulas.
+
+P:Lnn = PAPER.md line; R# = reading in DESIGN.md §3.
+"""
+import itertools
+
+import numpy as np
+import pytest
+
+import aceso_inputs as ai
+import oracle
+from aceso_inputs import profiles as P
+from tests.sim1f1b import simulate
+
+NF = 10
+FC, FM, BC, BM, ACT, KEEP, PEAK, RESH, P2PF, P2PB = range(NF)
+
+
+def mkprof(recs, op_type, n_tp=1, n_b=8, n_dp=1, G=1, C=1 << 40, Bg=8, wmem=None, dps=None):
+    """recs: dict type -> fn(tpl, b) -> list of NF values."""
+    T = len(recs)
+    rec = np.zeros((T, n_tp, n_b, NF), np.int64)
+    for t in range(T):
+        for tpl in range(n_tp):
+            for b in range(n_b):
+                rec[t, tpl, b] = recs[t](tpl, b)
+    wm = np.zeros((T, n_tp, 2), np.int64) if wmem is None else np.asarray(wmem, np.int64)
+    dp = np.zeros((T, n_tp, n_dp), np.int64) if dps is None else np.asarray(dps, np.int64)
+    return P.from_tables("hand", op_type, rec, wm, dp, G, C, Bg)
+
+
+def cand(stage_sizes, tpdp=None, rc=None):
+    """Row of codes for consecutive stages of the given sizes."""
+    out = []
+    j = 0
+    for i, n in enumerate(stage_sizes):
+        tpl, dpl = (tpdp[i] if tpdp else (0, 0))
+        for k in range(n):
+            r = rc[j] if rc else 0
+            out.append(ai.code(1 if k == 0 else 0, tpl, dpl, r))
+            j += 1
+    return out
+
+
+def ev(prof, rows, hdrs, full=True):
+    return oracle.evaluate(prof, np.array(rows, np.uint8), np.array(hdrs, np.uint64), full=full)
+
+
+# --------------------------------------------------------------------------
+# Eq. 2 (R1) and Eq. 1 (R2) against a discrete-event 1F1B simulation
+# --------------------------------------------------------------------------
+@pytest.mark.parametrize("p", [1, 2, 3, 4, 5])
+@pytest.mark.parametrize("mbs_log2", [0, 1, 2, 3])
+def test_uniform_pipeline_matches_1f1b_simulation(p, mbs_log2):
+    """Uniform stages: Eq. 2 (reading R1) gives the 1F1B makespan (N+p-1)(f+b)
+    and Eq. 1 gives min(p-i, N) in-flight activations on stage i."""
+    k = 3  # ops per stage
+    f_op, b_op = 7, 13
+    prof = mkprof({0: lambda tpl, b: [f_op, 0, b_op, 0, 1, 0, 0, 0, 0, 0]}, [0] * (p * k), G=p, Bg=8)
+    N = 8 >> mbs_log2
+    out = ev(prof, [cand([k] * p)], [ai.header(mbs_log2, p)])
+    assert out["info"][0] & oracle.INFO_INVALID == 0
+    mk, peak = simulate([f_op * k] * p, [b_op * k] * p, N)
+    assert int(out["iter"][0]) == mk == (N + p - 1) * (f_op + b_op) * k
+    for i in range(p):
+        assert int(out["stage_mem"][0, i]) == k * peak[i] == k * min(p - i, N)
+
+
+def test_inflight_rule_on_nonuniform_stages():
+    """The in-flight count min(p-i, N) of Eq. 1 (R2) is structural: it holds for any
+    stage times in the 1F1B simulation, so Mem_i/A_i must equal the simulated peak."""
+    rng = np.random.default_rng(5)
+    for _ in range(20):
+        p = int(rng.integers(1, 7))
+        sizes = [int(x) for x in rng.integers(1, 5, size=p)]
+        L = sum(sizes)
+        prof = mkprof({0: lambda tpl, b: [3, 0, 5, 0, 1, 0, 0, 0, 0, 0]}, [0] * L, G=p, Bg=16)
+        mbs_log2 = int(rng.integers(0, 5))
+        N = 16 >> mbs_log2
+        out = ev(prof, [cand(sizes)], [ai.header(mbs_log2, p)])
+        f = [float(rng.uniform(1, 9)) for _ in range(p)]
+        b = [float(rng.uniform(1, 9)) for _ in range(p)]
+        _, peak = simulate(f, b, N)
+        for i in range(p):
+            assert int(out["stage_mem"][0, i]) == sizes[i] * peak[i]
+
+
+def test_p1_is_gradient_accumulation():
+    """p = 1: T = N*S + D (N microbatches back to back, then the DP sync)."""
+    prof = mkprof({0: lambda tpl, b: [11 * (b + 1), 2, 23 * (b + 1), 3, 0, 0, 0, 0, 0, 0]},
+                  [0] * 5, n_b=2, n_dp=2, G=2, Bg=16, dps=[[[0, 1000]]])
+    # one stage, dp = 2, mbs = 4 -> per-GPU batch 2 (b index 1), N = 4
+    out = ev(prof, [cand([5], tpdp=[(0, 1)])], [ai.header(2, 1)])
+    mk, _ = simulate([5 * (22 + 2)], [5 * (46 + 3)], 4, sync=[5 * 1000])
+    assert int(out["iter"][0]) == mk
+
+
+def test_dp_sync_on_first_stage_matches_simulation():
+    """R6: the DP gradient sync is added once to its own stage. Stage 0 finishes last
+    in 1F1B, so a sync on stage 0 adds exactly to the simulated makespan."""
+    p, k = 3, 2
+    prof = mkprof({0: lambda tpl, b: [5, 0, 9, 0, 0, 0, 0, 0, 0, 0],
+                   1: lambda tpl, b: [5, 0, 9, 0, 0, 0, 0, 0, 0, 0]},
+                  [1, 1] + [0] * 4, n_dp=2, G=p, Bg=8,
+                  dps=[[[0, 0]], [[40, 40]]])
+    # op type 1 carries a DP sync only when dp > 1 ... stage 0 runs dp=1 -> use dps[1][0][0]
+    prof.dps[1, 0, 0] = 40
+    out = ev(prof, [cand([k] * p)], [ai.header(1, p)])
+    N = 4
+    mk, _ = simulate([5 * k] * p, [9 * k] * p, N, sync=[80, 0, 0])
+    assert int(out["iter"][0]) == mk
+
+
+# --------------------------------------------------------------------------
+# recomputation (R3, R7)
+# --------------------------------------------------------------------------
+def test_recompute_adds_forward_and_never_adds_memory():
+    """inc-rc on op j (Table 1 row 9: Comp up, Mem down): stage i's per-microbatch
+    time grows by F_j, so T_i grows by N*F_j and every other T_k by F_j (Eq. 2);
+    Mem_i does not grow (R3)."""
+    prof = P.toy_b()
+    codes, hdr = ai.search_shaped(prof, 11, 0, 400, group_size=16, invalid_permille=0)
+    base = oracle.evaluate(prof, codes, hdr, full=True)
+    rng = np.random.default_rng(3)
+    checked = 0
+    for c in range(len(hdr)):
+        if base["info"][c] & oracle.INFO_INVALID:
+            continue
+        j = int(rng.integers(0, prof.n_ops))
+        if codes[c, j] & 0x10:
+            continue
+        row = codes[c].copy()
+        row[j] |= 0x10
+        new = oracle.evaluate(prof, row[None, :], hdr[c:c + 1], full=True)
+        p = (int(hdr[c]) >> 8) & 0xFF
+        i = int(np.sum(codes[c, :j + 1] & 1)) - 1
+        mbs_log2 = int(hdr[c]) & 0xFF
+        N = prof.global_batch >> mbs_log2
+        tpl = (int(codes[c, j]) >> 1) & 7
+        dpl = (int(codes[c, j]) >> 5) & 7
+        r = prof.rec[prof.op_type[j], tpl, mbs_log2 - dpl]
+        F = int(r[FC] + r[FM])
+        for k in range(p):
+            d = int(new["stage_T"][0, k]) - int(base["stage_T"][c, k])
+            assert d == (N * F if k == i else F)
+        assert int(new["stage_mem"][0, i]) <= int(base["stage_mem"][c, i])
+        assert int(new["iter"][0]) >= int(base["iter"][c])
+        checked += 1
+    assert checked > 100
+
+
+# --------------------------------------------------------------------------
+# zero-cost operator invariance (north_star)
+# --------------------------------------------------------------------------
+def test_zero_cost_op_move_changes_nothing():
+    rng = np.random.default_rng(9)
+    recs = {0: lambda tpl, b: [0] * NF}
+    for t in range(1, 4):
+        vals = [int(x) for x in rng.integers(1, 1000, size=NF)]
+        vals[KEEP] = vals[ACT] // 2
+        vals[P2PF] = vals[P2PB] = 0
+        recs[t] = (lambda v: (lambda tpl, b: v))(vals)
+    op_type = [1, 2, 0, 3, 1, 0, 2, 3]
+    wm = np.zeros((4, 1, 2), np.int64)
+    wm[1:] = rng.integers(0, 100, size=(3, 1, 2))
+    dps = np.zeros((4, 1, 1), np.int64)
+    prof = mkprof(recs, op_type, G=2, Bg=8, wmem=wm, dps=dps, C=1 << 40)
+    # boundary before op 2 (zero op in stage 1) vs after it (zero op in stage 0)
+    a = ev(prof, [cand([2, 6])], [ai.header(1, 2)])
+    b = ev(prof, [cand([3, 5])], [ai.header(1, 2)])
+    for key in ["iter", "max_mem", "info", "stage_T", "stage_mem", "stage_comp", "stage_comm"]:
+        assert np.array_equal(a[key], b[key]), key
+
+
+# --------------------------------------------------------------------------
+# Heuristic-1 on the Fig. 3 scenario, worked by hand
+# --------------------------------------------------------------------------
+def fig3_profile():
+    # one op type; b index 0 = 1 sample/GPU, 1 = 2 samples/GPU; tpl 0/1
+    tab = {(0, 0): (100, 200, 10), (0, 1): (200, 400, 20), (1, 0): (60, 120, 5), (1, 1): (120, 240, 10)}
+
+    def r(tpl, b):
+        f, bw, a = tab[(tpl, b)]
+        return [f, 0, bw, 0, a, a, 0, 0, 0, 0]
+    return mkprof({0: r}, [0, 0, 0, 0], n_tp=2, n_b=2, n_dp=2, G=3, C=60, Bg=8)
+
+
+def test_fig3_scenario():
+    prof = fig3_profile()
+    rows = [cand([2, 2], tpdp=[(0, 0), (0, 1)]),   # (a) even ops; 1 GPU + 2 GPUs (dp=2)
+            cand([2, 2], tpdp=[(1, 0), (0, 0)]),   # (b) stage 0 gets 2 GPUs (tp=2)
+            cand([3, 1], tpdp=[(1, 0), (0, 0)])]   # (c) migrate one op to stage 0
+    out = ev(prof, rows, [ai.header(1, 2)] * 3)
+    info = out["info"]
+    # (a): Mem = (80, 20) > C=60 on stage 0 -> OOM, bottleneck stage 0 by memory
+    assert info[0] & oracle.INFO_OOM and info[0] & 0xFF == 0
+    assert list(out["stage_mem"][0, :2]) == [80, 20] and out["max_mem"][0] == 80
+    # (b): no OOM, stage 1 slowest -> bottleneck 1 by time; iter = 1920 + 3*1200
+    assert not info[1] & oracle.INFO_OOM and info[1] & 0xFF == 1
+    assert out["iter"][1] == 5520
+    # (c): balanced -> faster than (b): iter = 1680 + 3*1080
+    assert not info[2] & oracle.INFO_OOM and out["iter"][2] == 4920 < out["iter"][1]
+    # "better": feasible beats infeasible, then faster
+    assert oracle.select(out) == (0, 4920, 2)
+
+
+def test_bottleneck_ties_take_lowest_stage():
+    prof = mkprof({0: lambda tpl, b: [5, 0, 5, 0, 1, 1, 0, 0, 0, 0]}, [0] * 6, G=3, Bg=1, C=1 << 40)
+    out = ev(prof, [cand([2, 2, 2])], [ai.header(0, 3)])   # N = 1: equal T, equal Mem
+    assert out["info"][0] & 0xFF == 0
+    prof.mem_capacity = 0                                   # all stages OOM, equal Mem
+    out = ev(prof, [cand([2, 2, 2])], [ai.header(0, 3)])
+    assert out["info"][0] & oracle.INFO_OOM and out["info"][0] & 0xFF == 0
+
+
+# --------------------------------------------------------------------------
+# record lookup: which (type, tp, per-GPU batch) entry is read (R8)
+# --------------------------------------------------------------------------
+def test_lookup_fingerprint():
+    """Single-op model, one stage: T = N*F + D with only fwd_comp set to a fingerprint
+    of (type, tpl, b) and dps to a fingerprint of (type, tpl, dpl): a transposed index
+    or a wrong per-GPU batch (mbs/dp) shows up as a different number."""
+    n_tp = n_dp = 4
+    n_b = 4
+
+    def fp(t, tpl, b):
+        return 1 + b + 10 * tpl + 100 * t
+
+    recs = {t: (lambda t: (lambda tpl, b: [fp(t, tpl, b), 0, 0, 0, 0, 0, 0, 0, 0, 0]))(t) for t in range(2)}
+    dps = np.zeros((2, n_tp, n_dp), np.int64)
+    for t, tpl, dpl in itertools.product(range(2), range(n_tp), range(n_dp)):
+        dps[t, tpl, dpl] = 1000 * (1 + dpl + 10 * tpl + 100 * t)
+    for t in range(2):
+        for G in [1, 2, 4, 8]:
+            kG = G.bit_length() - 1
+            prof = mkprof(recs, [t], n_tp=n_tp, n_b=n_b, n_dp=n_dp, G=G, Bg=64, dps=dps)
+            rows, hdrs, exp = [], [], []
+            for tpl in range(kG + 1):
+                dpl = kG - tpl
+                for mbs_log2 in range(dpl, dpl + n_b):
+                    rows.append([ai.code(1, tpl, dpl, 0)])
+                    hdrs.append(ai.header(mbs_log2, 1))
+                    N = 64 >> mbs_log2
+                    exp.append(N * fp(t, tpl, mbs_log2 - dpl) + dps[t, tpl, dpl])
+            out = ev(prof, rows, hdrs)
+            assert [int(x) for x in out["iter"]] == exp
+
+
+def test_memory_terms_special_cases():
+    """One stage, N = 1: Mem = sum W + sum A + max_j peak (P:L229 + P:L234, R4)."""
+    vals = [(10, 3, 7, 5), (20, 20, 40, 1), (30, 0, 11, 9)]  # (act, keep, peak, W)
+    recs = {t: (lambda v: (lambda tpl, b: [1, 0, 1, 0, v[0], v[1], v[2], 0, 0, 0]))(v)
+            for t, v in enumerate(vals)}
+    wm = np.array([[[v[3], 0]] for v in vals], np.int64)
+    prof = mkprof(recs, [0, 1, 2], G=1, Bg=1, wmem=wm)
+    out = ev(prof, [cand([3])], [ai.header(0, 1)])
+    assert out["max_mem"][0] == (5 + 1 + 9) + (10 + 20 + 30) + 40
+    # recompute op 0: keeps 3 instead of 10, re-materialises 7 transiently (R3)
+    out = ev(prof, [cand([3], rc=[1, 0, 0])], [ai.header(0, 1)])
+    assert out["max_mem"][0] == 15 + (3 + 20 + 30) + max(7 + 7, 40, 11)
+
+
+# --------------------------------------------------------------------------
+# readings without an independent pin: worked examples (parity unpinned beyond these)
+# --------------------------------------------------------------------------
+def test_p2p_and_reshard_worked_example():
+    """R5: stage i pays p2p_fwd of its last op (i < p-1) and p2p_bwd of its first op
+    (i > 0). R13: an in-stage tp/dp change charges the receiving op's reshard."""
+    def r(tpl, b):
+        return [10, 0, 20, 0, 0, 0, 0, 100 + tpl, 1000 + tpl, 2000 + tpl]
+    prof = mkprof({0: r}, [0] * 4, n_tp=2, n_b=2, n_dp=2, G=4, Bg=4)
+    # stage 0: ops 0,1 at (tp2,dp1) then (tp1,dp2) -> reshard on op 1 (tpl 0): 100
+    # stage 1: ops 2,3 at (tp2,dp1)
+    row = [ai.code(1, 1, 0, 0), ai.code(0, 0, 1, 0), ai.code(1, 1, 0, 0), ai.code(0, 1, 0, 0)]
+    out = ev(prof, [row], [ai.header(1, 2)])
+    S0 = 30 + 30 + 100 + 1000  # + p2p_fwd of op 1 (tpl 0)
+    S1 = 30 + 30 + 2001        # + p2p_bwd of op 2 (tpl 1)
+    N = 2
+    assert list(out["stage_T"][0, :2]) == [S0 + S1 + (N - 1) * S0, S0 + S1 + (N - 1) * S1]
+    assert list(out["stage_comp"][0, :2]) == [N * 60, N * 60]
+    assert list(out["stage_comm"][0, :2]) == [N * 1100, N * 2001]
+
+
+# --------------------------------------------------------------------------
+# invalid encodings
+# --------------------------------------------------------------------------
+def test_invalid_reasons():
+    prof = mkprof({0: lambda tpl, b: [1] * 4 + [2, 1, 1, 1, 1, 1]}, [0] * 4, n_tp=3, n_b=2, n_dp=3,
+                  G=4, Bg=8)
+    R = {"HEAD0": 1, "NSTAGE": 2, "PRANGE": 4, "GSTAGE": 8, "GSUM": 16, "DPMBS": 32, "TABLE": 64,
+         "MBS": 128, "HDR": 256}
+    ok = cand([2, 2], tpdp=[(1, 0), (0, 1)])
+    cases = [
+        (ok, ai.header(1, 2), 0),
+        ([ok[0] & 0xFE] + ok[1:], ai.header(1, 2), R["HEAD0"] | R["NSTAGE"]),
+        (ok, ai.header(1, 3), R["NSTAGE"]),
+        (cand([1, 1, 1, 1]), ai.header(0, 4), 0),
+        (cand([1, 1, 1, 1]), ai.header(0, 5), R["NSTAGE"] | R["PRANGE"]),
+        ([ok[0], ai.code(0, 0, 0, 0)] + ok[2:], ai.header(1, 2), R["GSTAGE"]),
+        (cand([2, 2], tpdp=[(1, 0), (1, 0)]), ai.header(1, 2), 0),
+        (cand([2, 2], tpdp=[(1, 0), (0, 0)]), ai.header(1, 2), R["GSUM"]),
+        (ok, ai.header(0, 2), R["DPMBS"]),
+        (cand([4], tpdp=[(0, 2)]), ai.header(2, 1), 0),
+        (cand([4], tpdp=[(0, 2)]), ai.header(3, 1), 0),
+        (cand([2, 2], tpdp=[(1, 0), (0, 1)]), ai.header(3, 2), R["TABLE"]),  # b = 3 >= n_b
+        (cand([4], tpdp=[(3, 0)]), ai.header(0, 1), R["TABLE"] | R["GSUM"]),
+        (ok, ai.header(4, 2), R["MBS"] | R["TABLE"]),
+        (ok, ai.header(1, 2) | (1 << 40), R["HDR"]),
+    ]
+    rows = [c[0] for c in cases]
+    hdrs = [c[1] for c in cases]
+    out = ev(prof, rows, hdrs)
+    for k, (_, _, exp) in enumerate(cases):
+        info = int(out["info"][k])
+        assert (info >> 18) == exp, (k, info >> 18, exp)
+        assert bool(info & oracle.INFO_INVALID) == bool(exp)
+        if exp:
+            assert out["iter"][k] == 0 and out["max_mem"][k] == 0
+
+
+# --------------------------------------------------------------------------
+# selection: brute force over the exhaustively enumerated toy spaces
+# --------------------------------------------------------------------------
+def _brute_min(out, offset=0):
+    info = out["info"].astype(np.int64)
+    valid = (info & oracle.INFO_INVALID) == 0
+    if not valid.any():
+        return (-1, 0, -1)
+    cls = ((info & oracle.INFO_OOM) != 0).astype(np.int64)
+    cost = np.where(cls == 1, out["max_mem"], out["iter"]).astype(np.uint64)
+    idx = np.arange(len(info), dtype=np.int64) + offset
+    keys = [(int(c), int(v), int(i)) for c, v, i, ok in zip(cls, cost, idx, valid) if ok]
+    return min(keys)
+
+
+@pytest.mark.parametrize("name,per_op", [("toy-a", True), ("toy-b", False)])
+def test_select_is_exhaustive_optimum(name, per_op):
+    prof = P.WORKLOADS[name]()
+    codes, hdr = ai.exhaustive(prof, per_op=per_op)
+    assert len(hdr) == {"toy-a": 388800, "toy-b": 1388544}[name]
+    out = oracle.evaluate(prof, codes, hdr, threads=8)
+    best = oracle.select(out)
+    assert best == _brute_min(out)
+    # the optimum is a feasible configuration, and nothing feasible is faster
+    info = out["info"]
+    feas = ((info & (oracle.INFO_INVALID | oracle.INFO_OOM)) == 0)
+    assert best[0] == 0 and best[1] == int(out["iter"][feas].min())
+    # sharded selection with global offsets gives the same winner (§8e)
+    parts = np.array_split(np.arange(len(hdr)), 5)
+    res = []
+    for part in parts:
+        sub = {k: v[part] for k, v in out.items()}
+        res.append(oracle.select(sub, global_offset=int(part[0])))
+    res = [r for r in res if r[2] >= 0]
+    assert min(res) == best
+
+
+def test_select_orders_classes_then_cost_then_index():
+    out = dict(iter=np.array([50, 10, 10, 0, 10], np.uint64),
+               max_mem=np.array([5, 1, 9, 0, 9], np.uint64),
+               info=np.array([oracle.INFO_OOM, oracle.INFO_OOM, 0, oracle.INFO_INVALID, 0], np.uint32))
+    assert oracle.select(out) == (0, 10, 2)
+    assert oracle.select(out, global_offset=100) == (0, 10, 102)
+    out["info"][2] = out["info"][4] = oracle.INFO_OOM
+    assert oracle.select(out) == (1, 1, 1)
+    out["info"][:] = oracle.INFO_INVALID
+    assert oracle.select(out)[2] == -1
