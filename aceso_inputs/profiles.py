@@ -128,15 +128,22 @@ class OpCost:
     workspace: float = 0.0
 
 
+ALLOC_GRAIN = 512  # PyTorch's caching allocator rounds every block to 512 bytes
+
+
+def _mem(x):
+    return int(math.ceil(x / ALLOC_GRAIN)) * ALLOC_GRAIN
+
+
 def _record(hw, c: OpCost, tp, n_dev):
     cross_tp = tp > 8
     f_comp = hw.launch_f + _mm_time(hw, c.flops) + c.mbytes / hw.hbm
     b_comp = hw.launch_b + 2.0 * _mm_time(hw, c.flops) + 1.5 * c.mbytes / hw.hbm
     f_comm = _allreduce(hw, c.tp_fwd_bytes, tp, cross_tp) + _allgather(hw, c.tp_fwd_gather, tp, cross_tp)
     b_comm = _allreduce(hw, c.tp_bwd_bytes, tp, cross_tp) + _allgather(hw, c.tp_fwd_gather, tp, cross_tp)
-    act = int(c.act)
-    keep = int(c.act * c.keep_frac)
-    peak = int(c.out + c.workspace)
+    act = _mem(c.act)
+    keep = min(act, _mem(c.act * c.keep_frac))
+    peak = _mem(c.out + c.workspace)
     reshard = _allgather(hw, c.inp, 2 * tp, 2 * tp > 8)
     p2p_bw = hw.nvlink if n_dev <= 8 else hw.ib
     p2p_f = hw.alpha + c.out / p2p_bw
@@ -170,22 +177,25 @@ def _build(name, ops, type_of, n_devices, global_batch, n_b_max, hw, bytes_per_p
                     rec[t, tpl, b] = _record(hw, type_of[k](1 << b, 1 << tpl), 1 << tpl, n_devices)
         s_op = rec[..., 0] + rec[..., 1] + rec[..., 2] + rec[..., 3] + rec[..., 0] + rec[..., 1]
         e_op = rec[..., 6] + rec[..., 4] - rec[..., 5]
-        if (rec.max() <= U32 and s_op.max() <= U32 and e_op.max() <= U32) or n_b == 1:
+        times = rec[..., [0, 1, 2, 3, 7, 8, 9]]
+        # library range rules (include/aceso.h): times < 2^32 ns; memory < 2^32 allocator grains
+        if (times.max() <= U32 and s_op.max() <= U32 and e_op.max() // ALLOC_GRAIN <= U32
+                and rec[..., 4].max() // ALLOC_GRAIN <= U32) or n_b == 1:
             break
         n_b -= 1
-    assert rec.max() <= U32, name
+    assert rec[..., [0, 1, 2, 3, 7, 8, 9]].max() <= U32, name
     wmem = np.zeros((T, n_tp, 2), dtype=np.int64)
     dps = np.zeros((T, n_tp, n_dp), dtype=np.int64)
     for t, k in enumerate(keys):
         for tpl in range(n_tp):
             prm = type_of[k](1, 1 << tpl).params
-            wmem[t, tpl, 0] = int(prm * bytes_per_param)
-            wmem[t, tpl, 1] = int(prm * opt_per_param)
+            wmem[t, tpl, 0] = _mem(prm * bytes_per_param)
+            wmem[t, tpl, 1] = _mem(prm * opt_per_param)
             for dpl in range(n_dp):
                 dp = 1 << dpl
                 dps[t, tpl, dpl] = _ns(_allreduce(hw, prm * grad_bytes_per_param, dp,
                                                   (1 << tpl) * dp > 8))
-    assert wmem.max() <= U32 and dps.max() <= U32, name
+    assert wmem.sum(-1).max() // ALLOC_GRAIN <= U32 and dps.max() <= U32, name
     return Profile(name=name, op_type=op_type, type_names=[str(k) for k in keys], rec=rec, wmem=wmem,
                    dps=dps, n_devices=n_devices, mem_capacity=int(mem_capacity),
                    global_batch=int(global_batch))
@@ -276,7 +286,7 @@ def _xf_ops(h, a, ff, inner, s, V, dtype_b=2.0, s_kv=None):
     def emb(b, tp):
         t = b * s
         return OpCost(mbytes=2 * t * h * dtype_b, tp_fwd_bytes=t * h * dtype_b, act=t * 4.0,
-                      keep_frac=1.0, out=t * h * dtype_b, inp=t * 4.0, params=V * h / tp + s * h)
+                      keep_frac=1.0, out=t * h * dtype_b, inp=t * 4.0, params=V * h / tp)
 
     def head(b, tp):
         t = b * s

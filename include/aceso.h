@@ -84,10 +84,14 @@ typedef struct aceso_ctx aceso_ctx; /* opaque; owned by the library */
 
 /* Validates and packs the profile, uploads it to `cuda_device` and returns a
  * context. Synchronous. Range rules (ACESO_ERANGE on violation):
- *  - every rec/wmem/dps value in [0, 2^32);  keep <= act;  peak + act - keep < 2^32;
+ *  - time fields (ns) and dps in [0, 2^32); memory fields (act, keep, peak) and
+ *    each wmem entry in [0, 2^40];  keep <= act;
  *  - fwd_comp+fwd_comm+bwd_comp+bwd_comm + (fwd_comp+fwd_comm) < 2^32;
- *  - model-wide: L * max-per-op cost * Bg < 2^62 for time and memory, so that
- *    every iteration time and stage memory is < 2^62 (exact packed keys).
+ *  - memory is packed exactly in units of 2^m bytes, m = the largest power of two
+ *    (<= 16) dividing every memory value; act, peak + act - keep and
+ *    param+optimizer bytes must each be < 2^(32+m);
+ *  - model-wide: a conservative bound on every iteration time and stage memory
+ *    (L * max per-op cost * (Bg + 1)) is < 2^62, so packed keys are exact.
  * Returns ACESO_OK and sets *out, or a negative status (see aceso_last_error). */
 int aceso_load_profile(const aceso_profile_desc *desc, int cuda_device, aceso_ctx **out);
 

@@ -1,0 +1,10 @@
+"""B200-native batched evaluator of Aceso's performance/memory model (EuroSys '24).
+
+Public API (names follow include/aceso.h): Context (aceso_load_profile/aceso_free),
+Context.eval (aceso_eval), Context.select (aceso_select), Context.pack_rowmajor
+(aceso_pack_rowmajor), decode_key (aceso_decode_key), dist.global_select (NCCL
+all-reduce MIN of the packed key).
+"""
+from .api import AcesoError, Context, Outputs, Selection, as_u32, as_u64, decode_key, tiled_bytes, \
+    upload_candidates, version  # noqa: F401
+from .buildlib import LIB, build  # noqa: F401

@@ -1,0 +1,211 @@
+"""Python binding of libaceso (same names as the C-ABI; argument marshalling only).
+
+Every step of the evaluation path runs in the sm_100a kernels of libaceso.so;
+PyTorch only provides device memory and streams. There is no CPU fallback: if
+the library or a CUDA device is missing, these calls raise.
+
+Unsigned 64-bit device arrays are carried in torch.int64 tensors (same bits);
+`as_u64` / `as_u32` view them as numpy unsigned arrays on the host.
+"""
+from __future__ import annotations
+
+import ctypes
+import dataclasses
+
+import numpy as np
+import torch
+
+from . import _lib as L
+
+
+class AcesoError(RuntimeError):
+    pass
+
+
+def _check(rc, what):
+    if rc != L.ACESO_OK:
+        msg = L.load().aceso_last_error().decode()
+        raise AcesoError(f"{what} failed ({rc}): {msg}")
+
+
+def _ptr(t):
+    return None if t is None else ctypes.c_void_p(t.data_ptr())
+
+
+def _stream(stream):
+    if stream is None:
+        stream = torch.cuda.current_stream()
+    return ctypes.c_void_p(stream.cuda_stream)
+
+
+def version():
+    return L.load().aceso_version().decode()
+
+
+def tiled_bytes(n, n_ops):
+    return int(L.load().aceso_tiled_bytes(int(n), int(n_ops)))
+
+
+def as_u64(t):
+    return t.detach().cpu().numpy().view(np.uint64)
+
+
+def as_u32(t):
+    return t.detach().cpu().numpy().view(np.uint32)
+
+
+@dataclasses.dataclass
+class Outputs:
+    """Device output arrays of one batch (SoA). Stage arrays are [p_max, n]."""
+    iter_ns: torch.Tensor
+    max_mem: torch.Tensor
+    info: torch.Tensor
+    stage_T: torch.Tensor | None = None
+    stage_mem: torch.Tensor | None = None
+    stage_comp: torch.Tensor | None = None
+    stage_comm: torch.Tensor | None = None
+    p_max: int = 0
+
+    def c_struct(self):
+        return L.EvalOut(_ptr(self.iter_ns), _ptr(self.max_mem), _ptr(self.info), _ptr(self.stage_T),
+                         _ptr(self.stage_mem), _ptr(self.stage_comp), _ptr(self.stage_comm),
+                         int(self.p_max))
+
+
+@dataclasses.dataclass
+class Selection:
+    cls: int          # 0 feasible, 1 OOM, -1 nothing valid
+    cost: int         # iteration time (cls 0) or max stage memory (cls 1)
+    index: int        # global candidate index, -1 if nothing valid
+    key: int          # packed all-reduce key
+
+    @classmethod
+    def from_buffer(cls, sel: torch.Tensor):
+        raw = sel[:32].cpu().numpy()
+        key = int(raw[0:8].view(np.int64)[0])
+        cc = int(raw[8:16].view(np.uint64)[0])
+        idx = int(raw[16:24].view(np.int64)[0])
+        if idx < 0:
+            return cls(-1, 0, -1, key)
+        return cls(cc >> 62, cc & ((1 << 62) - 1), idx, key)
+
+
+class Context:
+    """aceso_load_profile / aceso_free: a packed, device-resident op-cost profile."""
+
+    def __init__(self, profile, device: int = 0):
+        lib = L.load()
+        self.device = int(device)
+        self.profile = profile
+        self._keep = [np.ascontiguousarray(profile.op_type, dtype=np.uint16),
+                      np.ascontiguousarray(profile.rec, dtype=np.int64),
+                      np.ascontiguousarray(profile.wmem, dtype=np.int64),
+                      np.ascontiguousarray(profile.dps, dtype=np.int64)]
+        ot, rec, wm, dps = self._keep
+        desc = L.ProfileDesc(int(ot.shape[0]), int(rec.shape[0]), int(rec.shape[1]), int(dps.shape[2]),
+                             int(rec.shape[2]), int(profile.n_devices), ot.ctypes.data, rec.ctypes.data,
+                             wm.ctypes.data, dps.ctypes.data, int(profile.mem_capacity),
+                             int(profile.global_batch))
+        h = ctypes.c_void_p()
+        _check(lib.aceso_load_profile(ctypes.byref(desc), self.device, ctypes.byref(h)),
+               "aceso_load_profile")
+        self._h = h
+        self.n_ops = int(ot.shape[0])
+        self.n_devices = int(profile.n_devices)
+        self._dev = torch.device("cuda", self.device)
+
+    def close(self):
+        if getattr(self, "_h", None):
+            L.load().aceso_free(self._h)
+            self._h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    # -- buffers --------------------------------------------------------------
+    def alloc_outputs(self, n: int, full: bool = False) -> Outputs:
+        d = self._dev
+        o = Outputs(torch.empty(n, dtype=torch.int64, device=d), torch.empty(n, dtype=torch.int64, device=d),
+                    torch.empty(n, dtype=torch.int32, device=d))
+        if full:
+            pm = self.n_devices
+            o.p_max = pm
+            o.stage_T = torch.zeros((pm, n), dtype=torch.int64, device=d)
+            o.stage_mem = torch.zeros((pm, n), dtype=torch.int64, device=d)
+            o.stage_comp = torch.zeros((pm, n), dtype=torch.int64, device=d)
+            o.stage_comm = torch.zeros((pm, n), dtype=torch.int64, device=d)
+        return o
+
+    def alloc_select(self, n: int = 0) -> torch.Tensor:
+        nb = int(L.load().aceso_select_buf_bytes(self._h, int(n)))
+        return torch.zeros(nb, dtype=torch.uint8, device=self._dev)
+
+    def alloc_tiled(self, n: int) -> torch.Tensor:
+        return torch.zeros(tiled_bytes(n, self.n_ops), dtype=torch.uint8, device=self._dev)
+
+    # -- C-ABI calls ------------------------------------------------------------
+    def pack_rowmajor(self, codes: torch.Tensor, tiled: torch.Tensor | None = None, stream=None):
+        """aceso_pack_rowmajor: device row-major [n, L] uint8 -> tiled layout."""
+        assert codes.is_cuda and codes.dtype == torch.uint8 and codes.dim() == 2
+        n = int(codes.shape[0])
+        if tiled is None:
+            tiled = self.alloc_tiled(n)
+        codes = codes.contiguous()
+        _check(L.load().aceso_pack_rowmajor(_ptr(codes), n, int(codes.shape[1]), _ptr(tiled),
+                                            _stream(stream)), "aceso_pack_rowmajor")
+        return tiled
+
+    def eval(self, codes: torch.Tensor, hdr: torch.Tensor, n: int | None = None, global_offset: int = 0,
+             n_total: int | None = None, summary: bool = True, full: bool = False, select: bool = True,
+             out: Outputs | None = None, sel: torch.Tensor | None = None, stream=None):
+        """aceso_eval on tiled device codes and int64 device headers.
+
+        Returns (out, sel): the output arrays (or None) and the select buffer (or None)."""
+        n = int(hdr.shape[0]) if n is None else int(n)
+        n_total = global_offset + n if n_total is None else int(n_total)
+        flags = (L.OUT_SUMMARY if summary else 0) | (L.OUT_FULL if full else 0) | (L.FUSED_SELECT if select else 0)
+        if (summary or full) and out is None:
+            out = self.alloc_outputs(n, full=full)
+        if select and sel is None:
+            sel = self.alloc_select(n)
+        cs = out.c_struct() if out is not None else None
+        rc = L.load().aceso_eval(self._h, _ptr(codes), _ptr(hdr), n, int(global_offset), n_total, flags,
+                                 ctypes.byref(cs) if cs is not None else None, _ptr(sel), _stream(stream))
+        _check(rc, "aceso_eval")
+        return out, sel
+
+    def select(self, out: Outputs, n: int | None = None, global_offset: int = 0,
+               n_total: int | None = None, sel: torch.Tensor | None = None, stream=None):
+        """aceso_select: argmin over an already written summary."""
+        n = int(out.iter_ns.shape[0]) if n is None else int(n)
+        n_total = global_offset + n if n_total is None else int(n_total)
+        if sel is None:
+            sel = self.alloc_select(n)
+        cs = out.c_struct()
+        _check(L.load().aceso_select(self._h, ctypes.byref(cs), n, int(global_offset), n_total, _ptr(sel),
+                                     _stream(stream)), "aceso_select")
+        return sel
+
+
+def decode_key(key: int, n_total: int):
+    """aceso_decode_key -> (cls, cost, index, saturated)."""
+    cls = ctypes.c_int()
+    cost = ctypes.c_uint64()
+    idx = ctypes.c_int64()
+    sat = ctypes.c_int()
+    _check(L.load().aceso_decode_key(int(key), int(n_total), ctypes.byref(cls), ctypes.byref(cost),
+                                     ctypes.byref(idx), ctypes.byref(sat)), "aceso_decode_key")
+    return cls.value, cost.value, idx.value, bool(sat.value)
+
+
+def upload_candidates(codes_tiled: np.ndarray, hdr: np.ndarray, device=0, pin=False):
+    """Host tiled codes + uint64 headers -> device tensors (tiled uint8, int64 headers)."""
+    c = torch.from_numpy(np.ascontiguousarray(codes_tiled, dtype=np.uint8))
+    h = torch.from_numpy(np.ascontiguousarray(hdr, dtype=np.uint64).view(np.int64))
+    if pin:
+        c, h = c.pin_memory(), h.pin_memory()
+    dev = torch.device("cuda", device)
+    return c.to(dev, non_blocking=pin), h.to(dev, non_blocking=pin)

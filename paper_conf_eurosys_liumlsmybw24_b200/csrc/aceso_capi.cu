@@ -1,0 +1,391 @@
+// aceso_capi.cu — the C-ABI of libaceso (include/aceso.h): profile validation and
+// packing, launches of the sm_100a kernels, error reporting. No computation of
+// the model happens on the host: every step of the evaluation path runs in the
+// kernels of eval_kernel.cuh / aux_kernels.cuh.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <string>
+#include <vector>
+
+#include "aux_kernels.cuh"
+#include "common.cuh"
+#include "eval_kernel.cuh"
+
+using namespace aceso;
+
+namespace {
+
+thread_local std::string g_err;
+
+int fail(int code, const char *fmt, ...) {
+  char buf[512];
+  va_list ap;
+  va_start(ap, fmt);
+  vsnprintf(buf, sizeof(buf), fmt, ap);
+  va_end(ap);
+  g_err = buf;
+  return code;
+}
+
+#define CUDA_TRY(expr)                                                                     \
+  do {                                                                                     \
+    cudaError_t e_ = (expr);                                                               \
+    if (e_ != cudaSuccess)                                                                 \
+      return fail(ACESO_ECUDA, "%s failed: %s", #expr, cudaGetErrorString(e_));            \
+  } while (0)
+
+template <uint32_t M>
+void *kernel_ptr() {
+  return reinterpret_cast<void *>(&eval_kernel<M>);
+}
+
+void *eval_kernel_for(uint32_t mode) {
+  switch (mode) {
+    case 1: return kernel_ptr<1>();
+    case 2: return kernel_ptr<2>();
+    case 3: return kernel_ptr<3>();
+    case 4: return kernel_ptr<4>();
+    case 5: return kernel_ptr<5>();
+    case 6: return kernel_ptr<6>();
+    case 7: return kernel_ptr<7>();
+    default: return nullptr;
+  }
+}
+
+uint32_t bitlen(uint64_t v) {
+  uint32_t b = 0;
+  while (v) { b++; v >>= 1; }
+  return b;
+}
+
+}  // namespace
+
+struct aceso_ctx {
+  int device;
+  int sms;
+  int32_t L, T, n_tp, n_dp, n_b, G;
+  uint64_t Bg, C;
+  uint32_t mem_shift;
+  Tables tab;
+  void *d_blob;
+  int max_ctas[8];  // per mode: resident CTAs (occupancy x SMs)
+  size_t smem[8];
+};
+
+extern "C" {
+
+const char *aceso_last_error(void) { return g_err.c_str(); }
+const char *aceso_version(void) { return "aceso-b200 0.1 (sm_100a)"; }
+
+size_t aceso_tiled_bytes(int64_t n, int32_t n_ops) {
+  if (n < 0 || n_ops < 1) return 0;
+  return (size_t)((n + 31) / 32) * (size_t)((n_ops + 15) / 16) * 512;
+}
+
+int aceso_load_profile(const aceso_profile_desc *d, int cuda_device, aceso_ctx **out) {
+  if (!d || !out) return fail(ACESO_EINVAL, "null argument");
+  *out = nullptr;
+  if (d->n_ops < 1 || d->n_ops > kMaxOps) return fail(ACESO_EINVAL, "n_ops %d outside [1, %d]", d->n_ops, kMaxOps);
+  if (d->n_types < 1 || d->n_types > 4096) return fail(ACESO_EINVAL, "n_types %d outside [1, 4096]", d->n_types);
+  if (d->n_tp < 1 || d->n_tp > 8 || d->n_dp < 1 || d->n_dp > 8)
+    return fail(ACESO_EINVAL, "n_tp/n_dp must be in [1, 8]");
+  if (d->n_b < 1 || d->n_b > 16) return fail(ACESO_EINVAL, "n_b %d outside [1, 16]", d->n_b);
+  if (d->n_devices < 1 || d->n_devices > 255) return fail(ACESO_EINVAL, "n_devices outside [1, 255]");
+  if (d->global_batch < 1 || d->global_batch > (1ll << 31)) return fail(ACESO_EINVAL, "global_batch outside [1, 2^31]");
+  if (d->mem_capacity < 0) return fail(ACESO_EINVAL, "negative mem_capacity");
+  if (!d->op_type || !d->rec || !d->wmem || !d->dps) return fail(ACESO_EINVAL, "null table");
+  const int L = d->n_ops, T = d->n_types, NT = d->n_tp, ND = d->n_dp, NB = d->n_b;
+  for (int j = 0; j < L; ++j)
+    if (d->op_type[j] >= T) return fail(ACESO_EINVAL, "op_type[%d] = %d >= n_types", j, d->op_type[j]);
+
+  const uint64_t U32 = 0xffffffffull;
+  auto R = [&](int t, int tp, int b, int f) { return d->rec[(((int64_t)t * NT + tp) * NB + b) * ACESO_REC_FIELDS + f]; };
+  uint64_t maxSop = 0, maxRes = 0, maxP2P = 0, maxA = 0, maxE = 0, maxW = 0, maxD = 0;
+  for (int t = 0; t < T; ++t)
+    for (int tp = 0; tp < NT; ++tp) {
+      for (int b = 0; b < NB; ++b) {
+        for (int f = 0; f < ACESO_REC_FIELDS; ++f) {
+          int64_t v = R(t, tp, b, f);
+          const bool memf = (f == ACESO_F_ACT || f == ACESO_F_KEEP || f == ACESO_F_PEAK);
+          if (v < 0 || (uint64_t)v > (memf ? (1ull << 40) : U32))
+            return fail(ACESO_ERANGE, "rec[%d][%d][%d][%d] = %lld out of range", t, tp, b, f, (long long)v);
+        }
+        uint64_t fc = R(t, tp, b, 0), fm = R(t, tp, b, 1), bc = R(t, tp, b, 2), bm = R(t, tp, b, 3);
+        uint64_t act = R(t, tp, b, 4), keep = R(t, tp, b, 5), peak = R(t, tp, b, 6);
+        if (keep > act) return fail(ACESO_ERANGE, "keep > act at rec[%d][%d][%d]", t, tp, b);
+        uint64_t s1 = 2 * (fc + fm) + bc + bm;
+        uint64_t e1 = peak + act - keep;
+        if (s1 > U32) return fail(ACESO_ERANGE, "recomputed op time > 2^32-1 at rec[%d][%d][%d]", t, tp, b);
+        maxSop = std::max(maxSop, s1);
+        maxRes = std::max(maxRes, (uint64_t)R(t, tp, b, 7));
+        maxP2P = std::max(maxP2P, (uint64_t)std::max(R(t, tp, b, 8), R(t, tp, b, 9)));
+        maxA = std::max(maxA, act);
+        maxE = std::max(maxE, e1);
+      }
+      int64_t pg = d->wmem[((int64_t)t * NT + tp) * 2], op = d->wmem[((int64_t)t * NT + tp) * 2 + 1];
+      if (pg < 0 || op < 0 || pg > (1ll << 40) || op > (1ll << 40)) return fail(ACESO_ERANGE, "wmem[%d][%d] not in [0, 2^40]", t, tp);
+      maxW = std::max(maxW, (uint64_t)(pg + op));
+      for (int dp = 0; dp < ND; ++dp) {
+        int64_t v = d->dps[((int64_t)t * NT + tp) * ND + dp];
+        if (v < 0 || (uint64_t)v > U32) return fail(ACESO_ERANGE, "dps[%d][%d][%d] not in [0, 2^32)", t, tp, dp);
+        maxD = std::max(maxD, (uint64_t)v);
+      }
+    }
+  // memory fields are packed in units of 2^ms bytes (exact): ms = common trailing zeros
+  uint32_t ms = 16;
+  {
+    auto tz = [&](int64_t v) { if (v != 0) ms = std::min<uint32_t>(ms, (uint32_t)__builtin_ctzll((uint64_t)v)); };
+    for (int t = 0; t < T; ++t)
+      for (int tp = 0; tp < NT; ++tp) {
+        for (int b = 0; b < NB; ++b) { tz(R(t, tp, b, 4)); tz(R(t, tp, b, 5)); tz(R(t, tp, b, 6)); }
+        tz(d->wmem[((int64_t)t * NT + tp) * 2]);
+        tz(d->wmem[((int64_t)t * NT + tp) * 2 + 1]);
+      }
+    if ((maxA >> ms) > U32) return fail(ACESO_ERANGE, "act exceeds 2^32 units of 2^%u bytes", ms);
+    if ((maxE >> ms) > U32) return fail(ACESO_ERANGE, "peak + act - keep exceeds 2^32 units of 2^%u bytes", ms);
+    if ((maxW >> ms) > U32) return fail(ACESO_ERANGE, "param+optimizer bytes exceed 2^32 units of 2^%u bytes", ms);
+  }
+  {
+    // model-wide bounds: every iteration time / stage memory < 2^62 (exact keys)
+    typedef unsigned __int128 u128;
+    const u128 lim = (u128)1 << 62;
+    u128 tb = ((u128)L * (maxSop + maxRes + maxD) + (u128)2 * d->n_devices * maxP2P) * ((u128)d->global_batch + 1);
+    u128 mb = (u128)L * maxW + (u128)d->global_batch * L * maxA + maxE;
+    if (tb >= lim) return fail(ACESO_ERANGE, "iteration-time bound exceeds 2^62");
+    if (mb >= lim) return fail(ACESO_ERANGE, "memory bound exceeds 2^62");
+  }
+
+  // ---- pack tables ----
+  const uint32_t S = kTypeStride;
+  const uint32_t bytesR = (uint32_t)NB * NT * T * S;
+  const uint32_t bytesD = (uint32_t)NT * T * S;
+  const uint32_t bytesT = (uint32_t)((L + 15) / 16) * 64;
+  const uint32_t bytesF = ((uint32_t)NB * NT * T * 8 + 15) / 16 * 16;
+  const uint32_t bytesK = (uint32_t)NB * NT * T * 16;
+  Tables tab;
+  tab.offR = 0;
+  tab.offD = bytesR;
+  tab.offT = tab.offD + bytesD;
+  tab.offF = tab.offT + bytesT;
+  tab.bytes = tab.offF;
+  tab.bytes_full = tab.offF + bytesF;
+  tab.offK = tab.bytes_full;
+  if (tab.bytes_full > 180u * 1024u) return fail(ACESO_EINVAL, "packed tables of %u bytes exceed shared memory", tab.bytes_full);
+  const uint32_t blob_bytes = tab.offK + bytesK;
+  std::vector<uint32_t> blob(blob_bytes / 4, 0u);
+  for (int b = 0; b < NB; ++b)
+    for (int tp = 0; tp < NT; ++tp)
+      for (int t = 0; t < T; ++t) {
+        const uint32_t rt = (uint32_t)(b * NT + tp) * T + t;  // (run, type) index
+        const uint32_t run = rt * S / 4;
+        uint64_t fc = R(t, tp, b, 0), fm = R(t, tp, b, 1), bc = R(t, tp, b, 2), bm = R(t, tp, b, 3);
+        uint64_t act = R(t, tp, b, 4), keep = R(t, tp, b, 5), peak = R(t, tp, b, 6);
+        uint64_t W = (uint64_t)d->wmem[((int64_t)t * NT + tp) * 2] + (uint64_t)d->wmem[((int64_t)t * NT + tp) * 2 + 1];
+        for (int rc = 0; rc < 2; ++rc) {
+          uint32_t *r = &blob[(tab.offR / 4) + run + rc * 4];
+          r[0] = (uint32_t)(fc + fm + bc + bm + (rc ? fc + fm : 0));
+          r[1] = (uint32_t)((rc ? keep : act) >> ms);
+          r[2] = (uint32_t)((peak + (rc ? act - keep : 0)) >> ms);
+          r[3] = (uint32_t)(W >> ms);
+          blob[(tab.offF / 4) + rt * 2 + rc] = (uint32_t)(fc + bc + (rc ? fc : 0));
+        }
+        uint32_t *k = &blob[(tab.offK / 4) + rt * 4];
+        k[0] = (uint32_t)R(t, tp, b, 7);
+        k[1] = (uint32_t)R(t, tp, b, 8);
+        k[2] = (uint32_t)R(t, tp, b, 9);
+      }
+  for (int j = 0; j < L; ++j) blob[tab.offT / 4 + j] = (uint32_t)d->op_type[j] * S;
+  for (int tp = 0; tp < NT; ++tp)
+    for (int t = 0; t < T; ++t)
+      for (int dp = 0; dp < ND; ++dp)
+        blob[(tab.offD + ((uint32_t)tp * T + t) * S) / 4 + dp] = (uint32_t)d->dps[((int64_t)t * NT + tp) * ND + dp];
+
+  // ---- device ----
+  int ndev = 0;
+  if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev == 0) return fail(ACESO_ENODEV, "no CUDA device");
+  if (cuda_device < 0 || cuda_device >= ndev || cuda_device >= 64) return fail(ACESO_EINVAL, "bad device %d", cuda_device);
+  int prev_dev = 0;
+  CUDA_TRY(cudaGetDevice(&prev_dev));
+  CUDA_TRY(cudaSetDevice(cuda_device));
+  cudaDeviceProp prop;
+  CUDA_TRY(cudaGetDeviceProperties(&prop, cuda_device));
+  if (prop.major != 10) {
+    cudaSetDevice(prev_dev);
+    return fail(ACESO_ENODEV, "device %d is sm_%d%d; libaceso is built for sm_100a", cuda_device, prop.major, prop.minor);
+  }
+  aceso_ctx *ctx = new aceso_ctx();
+  ctx->device = cuda_device;
+  ctx->sms = prop.multiProcessorCount;
+  ctx->L = L; ctx->T = T; ctx->n_tp = NT; ctx->n_dp = ND; ctx->n_b = NB; ctx->G = d->n_devices;
+  ctx->Bg = (uint64_t)d->global_batch;
+  ctx->C = (uint64_t)d->mem_capacity;
+  ctx->tab = tab;
+  ctx->mem_shift = ms;
+  ctx->d_blob = nullptr;
+  int rc = ACESO_OK;
+  do {
+    cudaStream_t st;
+    if (cudaStreamCreateWithFlags(&st, cudaStreamNonBlocking) != cudaSuccess) { rc = fail(ACESO_ECUDA, "stream create"); break; }
+    cudaError_t e = cudaMalloc(&ctx->d_blob, blob_bytes);
+    if (e == cudaSuccess) e = cudaMemcpyAsync(ctx->d_blob, blob.data(), blob_bytes, cudaMemcpyHostToDevice, st);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(st);
+    cudaStreamDestroy(st);
+    if (e != cudaSuccess) { rc = fail(e == cudaErrorMemoryAllocation ? ACESO_ENOMEM : ACESO_ECUDA, "upload: %s", cudaGetErrorString(e)); break; }
+    for (uint32_t mode = 1; mode < 8; ++mode) {
+      const size_t smem = ((mode & ACESO_OUT_FULL) ? tab.bytes_full : tab.bytes) + kRingBytesPerCta;
+      ctx->smem[mode] = smem;
+      void *k = eval_kernel_for(mode);
+      e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+      int occ = 0;
+      if (e == cudaSuccess) e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k, kThreads, smem);
+      if (e != cudaSuccess || occ < 1) { rc = fail(ACESO_ECUDA, "kernel setup (mode %u, %zu B smem): %s", mode, smem, cudaGetErrorString(e)); break; }
+      ctx->max_ctas[mode] = occ * ctx->sms;
+    }
+  } while (0);
+  cudaSetDevice(prev_dev);
+  if (rc != ACESO_OK) {
+    if (ctx->d_blob) cudaFree(ctx->d_blob);
+    delete ctx;
+    return rc;
+  }
+  *out = ctx;
+  return ACESO_OK;
+}
+
+void aceso_free(aceso_ctx *ctx) {
+  if (!ctx) return;
+  int prev = 0;
+  cudaGetDevice(&prev);
+  cudaSetDevice(ctx->device);
+  cudaFree(ctx->d_blob);
+  cudaSetDevice(prev);
+  delete ctx;
+}
+
+size_t aceso_select_buf_bytes(const aceso_ctx *ctx, int64_t n) {
+  (void)n;
+  if (!ctx) return 0;
+  int m = 0;
+  for (int k = 1; k < 8; ++k) m = std::max(m, ctx->max_ctas[k]);
+  m = std::max(m, 4 * ctx->sms);  // select kernel grid
+  return (size_t)kSelPartialOff + 16 * (size_t)m;
+}
+
+int aceso_eval(aceso_ctx *ctx, const uint8_t *d_codes, const uint64_t *d_hdr, int64_t n,
+               int64_t global_offset, int64_t n_total, uint32_t flags, const aceso_eval_out *out,
+               void *d_sel, void *stream) {
+  if (!ctx) return fail(ACESO_EINVAL, "null context");
+  if (n < 0 || global_offset < 0 || n_total < global_offset + n) return fail(ACESO_EINVAL, "bad n / global_offset / n_total");
+  if (n_total >= (1ll << 40)) return fail(ACESO_EINVAL, "n_total >= 2^40");
+  const uint32_t mode = flags & 7u;
+  if (mode == 0 || (flags & ~7u)) return fail(ACESO_EINVAL, "bad flags 0x%x", flags);
+  if (n > 0 && (!d_codes || !d_hdr)) return fail(ACESO_EINVAL, "null codes/headers");
+  if ((mode & (ACESO_OUT_SUMMARY | ACESO_OUT_FULL)) && !out) return fail(ACESO_EINVAL, "null outputs");
+  if ((mode & ACESO_OUT_SUMMARY) && n > 0 && (!out->iter_ns || !out->max_mem || !out->info)) return fail(ACESO_EINVAL, "null summary array");
+  if (mode & ACESO_OUT_FULL) {
+    if (out->p_max < ctx->G) return fail(ACESO_EINVAL, "p_max %d < n_devices %d", out->p_max, ctx->G);
+    if (n > 0 && (!out->stage_T || !out->stage_mem || !out->stage_comp || !out->stage_comm)) return fail(ACESO_EINVAL, "null stage array");
+  }
+  if ((mode & ACESO_FUSED_SELECT) && !d_sel) return fail(ACESO_EINVAL, "null select buffer");
+  if (((uintptr_t)d_codes & 15) != 0) return fail(ACESO_EINVAL, "codes not 16-byte aligned");
+
+  EvalParams P;
+  memset(&P, 0, sizeof(P));
+  P.codes = reinterpret_cast<const uint4 *>(d_codes);
+  P.hdr = d_hdr;
+  P.n = n;
+  P.gofs = global_offset;
+  P.n_tiles = (n + 31) / 32;
+  P.L = ctx->L;
+  P.nch = (ctx->L + 15) / 16;
+  P.T = ctx->T;
+  P.n_tp = ctx->n_tp;
+  P.n_dp = ctx->n_dp;
+  P.n_b = ctx->n_b;
+  P.G = ctx->G;
+  P.Bg = ctx->Bg;
+  P.C = ctx->C;
+  P.mem_shift = ctx->mem_shift;
+  P.blob = reinterpret_cast<const uint4 *>(ctx->d_blob);
+  P.tab = ctx->tab;
+  if (out) {
+    P.iter_ns = out->iter_ns;
+    P.max_mem = out->max_mem;
+    P.info = out->info;
+    P.stage_T = out->stage_T;
+    P.stage_mem = out->stage_mem;
+    P.stage_comp = out->stage_comp;
+    P.stage_comm = out->stage_comm;
+    P.p_max = out->p_max;
+  }
+  P.sel = reinterpret_cast<unsigned char *>(d_sel);
+  P.n_total = n_total;
+  P.ib = std::max(1u, bitlen((uint64_t)n_total));
+
+  const int64_t need = (P.n_tiles + kWarps - 1) / kWarps;
+  int grid = (int)std::max<int64_t>(1, std::min<int64_t>(need, ctx->max_ctas[mode]));
+  int prev = 0;
+  CUDA_TRY(cudaGetDevice(&prev));
+  if (prev != ctx->device) CUDA_TRY(cudaSetDevice(ctx->device));
+  void *args[] = {&P};
+  cudaError_t e = cudaLaunchKernel(eval_kernel_for(mode), dim3(grid), dim3(kThreads), args, ctx->smem[mode],
+                                   reinterpret_cast<cudaStream_t>(stream));
+  if (prev != ctx->device) cudaSetDevice(prev);
+  if (e != cudaSuccess) return fail(ACESO_ECUDA, "eval launch: %s", cudaGetErrorString(e));
+  return ACESO_OK;
+}
+
+int aceso_select(aceso_ctx *ctx, const aceso_eval_out *out, int64_t n, int64_t global_offset,
+                 int64_t n_total, void *d_sel, void *stream) {
+  if (!ctx || !d_sel) return fail(ACESO_EINVAL, "null argument");
+  if (n < 0 || global_offset < 0 || n_total < global_offset + n) return fail(ACESO_EINVAL, "bad n / global_offset / n_total");
+  if (n > 0 && (!out || !out->iter_ns || !out->max_mem || !out->info)) return fail(ACESO_EINVAL, "null summary");
+  const int64_t blocks = (n + 255) / 256;
+  const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(blocks, 4 * ctx->sms));
+  int prev = 0;
+  CUDA_TRY(cudaGetDevice(&prev));
+  if (prev != ctx->device) CUDA_TRY(cudaSetDevice(ctx->device));
+  select_kernel<<<grid, 256, 0, reinterpret_cast<cudaStream_t>(stream)>>>(
+      n ? out->iter_ns : nullptr, n ? out->max_mem : nullptr, n ? out->info : nullptr, n, global_offset,
+      reinterpret_cast<unsigned char *>(d_sel), n_total, std::max(1u, bitlen((uint64_t)n_total)));
+  cudaError_t e = cudaGetLastError();
+  if (prev != ctx->device) cudaSetDevice(prev);
+  if (e != cudaSuccess) return fail(ACESO_ECUDA, "select launch: %s", cudaGetErrorString(e));
+  return ACESO_OK;
+}
+
+int aceso_decode_key(int64_t key, int64_t n_total, int *cls, uint64_t *cost, int64_t *index,
+                     int *saturated) {
+  if (!cls || !cost || !index || !saturated || n_total < 0) return fail(ACESO_EINVAL, "bad argument");
+  if (key == INT64_MAX || key < 0) {
+    *cls = -1; *cost = 0; *index = -1; *saturated = 0;
+    return ACESO_OK;
+  }
+  const uint32_t ib = std::max(1u, bitlen((uint64_t)n_total));
+  const uint64_t k = (uint64_t)key;
+  const uint64_t cmax = (1ull << (62 - ib)) - 1;
+  *cls = (int)(k >> 62);
+  *cost = (k & ((1ull << 62) - 1)) >> ib;
+  *index = (int64_t)(k & ((1ull << ib) - 1));
+  *saturated = *cost == cmax;
+  return ACESO_OK;
+}
+
+int aceso_pack_rowmajor(const uint8_t *d_rowmajor, int64_t n, int32_t n_ops, uint8_t *d_tiled,
+                        void *stream) {
+  if (n < 0 || n_ops < 1 || (n > 0 && (!d_rowmajor || !d_tiled))) return fail(ACESO_EINVAL, "bad argument");
+  if (((uintptr_t)d_tiled & 15) != 0) return fail(ACESO_EINVAL, "tiled buffer not 16-byte aligned");
+  if (n == 0) return ACESO_OK;
+  const int64_t total_vec = (int64_t)aceso_tiled_bytes(n, n_ops) / 16;
+  const int grid = (int)std::min<int64_t>((total_vec + 255) / 256, 148 * 16);
+  pack_kernel<<<grid, 256, 0, reinterpret_cast<cudaStream_t>(stream)>>>(d_rowmajor, n, n_ops, reinterpret_cast<uint4 *>(d_tiled), total_vec);
+  cudaError_t e = cudaGetLastError();
+  if (e != cudaSuccess) return fail(ACESO_ECUDA, "pack launch: %s", cudaGetErrorString(e));
+  return ACESO_OK;
+}
+
+}  // extern "C"

@@ -1,0 +1,155 @@
+// common.cuh — shared device-side definitions of libaceso (sm_100a).
+//
+// Packed profile tables (built on the host by aceso_load_profile from the
+// int64 op-cost database of §3.3) and the kernel parameter block.
+// DESIGN.md §5 documents the layout; the encoding is the one of include/aceso.h.
+#pragma once
+#include <cstdint>
+
+#include "../../include/aceso.h"
+
+namespace aceso {
+
+constexpr int kWarps = 8;                    // warps per CTA in the eval kernel
+constexpr int kThreads = kWarps * 32;
+constexpr int kMaxOps = 16384;               // ops per model (per-op type offsets staged in smem)
+constexpr uint32_t kTypeStride = 32;         // bytes per op type in every smem table
+
+// Hot table R[b][tpl][type][rc] : 16-byte record (u32 each)
+//   x = S'  = fwd_comp + fwd_comm + bwd_comp + bwd_comm + rc*(fwd_comp + fwd_comm)   (R7)
+//   y = A   = rc ? keep : act                                                          (R3)
+//   z = e   = peak + rc*(act - keep)                                                   (R3, R4)
+//   w = W   = param+grad bytes + optimizer bytes at this tp
+// Memory fields (y, z, w) are stored in units of 2^mem_shift bytes, where mem_shift is
+// the largest power of two dividing every memory value of the profile (<= 2^16), so
+// the sums stay exact: Mem_i = (Wst + infl * A + E) << mem_shift.
+// DP table D[tpl][type][dpl] : u32 DP gradient all-reduce ns, 8 dpl slots per 32-byte entry
+// Type offsets O[j] : u32 type_j * 32 for every op (16-entry chunks, zero padded)
+// Full table F[b][tpl][type][rc] : u32 comp = fwd_comp + bwd_comp + rc*fwd_comp (8 B per type)
+// Cold table K[b][tpl][type] : 16 bytes {reshard, p2p_fwd, p2p_bwd, 0}  (R5, R13), read
+//   from global memory (L1/L2) at events only — after the shared blob in the same allocation
+struct Tables {
+  uint32_t offR, offD, offT, offF;  // byte offsets inside the staged blob (shared memory)
+  uint32_t bytes;                   // bytes staged to shared memory (multiple of 16)
+  uint32_t bytes_full;              // bytes staged including the F table
+  uint32_t offK;                    // byte offset of the cold table in the global blob
+};
+
+struct EvalParams {
+  const uint4 *codes;     // tiled op codes
+  const uint64_t *hdr;    // [n] headers
+  int64_t n;              // candidates in this call
+  int64_t gofs;           // global index of candidate 0
+  int64_t n_tiles;
+  int32_t L, nch, T, n_tp, n_dp, n_b, G;
+  uint64_t Bg, C;
+  uint32_t mem_shift;     // memory fields are stored >> mem_shift (exact)
+  const uint4 *blob;      // packed tables (global)
+  Tables tab;
+  // outputs
+  uint64_t *iter_ns, *max_mem;
+  uint32_t *info;
+  uint64_t *stage_T, *stage_mem, *stage_comp, *stage_comm;
+  int32_t p_max;
+  // selection
+  unsigned char *sel;     // aceso_select_result + counter + per-CTA partials
+  int64_t n_total;
+  uint32_t ib;            // index bits of the packed key
+};
+
+// select buffer layout: [0,32) result, [32,40) completion counter, [64, ...) partials (16 B each)
+constexpr int kSelCounterOff = 32;
+constexpr int kSelPartialOff = 64;
+
+__device__ __forceinline__ bool key_less(uint64_t a, int64_t ai, uint64_t b, int64_t bi) {
+  return a < b || (a == b && ai < bi);
+}
+
+// lexicographic argmin of (ck, idx) across the warp; result valid in every lane
+__device__ __forceinline__ void warp_argmin(uint64_t &ck, int64_t &idx) {
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) {
+    uint64_t ock = __shfl_xor_sync(0xffffffffu, ck, o);
+    int64_t oidx = __shfl_xor_sync(0xffffffffu, idx, o);
+    if (key_less(ock, oidx, ck, idx)) {
+      ck = ock;
+      idx = oidx;
+    }
+  }
+}
+
+// Block-level argmin + grid-level completion (last CTA reduces all partials and
+// writes the final result). Called by every thread of the CTA.
+__device__ __forceinline__ void block_select_finish(uint64_t ck, int64_t idx, unsigned char *sel,
+                                                    int64_t n_total, uint32_t ib,
+                                                    uint64_t *s_ck, int64_t *s_idx) {
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nw = blockDim.x >> 5;
+  warp_argmin(ck, idx);
+  if (lane == 0) {
+    s_ck[warp] = ck;
+    s_idx[warp] = idx;
+  }
+  __syncthreads();
+  __shared__ bool s_last;
+  if (warp == 0) {
+    ck = lane < nw ? s_ck[lane] : ~0ull;
+    idx = lane < nw ? s_idx[lane] : INT64_MAX;
+    warp_argmin(ck, idx);
+    if (lane == 0) {
+      uint64_t *part = reinterpret_cast<uint64_t *>(sel + kSelPartialOff) + 2 * blockIdx.x;
+      part[0] = ck;
+      part[1] = (uint64_t)idx;
+      __threadfence();
+      unsigned int *cnt = reinterpret_cast<unsigned int *>(sel + kSelCounterOff);
+      unsigned int t = atomicAdd(cnt, 1u);
+      s_last = (t == gridDim.x - 1);
+    }
+  }
+  __syncthreads();
+  if (!s_last) return;
+  __threadfence();
+  // last CTA: reduce all partials
+  const volatile uint64_t *parts = reinterpret_cast<const volatile uint64_t *>(sel + kSelPartialOff);
+  ck = ~0ull;
+  idx = INT64_MAX;
+  for (unsigned int b = threadIdx.x; b < gridDim.x; b += blockDim.x) {
+    uint64_t c2 = parts[2 * b];
+    int64_t i2 = (int64_t)parts[2 * b + 1];
+    if (key_less(c2, i2, ck, idx)) {
+      ck = c2;
+      idx = i2;
+    }
+  }
+  warp_argmin(ck, idx);
+  if (lane == 0) {
+    s_ck[warp] = ck;
+    s_idx[warp] = idx;
+  }
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    for (int w = 1; w < nw; ++w)
+      if (key_less(s_ck[w], s_idx[w], s_ck[0], s_idx[0])) {
+        s_ck[0] = s_ck[w];
+        s_idx[0] = s_idx[w];
+      }
+    ck = s_ck[0];
+    idx = s_idx[0];
+    aceso_select_result *res = reinterpret_cast<aceso_select_result *>(sel);
+    if (ck == ~0ull) {
+      res->key = INT64_MAX;
+      res->cls_cost = ~0ull;
+      res->index = -1;
+    } else {
+      uint64_t cls = ck >> 62, cost = ck & ((1ull << 62) - 1);
+      uint64_t cmax = (1ull << (62 - ib)) - 1;
+      uint64_t c = cost < cmax ? cost : cmax;
+      res->key = (int64_t)((cls << 62) | (c << ib) | (uint64_t)idx);
+      res->cls_cost = ck;
+      res->index = idx;
+    }
+    res->reserved = 0;
+    *reinterpret_cast<unsigned int *>(sel + kSelCounterOff) = 0;  // reusable
+  }
+}
+
+}  // namespace aceso

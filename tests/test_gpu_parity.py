@@ -1,0 +1,233 @@
+"""GPU parity: libaceso (sm_100a kernels, through the C-ABI) vs the CPU oracle.
+
+Bit-exact on every output (integer ns / bytes, bottleneck, status, reasons) and
+on the selected candidate; derived throughput Bg*1e9/iter agrees to 1e-12 rel.
+"""
+import numpy as np
+import pytest
+import torch
+
+import aceso_inputs as ai
+import oracle
+from aceso_inputs import profiles as P
+
+pytestmark = pytest.mark.gpu
+
+A = pytest.importorskip("paper_conf_eurosys_liumlsmybw24_b200")
+from paper_conf_eurosys_liumlsmybw24_b200.api import Selection, as_u32, as_u64  # noqa: E402
+
+SEED = 20240422
+
+
+@pytest.fixture(scope="module", autouse=True)
+def _need_gpu():
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+
+
+_ctx_cache = {}
+
+
+def ctx_for(prof):
+    key = id(prof)
+    if key not in _ctx_cache:
+        _ctx_cache[key] = (prof, A.Context(prof, 0))
+    return _ctx_cache[key][1]
+
+
+def run_gpu(prof, codes, hdr, full=False, gofs=0, n_total=None, pack_on_device=False, select=True):
+    ctx = ctx_for(prof)
+    n = len(hdr)
+    if pack_on_device:
+        tiled = ctx.pack_rowmajor(torch.from_numpy(np.ascontiguousarray(codes)).cuda())
+    else:
+        tiled = torch.from_numpy(ai.tile(codes)).cuda()
+    hd = torch.from_numpy(np.ascontiguousarray(hdr, np.uint64).view(np.int64)).cuda()
+    out, sel = ctx.eval(tiled, hd, n=n, global_offset=gofs, n_total=n_total, full=full, select=select)
+    torch.cuda.synchronize()
+    g = dict(iter=as_u64(out.iter_ns), max_mem=as_u64(out.max_mem), info=as_u32(out.info))
+    if full:
+        for k in ["stage_T", "stage_mem", "stage_comp", "stage_comm"]:
+            g[k] = as_u64(getattr(out, k)).reshape(out.p_max, n).T
+    return g, (Selection.from_buffer(sel) if select else None), out, ctx
+
+
+def compare(prof, codes, hdr, full=False, gofs=0, n_total=None, pack_on_device=False):
+    g, sel, out, ctx = run_gpu(prof, codes, hdr, full, gofs, n_total, pack_on_device)
+    o = oracle.evaluate(prof, codes, hdr, full=full, threads=8)
+    for k in ["iter", "max_mem", "info"]:
+        bad = np.nonzero(g[k] != o[k])[0]
+        assert bad.size == 0, (k, bad[:5], g[k][bad[:5]], o[k][bad[:5]])
+    if full:
+        valid = (o["info"] & oracle.INFO_INVALID) == 0
+        p = (o["info"] >> 8) & 0xFF
+        for k in ["stage_T", "stage_mem", "stage_comp", "stage_comm"]:
+            for c in np.nonzero(valid)[0]:
+                assert np.array_equal(g[k][c, :p[c]], o[k][c, :p[c]]), (k, c)
+    ocls, ocost, oidx = oracle.select(o, gofs)
+    assert (sel.cls, sel.cost, sel.index) == (ocls, ocost, oidx)
+    # derived throughput (samples/s), same IEEE division on both sides
+    valid = (o["info"] & oracle.INFO_INVALID) == 0
+    if valid.any():
+        tg = prof.global_batch * 1e9 / g["iter"][valid].astype(np.float64)
+        to = prof.global_batch * 1e9 / o["iter"][valid].astype(np.float64)
+        assert np.allclose(tg, to, rtol=1e-12, atol=0)
+    return g, o, sel, out, ctx
+
+
+# ---------------------------------------------------------------------------
+# exhaustive toy spaces (BASELINE.json configs[0])
+# ---------------------------------------------------------------------------
+@pytest.mark.parametrize("name,per_op", [("toy-a", True), ("toy-b", False)])
+def test_toy_exhaustive_parity_and_optimum(name, per_op):
+    prof = P.WORKLOADS[name]()
+    codes, hdr = ai.exhaustive(prof, per_op=per_op)
+    compare(prof, codes, hdr)
+
+
+def test_toy_exhaustive_full_mode():
+    prof = P.toy_a()
+    codes, hdr = ai.exhaustive(prof, per_op=True)
+    compare(prof, codes[:50000], hdr[:50000], full=True)
+
+
+# ---------------------------------------------------------------------------
+# paper-shaped workloads (configs[1..4]): search-shaped and adversarial batches
+# ---------------------------------------------------------------------------
+WL = ["gpt3-1.3b", "gpt3-13b", "t5", "wrn"]
+
+
+@pytest.mark.parametrize("name", WL)
+def test_search_shaped_parity(name):
+    prof = P.WORKLOADS[name]()
+    codes, hdr = ai.search_shaped(prof, SEED + 1, 0, 4099, group_size=64)
+    compare(prof, codes, hdr)
+
+
+@pytest.mark.parametrize("name", WL)
+def test_dense_random_parity(name):
+    prof = P.WORKLOADS[name]()
+    codes, hdr = ai.dense_random(prof, SEED + 2, 0, 2051)
+    compare(prof, codes, hdr)
+
+
+@pytest.mark.parametrize("name", WL)
+def test_full_mode_parity(name):
+    prof = P.WORKLOADS[name]()
+    codes, hdr = ai.search_shaped(prof, SEED + 3, 0, 1000, group_size=16)
+    compare(prof, codes, hdr, full=True)
+    codes, hdr = ai.dense_random(prof, SEED + 4, 0, 500)
+    compare(prof, codes, hdr, full=True)
+
+
+def test_gpt_1k_layers_parity():
+    prof = P.WORKLOADS["gpt-1k"]()
+    codes, hdr = ai.search_shaped(prof, SEED + 5, 0, 257, group_size=8)
+    compare(prof, codes, hdr, full=True)
+    codes, hdr = ai.dense_random(prof, SEED + 6, 0, 97)
+    compare(prof, codes, hdr)
+
+
+def test_bench_config_full_size_parity():
+    """The bench workload (GPT-3 1.3B, 8 devices, 65,536 candidates, bench seed) at full size."""
+    prof = P.WORKLOADS["gpt3-1.3b"]()
+    codes, hdr = ai.search_shaped(prof, SEED, 0, 65536, group_size=1024)
+    compare(prof, codes, hdr)
+
+
+# ---------------------------------------------------------------------------
+# edge cases
+# ---------------------------------------------------------------------------
+@pytest.mark.parametrize("n", [1, 2, 31, 32, 33, 63, 65, 257])
+def test_ragged_sizes(n):
+    prof = P.WORKLOADS["gpt3-1.3b"]()
+    codes, hdr = ai.search_shaped(prof, SEED + 7, 0, n, group_size=4)
+    compare(prof, codes, hdr, full=True)
+
+
+def test_empty_batch_selects_nothing():
+    prof = P.toy_a()
+    ctx = ctx_for(prof)
+    tiled = torch.zeros(512, dtype=torch.uint8, device="cuda")
+    hd = torch.zeros(1, dtype=torch.int64, device="cuda")
+    out, sel = ctx.eval(tiled, hd, n=0, summary=False, select=True)
+    s = Selection.from_buffer(sel)
+    assert s.index == -1 and s.key == (1 << 63) - 1
+
+
+def test_all_invalid_selects_nothing():
+    prof = P.toy_a()
+    codes, hdr = ai.search_shaped(prof, SEED, 0, 100)
+    hdr = hdr | np.uint64(1 << 40)  # reserved header byte set
+    g, o, sel, _, _ = compare(prof, codes, hdr)
+    assert sel.index == -1 and (g["info"] & oracle.INFO_INVALID).all()
+
+
+def test_global_offset_and_ties_take_lowest_index():
+    prof = P.WORKLOADS["gpt3-1.3b"]()
+    codes, hdr = ai.search_shaped(prof, SEED + 8, 0, 300, group_size=300)
+    codes = np.concatenate([codes, codes, codes])  # duplicates: equal cost
+    hdr = np.concatenate([hdr, hdr, hdr])
+    g, o, sel, _, _ = compare(prof, codes, hdr, gofs=1000, n_total=5000)
+    assert 1000 <= sel.index < 1300
+
+
+def test_device_pack_matches_host_tiling():
+    prof = P.WORKLOADS["t5"]()
+    codes, hdr = ai.search_shaped(prof, SEED + 9, 0, 333, group_size=8)
+    ctx = ctx_for(prof)
+    dev = ctx.pack_rowmajor(torch.from_numpy(codes).cuda()).cpu().numpy()
+    assert np.array_equal(dev, ai.tile(codes))
+    compare(prof, codes, hdr, pack_on_device=True)
+
+
+def test_standalone_select_matches_fused():
+    prof = P.WORKLOADS["wrn"]()
+    codes, hdr = ai.search_shaped(prof, SEED + 10, 0, 5000, group_size=32)
+    g, sel, out, ctx = run_gpu(prof, codes, hdr)
+    sel2 = Selection.from_buffer(ctx.select(out, global_offset=0))
+    assert (sel2.cls, sel2.cost, sel2.index, sel2.key) == (sel.cls, sel.cost, sel.index, sel.key)
+
+
+def test_select_buffer_reuse_and_streams():
+    prof = P.WORKLOADS["gpt3-1.3b"]()
+    ctx = ctx_for(prof)
+    s1 = torch.cuda.Stream()
+    sel = ctx.alloc_select()
+    results = []
+    for k in range(4):
+        codes, hdr = ai.search_shaped(prof, SEED + 20 + k, 0, 1000, group_size=50)
+        tiled = torch.from_numpy(ai.tile(codes)).cuda()
+        hd = torch.from_numpy(hdr.view(np.int64)).cuda()
+        torch.cuda.synchronize()
+        with torch.cuda.stream(s1):
+            ctx.eval(tiled, hd, summary=False, select=True, sel=sel, stream=s1)
+        s1.synchronize()
+        r = Selection.from_buffer(sel)
+        o = oracle.evaluate(prof, codes, hdr, threads=8)
+        assert (r.cls, r.cost, r.index) == oracle.select(o)
+        results.append(r.index)
+
+
+def test_stage_per_op_extremes():
+    """Every op its own stage (p = L) and one single stage (p = 1) on the toy model."""
+    prof = P.toy_a()
+    rows, hdrs = [], []
+    for mbs in range(0, 5):
+        rows.append([ai.code(1, 0, 0, j % 2) for j in range(4)] + [ai.code(0, 0, 0, 0)] * 2)
+        hdrs.append(ai.header(mbs, 4))
+        rows.append([ai.code(1, 1, 1, 1)] + [ai.code(0, 1, 1, 0)] * 5)
+        hdrs.append(ai.header(mbs, 1))
+        rows.append([ai.code(1, 2, 0, 1)] + [ai.code(0, 0, 2, 1)] * 5)  # tp<->dp change inside a stage
+        hdrs.append(ai.header(mbs, 1))
+    compare(prof, np.array(rows, np.uint8), np.array(hdrs, np.uint64), full=True)
+
+
+def test_random_bytes_never_crash_and_match():
+    """Arbitrary bytes (mostly invalid encodings) still match the oracle bit for bit."""
+    rng = np.random.default_rng(1)
+    for name in ["toy-b", "gpt3-1.3b"]:
+        prof = P.WORKLOADS[name]()
+        codes = rng.integers(0, 256, size=(3000, prof.n_ops), dtype=np.uint8)
+        hdr = rng.integers(0, 1 << 16, size=3000, dtype=np.uint64)
+        compare(prof, codes, hdr, full=True)
