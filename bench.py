@@ -246,8 +246,9 @@ def main():
     # The K timed steps are captured once into a CUDA graph (64K-candidate batches
     # take microseconds; host launch overhead must not pace the GPU), then the
     # graph is replayed once inside the timed region: exactly K steps.
-    ev_s = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps)]
-    ev_k = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps)]
+    # per-launch kernel times: external timing events captured as graph nodes
+    ev_s = [torch.cuda.Event(enable_timing=True, external=True) for _ in range(args.steps)]
+    ev_k = [torch.cuda.Event(enable_timing=True, external=True) for _ in range(args.steps)]
     graph = torch.cuda.CUDAGraph()
     if world > 1:
         dist.barrier()

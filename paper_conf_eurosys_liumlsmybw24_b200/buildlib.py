@@ -8,6 +8,7 @@ SRC = os.path.join(HERE, "csrc", "aceso_capi.cu")
 DEPS = [os.path.join(HERE, "csrc", f) for f in os.listdir(os.path.join(HERE, "csrc"))] + [
     os.path.join(os.path.dirname(HERE), "include", "aceso.h")]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
+EXTRA = os.environ.get("ACESO_NVCC_EXTRA", "").split()
 FLAGS = ["-gencode", "arch=compute_100a,code=sm_100a", "-O3", "-lineinfo", "-std=c++17",
          "-Xcompiler", "-fPIC", "-shared", "-Xptxas", "-warn-spills"]
 
@@ -21,7 +22,7 @@ def stale():
 
 def build(force=False, verbose=False):
     if force or stale():
-        cmd = [NVCC] + FLAGS + ["-o", LIB + ".tmp", SRC]
+        cmd = [NVCC] + FLAGS + EXTRA + ["-o", LIB + ".tmp", SRC]
         if verbose:
             print(" ".join(cmd))
         subprocess.check_call(cmd)

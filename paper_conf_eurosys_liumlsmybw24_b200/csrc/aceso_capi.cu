@@ -7,6 +7,7 @@
 #include <algorithm>
 #include <cstdarg>
 #include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <string>
 #include <vector>
@@ -38,22 +39,27 @@ int fail(int code, const char *fmt, ...) {
       return fail(ACESO_ECUDA, "%s failed: %s", #expr, cudaGetErrorString(e_));            \
   } while (0)
 
-template <uint32_t M>
+template <uint32_t M, int S>
 void *kernel_ptr() {
-  return reinterpret_cast<void *>(&eval_kernel<M>);
+  return reinterpret_cast<void *>(&eval_kernel<M, S>);
 }
 
-void *eval_kernel_for(uint32_t mode) {
+template <int S>
+void *eval_kernel_split(uint32_t mode) {
   switch (mode) {
-    case 1: return kernel_ptr<1>();
-    case 2: return kernel_ptr<2>();
-    case 3: return kernel_ptr<3>();
-    case 4: return kernel_ptr<4>();
-    case 5: return kernel_ptr<5>();
-    case 6: return kernel_ptr<6>();
-    case 7: return kernel_ptr<7>();
+    case 1: return kernel_ptr<1, S>();
+    case 2: return kernel_ptr<2, S>();
+    case 3: return kernel_ptr<3, S>();
+    case 4: return kernel_ptr<4, S>();
+    case 5: return kernel_ptr<5, S>();
+    case 6: return kernel_ptr<6, S>();
+    case 7: return kernel_ptr<7, S>();
     default: return nullptr;
   }
+}
+
+void *eval_kernel_for(uint32_t mode, int split) {
+  return split == 2 ? eval_kernel_split<2>(mode) : eval_kernel_split<1>(mode);
 }
 
 uint32_t bitlen(uint64_t v) {
@@ -72,6 +78,7 @@ struct aceso_ctx {
   uint32_t mem_shift;
   Tables tab;
   void *d_blob;
+  int split;        // warps per tile (1 or 2)
   int max_ctas[8];  // per mode: resident CTAs (occupancy x SMs)
   size_t smem[8];
 };
@@ -174,6 +181,9 @@ int aceso_load_profile(const aceso_profile_desc *d, int cuda_device, aceso_ctx *
   tab.bytes = tab.offF;
   tab.bytes_full = tab.offF + bytesF;
   tab.offK = tab.bytes_full;
+  tab.bytesK = bytesK;
+  // stage the cold table too when shared memory allows ~2 CTAs per SM
+  tab.k_smem = (tab.bytes_full + bytesK + kRingBytesPerCta + 16384u <= 100u * 1024u) ? 1u : 0u;
   if (tab.bytes_full > 180u * 1024u) return fail(ACESO_EINVAL, "packed tables of %u bytes exceed shared memory", tab.bytes_full);
   const uint32_t blob_bytes = tab.offK + bytesK;
   std::vector<uint32_t> blob(blob_bytes / 4, 0u);
@@ -235,10 +245,18 @@ int aceso_load_profile(const aceso_profile_desc *d, int cuda_device, aceso_ctx *
     if (e == cudaSuccess) e = cudaStreamSynchronize(st);
     cudaStreamDestroy(st);
     if (e != cudaSuccess) { rc = fail(e == cudaErrorMemoryAllocation ? ACESO_ENOMEM : ACESO_ECUDA, "upload: %s", cudaGetErrorString(e)); break; }
+    const int nch = (L + 15) / 16;
+    ctx->split = nch >= 2 ? 2 : 1;
+    if (const char *env = getenv("ACESO_SPLIT")) {
+      int v = atoi(env);
+      if (v == 1 || (v == 2 && nch >= 2)) ctx->split = v;
+    }
     for (uint32_t mode = 1; mode < 8; ++mode) {
-      const size_t smem = ((mode & ACESO_OUT_FULL) ? tab.bytes_full : tab.bytes) + kRingBytesPerCta;
+      const size_t smem = ((mode & ACESO_OUT_FULL) ? tab.bytes_full : tab.bytes) +
+                          (tab.k_smem ? bytesK : 0u) + kRingBytesPerCta +
+                          (ctx->split == 2 ? (size_t)(kWarps / 2) * 32 * sizeof(Xchg) : 0);
       ctx->smem[mode] = smem;
-      void *k = eval_kernel_for(mode);
+      void *k = eval_kernel_for(mode, ctx->split);
       e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
       int occ = 0;
       if (e == cudaSuccess) e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k, kThreads, smem);
@@ -326,13 +344,14 @@ int aceso_eval(aceso_ctx *ctx, const uint8_t *d_codes, const uint64_t *d_hdr, in
   P.n_total = n_total;
   P.ib = std::max(1u, bitlen((uint64_t)n_total));
 
-  const int64_t need = (P.n_tiles + kWarps - 1) / kWarps;
+  const int tiles_per_cta = kWarps / ctx->split;
+  const int64_t need = (P.n_tiles + tiles_per_cta - 1) / tiles_per_cta;
   int grid = (int)std::max<int64_t>(1, std::min<int64_t>(need, ctx->max_ctas[mode]));
   int prev = 0;
   CUDA_TRY(cudaGetDevice(&prev));
   if (prev != ctx->device) CUDA_TRY(cudaSetDevice(ctx->device));
   void *args[] = {&P};
-  cudaError_t e = cudaLaunchKernel(eval_kernel_for(mode), dim3(grid), dim3(kThreads), args, ctx->smem[mode],
+  cudaError_t e = cudaLaunchKernel(eval_kernel_for(mode, ctx->split), dim3(grid), dim3(kThreads), args, ctx->smem[mode],
                                    reinterpret_cast<cudaStream_t>(stream));
   if (prev != ctx->device) cudaSetDevice(prev);
   if (e != cudaSuccess) return fail(ACESO_ECUDA, "eval launch: %s", cudaGetErrorString(e));

@@ -33,6 +33,8 @@ struct Tables {
   uint32_t bytes;                   // bytes staged to shared memory (multiple of 16)
   uint32_t bytes_full;              // bytes staged including the F table
   uint32_t offK;                    // byte offset of the cold table in the global blob
+  uint32_t bytesK;                  // bytes of the cold table
+  uint32_t k_smem;                  // 1: the cold table is staged to shared memory too
 };
 
 struct EvalParams {

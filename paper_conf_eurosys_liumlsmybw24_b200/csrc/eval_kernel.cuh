@@ -1,15 +1,26 @@
 // eval_kernel.cuh — batched evaluation of Aceso's performance/memory model (sm_100a).
 //
-// One thread per candidate configuration; a warp owns a tile of 32 candidates
-// (tiled layout of include/aceso.h) and streams its 16-op chunks from HBM into a
-// per-warp shared-memory ring with cp.async.bulk (TMA bulk copies, mbarrier
-// completion). The packed profile tables are staged into shared memory once per
-// CTA, also with cp.async.bulk. Per op the thread gathers its 16-byte record and
-// the DP record from shared memory and accumulates the stage sums; stage heads and
-// in-stage tp/dp changes ("events") are detected per chunk with SWAR byte tricks
-// so that event-free chunks run a branch-free path. Stage close applies Eq. 1/2,
-// OOM flag and Heuristic-1; the candidate epilogue writes the SoA summary and
-// folds the candidate into the fused argmin (K2, common.cuh).
+// Work decomposition. A tile holds 32 candidates (tiled layout of include/aceso.h);
+// thread = candidate. With SPLIT = 2 a tile is processed by a PAIR of warps: part 0
+// walks ops [0, M) forward, part 1 walks ops [M, L) BACKWARD. Walking backward from
+// the last stage (index p-1), part 1 knows every stage's absolute index without a
+// pre-scan, so Eq. 1's in-flight factor min(p - i, N) is available when it closes a
+// stage. The stage that spans M is closed by part 0 after part 1 hands over its
+// partial sums through shared memory (named barrier per warp pair). SPLIT = 1 runs
+// one forward warp per tile (short models).
+//
+// Data movement. The packed profile tables are staged into shared memory once per
+// CTA with one cp.async.bulk (TMA bulk copy, mbarrier completion); each warp streams
+// its chunks (512 B = 32 candidates x 16 ops) from HBM into a private 4-slot ring
+// with cp.async.bulk, so loads run several chunks ahead of the math.
+//
+// Per op. A 16-byte record {S', A, e, W} is gathered from shared memory at
+// run_base + type_offset + rc*16 plus the DP record; the sums are u64. Stage heads
+// and in-stage tp/dp changes ("events") are detected per chunk with SWAR byte
+// tricks and OR-reduced across the warp; a 4-op group without events in any lane
+// runs branch-free, otherwise each op tests the warp-uniform union and only lanes
+// with an event run the handler (stage close: Eq. 1/2, OOM, Heuristic-1 bookkeeping;
+// run open: validity, table bases, reshard / p2p terms).
 //
 // Paper: configuration (§3.1), Heuristic-1, memory Eq. 1
 // (P:L225-234), time Eq. 2; readings R1-R13 in DESIGN.md §3.
@@ -24,9 +35,13 @@ constexpr int kRingSlots = 4;    // per-warp ring depth
 constexpr int kSlotChunks = 2;   // 16-op chunks per ring slot (1 KB)
 constexpr int kSlotBytes = kSlotChunks * 512;
 constexpr int kRingBytesPerCta = kWarps * kRingSlots * kSlotBytes;
+constexpr uint32_t kNone = 0xffffffffu;
+#ifndef ACESO_MINB
+#define ACESO_MINB 2  // resident CTAs per SM the register allocation targets
+#endif
 
 // ---------------------------------------------------------------------------
-// PTX helpers: mbarrier + cp.async.bulk (TMA bulk copy)
+// PTX helpers: mbarrier + cp.async.bulk (TMA bulk copy), shared loads
 // ---------------------------------------------------------------------------
 __device__ __forceinline__ uint32_t smem_addr(const void *p) {
   return (uint32_t)__cvta_generic_to_shared(p);
@@ -63,120 +78,174 @@ __device__ __forceinline__ void mbar_wait(uint32_t bar, uint32_t parity) {
       "r"(parity)
       : "memory");
 }
-
-// shared-memory loads by absolute shared address (no generic-pointer arithmetic)
-__device__ __forceinline__ uint4 lds128(const unsigned char *, uint32_t a) {
+// named barrier of a warp pair (immediate ids 1..4 so ptxas reserves only those)
+__device__ __forceinline__ void pair_bar_sync(int pair) {
+  switch (pair) {
+    case 0: asm volatile("bar.sync 1, 64;" ::: "memory"); break;
+    case 1: asm volatile("bar.sync 2, 64;" ::: "memory"); break;
+    case 2: asm volatile("bar.sync 3, 64;" ::: "memory"); break;
+    default: asm volatile("bar.sync 4, 64;" ::: "memory"); break;
+  }
+}
+__device__ __forceinline__ uint4 lds128(uint32_t a) {
   uint4 v;
   asm volatile("ld.shared.v4.u32 {%0, %1, %2, %3}, [%4];"
                : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w)
                : "r"(a));
   return v;
 }
-__device__ __forceinline__ uint32_t lds32(const unsigned char *, uint32_t a) {
+__device__ __forceinline__ uint32_t lds32(uint32_t a) {
   uint32_t v;
   asm volatile("ld.shared.u32 %0, [%1];" : "=r"(v) : "r"(a));
   return v;
 }
 
 // ---------------------------------------------------------------------------
-// per-candidate state (registers)
+// state
 // ---------------------------------------------------------------------------
-struct Cand {
-  // current stage (per-microbatch sums, R5/R13 terms included in S)
-  uint64_t S, A, W, D, comp;
-  uint32_t E;
-  // current run (ops with equal (tp, dp) inside one stage): absolute shared addresses,
-  // kbase: offset of the run in the global cold table (16 B per type)
-  uint32_t rbase, dbase, kbase, fbase, gst;
-  // candidate-level
-  uint64_t sumS, bestT, bestM;
-  uint32_t bt, bm, oom, i, gsum, reasons, head0;
-  uint32_t mbs, p;
-  uint64_t N;
-};
-
-// absolute shared addresses of the staged tables
 struct Smem {
-  uint32_t R, D, F, T;
-  const unsigned char *K;  // global cold table
+  uint32_t R, D, F, T, K;   // shared addresses of the staged tables (K valid if k_smem)
+  const unsigned char *Kg;  // cold table in global memory
+  uint32_t k_smem;
+  uint32_t TS;              // T * 32: bytes of one (b, tpl) block of R
 };
 
 __device__ __forceinline__ uint32_t ldk(const Smem &sm, uint32_t off) {
-  return __ldg(reinterpret_cast<const uint32_t *>(sm.K + off));
+  return sm.k_smem ? lds32(sm.K + off) : __ldg(reinterpret_cast<const uint32_t *>(sm.Kg + off));
 }
 
+struct Cand {
+  // current stage: per-microbatch sums (R5/R13 terms included in S)
+  uint64_t S, A, W, D, comp;
+  uint32_t E;
+  // current run (ops of equal (tp, dp) inside one stage)
+  uint32_t rbase, dbase, kbase, fbase, gst;
+  // candidate-level aggregates
+  uint64_t sumS, bestT, bestM;
+  uint32_t bt, bm, oom, i, gsum, reasons, nheads, head0;
+  uint32_t mbs, p, N;
+};
+
+// hand-over record, part 1 -> part 0 (one per candidate of a tile)
+struct Xchg {
+  uint64_t S, A, W, D, comp, sumS, bestT, bestM;
+  uint32_t E, bt, bm, flags, gsum, reasons, nheads, pad;
+};
+
+// Closes the current stage i: Eq. 2 key, Eq. 1 memory, OOM, Heuristic-1 maxima.
 template <uint32_t MODE>
-__device__ __forceinline__ void close_stage(Cand &s, const Smem &sm, const EvalParams &P,
-                                            uint32_t toff_last, int64_t c, bool active) {
-  // R5: a non-last stage pays the forward send of its last op
-  if (s.i + 1 < s.p) s.S += ldk(sm, s.kbase + (toff_last >> 1) + 4);
+__device__ __forceinline__ void stage_commit(Cand &s, const EvalParams &P, int64_t c, bool active,
+                                             bool reverse) {
   s.sumS += s.S;
-  const uint64_t tk = (s.N - 1) * s.S + s.D;  // T_i - sum_k S_k   (Eq. 2, R1, R6)
-  if (s.i == 0 || tk > s.bestT) { s.bestT = tk; s.bt = s.i; }
-  const uint64_t infl = s.p > s.i ? min((uint64_t)(s.p - s.i), s.N) : 0ull;  // R2
-  const uint64_t M = (s.W + infl * s.A + s.E) << P.mem_shift;                 // Eq. 1
-  if (s.i == 0 || M > s.bestM) { s.bestM = M; s.bm = s.i; }
+  const uint64_t tk = (uint64_t)(s.N - 1) * s.S + s.D;  // T_i - sum_k S_k (Eq. 2, R1, R6)
+  const uint64_t infl = s.p > s.i ? (uint64_t)min(s.p - s.i, s.N) : 0ull;  // R2
+  const uint64_t M = (s.W + infl * s.A + s.E) << P.mem_shift;              // Eq. 1 (R3, R4)
+  // argmax with the lowest stage index on ties (R11): forward visits ascending
+  // indices (strict >), the reverse part descending ones (>=, kNone = nothing yet)
+  if (reverse ? (tk >= s.bestT || s.bt == kNone) : (tk > s.bestT)) { s.bestT = tk; s.bt = s.i; }
+  if (reverse ? (M >= s.bestM || s.bm == kNone) : (M > s.bestM)) { s.bestM = M; s.bm = s.i; }
   s.oom |= (M > P.C) ? 1u : 0u;  // R10
   if (MODE & kFull) {
     if (active && s.i < (uint32_t)P.p_max) {
       const int64_t o = (int64_t)s.i * P.n + c;
       P.stage_T[o] = tk;  // + sum_k S_k in the epilogue
       P.stage_mem[o] = M;
-      P.stage_comp[o] = s.N * s.comp;
-      P.stage_comm[o] = s.N * (s.S - s.comp) + s.D;
+      P.stage_comp[o] = (uint64_t)s.N * s.comp;
+      P.stage_comm[o] = (uint64_t)s.N * (s.S - s.comp) + s.D;
     }
   }
-  s.i += 1;
   s.S = s.A = s.W = s.D = s.comp = 0;
   s.E = 0;
 }
 
-// Event at op j: stage head and/or change of (tp, dp). Opens the new run.
+// Opens the run of op code c: validity checks and table bases for its (tp, dp).
 template <uint32_t MODE>
-__device__ __forceinline__ void on_event(Cand &s, const Smem &sm, const EvalParams &P, uint32_t j,
-                                      uint32_t c, uint32_t toff, uint32_t toff_prev, int64_t cand,
-                                      bool active) {
-  const uint32_t head = c & 1u;
-  if (head && j > 0) close_stage<MODE>(s, sm, P, toff_prev, cand, active);
+__device__ __forceinline__ void open_run(Cand &s, const Smem &sm, const EvalParams &P, uint32_t c) {
   const uint32_t tpl = (c >> 1) & 7u, dpl = c >> 5;
   if (dpl > s.mbs) s.reasons |= ACESO_R_DPMBS;
-  if (tpl >= (uint32_t)P.n_tp || dpl >= (uint32_t)P.n_dp) s.reasons |= ACESO_R_TABLE;
-  else if (dpl <= s.mbs && s.mbs - dpl >= (uint32_t)P.n_b) s.reasons |= ACESO_R_TABLE;
+  const bool tab = tpl >= (uint32_t)P.n_tp || dpl >= (uint32_t)P.n_dp ||
+                   (dpl <= s.mbs && s.mbs - dpl >= (uint32_t)P.n_b);
+  if (tab) s.reasons |= ACESO_R_TABLE;
   // clamped indices keep every gather inside the tables for invalid encodings
-  uint32_t b = dpl <= s.mbs ? s.mbs - dpl : 0u;
-  b = min(b, (uint32_t)P.n_b - 1);
+  const uint32_t b = min(dpl <= s.mbs ? s.mbs - dpl : 0u, (uint32_t)P.n_b - 1);
   const uint32_t tplc = min(tpl, (uint32_t)P.n_tp - 1);
-  const uint32_t run = (b * (uint32_t)P.n_tp + tplc) * (uint32_t)P.T;
-  s.rbase = sm.R + run * kTypeStride;
-  s.kbase = run * 16u;
-  if (MODE & kFull) s.fbase = sm.F + run * 8u;
-  s.dbase = sm.D + tplc * (uint32_t)P.T * kTypeStride + dpl * 4u;
-  const uint32_t g = tpl + dpl;
-  if (head || j == 0) {
-    s.gst = g;
-    s.gsum += 1u << g;  // R9: sum_i tp_i * dp_i
-    if (s.i > 0) s.S += ldk(sm, s.kbase + (toff >> 1) + 8);  // R5: backward send of the first op
-  } else {
-    if (g != s.gst) s.reasons |= ACESO_R_GSTAGE;  // P:L151 in-stage symmetry
-    s.S += ldk(sm, s.kbase + (toff >> 1));       // R13: reshard into this op
-  }
+  const uint32_t run = b * (uint32_t)P.n_tp + tplc;
+  s.rbase = sm.R + run * sm.TS;
+  s.kbase = run * (sm.TS >> 1);
+  if (MODE & kFull) s.fbase = sm.F + run * (sm.TS >> 2);
+  s.dbase = sm.D + tplc * sm.TS + dpl * 4u;
 }
 
 template <uint32_t MODE>
-__device__ __forceinline__ void accumulate(Cand &s, const Smem &sm, uint32_t rcoff, uint32_t toff) {
+__device__ __forceinline__ void accumulate(Cand &s, uint32_t rcoff, uint32_t toff) {
   const uint32_t ra = s.rbase + toff + rcoff;
-  const uint4 r = lds128(nullptr, ra);
-  const uint32_t d = lds32(nullptr, s.dbase + toff);
+  const uint4 r = lds128(ra);
+  const uint32_t d = lds32(s.dbase + toff);
   s.S += r.x;
   s.A += r.y;
   s.E = max(s.E, r.z);
   s.W += r.w;
   s.D += d;
-  if (MODE & kFull) s.comp += lds32(nullptr, s.fbase + (toff >> 2) + (rcoff >> 2));
+  if (MODE & kFull) s.comp += lds32(s.fbase + (toff >> 2) + (rcoff >> 2));
 }
 
+// forward event at op j (before accumulating op j): stage head and/or tp/dp change
 template <uint32_t MODE>
-__device__ __forceinline__ void init_cand(Cand &s, const Smem &sm, const EvalParams &P, uint64_t h) {
+__device__ __forceinline__ void fwd_event(Cand &s, const Smem &sm, const EvalParams &P, uint32_t j,
+                                          uint32_t c, uint32_t toff, uint32_t toff_prev, int64_t cand,
+                                          bool active) {
+  const uint32_t head = c & 1u;
+  if (head && j > 0) {
+    s.S += ldk(sm, s.kbase + (toff_prev >> 1) + 4);  // R5: p2p_fwd of the stage's last op
+    stage_commit<MODE>(s, P, cand, active, false);
+    s.i += 1;
+  }
+  const uint32_t g = ((c >> 1) & 7u) + (c >> 5);
+  open_run<MODE>(s, sm, P, c);
+  if (head || j == 0) {
+    s.gst = g;
+    s.gsum += 1u << g;  // R9
+    s.nheads += head;
+    if (head && j > 0) s.S += ldk(sm, s.kbase + (toff >> 1) + 8);  // R5: p2p_bwd of the first op
+  } else {
+    if (g != s.gst) s.reasons |= ACESO_R_GSTAGE;  // P:L151 in-stage symmetry
+    s.S += ldk(sm, s.kbase + (toff >> 1));        // R13: reshard into this op
+  }
+}
+
+// reverse "pre" event at op j (before accumulating op j): op j+1 opened a run
+// (cn = code of op j+1, tn = its type offset), or j is the model's last op.
+template <uint32_t MODE>
+__device__ __forceinline__ void rev_pre(Cand &s, const Smem &sm, const EvalParams &P, uint32_t j,
+                                        uint32_t c, uint32_t cn, uint32_t toff, uint32_t tn) {
+  const uint32_t g = ((c >> 1) & 7u) + (c >> 5);
+  if (j + 1 == (uint32_t)P.L) {  // the last stage (p - 1), visited first
+    open_run<MODE>(s, sm, P, c);
+    s.gst = g;
+  } else if (cn & 1u) {  // op j+1 was a head: op j is the last op of the previous stage
+    open_run<MODE>(s, sm, P, c);
+    s.gst = g;
+    s.S += ldk(sm, s.kbase + (toff >> 1) + 4);  // R5: p2p_fwd of the last op
+  } else {               // tp/dp change at op j+1 inside a stage
+    s.S += ldk(sm, s.kbase + (tn >> 1));         // R13: reshard into op j+1 (its run)
+    if (g != s.gst) s.reasons |= ACESO_R_GSTAGE;
+    open_run<MODE>(s, sm, P, c);
+  }
+}
+
+// reverse "post" event at op j (after accumulating op j): op j is a stage head
+template <uint32_t MODE>
+__device__ __forceinline__ void rev_post(Cand &s, const Smem &sm, const EvalParams &P, uint32_t c,
+                                         uint32_t toff, int64_t cand, bool active) {
+  s.S += ldk(sm, s.kbase + (toff >> 1) + 8);  // R5: p2p_bwd of the first op (j >= M > 0)
+  s.gsum += 1u << (((c >> 1) & 7u) + (c >> 5));
+  s.nheads += 1;
+  stage_commit<MODE>(s, P, cand, active, true);
+  s.i -= 1;
+}
+
+__device__ __forceinline__ void init_cand(Cand &s, const Smem &sm, const EvalParams &P, uint64_t h,
+                                          bool reverse) {
   s.mbs = (uint32_t)(h & 0xff);
   s.p = (uint32_t)((h >> 8) & 0xff);
   s.reasons = (h >> 16) ? ACESO_R_HDR : 0u;
@@ -184,13 +253,14 @@ __device__ __forceinline__ void init_cand(Cand &s, const Smem &sm, const EvalPar
   if (s.mbs >= 62 || (1ull << s.mbs) > P.Bg || (P.Bg & ((1ull << s.mbs) - 1)) != 0)
     s.reasons |= ACESO_R_MBS;
   else
-    s.N = P.Bg >> s.mbs;
+    s.N = (uint32_t)(P.Bg >> s.mbs);
   if (s.p == 0 || s.p > (uint32_t)P.G) s.reasons |= ACESO_R_PRANGE;
   s.S = s.A = s.W = s.D = s.comp = 0;
   s.E = 0;
   s.sumS = s.bestT = s.bestM = 0;
-  s.bt = s.bm = s.oom = s.i = s.gsum = 0;
-  s.head0 = 0;
+  s.bt = s.bm = reverse ? kNone : 0u;
+  s.oom = s.gsum = s.nheads = s.head0 = 0;
+  s.i = reverse ? s.p - 1 : 0u;
   s.rbase = sm.R;
   s.dbase = sm.D;
   s.kbase = 0;
@@ -198,72 +268,103 @@ __device__ __forceinline__ void init_cand(Cand &s, const Smem &sm, const EvalPar
   s.gst = 0;
 }
 
-// Process one 16-op chunk of the lane's candidate. v = the lane's 16 code bytes.
+// ---------------------------------------------------------------------------
+// 4-op groups ("quads"): the unit of the warp-uniform event test. One call site
+// per direction keeps the kernel small enough for the instruction cache.
+// ---------------------------------------------------------------------------
+// forward quad qg (ops 4qg..4qg+3); w = the lane's 4 code bytes; pw = previous word
 template <uint32_t MODE>
-__device__ __forceinline__ void process_chunk(Cand &s, const Smem &sm, const EvalParams &P, uint4 v,
-                                              uint32_t ch, uint32_t &prevw, int64_t cand,
-                                              bool active) {
-  const uint32_t w[4] = {v.x, v.y, v.z, v.w};
-  uint32_t x[4];
-  uint32_t pw = prevw;
-#pragma unroll
-  for (int q = 0; q < 4; ++q) {
-    // previous op's byte under each byte: funnel shift of (previous word, word)
-    const uint32_t sh = __funnelshift_l(pw, w[q], 8);
-    x[q] = ((w[q] ^ sh) & 0xEEEEEEEEu) | (w[q] & 0x01010101u);  // tp/dp change | head
-    pw = w[q];
+__device__ __forceinline__ void quad_fwd(Cand &s, const Smem &sm, const EvalParams &P, uint32_t w,
+                                         uint32_t &pw, uint32_t qg, int64_t cand, bool active) {
+  const uint32_t sh = __funnelshift_l(pw, w, 8);  // previous op's byte under each byte
+  uint32_t x = ((w ^ sh) & 0xEEEEEEEEu) | (w & 0x01010101u);  // tp/dp change | head
+  pw = w;
+  if (qg == 0) {
+    x |= 0xffu;  // op 0 always opens the first run
+    s.head0 = w & 1u;
   }
-  prevw = pw;
-  const uint32_t j0 = ch * 16u;
-  if (ch == 0) {
-    x[0] |= 0xffu;  // op 0 always opens the first run
-    s.head0 = w[0] & 1u;
-  }
-  const bool last = (j0 + 16u >= (uint32_t)P.L);
-  const uint32_t ev = x[0] | x[1] | x[2] | x[3];
-  const uint32_t ta = sm.T + j0 * 4u;  // this chunk's 16 type offsets (broadcast loads)
-  if (!last && !__any_sync(0xffffffffu, ev != 0)) {
-    // fast path: no head, no tp/dp change in any lane of the warp
-#pragma unroll
-    for (int q = 0; q < 4; ++q) {
-      const uint4 t4 = lds128(nullptr, ta + 16u * q);
-      const uint32_t t[4] = {t4.x, t4.y, t4.z, t4.w};
-      const uint32_t rcw = w[q] & 0x10101010u;  // rc * 16 per byte
-#pragma unroll
-      for (int k = 0; k < 4; ++k) accumulate<MODE>(s, sm, __byte_perm(rcw, 0, 0x4440 + k), t[k]);
-    }
-    return;
-  }
-  // general path: per-op event test
-  const uint32_t kmax = last ? (uint32_t)P.L - j0 : 16u;
-#pragma unroll
-  for (int q = 0; q < 4; ++q) {
-    uint32_t ww = w[q], xx = x[q];
+  const uint32_t j0 = qg * 4u;
+  const uint32_t nvalid = min(4u, (uint32_t)P.L - j0);
+  if (nvalid < 4u) x &= 0xffffffffu >> (8 * (4u - nvalid));
+  const uint32_t U = __reduce_or_sync(0xffffffffu, x);
+  const uint32_t ta = sm.T + j0 * 4u;  // type offsets of these ops (broadcast loads)
+  if (U == 0u && nvalid == 4u) {
+    // no head, no tp/dp change in any lane: branch-free
+    const uint4 t4 = lds128(ta);
+    const uint32_t rcw = w & 0x10101010u;  // rc * 16 per byte
+    accumulate<MODE>(s, __byte_perm(rcw, 0, 0x4440), t4.x);
+    accumulate<MODE>(s, __byte_perm(rcw, 0, 0x4441), t4.y);
+    accumulate<MODE>(s, __byte_perm(rcw, 0, 0x4442), t4.z);
+    accumulate<MODE>(s, __byte_perm(rcw, 0, 0x4443), t4.w);
+  } else {
+    uint32_t tprev = j0 > 0 ? lds32(ta - 4u) : 0u;
 #pragma unroll 1
-    for (int k = 0; k < 4; ++k) {
-      const uint32_t kk = 4 * q + k;
-      if (kk >= kmax) break;
-      const uint32_t j = j0 + kk;
-      const uint32_t toff = lds32(nullptr, ta + 4u * kk);
-      const uint32_t c = ww & 0xffu;
-      if (xx & 0xffu) {
-        const uint32_t toff_prev = j > 0 ? lds32(nullptr, ta + 4u * kk - 4u) : 0u;
-        on_event<MODE>(s, sm, P, j, c, toff, toff_prev, cand, active);
+    for (uint32_t k = 0; k < nvalid; ++k) {
+      const uint32_t toff = lds32(ta + 4u * k);
+      const uint32_t c = (w >> (8 * k)) & 0xffu;
+      if ((U >> (8 * k)) & 0xffu) {
+        if ((x >> (8 * k)) & 0xffu) fwd_event<MODE>(s, sm, P, j0 + k, c, toff, tprev, cand, active);
       }
-      accumulate<MODE>(s, sm, c & 0x10u, toff);
-      ww >>= 8;
-      xx >>= 8;
+      accumulate<MODE>(s, c & 0x10u, toff);
+      tprev = toff;
     }
   }
 }
 
+// reverse quad qg, ops visited from the highest down; nw = code word of the next quad
+// (visited before this one), tn = type offset of op 4qg+4. On return nw = w and
+// tn = type offset of op 4qg.
 template <uint32_t MODE>
-__device__ __forceinline__ void finish_cand(Cand &s, const Smem &sm, const EvalParams &P, int64_t c,
-                                            bool active, uint64_t &best_ck, int64_t &best_idx) {
-  close_stage<MODE>(s, sm, P, lds32(nullptr, sm.T + 4u * (uint32_t)(P.L - 1)), c, active);
-  const uint32_t nheads = s.i - 1 + s.head0;
+__device__ __forceinline__ void quad_rev(Cand &s, const Smem &sm, const EvalParams &P, uint32_t w,
+                                         uint32_t &nw, uint32_t &tn, uint32_t qg, int64_t cand,
+                                         bool active) {
+  const uint32_t nb = __funnelshift_r(w, nw, 8);  // next op's byte under each byte
+  // bits 1-3, 5-7: op j+1 opens a run (tp/dp change, or bit 1 = head of op j+1);
+  // bit 0: op j is a stage head
+  uint32_t x = ((w ^ nb) & 0xEEEEEEEEu) | ((nb & 0x01010101u) << 1) | (w & 0x01010101u);
+  const uint32_t j0 = qg * 4u;
+  const uint32_t nvalid = min(4u, (uint32_t)P.L - j0);
+  if (j0 + nvalid == (uint32_t)P.L) x |= 0x80u << (8 * (nvalid - 1));  // last op: last stage
+  if (nvalid < 4u) x &= 0xffffffffu >> (8 * (4u - nvalid));
+  const uint32_t U = __reduce_or_sync(0xffffffffu, x);
+  const uint32_t ta = sm.T + j0 * 4u;
+  if (U == 0u && nvalid == 4u) {
+    const uint4 t4 = lds128(ta);
+    const uint32_t rcw = w & 0x10101010u;
+    accumulate<MODE>(s, __byte_perm(rcw, 0, 0x4440), t4.x);
+    accumulate<MODE>(s, __byte_perm(rcw, 0, 0x4441), t4.y);
+    accumulate<MODE>(s, __byte_perm(rcw, 0, 0x4442), t4.z);
+    accumulate<MODE>(s, __byte_perm(rcw, 0, 0x4443), t4.w);
+    tn = t4.x;
+  } else {
+#pragma unroll 1
+    for (int k = (int)nvalid - 1; k >= 0; --k) {
+      const uint32_t toff = lds32(ta + 4u * k);
+      const uint32_t c = (w >> (8 * k)) & 0xffu;
+      const uint32_t e = (x >> (8 * k)) & 0xffu;
+      const uint32_t u = (U >> (8 * k)) & 0xffu;
+      if (u & 0xfeu) {
+        if (e & 0xfeu) {
+          const uint32_t cn = k < 3 ? (w >> (8 * k + 8)) & 0xffu : nw & 0xffu;
+          rev_pre<MODE>(s, sm, P, j0 + k, c, cn, toff, tn);
+        }
+      }
+      accumulate<MODE>(s, c & 0x10u, toff);
+      if (u & 1u) {
+        if (e & 1u) rev_post<MODE>(s, sm, P, c, toff, cand, active);
+      }
+      tn = toff;
+    }
+  }
+  nw = w;
+}
+
+// Candidate epilogue (forward part): validity, summary outputs, fused argmin.
+template <uint32_t MODE>
+__device__ __forceinline__ void finish_cand(Cand &s, const EvalParams &P, int64_t c, bool active,
+                                            uint64_t &best_ck, int64_t &best_idx) {
   if (!s.head0) s.reasons |= ACESO_R_HEAD0;
-  if (nheads != s.p) s.reasons |= ACESO_R_NSTAGE;
+  if (s.nheads != s.p) s.reasons |= ACESO_R_NSTAGE;
   if (s.gsum != (uint32_t)P.G) s.reasons |= ACESO_R_GSUM;
   const bool invalid = s.reasons != 0;
   const uint64_t iter = invalid ? 0ull : s.sumS + s.bestT;  // max_i T_i (Eq. 2)
@@ -278,7 +379,7 @@ __device__ __forceinline__ void finish_cand(Cand &s, const Smem &sm, const EvalP
       P.info[c] = info;
     }
     if ((MODE & kFull) && !invalid) {
-      const uint32_t ns = min(s.i, (uint32_t)P.p_max);
+      const uint32_t ns = min(s.p, (uint32_t)P.p_max);
       for (uint32_t k = 0; k < ns; ++k) P.stage_T[(int64_t)k * P.n + c] += s.sumS;
     }
     if ((MODE & kSelect) && !invalid) {
@@ -293,8 +394,11 @@ __device__ __forceinline__ void finish_cand(Cand &s, const Smem &sm, const EvalP
   }
 }
 
-template <uint32_t MODE>
-__global__ void __launch_bounds__(kThreads) eval_kernel(const __grid_constant__ EvalParams P) {
+// ---------------------------------------------------------------------------
+// kernel
+// ---------------------------------------------------------------------------
+template <uint32_t MODE, int SPLIT>
+__global__ void __launch_bounds__(kThreads, ACESO_MINB) eval_kernel(const __grid_constant__ EvalParams P) {
   extern __shared__ __align__(128) unsigned char sm_raw[];
   __shared__ __align__(8) uint64_t s_tbar;
   __shared__ __align__(8) uint64_t s_ring_bar[kWarps][kRingSlots];
@@ -302,6 +406,9 @@ __global__ void __launch_bounds__(kThreads) eval_kernel(const __grid_constant__ 
   __shared__ int64_t s_idx[kWarps];
 
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const int npairs = kWarps / SPLIT;
+  const int pair = SPLIT == 2 ? (warp >> 1) : warp;
+  const int part = SPLIT == 2 ? (warp & 1) : 0;
   const uint32_t tab_bytes = (MODE & kFull) ? P.tab.bytes_full : P.tab.bytes;
   const uint32_t sb = smem_addr(sm_raw);
   Smem sm;
@@ -309,10 +416,15 @@ __global__ void __launch_bounds__(kThreads) eval_kernel(const __grid_constant__ 
   sm.D = sb + P.tab.offD;
   sm.T = sb + P.tab.offT;
   sm.F = sb + P.tab.offF;
-  sm.K = reinterpret_cast<const unsigned char *>(P.blob) + P.tab.offK;
-  const uint32_t ring = sb + tab_bytes + (uint32_t)warp * kRingSlots * kSlotBytes;
+  sm.K = sb + tab_bytes;  // cold table staged after the other tables when k_smem
+  sm.Kg = reinterpret_cast<const unsigned char *>(P.blob) + P.tab.offK;
+  sm.k_smem = P.tab.k_smem;
+  sm.TS = (uint32_t)P.T * kTypeStride;
+  const uint32_t stage_bytes = tab_bytes + (P.tab.k_smem ? P.tab.bytesK : 0u);
+  const uint32_t ring = sb + stage_bytes + (uint32_t)warp * kRingSlots * kSlotBytes;
+  Xchg *xch = reinterpret_cast<Xchg *>(sm_raw + stage_bytes + kRingBytesPerCta) + pair * 32;
 
-  // ---- stage the packed tables (one bulk copy, TMA) ----
+  // ---- stage the packed tables (TMA bulk copies) ----
   if (threadIdx.x == 0) {
     mbar_init(smem_addr(&s_tbar), 1);
     fence_barrier_init();
@@ -324,32 +436,47 @@ __global__ void __launch_bounds__(kThreads) eval_kernel(const __grid_constant__ 
   __syncthreads();
   if (threadIdx.x == 0) {
     const uint32_t bar = smem_addr(&s_tbar);
-    mbar_expect_tx(bar, tab_bytes);
+    mbar_expect_tx(bar, stage_bytes);
     bulk_g2s(sb, P.blob, tab_bytes, bar);
+    if (P.tab.k_smem) bulk_g2s(sb + tab_bytes, sm.Kg, P.tab.bytesK, bar);
   }
 
-  // ---- this warp's stream of units (tile, group of kSlotChunks chunks) ----
-  const int64_t first_tile = (int64_t)blockIdx.x * kWarps + warp;
-  const int64_t tile_stride = (int64_t)gridDim.x * kWarps;
+  // ---- this warp's part of every tile it owns ----
+  const uint32_t nch = (uint32_t)P.nch;
+  const uint32_t nch0 = SPLIT == 2 ? (nch + 1) / 2 : nch;
+  const uint32_t c_lo = part ? nch0 : 0u, c_hi = part ? nch : nch0;
+  const uint32_t ngroups = (c_hi - c_lo + kSlotChunks - 1) / kSlotChunks;
+  const int64_t first_tile = (int64_t)blockIdx.x * npairs + pair;
+  const int64_t tile_stride = (int64_t)gridDim.x * npairs;
   const int64_t my_tiles =
       first_tile < P.n_tiles ? (P.n_tiles - first_tile + tile_stride - 1) / tile_stride : 0;
-  const uint32_t ngroups = ((uint32_t)P.nch + kSlotChunks - 1) / kSlotChunks;
   const int64_t units = my_tiles * ngroups;
+  const unsigned char *codes = reinterpret_cast<const unsigned char *>(P.codes);
 
-  auto issue = [&](int64_t u) {
-    const int64_t t = first_tile + (u / ngroups) * tile_stride;
-    const uint32_t g = (uint32_t)(u % ngroups);
-    const uint32_t c0 = g * kSlotChunks;
-    const uint32_t nc = min((uint32_t)kSlotChunks, (uint32_t)P.nch - c0);
-    const int slot = (int)(u % kRingSlots);
+  // chunk range of group g of this part (ascending addresses)
+  auto group_lo = [&](uint32_t g) {
+    return part ? (c_hi >= kSlotChunks * (g + 1) + c_lo ? c_hi - kSlotChunks * (g + 1) : c_lo)
+                : c_lo + kSlotChunks * g;
+  };
+  auto group_hi = [&](uint32_t g) {
+    return part ? c_hi - kSlotChunks * g : min(c_lo + kSlotChunks * (g + 1), c_hi);
+  };
+  // issue cursor (lane 0)
+  int64_t it_tile = first_tile;
+  uint32_t it_g = 0;
+  auto issue_next = [&](int slot) {
+    const uint32_t a = group_lo(it_g), b = group_hi(it_g);
     const uint32_t bar = smem_addr(&s_ring_bar[warp][slot]);
-    const unsigned char *src =
-        reinterpret_cast<const unsigned char *>(P.codes) + ((size_t)t * P.nch + c0) * 512;
-    mbar_expect_tx(bar, nc * 512u);
-    bulk_g2s(ring + slot * kSlotBytes, src, nc * 512u, bar);
+    mbar_expect_tx(bar, (b - a) * 512u);
+    bulk_g2s(ring + slot * kSlotBytes, codes + ((size_t)it_tile * nch + a) * 512, (b - a) * 512u,
+             bar);
+    if (++it_g == ngroups) {
+      it_g = 0;
+      it_tile += tile_stride;
+    }
   };
   if (lane == 0) {
-    for (int64_t u = 0; u < units && u < kRingSlots; ++u) issue(u);
+    for (int64_t u = 0; u < units && u < kRingSlots; ++u) issue_next((int)u);
   }
   __syncwarp();
 
@@ -358,33 +485,101 @@ __global__ void __launch_bounds__(kThreads) eval_kernel(const __grid_constant__ 
   uint64_t best_ck = ~0ull;
   int64_t best_idx = INT64_MAX;
   Cand s;
-  uint32_t prevw = 0;
+  uint32_t cw = 0, ct = 0;  // forward: previous word; reverse: next word / next type offset
+  uint32_t cM = 0, tM = 0;  // reverse: code and type offset of op M (the part's first op)
+  int64_t tile = first_tile;
+  uint32_t g = 0;
+  int slot = 0;
+  uint32_t phase = 0;
   int64_t cand = 0;
   bool active = false;
   for (int64_t u = 0; u < units; ++u) {
-    const int64_t t = first_tile + (u / ngroups) * tile_stride;
-    const uint32_t g = (uint32_t)(u % ngroups);
-    const int slot = (int)(u % kRingSlots);
     if (g == 0) {
-      cand = t * 32 + lane;
+      cand = tile * 32 + lane;
       active = cand < P.n;
-      init_cand<MODE>(s, sm, P, active ? __ldg(P.hdr + cand) : 0ull);
-      prevw = 0;
+      init_cand(s, sm, P, active ? __ldg(P.hdr + cand) : 0ull, part == 1);
+      cw = 0;
+      ct = 0;
     }
-    mbar_wait(smem_addr(&s_ring_bar[warp][slot]), (uint32_t)((u / kRingSlots) & 1));
-    const uint32_t c0 = g * kSlotChunks;
-    const uint32_t nc = min((uint32_t)kSlotChunks, (uint32_t)P.nch - c0);
+    mbar_wait(smem_addr(&s_ring_bar[warp][slot]), phase);
+    const uint32_t a = group_lo(g), b = group_hi(g);
     const uint32_t slot_a = ring + slot * kSlotBytes + lane * 16;
-    for (uint32_t k = 0; k < nc; ++k) {
-      const uint4 v = lds128(nullptr, slot_a + k * 512);
-      process_chunk<MODE>(s, sm, P, v, c0 + k, prevw, cand, active);
+    const uint32_t nq = (b - a) * 4u;  // quads in this slot
+    if (part == 0) {
+#pragma unroll 1
+      for (uint32_t qq = 0; qq < nq; ++qq) {
+        const uint32_t qg = a * 4u + qq;
+        if (qg * 4u >= (uint32_t)P.L) break;
+        const uint32_t w = lds32(slot_a + (qq >> 2) * 512u + (qq & 3u) * 4u);
+        quad_fwd<MODE>(s, sm, P, w, cw, qg, cand, active);
+      }
+    } else {
+#pragma unroll 1
+      for (uint32_t qq = nq; qq-- > 0;) {
+        const uint32_t qg = a * 4u + qq;
+        if (qg * 4u >= (uint32_t)P.L) continue;
+        const uint32_t w = lds32(slot_a + (qq >> 2) * 512u + (qq & 3u) * 4u);
+        quad_rev<MODE>(s, sm, P, w, cw, ct, qg, cand, active);
+        if (qg == c_lo * 4u) {
+          cM = w & 0xffu;
+          tM = ct;
+        }
+      }
     }
     __syncwarp();
     if (lane == 0 && u + kRingSlots < units) {
       fence_proxy_async();
-      issue(u + kRingSlots);
+      issue_next(slot);
     }
-    if (g == ngroups - 1) finish_cand<MODE>(s, sm, P, cand, active, best_ck, best_idx);
+    if (++slot == kRingSlots) {
+      slot = 0;
+      phase ^= 1u;
+    }
+    if (++g == ngroups) {
+      // ---- tile epilogue ----
+      if (SPLIT == 1) {
+        stage_commit<MODE>(s, P, cand, active, false);  // last stage: no p2p_fwd
+        finish_cand<MODE>(s, P, cand, active, best_ck, best_idx);
+      } else {
+        const uint32_t M = nch0 * 16u;
+        if (part == 1) {
+          // boundary pair (M-1, M): in-stage tp/dp change -> reshard of op M, symmetry
+          const uint32_t cb = codes[((size_t)tile * nch + (nch0 - 1)) * 512 + lane * 16 + 15];
+          if (!(cM & 1u) && ((cM ^ cb) & 0xEEu)) {
+            s.S += ldk(sm, s.kbase + (tM >> 1));
+            if ((((cb >> 1) & 7u) + (cb >> 5)) != s.gst) s.reasons |= ACESO_R_GSTAGE;
+          }
+          Xchg &xr = xch[lane];
+          xr.S = s.S; xr.A = s.A; xr.W = s.W; xr.D = s.D; xr.comp = s.comp; xr.E = s.E;
+          xr.sumS = s.sumS; xr.bestT = s.bestT; xr.bestM = s.bestM; xr.bt = s.bt; xr.bm = s.bm;
+          xr.flags = s.oom | ((cM & 1u) << 1);
+          xr.gsum = s.gsum; xr.reasons = s.reasons; xr.nheads = s.nheads;
+        }
+        pair_bar_sync(pair);
+        if (part == 0) {
+          const Xchg &xr = xch[lane];
+          if (xr.flags & 2u) {
+            // op M is a head: part 0's open stage ends at M-1 and is followed by a stage
+            s.S += ldk(sm, s.kbase + (lds32(sm.T + (M - 1) * 4u) >> 1) + 4);  // R5 p2p_fwd
+          } else {
+            s.S += xr.S; s.A += xr.A; s.W += xr.W; s.D += xr.D; s.comp += xr.comp;
+            s.E = max(s.E, xr.E);
+          }
+          stage_commit<MODE>(s, P, cand, active, false);  // the stage spanning M
+          s.sumS += xr.sumS;
+          if (xr.bt != kNone && xr.bestT > s.bestT) { s.bestT = xr.bestT; s.bt = xr.bt; }
+          if (xr.bm != kNone && xr.bestM > s.bestM) { s.bestM = xr.bestM; s.bm = xr.bm; }
+          s.oom |= xr.flags & 1u;
+          s.gsum += xr.gsum;
+          s.reasons |= xr.reasons;
+          s.nheads += xr.nheads;
+          finish_cand<MODE>(s, P, cand, active, best_ck, best_idx);
+        }
+        pair_bar_sync(pair);  // hand-over record free for the next tile
+      }
+      g = 0;
+      tile += tile_stride;
+    }
   }
 
   if (MODE & kSelect)
