@@ -42,6 +42,8 @@ def parse():
     ap.add_argument("--group", type=int, default=1024, help="candidates sharing a base config")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--streams", type=int, default=1,
+                    help="independent batches in flight (steps round-robin over streams)")
     return ap.parse_args()
 
 
@@ -253,17 +255,30 @@ def main():
     if world > 1:
         dist.barrier()
     torch.cuda.synchronize()
+    nstr = max(1, min(args.streams, nbuf))
+    outs = [out] + [ctx.alloc_outputs(n) for _ in range(nstr - 1)]
+    side = [torch.cuda.Stream() for _ in range(nstr)]
     with torch.cuda.graph(graph):
         cs = torch.cuda.current_stream()
+        fork = torch.cuda.Event()
+        fork.record(cs)
+        for st in side:
+            st.wait_event(fork)
         for s in range(args.steps):
             b = s % nbuf
+            st = side[s % nstr] if nstr > 1 else cs
             codes_d, hdr_d = dev_batches[b]
-            ev_s[s].record(cs)
+            ev_s[s].record(st)
             ctx.eval(codes_d, hdr_d, n=n, global_offset=rank * n, n_total=n_total, summary=True,
-                     select=True, out=out, sel=sels[b], stream=cs)
-            ev_k[s].record(cs)
+                     select=True, out=outs[s % nstr], sel=sels[b], stream=st)
+            ev_k[s].record(st)
             if world > 1:
-                dist.all_reduce(sels[b][0:8].view(torch.int64), op=dist.ReduceOp.MIN)
+                with torch.cuda.stream(st):
+                    dist.all_reduce(sels[b][0:8].view(torch.int64), op=dist.ReduceOp.MIN)
+        for st in side:
+            j = torch.cuda.Event()
+            j.record(st)
+            cs.wait_event(j)
     torch.cuda.synchronize()
     graph.replay()  # one untimed replay (graph upload)
     torch.cuda.synchronize()

@@ -5,6 +5,8 @@
 #include <cuda_runtime.h>
 
 #include <algorithm>
+#include <array>
+#include <map>
 #include <cstdarg>
 #include <cstdio>
 #include <cstdlib>
@@ -168,51 +170,136 @@ int aceso_load_profile(const aceso_profile_desc *d, int cuda_device, aceso_ctx *
 
   // ---- pack tables ----
   const uint32_t S = kTypeStride;
-  const uint32_t bytesR = (uint32_t)NB * NT * T * S;
+  const uint32_t RUNS = (uint32_t)NB * NT;
+  const int nch = (L + 15) / 16;
+  const int nquads = nch * 4;  // quads incl. the zero-padded tail
+  auto a16 = [](uint32_t v) { return (v + 15u) & ~15u; };
+  // quad signatures: distinct type 4-tuples of the full quads
+  std::vector<int> qsig(nquads, -1);
+  std::vector<std::array<uint16_t, 4>> sigs;
+  {
+    std::map<std::array<uint16_t, 4>, int> seen;
+    for (int q = 0; q < nquads; ++q) {
+      if (4 * q + 4 > L) continue;
+      std::array<uint16_t, 4> key = {d->op_type[4 * q], d->op_type[4 * q + 1], d->op_type[4 * q + 2], d->op_type[4 * q + 3]};
+      auto it = seen.find(key);
+      if (it == seen.end()) {
+        it = seen.emplace(key, (int)sigs.size()).first;
+        sigs.push_back(key);
+      }
+      qsig[q] = it->second;
+    }
+  }
+  const uint32_t NS = (uint32_t)sigs.size();
+  const uint32_t bytesR = RUNS * T * S;
   const uint32_t bytesD = (uint32_t)NT * T * S;
-  const uint32_t bytesT = (uint32_t)((L + 15) / 16) * 64;
-  const uint32_t bytesF = ((uint32_t)NB * NT * T * 8 + 15) / 16 * 16;
-  const uint32_t bytesK = (uint32_t)NB * NT * T * 16;
+  const uint32_t bytesT = a16((uint32_t)nch * 16 * 2);
+  const uint32_t bytesQO = (uint32_t)nquads * 8;
+  const uint32_t bytesQT = NS * RUNS * 32;
+  const uint32_t bytesQD = NS * (uint32_t)NT * 32;
+  const uint32_t bytesF = a16(RUNS * T * 8);
+  const uint32_t bytesQF = a16(NS * RUNS * 8);
+  const uint32_t bytesK = RUNS * T * 16;
   Tables tab;
+  memset(&tab, 0, sizeof(tab));
   tab.offR = 0;
-  tab.offD = bytesR;
+  tab.offD = tab.offR + bytesR;
   tab.offT = tab.offD + bytesD;
-  tab.offF = tab.offT + bytesT;
-  tab.bytes = tab.offF;
-  tab.bytes_full = tab.offF + bytesF;
+  tab.offQO = tab.offT + bytesT;
+  tab.offQT = tab.offQO + bytesQO;
+  tab.offQD = tab.offQT + bytesQT;
+  tab.bytes = tab.offQD + bytesQD;
+  tab.offF = tab.bytes;
+  tab.offQF = tab.offF + bytesF;
+  tab.bytes_full = tab.offQF + bytesQF;
   tab.offK = tab.bytes_full;
   tab.bytesK = bytesK;
   // stage the cold table too when shared memory allows ~2 CTAs per SM
   tab.k_smem = (tab.bytes_full + bytesK + kRingBytesPerCta + 16384u <= 100u * 1024u) ? 1u : 0u;
-  if (tab.bytes_full > 180u * 1024u) return fail(ACESO_EINVAL, "packed tables of %u bytes exceed shared memory", tab.bytes_full);
+  if (tab.bytes_full + kRingBytesPerCta + 16384u > 220u * 1024u)
+    return fail(ACESO_EINVAL, "packed tables of %u bytes exceed shared memory", tab.bytes_full);
   const uint32_t blob_bytes = tab.offK + bytesK;
   std::vector<uint32_t> blob(blob_bytes / 4, 0u);
+  auto rec_S = [&](int t, int tp, int b, int rc) -> uint64_t {
+    uint64_t F = (uint64_t)R(t, tp, b, 0) + R(t, tp, b, 1);
+    return F + R(t, tp, b, 2) + R(t, tp, b, 3) + (rc ? F : 0);
+  };
+  auto rec_A = [&](int t, int tp, int b, int rc) -> uint64_t { return (uint64_t)(rc ? R(t, tp, b, 5) : R(t, tp, b, 4)) >> ms; };
+  auto rec_e = [&](int t, int tp, int b, int rc) -> uint64_t {
+    return ((uint64_t)R(t, tp, b, 6) + (rc ? (uint64_t)(R(t, tp, b, 4) - R(t, tp, b, 5)) : 0)) >> ms;
+  };
+  auto rec_W = [&](int t, int tp) -> uint64_t {
+    return ((uint64_t)d->wmem[((int64_t)t * NT + tp) * 2] + (uint64_t)d->wmem[((int64_t)t * NT + tp) * 2 + 1]) >> ms;
+  };
+  auto rec_C = [&](int t, int tp, int b, int rc) -> uint64_t {
+    return (uint64_t)R(t, tp, b, 0) + R(t, tp, b, 2) + (rc ? (uint64_t)R(t, tp, b, 0) : 0);
+  };
+  auto dps_of = [&](int t, int tp, int dp) -> uint64_t { return (uint64_t)d->dps[((int64_t)t * NT + tp) * ND + dp]; };
   for (int b = 0; b < NB; ++b)
     for (int tp = 0; tp < NT; ++tp)
       for (int t = 0; t < T; ++t) {
         const uint32_t rt = (uint32_t)(b * NT + tp) * T + t;  // (run, type) index
-        const uint32_t run = rt * S / 4;
-        uint64_t fc = R(t, tp, b, 0), fm = R(t, tp, b, 1), bc = R(t, tp, b, 2), bm = R(t, tp, b, 3);
-        uint64_t act = R(t, tp, b, 4), keep = R(t, tp, b, 5), peak = R(t, tp, b, 6);
-        uint64_t W = (uint64_t)d->wmem[((int64_t)t * NT + tp) * 2] + (uint64_t)d->wmem[((int64_t)t * NT + tp) * 2 + 1];
         for (int rc = 0; rc < 2; ++rc) {
-          uint32_t *r = &blob[(tab.offR / 4) + run + rc * 4];
-          r[0] = (uint32_t)(fc + fm + bc + bm + (rc ? fc + fm : 0));
-          r[1] = (uint32_t)((rc ? keep : act) >> ms);
-          r[2] = (uint32_t)((peak + (rc ? act - keep : 0)) >> ms);
-          r[3] = (uint32_t)(W >> ms);
-          blob[(tab.offF / 4) + rt * 2 + rc] = (uint32_t)(fc + bc + (rc ? fc : 0));
+          uint32_t *r = &blob[(tab.offR / 4) + rt * (S / 4) + rc * 4];
+          r[0] = (uint32_t)rec_S(t, tp, b, rc);
+          r[1] = (uint32_t)rec_A(t, tp, b, rc);
+          r[2] = (uint32_t)rec_e(t, tp, b, rc);
+          r[3] = (uint32_t)rec_W(t, tp);
+          blob[(tab.offF / 4) + rt * 2 + rc] = (uint32_t)rec_C(t, tp, b, rc);
         }
         uint32_t *k = &blob[(tab.offK / 4) + rt * 4];
         k[0] = (uint32_t)R(t, tp, b, 7);
         k[1] = (uint32_t)R(t, tp, b, 8);
         k[2] = (uint32_t)R(t, tp, b, 9);
       }
-  for (int j = 0; j < L; ++j) blob[tab.offT / 4 + j] = (uint32_t)d->op_type[j] * S;
   for (int tp = 0; tp < NT; ++tp)
     for (int t = 0; t < T; ++t)
       for (int dp = 0; dp < ND; ++dp)
-        blob[(tab.offD + ((uint32_t)tp * T + t) * S) / 4 + dp] = (uint32_t)d->dps[((int64_t)t * NT + tp) * ND + dp];
+        blob[(tab.offD + ((uint32_t)tp * T + t) * S) / 4 + dp] = (uint32_t)dps_of(t, tp, dp);
+  {
+    uint16_t *tt = reinterpret_cast<uint16_t *>(&blob[tab.offT / 4]);
+    for (int j = 0; j < L; ++j) tt[j] = d->op_type[j];
+  }
+  // quad sums; a signature whose sums do not fit 32 bits is not used (per-op path)
+  std::vector<char> sig_ok(NS, 1);
+  for (uint32_t sg = 0; sg < NS; ++sg) {
+    const auto &ty = sigs[sg];
+    for (int b = 0; b < NB; ++b)
+      for (int tp = 0; tp < NT; ++tp) {
+        const uint32_t run = (uint32_t)(b * NT + tp);
+        for (int rc = 0; rc < 2; ++rc) {
+          uint64_t sS = 0, sA = 0, mE = 0, sW = 0, sC = 0;
+          for (int k = 0; k < 4; ++k) {
+            sS += rec_S(ty[k], tp, b, rc);
+            sA += rec_A(ty[k], tp, b, rc);
+            mE = std::max(mE, rec_e(ty[k], tp, b, rc));
+            sW += rec_W(ty[k], tp);
+            sC += rec_C(ty[k], tp, b, rc);
+          }
+          if (sS > U32 || sA > U32 || sW > U32 || sC > U32) sig_ok[sg] = 0;
+          uint32_t *q = &blob[(tab.offQT / 4) + (sg * RUNS + run) * 8 + rc * 4];
+          q[0] = (uint32_t)sS; q[1] = (uint32_t)sA; q[2] = (uint32_t)mE; q[3] = (uint32_t)sW;
+          blob[(tab.offQF / 4) + (sg * RUNS + run) * 2 + rc] = (uint32_t)sC;
+        }
+      }
+    for (int tp = 0; tp < NT; ++tp)
+      for (int dp = 0; dp < ND; ++dp) {
+        uint64_t sD = 0;
+        for (int k = 0; k < 4; ++k) sD += dps_of(ty[k], tp, dp);
+        if (sD > U32) sig_ok[sg] = 0;
+        blob[(tab.offQD / 4) + (sg * NT + tp) * 8 + dp] = (uint32_t)sD;
+      }
+  }
+  for (int q = 0; q < nquads; ++q) {
+    uint32_t *o = &blob[(tab.offQO / 4) + q * 2];
+    if (qsig[q] >= 0 && sig_ok[qsig[q]]) {
+      o[0] = (uint32_t)qsig[q] * RUNS * 32;
+      o[1] = (uint32_t)qsig[q] * NT * 32;
+    } else {
+      o[0] = 0xffffffffu;
+      o[1] = 0;
+    }
+  }
 
   // ---- device ----
   int ndev = 0;
@@ -246,7 +333,7 @@ int aceso_load_profile(const aceso_profile_desc *d, int cuda_device, aceso_ctx *
     cudaStreamDestroy(st);
     if (e != cudaSuccess) { rc = fail(e == cudaErrorMemoryAllocation ? ACESO_ENOMEM : ACESO_ECUDA, "upload: %s", cudaGetErrorString(e)); break; }
     const int nch = (L + 15) / 16;
-    ctx->split = nch >= 2 ? 2 : 1;
+    ctx->split = 1;  // one warp per tile; ACESO_SPLIT=2 selects the forward/reverse warp pair
     if (const char *env = getenv("ACESO_SPLIT")) {
       int v = atoi(env);
       if (v == 1 || (v == 2 && nch >= 2)) ctx->split = v;

@@ -24,12 +24,18 @@ constexpr uint32_t kTypeStride = 32;         // bytes per op type in every smem 
 // the largest power of two dividing every memory value of the profile (<= 2^16), so
 // the sums stay exact: Mem_i = (Wst + infl * A + E) << mem_shift.
 // DP table D[tpl][type][dpl] : u32 DP gradient all-reduce ns, 8 dpl slots per 32-byte entry
-// Type offsets O[j] : u32 type_j * 32 for every op (16-entry chunks, zero padded)
+// Type table T[j] : u16 type_j for every op (16-entry chunks, zero padded)
+// Quad tables (4 consecutive ops j = 4q..4q+3 with the same run and rc; sums exact in u32):
+//   QO[q]            : {sig * RUNS * 32, sig * n_tp * 32} or {kNone, 0} (no quad sums)
+//   QT[sig][run][rc] : 16 B {sum S', sum A, max e, sum W} over the quad's 4 op types
+//   QD[sig][tpl][dpl]: u32 sum of DP all-reduce ns (8 dpl slots)
+//   QF[sig][run][rc] : u32 sum of comp (FULL only)
 // Full table F[b][tpl][type][rc] : u32 comp = fwd_comp + bwd_comp + rc*fwd_comp (8 B per type)
 // Cold table K[b][tpl][type] : 16 bytes {reshard, p2p_fwd, p2p_bwd, 0}  (R5, R13), read
 //   from global memory (L1/L2) at events only — after the shared blob in the same allocation
 struct Tables {
-  uint32_t offR, offD, offT, offF;  // byte offsets inside the staged blob (shared memory)
+  uint32_t offR, offD, offT, offQO, offQT, offQD;  // byte offsets in the staged blob (smem)
+  uint32_t offF, offQF;                            // FULL-only tables (staged after bytes)
   uint32_t bytes;                   // bytes staged to shared memory (multiple of 16)
   uint32_t bytes_full;              // bytes staged including the F table
   uint32_t offK;                    // byte offset of the cold table in the global blob

@@ -99,12 +99,25 @@ __device__ __forceinline__ uint32_t lds32(uint32_t a) {
   asm volatile("ld.shared.u32 %0, [%1];" : "=r"(v) : "r"(a));
   return v;
 }
+__device__ __forceinline__ uint2 lds64(uint32_t a) {
+  uint2 v;
+  asm volatile("ld.shared.v2.u32 {%0, %1}, [%2];" : "=r"(v.x), "=r"(v.y) : "r"(a));
+  return v;
+}
+__device__ __forceinline__ uint32_t lds16(uint32_t a) {
+  uint16_t v;
+  asm volatile("ld.shared.u16 %0, [%1];" : "=h"(v) : "r"(a));
+  return v;
+}
+// type offset (type * 32) of op j from the u16 type table
+__device__ __forceinline__ uint32_t toff_of(uint32_t T, uint32_t j) { return lds16(T + 2u * j) << 5; }
 
 // ---------------------------------------------------------------------------
 // state
 // ---------------------------------------------------------------------------
 struct Smem {
   uint32_t R, D, F, T, K;   // shared addresses of the staged tables (K valid if k_smem)
+  uint32_t QO, QT, QD, QF;  // quad tables: per-quad offsets, sums, DP sums, comp sums
   const unsigned char *Kg;  // cold table in global memory
   uint32_t k_smem;
   uint32_t TS;              // T * 32: bytes of one (b, tpl) block of R
@@ -118,8 +131,9 @@ struct Cand {
   // current stage: per-microbatch sums (R5/R13 terms included in S)
   uint64_t S, A, W, D, comp;
   uint32_t E;
-  // current run (ops of equal (tp, dp) inside one stage)
+  // current run (ops of equal (tp, dp) inside one stage): per-op and per-quad table bases
   uint32_t rbase, dbase, kbase, fbase, gst;
+  uint32_t qrun, qd, qf;
   // candidate-level aggregates
   uint64_t sumS, bestT, bestM;
   uint32_t bt, bm, oom, i, gsum, reasons, nheads, head0;
@@ -174,6 +188,23 @@ __device__ __forceinline__ void open_run(Cand &s, const Smem &sm, const EvalPara
   s.kbase = run * (sm.TS >> 1);
   if (MODE & kFull) s.fbase = sm.F + run * (sm.TS >> 2);
   s.dbase = sm.D + tplc * sm.TS + dpl * 4u;
+  s.qrun = sm.QT + run * 32u;
+  s.qd = sm.QD + tplc * 32u + dpl * 4u;
+  if (MODE & kFull) s.qf = sm.QF + run * 8u;
+}
+
+// a whole quad from the quad tables: o = {sig * quad-sum stride, sig * DP stride},
+// rsel = rc * 16 (uniform rc inside the quad)
+template <uint32_t MODE>
+__device__ __forceinline__ void accumulate_quad(Cand &s, uint2 o, uint32_t rsel) {
+  const uint4 r = lds128(s.qrun + o.x + rsel);
+  const uint32_t d = lds32(s.qd + o.y);
+  s.S += r.x;
+  s.A += r.y;
+  s.E = max(s.E, r.z);
+  s.W += r.w;
+  s.D += d;
+  if (MODE & kFull) s.comp += lds32(s.qf + (o.x >> 2) + (rsel >> 2));
 }
 
 template <uint32_t MODE>
@@ -265,6 +296,9 @@ __device__ __forceinline__ void init_cand(Cand &s, const Smem &sm, const EvalPar
   s.dbase = sm.D;
   s.kbase = 0;
   s.fbase = sm.F;
+  s.qrun = sm.QT;
+  s.qd = sm.QD;
+  s.qf = sm.QF;
   s.gst = 0;
 }
 
@@ -277,36 +311,33 @@ template <uint32_t MODE>
 __device__ __forceinline__ void quad_fwd(Cand &s, const Smem &sm, const EvalParams &P, uint32_t w,
                                          uint32_t &pw, uint32_t qg, int64_t cand, bool active) {
   const uint32_t sh = __funnelshift_l(pw, w, 8);  // previous op's byte under each byte
-  uint32_t x = ((w ^ sh) & 0xEEEEEEEEu) | (w & 0x01010101u);  // tp/dp change | head
+  // per byte: bit 0 = head; bits 1-7 = difference to the previous op's code. For op 0 of
+  // a tile the caller seeds pw so that op 0 always shows a tp/dp difference (opens a run).
+  uint32_t d;
+  asm("lop3.b32 %0, %1, %2, %3, 0xB4;" : "=r"(d) : "r"(w), "r"(sh), "r"(0x01010101u));  // c ? w : w^sh
+  d &= 0xffffffefu;  // an rc change at the quad's first op does not make it mixed
   pw = w;
-  if (qg == 0) {
-    x |= 0xffu;  // op 0 always opens the first run
-    s.head0 = w & 1u;
+  const uint2 o = lds64(sm.QO + 8u * qg);  // quad signature offsets (kNone: no quad sums)
+  // clean lane (no head, no tp/dp change, uniform rc) -> one quad-table gather
+  if (d == 0u && o.x != kNone) {
+    accumulate_quad<MODE>(s, o, w & 0x10u);
+    return;
   }
+  const uint32_t x = d & 0xefefefefu;  // events: head or tp/dp change
   const uint32_t j0 = qg * 4u;
   const uint32_t nvalid = min(4u, (uint32_t)P.L - j0);
-  if (nvalid < 4u) x &= 0xffffffffu >> (8 * (4u - nvalid));
-  const uint32_t U = __reduce_or_sync(0xffffffffu, x);
-  const uint32_t ta = sm.T + j0 * 4u;  // type offsets of these ops (broadcast loads)
-  if (U == 0u && nvalid == 4u) {
-    // no head, no tp/dp change in any lane: branch-free
-    const uint4 t4 = lds128(ta);
-    const uint32_t rcw = w & 0x10101010u;  // rc * 16 per byte
-    accumulate<MODE>(s, __byte_perm(rcw, 0, 0x4440), t4.x);
-    accumulate<MODE>(s, __byte_perm(rcw, 0, 0x4441), t4.y);
-    accumulate<MODE>(s, __byte_perm(rcw, 0, 0x4442), t4.z);
-    accumulate<MODE>(s, __byte_perm(rcw, 0, 0x4443), t4.w);
-  } else {
-    uint32_t tprev = j0 > 0 ? lds32(ta - 4u) : 0u;
-#pragma unroll 1
-    for (uint32_t k = 0; k < nvalid; ++k) {
-      const uint32_t toff = lds32(ta + 4u * k);
-      const uint32_t c = (w >> (8 * k)) & 0xffu;
-      if ((U >> (8 * k)) & 0xffu) {
-        if ((x >> (8 * k)) & 0xffu) fwd_event<MODE>(s, sm, P, j0 + k, c, toff, tprev, cand, active);
+  const uint2 tt = lds64(sm.T + 2u * j0);  // the quad's 4 u16 types
+  const uint32_t t4[4] = {(tt.x & 0xffffu) << 5, (tt.x >> 16) << 5, (tt.y & 0xffffu) << 5,
+                          (tt.y >> 16) << 5};
+  const uint32_t rc4 = w & 0x10101010u;
+#pragma unroll
+  for (int k = 0; k < 4; ++k) {
+    if ((uint32_t)k < nvalid) {
+      if ((x >> (8 * k)) & 0xffu) {
+        const uint32_t tprev = k > 0 ? t4[k - 1] : (j0 > 0 ? toff_of(sm.T, j0 - 1) : 0u);
+        fwd_event<MODE>(s, sm, P, j0 + k, (w >> (8 * k)) & 0xffu, t4[k], tprev, cand, active);
       }
-      accumulate<MODE>(s, c & 0x10u, toff);
-      tprev = toff;
+      accumulate<MODE>(s, __byte_perm(rc4, 0, 0x4440 + k), t4[k]);
     }
   }
 }
@@ -325,37 +356,39 @@ __device__ __forceinline__ void quad_rev(Cand &s, const Smem &sm, const EvalPara
   const uint32_t j0 = qg * 4u;
   const uint32_t nvalid = min(4u, (uint32_t)P.L - j0);
   if (j0 + nvalid == (uint32_t)P.L) x |= 0x80u << (8 * (nvalid - 1));  // last op: last stage
-  if (nvalid < 4u) x &= 0xffffffffu >> (8 * (4u - nvalid));
-  const uint32_t U = __reduce_or_sync(0xffffffffu, x);
-  const uint32_t ta = sm.T + j0 * 4u;
-  if (U == 0u && nvalid == 4u) {
-    const uint4 t4 = lds128(ta);
-    const uint32_t rcw = w & 0x10101010u;
-    accumulate<MODE>(s, __byte_perm(rcw, 0, 0x4440), t4.x);
-    accumulate<MODE>(s, __byte_perm(rcw, 0, 0x4441), t4.y);
-    accumulate<MODE>(s, __byte_perm(rcw, 0, 0x4442), t4.z);
-    accumulate<MODE>(s, __byte_perm(rcw, 0, 0x4443), t4.w);
-    tn = t4.x;
-  } else {
-#pragma unroll 1
-    for (int k = (int)nvalid - 1; k >= 0; --k) {
-      const uint32_t toff = lds32(ta + 4u * k);
+  const uint2 o = lds64(sm.QO + 8u * qg);
+  const uint32_t rcw = w & 0x10101010u;
+  const uint32_t mix = rcw ^ __byte_perm(rcw, 0, 0x0000);
+  if (o.x != kNone && !__any_sync(0xffffffffu, (x | mix) != 0u)) {
+    accumulate_quad<MODE>(s, o, rcw & 0x10u);
+    tn = toff_of(sm.T, j0);
+    nw = w;
+    return;
+  }
+  if (o.x != kNone && (x | mix) == 0u) {
+    accumulate_quad<MODE>(s, o, rcw & 0x10u);
+    tn = toff_of(sm.T, j0);
+    nw = w;
+    return;
+  }
+  const uint2 tt = lds64(sm.T + 2u * j0);
+  const uint32_t t4[4] = {(tt.x & 0xffffu) << 5, (tt.x >> 16) << 5, (tt.y & 0xffffu) << 5,
+                          (tt.y >> 16) << 5};
+  const uint32_t rc4 = w & 0x10101010u;
+#pragma unroll
+  for (int k = 3; k >= 0; --k) {
+    if ((uint32_t)k < nvalid) {
       const uint32_t c = (w >> (8 * k)) & 0xffu;
       const uint32_t e = (x >> (8 * k)) & 0xffu;
-      const uint32_t u = (U >> (8 * k)) & 0xffu;
-      if (u & 0xfeu) {
-        if (e & 0xfeu) {
-          const uint32_t cn = k < 3 ? (w >> (8 * k + 8)) & 0xffu : nw & 0xffu;
-          rev_pre<MODE>(s, sm, P, j0 + k, c, cn, toff, tn);
-        }
+      if (e & 0xfeu) {
+        const uint32_t cn = k < 3 ? (w >> (8 * k + 8)) & 0xffu : nw & 0xffu;
+        rev_pre<MODE>(s, sm, P, j0 + k, c, cn, t4[k], k < 3 ? t4[k + 1] : tn);
       }
-      accumulate<MODE>(s, c & 0x10u, toff);
-      if (u & 1u) {
-        if (e & 1u) rev_post<MODE>(s, sm, P, c, toff, cand, active);
-      }
-      tn = toff;
+      accumulate<MODE>(s, __byte_perm(rc4, 0, 0x4440 + k), t4[k]);
+      if (e & 1u) rev_post<MODE>(s, sm, P, c, t4[k], cand, active);
     }
   }
+  tn = t4[0];
   nw = w;
 }
 
@@ -416,6 +449,10 @@ __global__ void __launch_bounds__(kThreads, ACESO_MINB) eval_kernel(const __grid
   sm.D = sb + P.tab.offD;
   sm.T = sb + P.tab.offT;
   sm.F = sb + P.tab.offF;
+  sm.QO = sb + P.tab.offQO;
+  sm.QT = sb + P.tab.offQT;
+  sm.QD = sb + P.tab.offQD;
+  sm.QF = sb + P.tab.offQF;
   sm.K = sb + tab_bytes;  // cold table staged after the other tables when k_smem
   sm.Kg = reinterpret_cast<const unsigned char *>(P.blob) + P.tab.offK;
   sm.k_smem = P.tab.k_smem;
@@ -504,24 +541,34 @@ __global__ void __launch_bounds__(kThreads, ACESO_MINB) eval_kernel(const __grid
     mbar_wait(smem_addr(&s_ring_bar[warp][slot]), phase);
     const uint32_t a = group_lo(g), b = group_hi(g);
     const uint32_t slot_a = ring + slot * kSlotBytes + lane * 16;
-    const uint32_t nq = (b - a) * 4u;  // quads in this slot
+    if (g == 0 && part == 0) {
+      // seed the previous word so that op 0 always opens the first run
+      const uint32_t w0 = lds32(slot_a);
+      cw = ((w0 & 0xffu) ^ 0x02u) << 24;
+      s.head0 = w0 & 1u;
+    }
     if (part == 0) {
 #pragma unroll 1
-      for (uint32_t qq = 0; qq < nq; ++qq) {
-        const uint32_t qg = a * 4u + qq;
-        if (qg * 4u >= (uint32_t)P.L) break;
-        const uint32_t w = lds32(slot_a + (qq >> 2) * 512u + (qq & 3u) * 4u);
-        quad_fwd<MODE>(s, sm, P, w, cw, qg, cand, active);
+      for (uint32_t ch = a; ch < b; ++ch) {
+        const uint32_t nqc = min(4u, ((uint32_t)P.L - ch * 16u + 3u) >> 2);  // quads inside L
+        uint32_t wa = slot_a + (ch - a) * 512u;
+#pragma unroll 1
+        for (uint32_t q = 0; q < nqc; ++q, wa += 4u)
+          quad_fwd<MODE>(s, sm, P, lds32(wa), cw, ch * 4u + q, cand, active);
       }
     } else {
 #pragma unroll 1
-      for (uint32_t qq = nq; qq-- > 0;) {
-        const uint32_t qg = a * 4u + qq;
-        if (qg * 4u >= (uint32_t)P.L) continue;
-        const uint32_t w = lds32(slot_a + (qq >> 2) * 512u + (qq & 3u) * 4u);
-        quad_rev<MODE>(s, sm, P, w, cw, ct, qg, cand, active);
-        if (qg == c_lo * 4u) {
-          cM = w & 0xffu;
+      for (uint32_t ch = b; ch-- > a;) {
+        const uint32_t nqc = min(4u, ((uint32_t)P.L - ch * 16u + 3u) >> 2);
+        uint32_t wa = slot_a + (ch - a) * 512u + 4u * nqc;
+#pragma unroll 1
+        for (uint32_t q = nqc; q-- > 0;) {
+          wa -= 4u;
+          const uint32_t w = lds32(wa);
+          quad_rev<MODE>(s, sm, P, w, cw, ct, ch * 4u + q, cand, active);
+        }
+        if (ch == c_lo) {
+          cM = lds32(slot_a + (ch - a) * 512u) & 0xffu;
           tM = ct;
         }
       }
@@ -560,7 +607,7 @@ __global__ void __launch_bounds__(kThreads, ACESO_MINB) eval_kernel(const __grid
           const Xchg &xr = xch[lane];
           if (xr.flags & 2u) {
             // op M is a head: part 0's open stage ends at M-1 and is followed by a stage
-            s.S += ldk(sm, s.kbase + (lds32(sm.T + (M - 1) * 4u) >> 1) + 4);  // R5 p2p_fwd
+            s.S += ldk(sm, s.kbase + (toff_of(sm.T, M - 1) >> 1) + 4);  // R5 p2p_fwd
           } else {
             s.S += xr.S; s.A += xr.A; s.W += xr.W; s.D += xr.D; s.comp += xr.comp;
             s.E = max(s.E, xr.E);
