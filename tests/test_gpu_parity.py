@@ -231,3 +231,51 @@ def test_random_bytes_never_crash_and_match():
         codes = rng.integers(0, 256, size=(3000, prof.n_ops), dtype=np.uint8)
         hdr = rng.integers(0, 1 << 16, size=3000, dtype=np.uint64)
         compare(prof, codes, hdr, full=True)
+
+
+# ---------------------------------------------------------------------------
+# both work decompositions (one warp per tile / forward+reverse warp pair)
+# ---------------------------------------------------------------------------
+@pytest.mark.parametrize("split", ["1", "2"])
+@pytest.mark.parametrize("name", ["gpt3-1.3b", "t5", "wrn", "gpt3-13b"])
+def test_split_modes_parity(split, name, monkeypatch):
+    monkeypatch.setenv("ACESO_SPLIT", split)
+    prof = P.WORKLOADS[name]()
+    ctx = A.Context(prof, 0)  # the decomposition is fixed at load time
+    _ctx_cache[id(prof)] = (prof, ctx)
+    try:
+        codes, hdr = ai.search_shaped(prof, SEED + 30, 0, 2113, group_size=16)
+        compare(prof, codes, hdr, full=True)
+        codes, hdr = ai.dense_random(prof, SEED + 31, 0, 700)
+        compare(prof, codes, hdr, full=True)
+        rng = np.random.default_rng(5)
+        codes = rng.integers(0, 256, size=(500, prof.n_ops), dtype=np.uint8)
+        hdr = rng.integers(0, 1 << 16, size=500, dtype=np.uint64)
+        compare(prof, codes, hdr, full=True)
+    finally:
+        _ctx_cache.pop(id(prof), None)
+        ctx.close()
+
+
+def test_nccl_allreduce_min_single_rank():
+    """dist.global_select over a one-rank NCCL group on the device select buffer."""
+    import socket
+    import torch.distributed as dist
+    from paper_conf_eurosys_liumlsmybw24_b200 import dist as adist
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    port = s.getsockname()[1]
+    s.close()
+    dist.init_process_group("nccl", init_method=f"tcp://127.0.0.1:{port}", rank=0, world_size=1)
+    try:
+        prof = P.WORKLOADS["gpt3-1.3b"]()
+        codes, hdr = ai.search_shaped(prof, SEED + 40, 0, 3000, group_size=64)
+        ctx = ctx_for(prof)
+        tiled = torch.from_numpy(ai.tile(codes)).cuda()
+        hd = torch.from_numpy(hdr.view(np.int64)).cuda()
+        _, sel = ctx.eval(tiled, hd, summary=False, select=True, n_total=3000)
+        got = adist.global_select(sel, 3000)
+        o = oracle.evaluate(prof, codes, hdr, threads=8)
+        assert (got.cls, got.cost, got.index) == oracle.select(o)
+    finally:
+        dist.destroy_process_group()

@@ -7,7 +7,7 @@ for minb in 2 3; do
   for split in 1 2; do
     for dist in search dense; do
       r=$(ACESO_SPLIT=$split timeout 300 python bench.py --steps 200 --warmup 20 --no-cpu --no-e2e --dist $dist 2>&1 | tail -1)
-      echo "minb=$minb split=$split $dist: $(echo "$r" | python -c "import json,sys; d=json.load(sys.stdin); print('%.3f Gcfg/s  kernel %.1f us  frac %.3f' % (d['value']/1e9, d['roofline']['kernel_ms']*1e3, d['roofline']['frac']))" 2>&1 | tail -1)"
+      echo "minb=$minb split=$split $dist: $(echo "$r" | python -c "import json,sys; d=json.load(sys.stdin); print('%.3f Gcfg/s  kernel %.1f us  frac %.3f' % (d['value']/1e9, d['roofline']['kernel_ms_serial']*1e3, d['roofline']['frac']))" 2>&1 | tail -1)"
     done
   done
 done
