@@ -309,7 +309,8 @@ __device__ __forceinline__ void init_cand(Cand &s, const Smem &sm, const EvalPar
 // forward quad qg (ops 4qg..4qg+3); w = the lane's 4 code bytes; pw = previous word
 template <uint32_t MODE>
 __device__ __forceinline__ void quad_fwd(Cand &s, const Smem &sm, const EvalParams &P, uint32_t w,
-                                         uint32_t &pw, uint32_t qg, int64_t cand, bool active) {
+                                         uint2 o, uint32_t &pw, uint32_t qg, int64_t cand,
+                                         bool active) {
   const uint32_t sh = __funnelshift_l(pw, w, 8);  // previous op's byte under each byte
   // per byte: bit 0 = head; bits 1-7 = difference to the previous op's code. For op 0 of
   // a tile the caller seeds pw so that op 0 always shows a tp/dp difference (opens a run).
@@ -317,7 +318,6 @@ __device__ __forceinline__ void quad_fwd(Cand &s, const Smem &sm, const EvalPara
   asm("lop3.b32 %0, %1, %2, %3, 0xB4;" : "=r"(d) : "r"(w), "r"(sh), "r"(0x01010101u));  // c ? w : w^sh
   d &= 0xffffffefu;  // an rc change at the quad's first op does not make it mixed
   pw = w;
-  const uint2 o = lds64(sm.QO + 8u * qg);  // quad signature offsets (kNone: no quad sums)
   // clean lane (no head, no tp/dp change, uniform rc) -> one quad-table gather
   if (d == 0u && o.x != kNone) {
     accumulate_quad<MODE>(s, o, w & 0x10u);
@@ -552,9 +552,23 @@ __global__ void __launch_bounds__(kThreads, ACESO_MINB) eval_kernel(const __grid
       for (uint32_t ch = a; ch < b; ++ch) {
         const uint32_t nqc = min(4u, ((uint32_t)P.L - ch * 16u + 3u) >> 2);  // quads inside L
         uint32_t wa = slot_a + (ch - a) * 512u;
+        uint32_t oa = sm.QO + 8u * (ch * 4u);
+        // software pipeline: the next quad's code word and signature offsets load while
+        // this quad is processed
+        uint32_t wn = lds32(wa);
+        uint2 on = lds64(oa);
 #pragma unroll 1
-        for (uint32_t q = 0; q < nqc; ++q, wa += 4u)
-          quad_fwd<MODE>(s, sm, P, lds32(wa), cw, ch * 4u + q, cand, active);
+        for (uint32_t q = 0; q < nqc; ++q) {
+          const uint32_t w = wn;
+          const uint2 o = on;
+          wa += 4u;
+          oa += 8u;
+          if (q + 1 < nqc) {
+            wn = lds32(wa);
+            on = lds64(oa);
+          }
+          quad_fwd<MODE>(s, sm, P, w, o, cw, ch * 4u + q, cand, active);
+        }
       }
     } else {
 #pragma unroll 1
