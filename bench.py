@@ -42,6 +42,8 @@ def parse():
     ap.add_argument("--group", type=int, default=1024, help="candidates sharing a base config")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--search-budget", type=float, default=20.0,
+                    help="seconds for the search-time measurement (0: skip)")
     ap.add_argument("--streams", type=int, default=4,
                     help="independent batches in flight (steps round-robin over streams)")
     return ap.parse_args()
@@ -425,6 +427,28 @@ def main():
         }
         if e2e is not None:
             line["e2e"] = e2e
+        if args.search_budget > 0 and world == 1:
+            from paper_conf_eurosys_liumlsmybw24_b200 import search as S
+            ev = S.GPUEvaluator(ctx)
+            res, st = S.search(prof, ev, budget_s=args.search_budget, patience=8)
+            init_best = None
+            for p in [1, 2, 4, 8, 16, 32, 64]:
+                r0 = S.initial_config(prof, p) if p <= prof.n_devices else None
+                if r0 is None:
+                    continue
+                o = ev.evaluate(r0[0][None, :], np.array([S.header(r0[1], p)], np.uint64))
+                pf = S.perf_of(int(o["info"][0]), o["iter"][0], o["max_mem"][0])
+                init_best = pf if init_best is None or pf < init_best else init_best
+            line["search"] = {
+                "time_s": st["time_s"], "time_to_best_s": st["time_to_best_s"],
+                "evaluated": st["evaluated"], "batches": st["batches"],
+                "improvements": st["improvements"],
+                "best": {"class": res.perf[0], "cost": res.perf[1], "iter_ns": res.iter_ns,
+                         "p": int((res.codes & 1).sum()), "mbs_log2": res.mbs},
+                "initial_best": {"class": init_best[0], "cost": init_best[1]},
+                "note": "batched Alg. 1/2 (MaxHops 7, beam 4) over all stage counts, stops "
+                        "after 8 hops without a new best or at the budget; context: the "
+                        "paper's searches use a 200 s budget (P:L313)"}
         if not args.no_cpu and world == 1:
             import aceso_inputs as ai  # noqa: F811
             rowm = []

@@ -1,0 +1,439 @@
+"""Thin host search driver: Aceso's iterative bottleneck alleviation (Alg. 1/2,
+P:L521-593) on top of the batched evaluator.
+
+The paper estimates one candidate at a time. Here every hop of the
+multi-hop search applies all eligible reconfiguration primitives (Table 1,
+P:L163-176) with all their argument values to the current frontier, evaluates
+them as ONE batch (the evaluator is `aceso_eval`), and keeps the best ones:
+  - Heuristic-1: the bottleneck stage comes from the evaluator's info
+    word (largest memory if OOM, else longest time);
+  - Heuristic-2: the resource with the highest consumption
+    proportion (stage share of the total, from the FULL per-stage outputs)
+    selects the eligible primitives; "best performance first" orders the
+    frontier of the next hop;
+  - primitives: inc/dec-op# at both stage edges with relay along neighbours
+    (P:L253), inc/dec-mbs, dp/tp trades inside the stage and with a
+    partner stage, greedy inc/dec-rc of the largest-activation ops
+    (P:L255), op-level tp/dp fine-tuning from op k to the stage end;
+  - Alg. 1: restart from the improved config; on failure within MaxHops (7,
+    P:L313) continue from GetBestOf(unexplored) (reading R16: keep the
+    better of best and new);
+  - parallel search per pipeline-stage count: the searches of all
+    stage counts are stepped together and share each evaluation batch.
+Configurations are deduplicated by their encoding.
+
+The evaluator is any object with `evaluate(codes[n][L] u8, hdr[n] u64) ->
+dict(iter, max_mem, info, stage_comp, stage_comm, stage_mem, stage_T [n][G])`:
+`GPUEvaluator` below calls libaceso; tests may pass a CPU evaluator.
+"""
+from __future__ import annotations
+
+import dataclasses
+import math
+import time
+
+import numpy as np
+import torch
+
+INFO_OOM = 1 << 16
+INFO_INVALID = 1 << 17
+
+
+# ---------------------------------------------------------------------------
+# configurations (encoding of include/aceso.h)
+# ---------------------------------------------------------------------------
+def encode(head, tpl, dpl, rc):
+    return (head & 1) | ((tpl & 7) << 1) | ((rc & 1) << 4) | ((dpl & 7) << 5)
+
+
+def header(mbs, p):
+    return (mbs & 0xFF) | ((p & 0xFF) << 8)
+
+
+def stages_of(codes):
+    heads = np.flatnonzero(codes & 1)
+    ends = np.append(heads[1:], len(codes))
+    return heads, ends
+
+
+def _split_devices(p, G):
+    g = [1] * p
+    rem = G - p
+    while rem > 0:
+        cand = [i for i in range(p) if g[i] <= rem]
+        if not cand:
+            break
+        i = min(cand, key=lambda k: g[k])
+        rem -= g[i]
+        g[i] *= 2
+    return [int(math.log2(x)) for x in g]
+
+
+def initial_config(prof, p):
+    """Even partition, balanced devices, data parallelism first, minimum microbatch."""
+    L, G = prof.n_ops, prof.n_devices
+    k = _split_devices(p, G)
+    if sum(1 << x for x in k) != G:
+        return None
+    codes = np.zeros(L, np.uint8)
+    starts = [L * i // p for i in range(p)] + [L]
+    for i in range(p):
+        d = min(k[i], prof.n_dp - 1)
+        t = k[i] - d
+        if t >= prof.n_tp:
+            return None
+        a, b = starts[i], starts[i + 1]
+        codes[a:b] = encode(0, t, d, 0)
+        codes[a] |= 1
+    dmax = int(max((codes >> 5) & 7))
+    return codes, dmax
+
+
+@dataclasses.dataclass
+class Result:
+    codes: np.ndarray
+    mbs: int
+    perf: tuple
+    iter_ns: int
+    max_mem: int
+    info: int
+
+
+def perf_of(info, it, mem):
+    """(class, cost): feasible by iteration time before OOM by memory (R12)."""
+    if info & INFO_INVALID:
+        return (2, 0)
+    if info & INFO_OOM:
+        return (1, int(mem))
+    return (0, int(it))
+
+
+# ---------------------------------------------------------------------------
+# reconfiguration primitives (Table 1) applied to one configuration
+# ---------------------------------------------------------------------------
+def _move_front(codes, s, k):
+    """dec-op# of stage s / inc-op# of s-1: first k ops of stage s join stage s-1."""
+    heads, ends = stages_of(codes)
+    a, e = heads[s], ends[s]
+    if s == 0 or k < 1 or k >= e - a:
+        return None
+    c = codes.copy()
+    prev = c[a - 1] & 0xEE
+    c[a:a + k] = (c[a:a + k] & 0x10) | prev
+    c[a + k] = (c[a + k] & 0xFE) | 1
+    return c
+
+
+def _move_back(codes, s, k):
+    """dec-op# of stage s / inc-op# of s+1: last k ops of stage s join stage s+1."""
+    heads, ends = stages_of(codes)
+    p = len(heads)
+    a, e = heads[s], ends[s]
+    if s >= p - 1 or k < 1 or k >= e - a:
+        return None
+    c = codes.copy()
+    nxt = c[e] & 0xEE
+    c[e] &= 0xFE
+    c[e - k:e] = (c[e - k:e] & 0x10) | nxt
+    c[e - k] |= 1
+    return c
+
+
+def _recode_stage(codes, s, dt, dd, from_op=None):
+    heads, ends = stages_of(codes)
+    a, e = heads[s], ends[s]
+    lo = a if from_op is None else from_op
+    c = codes.copy()
+    tpl = ((c[lo:e] >> 1) & 7).astype(np.int16) + dt
+    dpl = ((c[lo:e] >> 5) & 7).astype(np.int16) + dd
+    if tpl.min() < 0 or dpl.min() < 0 or tpl.max() > 7 or dpl.max() > 7:
+        return None
+    c[lo:e] = (c[lo:e] & 0x11) | ((tpl.astype(np.uint8) & 7) << 1) | ((dpl.astype(np.uint8) & 7) << 5)
+    return c
+
+
+def _rc_order(prof, codes, s, mbs):
+    """Ops of stage s by activation size at their partition, largest first."""
+    heads, ends = stages_of(codes)
+    a, e = heads[s], ends[s]
+    j = np.arange(a, e)
+    tpl = (codes[a:e] >> 1) & 7
+    dpl = (codes[a:e] >> 5) & 7
+    b = np.clip(mbs - dpl.astype(np.int64), 0, prof.n_b - 1)
+    act = prof.rec[prof.op_type[a:e], np.minimum(tpl, prof.n_tp - 1), b, 4]
+    return j[np.argsort(-act, kind="stable")]
+
+
+class Primitives:
+    def __init__(self, prof, heuristic2=True, max_k=None):
+        self.prof = prof
+        self.heuristic2 = heuristic2
+        self.max_k = max_k
+
+    def apply_all(self, codes, mbs, info, comp, comm, stage_time):
+        """All eligible primitives on the Heuristic-1 bottleneck stage of (codes, mbs).
+        Returns a list of (codes, mbs)."""
+        prof = self.prof
+        heads, ends = stages_of(codes)
+        p = len(heads)
+        bn = int(info & 0xFF)
+        if bn >= p:
+            bn = 0
+        oom = bool(info & INFO_OOM)
+        # Heuristic-2: the resource with the highest consumption proportion of stage bn
+        if oom:
+            want = {"mem"}
+        else:
+            cs, ms = max(int(comp[:p].sum()), 1), max(int(comm[:p].sum()), 1)
+            want = {"comp"} if comp[bn] / cs >= comm[bn] / ms else {"comm"}
+        if not self.heuristic2:
+            want = {"mem", "comp", "comm"}
+        out = []
+        size = ends[bn] - heads[bn]
+        kmax = size - 1 if self.max_k is None else min(size - 1, self.max_k)
+        # inc/dec-op#: move ops out of the bottleneck at either edge (every resource),
+        # with a relay toward the idlest stage
+        idle = int(np.argmin(stage_time[:p])) if p > 1 else bn
+        for k in range(1, kmax + 1):
+            c = _move_front(codes, bn, k)
+            if c is not None:
+                out.append((c, mbs))
+                if idle < bn - 1:
+                    c2 = _move_front(c, bn - 1, k)
+                    if c2 is not None:
+                        out.append((c2, mbs))
+            c = _move_back(codes, bn, k)
+            if c is not None:
+                out.append((c, mbs))
+                if idle > bn + 1:
+                    c2 = _move_back(c, bn + 1, k)
+                    if c2 is not None:
+                        out.append((c2, mbs))
+        log2bg = int(math.log2(prof.global_batch & -prof.global_batch))
+        dmax = int(((codes >> 5) & 7).max())
+        # inc/dec-mbs (model level): memory down / computation efficiency up
+        if ("mem" in want or "comm" in want) and mbs - 1 >= dmax:
+            out.append((codes, mbs - 1))
+        if ("comp" in want) and mbs + 1 <= log2bg:
+            out.append((codes, mbs + 1))
+        # tp <-> dp inside the stage (same devices): inc-tp/dec-dp and dec-tp/inc-dp
+        for dt in (1, -1):
+            c = _recode_stage(codes, bn, dt, -dt)
+            if c is not None:
+                out.append((c, max(mbs, int(((c >> 5) & 7).max()))))
+        # inc-dp / inc-tp with a partner stage holding twice the devices
+        kb = ((codes[heads[bn]] >> 1) & 7) + ((codes[heads[bn]] >> 5) & 7)
+        for q in range(p):
+            if q == bn:
+                continue
+            kq = ((codes[heads[q]] >> 1) & 7) + ((codes[heads[q]] >> 5) & 7)
+            if kq == kb + 1 and ("comp" in want or "mem" in want):
+                for dtb, ddb in ((1, 0), (0, 1)):
+                    for dtq, ddq in ((-1, 0), (0, -1)):
+                        c = _recode_stage(codes, bn, dtb, ddb)
+                        c = _recode_stage(c, q, dtq, ddq) if c is not None else None
+                        if c is not None:
+                            out.append((c, max(mbs, int(((c >> 5) & 7).max()))))
+            if kq + 1 == kb and "comm" in want:  # give devices away (dec-dp/tp on the bottleneck)
+                for dtb, ddb in ((-1, 0), (0, -1)):
+                    for dtq, ddq in ((1, 0), (0, 1)):
+                        c = _recode_stage(codes, bn, dtb, ddb)
+                        c = _recode_stage(c, q, dtq, ddq) if c is not None else None
+                        if c is not None:
+                            out.append((c, max(mbs, int(((c >> 5) & 7).max()))))
+        # greedy inc-rc (memory) / dec-rc (computation) on the largest-activation ops
+        order = _rc_order(prof, codes, bn, mbs)
+        rc = (codes[order] >> 4) & 1
+        if "mem" in want:
+            todo = order[rc == 0]
+            for k in range(1, len(todo) + 1):
+                c = codes.copy()
+                c[todo[:k]] |= 0x10
+                out.append((c, mbs))
+        if "comp" in want:
+            have = order[rc == 1][::-1]
+            for k in range(1, len(have) + 1):
+                c = codes.copy()
+                c[have[:k]] &= 0xEF
+                out.append((c, mbs))
+        # op-level fine-tune: tp/dp change from op k to the end of the stage
+        for j in range(heads[bn] + 1, ends[bn]):
+            for dt in (1, -1):
+                c = _recode_stage(codes, bn, dt, -dt, from_op=j)
+                if c is not None:
+                    out.append((c, max(mbs, int(((c >> 5) & 7).max()))))
+        return out
+
+
+# ---------------------------------------------------------------------------
+# evaluators
+# ---------------------------------------------------------------------------
+class GPUEvaluator:
+    """aceso_eval in FULL mode on the device; uploads row-major codes and packs them."""
+
+    def __init__(self, ctx):
+        self.ctx = ctx
+        self.calls = 0
+        self.evaluated = 0
+
+    def evaluate(self, codes, hdr):
+        from .api import as_u32, as_u64
+        n = int(hdr.shape[0])
+        self.calls += 1
+        self.evaluated += n
+        dev = torch.device("cuda", self.ctx.device)
+        c = torch.from_numpy(np.ascontiguousarray(codes)).to(dev)
+        h = torch.from_numpy(np.ascontiguousarray(hdr, np.uint64).view(np.int64)).to(dev)
+        tiled = self.ctx.pack_rowmajor(c)
+        out, _ = self.ctx.eval(tiled, h, n=n, full=True, select=False)
+        res = dict(iter=as_u64(out.iter_ns), max_mem=as_u64(out.max_mem), info=as_u32(out.info))
+        for k in ["stage_T", "stage_mem", "stage_comp", "stage_comm"]:
+            res[k] = as_u64(getattr(out, k)).reshape(out.p_max, n).T
+        return res
+
+
+# ---------------------------------------------------------------------------
+# Alg. 1 / Alg. 2, batched
+# ---------------------------------------------------------------------------
+@dataclasses.dataclass
+class _Node:
+    codes: np.ndarray
+    mbs: int
+    perf: tuple
+    info: int
+    comp: np.ndarray
+    comm: np.ndarray
+    time: np.ndarray
+    iter_ns: int
+    max_mem: int
+
+
+class _Search:
+    """One AcesoSearch (Alg. 1) for one stage count, stepped one hop at a time."""
+
+    def __init__(self, start: _Node):
+        self.cur = start
+        self.best = start
+        self.init_perf = start.perf
+        self.frontier = [start]
+        self.hop = 0
+        self.unexplored = {}
+        self.done = False
+        self.improvements = 0
+
+
+def search(prof, evaluator, p_values=None, budget_s=10.0, max_hops=7, beam=4, heuristic2=True,
+           max_batch=200000, max_k=None, patience=None):
+    """Runs the batched Aceso search. Returns (best Result, stats dict)."""
+    t0 = time.perf_counter()
+    prims = Primitives(prof, heuristic2=heuristic2, max_k=max_k)
+    if p_values is None:
+        p_values = [p for p in (1, 2, 3, 4, 6, 8, 12, 16, 24, 32, 48, 64) if p <= min(prof.n_devices, prof.n_ops)]
+    visited = set()
+    # initial configurations, one search per stage count
+    init = []
+    for p in p_values:
+        r = initial_config(prof, p)
+        if r is not None:
+            init.append(r)
+    codes = np.stack([c for c, _ in init])
+    mbs = np.array([m for _, m in init])
+    res = evaluator.evaluate(codes, np.array([header(int(m), int((c & 1).sum())) for c, m in init], np.uint64))
+
+    def node(i, cds, mb, r):
+        info = int(r["info"][i])
+        return _Node(cds, int(mb), perf_of(info, r["iter"][i], r["max_mem"][i]), info,
+                     r["stage_comp"][i], r["stage_comm"][i], r["stage_T"][i], int(r["iter"][i]),
+                     int(r["max_mem"][i]))
+
+    searches = []
+    for i in range(len(init)):
+        n0 = node(i, codes[i], mbs[i], res)
+        visited.add((codes[i].tobytes(), int(mbs[i])))
+        searches.append(_Search(n0))
+    best = min((s.best for s in searches), key=lambda n: n.perf)
+    t_best = time.perf_counter() - t0
+    batches = 0
+    evaluated = len(init)
+    history = [(t_best, best.perf)]
+    stale = 0
+    while time.perf_counter() - t0 < budget_s and any(not s.done for s in searches):
+        # one hop of every active search, generated into one batch
+        owners, cand_codes, cand_mbs = [], [], []
+        for si, s in enumerate(searches):
+            if s.done:
+                continue
+            for nd in s.frontier:
+                if nd.perf[0] == 2:
+                    continue
+                for c, m in prims.apply_all(nd.codes, nd.mbs, nd.info, nd.comp, nd.comm, nd.time):
+                    key = (c.tobytes(), int(m))
+                    if key in visited:
+                        continue
+                    visited.add(key)
+                    owners.append(si)
+                    cand_codes.append(c)
+                    cand_mbs.append(m)
+                    if len(cand_codes) >= max_batch:
+                        break
+        if not cand_codes:
+            for s in searches:
+                s.done = True
+            break
+        cc = np.stack(cand_codes)
+        hdr = np.array([header(int(m), int((c & 1).sum())) for c, m in zip(cand_codes, cand_mbs)], np.uint64)
+        r = evaluator.evaluate(cc, hdr)
+        batches += 1
+        evaluated += len(cand_codes)
+        per = {}
+        for i, si in enumerate(owners):
+            per.setdefault(si, []).append(node(i, cc[i], cand_mbs[i], r))
+        improved_any = False
+        for si, s in enumerate(searches):
+            if s.done:
+                continue
+            new = per.get(si, [])
+            new.sort(key=lambda n: n.perf)  # Heuristic-2: best estimated performance first
+            for nd in new:
+                s.unexplored[(nd.codes.tobytes(), nd.mbs)] = nd
+            if new and new[0].perf < s.init_perf:
+                # Alg. 2 returns the improved configuration; Alg. 1 restarts from it
+                s.cur = new[0]
+                if new[0].perf < s.best.perf:
+                    s.best = new[0]
+                s.init_perf = new[0].perf
+                s.frontier = [new[0]]
+                s.hop = 0
+                s.improvements += 1
+                s.unexplored.pop((new[0].codes.tobytes(), new[0].mbs), None)
+                improved_any = True
+                continue
+            s.hop += 1
+            if s.hop < max_hops and new:
+                s.frontier = new[:beam]
+                continue
+            # MultiHop failed within MaxHops: Alg. 1 continues from GetBestOf(unexplored)
+            if not s.unexplored:
+                s.done = True
+                continue
+            k_best = min(s.unexplored, key=lambda k: s.unexplored[k].perf)
+            nd = s.unexplored.pop(k_best)
+            s.cur = nd
+            s.init_perf = nd.perf
+            s.frontier = [nd]
+            s.hop = 0
+        cur_best = min((s.best for s in searches), key=lambda n: n.perf)
+        if cur_best.perf < best.perf:
+            best = cur_best
+            t_best = time.perf_counter() - t0
+            history.append((t_best, best.perf))
+            stale = 0
+        else:
+            stale += 1
+        if patience is not None and stale >= patience:
+            break
+    total = time.perf_counter() - t0
+    stats = dict(time_s=total, time_to_best_s=t_best, batches=batches, evaluated=evaluated,
+                 searches=len(searches), history=history,
+                 improvements=sum(s.improvements for s in searches))
+    return Result(best.codes, best.mbs, best.perf, best.iter_ns, best.max_mem, best.info), stats

@@ -1,0 +1,84 @@
+"""Search driver (Alg. 1/2, Heuristic-1/2, Table 1 primitives) with a CPU
+evaluator built on the oracle (tests only); the product runs it with GPUEvaluator."""
+import numpy as np
+import pytest
+
+import aceso_inputs as ai
+import oracle
+from aceso_inputs import profiles as P
+from paper_conf_eurosys_liumlsmybw24_b200 import search as S
+
+
+class OracleEvaluator:
+    def __init__(self, prof):
+        self.prof = prof
+        self.evaluated = 0
+
+    def evaluate(self, codes, hdr):
+        self.evaluated += len(hdr)
+        return oracle.evaluate(self.prof, codes, hdr, full=True, threads=8)
+
+
+def perf_tuple(out, i):
+    return S.perf_of(int(out["info"][i]), out["iter"][i], out["max_mem"][i])
+
+
+def test_primitives_keep_encodings_valid_structure():
+    prof = P.WORKLOADS["gpt3-1.3b"]()
+    codes, mbs = S.initial_config(prof, 4)
+    ev = OracleEvaluator(prof)
+    base = ev.evaluate(codes[None, :], np.array([S.header(mbs, 4)], np.uint64))
+    prim = S.Primitives(prof, heuristic2=False)
+    cands = prim.apply_all(codes, mbs, int(base["info"][0]), base["stage_comp"][0],
+                           base["stage_comm"][0], base["stage_T"][0])
+    assert len(cands) > 100
+    cc = np.stack([c for c, _ in cands])
+    hdr = np.array([S.header(int(m), int((c & 1).sum())) for c, m in cands], np.uint64)
+    out = ev.evaluate(cc, hdr)
+    # op moves / trades preserve the device sum and the head count: almost all valid
+    valid = (out["info"] & oracle.INFO_INVALID) == 0
+    assert valid.mean() > 0.9
+    # every candidate differs from the base
+    assert all(not (np.array_equal(c, codes) and m == mbs) for c, m in cands)
+
+
+def test_initial_configs_are_valid():
+    for name in ["toy-a", "gpt3-1.3b", "gpt3-13b", "t5", "wrn"]:
+        prof = P.WORKLOADS[name]()
+        for p in [1, 2, 4]:
+            r = S.initial_config(prof, p)
+            assert r is not None
+            codes, mbs = r
+            out = oracle.evaluate(prof, codes[None, :], np.array([S.header(mbs, p)], np.uint64))
+            assert not out["info"][0] & oracle.INFO_INVALID, (name, p, out["info"][0] >> 18)
+
+
+def test_search_improves_and_is_deterministic():
+    prof = P.WORKLOADS["gpt3-1.3b"]()
+    r1, st1 = S.search(prof, OracleEvaluator(prof), p_values=[2, 4], budget_s=60, max_hops=3, beam=2,
+                       max_k=8, patience=4)
+    r2, st2 = S.search(prof, OracleEvaluator(prof), p_values=[2, 4], budget_s=60, max_hops=3, beam=2,
+                       max_k=8, patience=4)
+    assert r1.perf == r2.perf and np.array_equal(r1.codes, r2.codes)
+    # better than every initial configuration ("better")
+    inits = []
+    for p in [2, 4]:
+        c, m = S.initial_config(prof, p)
+        o = oracle.evaluate(prof, c[None, :], np.array([S.header(m, p)], np.uint64))
+        inits.append(perf_tuple(o, 0))
+    assert r1.perf < min(inits)
+    assert st1["improvements"] > 0
+    # the returned configuration re-evaluates to the reported performance
+    o = oracle.evaluate(prof, r1.codes[None, :], np.array([S.header(r1.mbs, int((r1.codes & 1).sum()))], np.uint64))
+    assert perf_tuple(o, 0) == r1.perf
+
+
+def test_search_on_toy_reaches_a_feasible_near_optimum():
+    """toy-A: the exhaustive optimum is known (388,800 configurations); the search
+    finds a feasible configuration within 10% of it (not guaranteed to be optimal)."""
+    prof = P.toy_a()
+    codes, hdr = ai.exhaustive(prof, per_op=True)
+    best = oracle.select(oracle.evaluate(prof, codes, hdr, threads=8))
+    r, st = S.search(prof, OracleEvaluator(prof), budget_s=30, max_hops=7, beam=4)
+    assert r.perf[0] == 0
+    assert r.perf[1] <= best[1] * 1.10
