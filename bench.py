@@ -267,24 +267,34 @@ def main():
     nstr = max(1, min(args.streams, nbuf))
     outs = [out] + [ctx.alloc_outputs(n) for _ in range(nstr - 1)]
     side = [torch.cuda.Stream() for _ in range(nstr)]
+    comm = torch.cuda.Stream()  # all-reduces in step order on one stream (same on every rank)
     with torch.cuda.graph(graph):
         cs = torch.cuda.current_stream()
         fork = torch.cuda.Event()
         fork.record(cs)
-        for st in side:
+        for st in side + [comm]:
             st.wait_event(fork)
+        comm_done = {}
         for s in range(args.steps):
             b = s % nbuf
             st = side[s % nstr] if nstr > 1 else cs
             codes_d, hdr_d = dev_batches[b]
+            if s - nbuf in comm_done:  # the select buffer's previous all-reduce has read it
+                st.wait_event(comm_done.pop(s - nbuf))
             ev_s[s].record(st)
             ctx.eval(codes_d, hdr_d, n=n, global_offset=rank * n, n_total=n_total, summary=True,
                      select=True, out=outs[s % nstr], sel=sels[b], stream=st)
             ev_k[s].record(st)
             if world > 1:
-                with torch.cuda.stream(st):
+                done = torch.cuda.Event()
+                done.record(st)
+                comm.wait_event(done)
+                with torch.cuda.stream(comm):
                     dist.all_reduce(sels[b][0:8].view(torch.int64), op=dist.ReduceOp.MIN)
-        for st in side:
+                cd = torch.cuda.Event()
+                cd.record(comm)
+                comm_done[s] = cd
+        for st in side + [comm]:
             j = torch.cuda.Event()
             j.record(st)
             cs.wait_event(j)
