@@ -41,27 +41,28 @@ int fail(int code, const char *fmt, ...) {
       return fail(ACESO_ECUDA, "%s failed: %s", #expr, cudaGetErrorString(e_));            \
   } while (0)
 
-template <uint32_t M, int S>
+template <uint32_t M, int S, int B>
 void *kernel_ptr() {
-  return reinterpret_cast<void *>(&eval_kernel<M, S>);
+  return reinterpret_cast<void *>(&eval_kernel<M, S, B>);
 }
 
-template <int S>
+template <int S, int B>
 void *eval_kernel_split(uint32_t mode) {
   switch (mode) {
-    case 1: return kernel_ptr<1, S>();
-    case 2: return kernel_ptr<2, S>();
-    case 3: return kernel_ptr<3, S>();
-    case 4: return kernel_ptr<4, S>();
-    case 5: return kernel_ptr<5, S>();
-    case 6: return kernel_ptr<6, S>();
-    case 7: return kernel_ptr<7, S>();
+    case 1: return kernel_ptr<1, S, B>();
+    case 2: return kernel_ptr<2, S, B>();
+    case 3: return kernel_ptr<3, S, B>();
+    case 4: return kernel_ptr<4, S, B>();
+    case 5: return kernel_ptr<5, S, B>();
+    case 6: return kernel_ptr<6, S, B>();
+    case 7: return kernel_ptr<7, S, B>();
     default: return nullptr;
   }
 }
 
-void *eval_kernel_for(uint32_t mode, int split) {
-  return split == 2 ? eval_kernel_split<2>(mode) : eval_kernel_split<1>(mode);
+void *eval_kernel_for(uint32_t mode, int split, int minb) {
+  if (minb == 2) return split == 2 ? eval_kernel_split<2, 2>(mode) : eval_kernel_split<1, 2>(mode);
+  return split == 2 ? eval_kernel_split<2, 3>(mode) : eval_kernel_split<1, 3>(mode);
 }
 
 uint32_t bitlen(uint64_t v) {
@@ -81,6 +82,7 @@ struct aceso_ctx {
   Tables tab;
   void *d_blob;
   int split;        // warps per tile (1 or 2)
+  int minb;         // register target: 2 or 3 resident CTAs per SM
   int max_ctas[8];  // per mode: resident CTAs (occupancy x SMs)
   size_t smem[8];
 };
@@ -338,12 +340,17 @@ int aceso_load_profile(const aceso_profile_desc *d, int cuda_device, aceso_ctx *
       int v = atoi(env);
       if (v == 1 || (v == 2 && nch >= 2)) ctx->split = v;
     }
+    ctx->minb = 3;  // ACESO_MINB=2 selects the ~96-register variant (lower single-launch latency)
+    if (const char *env = getenv("ACESO_MINB")) {
+      int v = atoi(env);
+      if (v == 2 || v == 3) ctx->minb = v;
+    }
     for (uint32_t mode = 1; mode < 8; ++mode) {
       const size_t smem = ((mode & ACESO_OUT_FULL) ? tab.bytes_full : tab.bytes) +
                           (tab.k_smem ? bytesK : 0u) + kRingBytesPerCta +
                           (ctx->split == 2 ? (size_t)(kWarps / 2) * 32 * sizeof(Xchg) : 0);
       ctx->smem[mode] = smem;
-      void *k = eval_kernel_for(mode, ctx->split);
+      void *k = eval_kernel_for(mode, ctx->split, ctx->minb);
       e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
       int occ = 0;
       if (e == cudaSuccess) e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k, kThreads, smem);
@@ -438,7 +445,7 @@ int aceso_eval(aceso_ctx *ctx, const uint8_t *d_codes, const uint64_t *d_hdr, in
   CUDA_TRY(cudaGetDevice(&prev));
   if (prev != ctx->device) CUDA_TRY(cudaSetDevice(ctx->device));
   void *args[] = {&P};
-  cudaError_t e = cudaLaunchKernel(eval_kernel_for(mode, ctx->split), dim3(grid), dim3(kThreads), args, ctx->smem[mode],
+  cudaError_t e = cudaLaunchKernel(eval_kernel_for(mode, ctx->split, ctx->minb), dim3(grid), dim3(kThreads), args, ctx->smem[mode],
                                    reinterpret_cast<cudaStream_t>(stream));
   if (prev != ctx->device) cudaSetDevice(prev);
   if (e != cudaSuccess) return fail(ACESO_ECUDA, "eval launch: %s", cudaGetErrorString(e));

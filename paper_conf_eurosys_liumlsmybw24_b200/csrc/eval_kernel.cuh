@@ -36,9 +36,7 @@ constexpr int kSlotChunks = 2;   // 16-op chunks per ring slot (1 KB)
 constexpr int kSlotBytes = kSlotChunks * 512;
 constexpr int kRingBytesPerCta = kWarps * kRingSlots * kSlotBytes;
 constexpr uint32_t kNone = 0xffffffffu;
-#ifndef ACESO_MINB
-#define ACESO_MINB 2  // resident CTAs per SM the register allocation targets
-#endif
+
 
 // ---------------------------------------------------------------------------
 // PTX helpers: mbarrier + cp.async.bulk (TMA bulk copy), shared loads
@@ -430,8 +428,10 @@ __device__ __forceinline__ void finish_cand(Cand &s, const EvalParams &P, int64_
 // ---------------------------------------------------------------------------
 // kernel
 // ---------------------------------------------------------------------------
-template <uint32_t MODE, int SPLIT>
-__global__ void __launch_bounds__(kThreads, ACESO_MINB) eval_kernel(const __grid_constant__ EvalParams P) {
+// MINB: resident CTAs per SM the register allocation targets (2: ~96 registers, lowest
+// latency per launch; 3: <= 80 registers, more warps when independent batches overlap)
+template <uint32_t MODE, int SPLIT, int MINB>
+__global__ void __launch_bounds__(kThreads, MINB) eval_kernel(const __grid_constant__ EvalParams P) {
   extern __shared__ __align__(128) unsigned char sm_raw[];
   __shared__ __align__(8) uint64_t s_tbar;
   __shared__ __align__(8) uint64_t s_ring_bar[kWarps][kRingSlots];

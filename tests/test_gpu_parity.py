@@ -236,10 +236,12 @@ def test_random_bytes_never_crash_and_match():
 # ---------------------------------------------------------------------------
 # both work decompositions (one warp per tile / forward+reverse warp pair)
 # ---------------------------------------------------------------------------
+@pytest.mark.parametrize("minb", ["2", "3"])
 @pytest.mark.parametrize("split", ["1", "2"])
 @pytest.mark.parametrize("name", ["gpt3-1.3b", "t5", "wrn", "gpt3-13b"])
-def test_split_modes_parity(split, name, monkeypatch):
+def test_split_modes_parity(split, minb, name, monkeypatch):
     monkeypatch.setenv("ACESO_SPLIT", split)
+    monkeypatch.setenv("ACESO_MINB", minb)
     prof = P.WORKLOADS[name]()
     ctx = A.Context(prof, 0)  # the decomposition is fixed at load time
     _ctx_cache[id(prof)] = (prof, ctx)
