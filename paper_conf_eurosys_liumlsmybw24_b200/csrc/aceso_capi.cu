@@ -17,6 +17,7 @@
 #include "aux_kernels.cuh"
 #include "common.cuh"
 #include "eval_kernel.cuh"
+#include "event_kernel.cuh"
 
 using namespace aceso;
 
@@ -60,7 +61,23 @@ void *eval_kernel_split(uint32_t mode) {
   }
 }
 
-void *eval_kernel_for(uint32_t mode, int split, int minb) {
+template <int B>
+void *event_kernel_for(uint32_t mode) {
+  switch (mode) {
+    case 1: return reinterpret_cast<void *>(&event_kernel<1, B>);
+    case 2: return reinterpret_cast<void *>(&event_kernel<2, B>);
+    case 3: return reinterpret_cast<void *>(&event_kernel<3, B>);
+    case 4: return reinterpret_cast<void *>(&event_kernel<4, B>);
+    case 5: return reinterpret_cast<void *>(&event_kernel<5, B>);
+    case 6: return reinterpret_cast<void *>(&event_kernel<6, B>);
+    case 7: return reinterpret_cast<void *>(&event_kernel<7, B>);
+    default: return nullptr;
+  }
+}
+
+// kernel 0: per-op/quad kernel (eval_kernel.cuh); kernel 1: event kernel (event_kernel.cuh)
+void *eval_kernel_for(uint32_t mode, int split, int minb, int kernel) {
+  if (kernel == 1) return minb == 2 ? event_kernel_for<2>(mode) : event_kernel_for<3>(mode);
   if (minb == 2) return split == 2 ? eval_kernel_split<2, 2>(mode) : eval_kernel_split<1, 2>(mode);
   return split == 2 ? eval_kernel_split<2, 3>(mode) : eval_kernel_split<1, 3>(mode);
 }
@@ -81,6 +98,12 @@ struct aceso_ctx {
   uint32_t mem_shift;
   Tables tab;
   void *d_blob;
+  int kernel;       // 0: quad kernel, 1: event kernel (default; ACESO_KERNEL=quad|events)
+  void *d_ev;       // event-kernel tables
+  uint32_t qo_off, qo_bytes;
+  const uint4 *px, *kx, *qr;
+  const uint64_t *pd;
+  const uint32_t *st;
   int split;        // warps per tile (1 or 2)
   int minb;         // register target: 2 or 3 resident CTAs per SM
   int max_ctas[8];  // per mode: resident CTAs (occupancy x SMs)
@@ -303,6 +326,97 @@ int aceso_load_profile(const aceso_profile_desc *d, int cuda_device, aceso_ctx *
     }
   }
 
+  // ---- event-kernel tables (event_kernel.cuh): position prefixes per run ----
+  const uint32_t Lp1 = (uint32_t)L + 1u;
+  const int levels = 32 - __builtin_clz((unsigned)L);  // floor(log2 L) + 1
+  const int nq = (L + 3) / 4;
+  std::vector<uint32_t> eqo(nq);
+  std::vector<std::array<int, 4>> esigs;
+  {
+    std::map<std::array<int, 4>, int> seen;
+    for (int q = 0; q < nq; ++q) {
+      std::array<int, 4> key;
+      for (int k = 0; k < 4; ++k) key[k] = 4 * q + k < L ? (int)d->op_type[4 * q + k] : -1;
+      auto it = seen.find(key);
+      if (it == seen.end()) {
+        it = seen.emplace(key, (int)esigs.size()).first;
+        esigs.push_back(key);
+      }
+      eqo[q] = (uint32_t)it->second * RUNS * 16u;
+    }
+  }
+  auto al = [](size_t v) { return (v + 255) & ~(size_t)255; };
+  const size_t ev_px = 0;
+  const size_t ev_kx = al(ev_px + (size_t)RUNS * Lp1 * 32);
+  const size_t ev_pd = al(ev_kx + (size_t)RUNS * Lp1 * 16);
+  const size_t ev_st = al(ev_pd + (size_t)NT * ND * Lp1 * 8);
+  const size_t ev_qr = al(ev_st + (size_t)levels * RUNS * L * 4);
+  const size_t ev_qo = al(ev_qr + esigs.size() * RUNS * 16 * 32);
+  const uint32_t qo_bytes = a16((uint32_t)nq * 4u);
+  const size_t ev_bytes = al(ev_qo + qo_bytes);
+  std::vector<unsigned char> ev(ev_bytes, 0);
+  {
+    auto put64 = [&](size_t off, uint64_t v) { memcpy(&ev[off], &v, 8); };
+    auto put32 = [&](size_t off, uint32_t v) { memcpy(&ev[off], &v, 4); };
+    for (int b = 0; b < NB; ++b)
+      for (int tp = 0; tp < NT; ++tp) {
+        const uint32_t rr = (uint32_t)(b * NT + tp);
+        uint64_t PS = 0, PA = 0, PW = 0, PC = 0;
+        for (uint32_t j = 0; j <= (uint32_t)L; ++j) {
+          const size_t o = (size_t)rr * Lp1 + j;
+          put64(ev_px + o * 32, PS);
+          put64(ev_px + o * 32 + 8, PA);
+          put64(ev_px + o * 32 + 16, PW);
+          put64(ev_px + o * 32 + 24, PC);
+          if (j < (uint32_t)L) {
+            const int t = d->op_type[j];
+            PS += rec_S(t, tp, b, 0);
+            PA += rec_A(t, tp, b, 0);
+            PW += rec_W(t, tp);
+            PC += rec_C(t, tp, b, 0);
+            put32(ev_kx + o * 16, (uint32_t)R(t, tp, b, ACESO_F_RESHARD));
+            put32(ev_kx + o * 16 + 4, (uint32_t)R(t, tp, b, ACESO_F_P2P_BWD));
+            put32(ev_st + ((size_t)rr * L + j) * 4, (uint32_t)rec_e(t, tp, b, 0));
+          }
+          if (j > 0) put32(ev_kx + o * 16 + 8, (uint32_t)R(d->op_type[j - 1], tp, b, ACESO_F_P2P_FWD));
+        }
+        for (int k = 1; k < levels; ++k)
+          for (int j = 0; j < L; ++j) {
+            const int j2 = std::min(j + (1 << (k - 1)), L - 1);
+            uint32_t v1, v2;
+            memcpy(&v1, &ev[ev_st + (((size_t)(k - 1) * RUNS + rr) * L + j) * 4], 4);
+            memcpy(&v2, &ev[ev_st + (((size_t)(k - 1) * RUNS + rr) * L + j2) * 4], 4);
+            put32(ev_st + (((size_t)k * RUNS + rr) * L + j) * 4, std::max(v1, v2));
+          }
+        for (size_t sg = 0; sg < esigs.size(); ++sg)
+          for (uint32_t m = 1; m < 16; ++m) {
+            uint64_t dS = 0, dA = 0, dC = 0, E1 = 0;
+            for (int k = 0; k < 4; ++k) {
+              const int t = esigs[sg][k];
+              if (t < 0 || !((m >> k) & 1u)) continue;
+              dS += (uint64_t)R(t, tp, b, ACESO_F_FWD_COMP) + R(t, tp, b, ACESO_F_FWD_COMM);
+              dA += (uint64_t)(R(t, tp, b, ACESO_F_ACT) - R(t, tp, b, ACESO_F_KEEP)) >> ms;
+              dC += (uint64_t)R(t, tp, b, ACESO_F_FWD_COMP);
+              E1 = std::max(E1, rec_e(t, tp, b, 1));
+            }
+            const size_t o = ev_qr + (((size_t)sg * RUNS + rr) * 16 + m) * 32;
+            put64(o, dS);
+            put64(o + 8, dA);
+            put32(o + 16, (uint32_t)E1);
+            put64(o + 24, dC);
+          }
+      }
+    for (int tp = 0; tp < NT; ++tp)
+      for (int dp = 0; dp < ND; ++dp) {
+        uint64_t s = 0;
+        for (uint32_t j = 0; j <= (uint32_t)L; ++j) {
+          put64(ev_pd + (((size_t)tp * ND + dp) * Lp1 + j) * 8, s);
+          if (j < (uint32_t)L) s += dps_of(d->op_type[j], tp, dp);
+        }
+      }
+    for (int q = 0; q < nq; ++q) put32(ev_qo + (size_t)q * 4, eqo[q]);
+  }
+
   // ---- device ----
   int ndev = 0;
   if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev == 0) return fail(ACESO_ENODEV, "no CUDA device");
@@ -325,12 +439,22 @@ int aceso_load_profile(const aceso_profile_desc *d, int cuda_device, aceso_ctx *
   ctx->tab = tab;
   ctx->mem_shift = ms;
   ctx->d_blob = nullptr;
+  ctx->d_ev = nullptr;
+  ctx->kernel = 1;
+  if (const char *env = getenv("ACESO_KERNEL")) {
+    if (!strcmp(env, "quad")) ctx->kernel = 0;
+    else if (!strcmp(env, "events")) ctx->kernel = 1;
+  }
+  ctx->qo_off = (uint32_t)ev_qo;
+  ctx->qo_bytes = qo_bytes;
   int rc = ACESO_OK;
   do {
     cudaStream_t st;
     if (cudaStreamCreateWithFlags(&st, cudaStreamNonBlocking) != cudaSuccess) { rc = fail(ACESO_ECUDA, "stream create"); break; }
     cudaError_t e = cudaMalloc(&ctx->d_blob, blob_bytes);
     if (e == cudaSuccess) e = cudaMemcpyAsync(ctx->d_blob, blob.data(), blob_bytes, cudaMemcpyHostToDevice, st);
+    if (e == cudaSuccess) e = cudaMalloc(&ctx->d_ev, ev_bytes);
+    if (e == cudaSuccess) e = cudaMemcpyAsync(ctx->d_ev, ev.data(), ev_bytes, cudaMemcpyHostToDevice, st);
     if (e == cudaSuccess) e = cudaStreamSynchronize(st);
     cudaStreamDestroy(st);
     if (e != cudaSuccess) { rc = fail(e == cudaErrorMemoryAllocation ? ACESO_ENOMEM : ACESO_ECUDA, "upload: %s", cudaGetErrorString(e)); break; }
@@ -345,12 +469,23 @@ int aceso_load_profile(const aceso_profile_desc *d, int cuda_device, aceso_ctx *
       int v = atoi(env);
       if (v == 2 || v == 3) ctx->minb = v;
     }
+    {
+      const unsigned char *eb = reinterpret_cast<const unsigned char *>(ctx->d_ev);
+      ctx->px = reinterpret_cast<const uint4 *>(eb + ev_px);
+      ctx->kx = reinterpret_cast<const uint4 *>(eb + ev_kx);
+      ctx->pd = reinterpret_cast<const uint64_t *>(eb + ev_pd);
+      ctx->st = reinterpret_cast<const uint32_t *>(eb + ev_st);
+      ctx->qr = reinterpret_cast<const uint4 *>(eb + ev_qr);
+    }
+    if (ctx->kernel == 1) ctx->split = 1;
     for (uint32_t mode = 1; mode < 8; ++mode) {
-      const size_t smem = ((mode & ACESO_OUT_FULL) ? tab.bytes_full : tab.bytes) +
-                          (tab.k_smem ? bytesK : 0u) + kRingBytesPerCta +
-                          (ctx->split == 2 ? (size_t)(kWarps / 2) * 32 * sizeof(Xchg) : 0);
+      const size_t smem =
+          ctx->kernel == 1
+              ? (size_t)qo_bytes + ev_ring_bytes() + ev_list_bytes() + ev_snap_bytes(mode & ACESO_OUT_FULL)
+              : ((mode & ACESO_OUT_FULL) ? tab.bytes_full : tab.bytes) + (tab.k_smem ? bytesK : 0u) +
+                    kRingBytesPerCta + (ctx->split == 2 ? (size_t)(kWarps / 2) * 32 * sizeof(Xchg) : 0);
       ctx->smem[mode] = smem;
-      void *k = eval_kernel_for(mode, ctx->split, ctx->minb);
+      void *k = eval_kernel_for(mode, ctx->split, ctx->minb, ctx->kernel);
       e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
       int occ = 0;
       if (e == cudaSuccess) e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k, kThreads, smem);
@@ -361,6 +496,7 @@ int aceso_load_profile(const aceso_profile_desc *d, int cuda_device, aceso_ctx *
   cudaSetDevice(prev_dev);
   if (rc != ACESO_OK) {
     if (ctx->d_blob) cudaFree(ctx->d_blob);
+    if (ctx->d_ev) cudaFree(ctx->d_ev);
     delete ctx;
     return rc;
   }
@@ -374,6 +510,7 @@ void aceso_free(aceso_ctx *ctx) {
   cudaGetDevice(&prev);
   cudaSetDevice(ctx->device);
   cudaFree(ctx->d_blob);
+  cudaFree(ctx->d_ev);
   cudaSetDevice(prev);
   delete ctx;
 }
@@ -437,6 +574,15 @@ int aceso_eval(aceso_ctx *ctx, const uint8_t *d_codes, const uint64_t *d_hdr, in
   P.sel = reinterpret_cast<unsigned char *>(d_sel);
   P.n_total = n_total;
   P.ib = std::max(1u, bitlen((uint64_t)n_total));
+  P.px = ctx->px;
+  P.kx = ctx->kx;
+  P.pd = ctx->pd;
+  P.st = ctx->st;
+  P.qr = ctx->qr;
+  P.runs = (uint32_t)(ctx->n_b * ctx->n_tp);
+  P.qo_bytes = ctx->qo_bytes;
+  P.qo_off = ctx->qo_off;
+  P.evblob = reinterpret_cast<const unsigned char *>(ctx->d_ev);
 
   const int tiles_per_cta = kWarps / ctx->split;
   const int64_t need = (P.n_tiles + tiles_per_cta - 1) / tiles_per_cta;
@@ -445,7 +591,7 @@ int aceso_eval(aceso_ctx *ctx, const uint8_t *d_codes, const uint64_t *d_hdr, in
   CUDA_TRY(cudaGetDevice(&prev));
   if (prev != ctx->device) CUDA_TRY(cudaSetDevice(ctx->device));
   void *args[] = {&P};
-  cudaError_t e = cudaLaunchKernel(eval_kernel_for(mode, ctx->split, ctx->minb), dim3(grid), dim3(kThreads), args, ctx->smem[mode],
+  cudaError_t e = cudaLaunchKernel(eval_kernel_for(mode, ctx->split, ctx->minb, ctx->kernel), dim3(grid), dim3(kThreads), args, ctx->smem[mode],
                                    reinterpret_cast<cudaStream_t>(stream));
   if (prev != ctx->device) cudaSetDevice(prev);
   if (e != cudaSuccess) return fail(ACESO_ECUDA, "eval launch: %s", cudaGetErrorString(e));

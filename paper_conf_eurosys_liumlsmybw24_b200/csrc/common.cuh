@@ -63,6 +63,16 @@ struct EvalParams {
   unsigned char *sel;     // aceso_select_result + counter + per-CTA partials
   int64_t n_total;
   uint32_t ib;            // index bits of the packed key
+  // event kernel (event_kernel.cuh): position-prefix tables in global memory, see EvTables
+  const uint4 *px;        // [RUNS][L+1] x 2: {PS, PA} {PW, PC}   (u64 prefix sums, rc = 0)
+  const uint4 *kx;        // [RUNS][L+1]    : {reshard_j, p2p_bwd_j, p2p_fwd_{j-1}, 0}
+  const uint64_t *pd;     // [n_tp * n_dp][L+1] DP all-reduce prefix sums
+  const uint32_t *st;     // [levels][RUNS][L] sparse table of e0 = peak (range max)
+  const uint4 *qr;        // [nsig][RUNS][16] x 2: {dS, dA} {E1, 0, dC} rc deltas of a quad pattern
+  uint32_t runs;          // RUNS = n_b * n_tp
+  uint32_t qo_bytes;      // bytes of the per-quad signature table staged to shared memory
+  uint32_t qo_off;        // its byte offset in the event blob
+  const unsigned char *evblob;
 };
 
 // select buffer layout: [0,32) result, [32,40) completion counter, [64, ...) partials (16 B each)

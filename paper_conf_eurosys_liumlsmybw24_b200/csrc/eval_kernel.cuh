@@ -145,8 +145,8 @@ struct Xchg {
 };
 
 // Closes the current stage i: Eq. 2 key, Eq. 1 memory, OOM, Heuristic-1 maxima.
-template <uint32_t MODE>
-__device__ __forceinline__ void stage_commit(Cand &s, const EvalParams &P, int64_t c, bool active,
+template <uint32_t MODE, class St>
+__device__ __forceinline__ void stage_commit(St &s, const EvalParams &P, int64_t c, bool active,
                                              bool reverse) {
   s.sumS += s.S;
   const uint64_t tk = (uint64_t)(s.N - 1) * s.S + s.D;  // T_i - sum_k S_k (Eq. 2, R1, R6)
@@ -391,8 +391,8 @@ __device__ __forceinline__ void quad_rev(Cand &s, const Smem &sm, const EvalPara
 }
 
 // Candidate epilogue (forward part): validity, summary outputs, fused argmin.
-template <uint32_t MODE>
-__device__ __forceinline__ void finish_cand(Cand &s, const EvalParams &P, int64_t c, bool active,
+template <uint32_t MODE, class St>
+__device__ __forceinline__ void finish_cand(St &s, const EvalParams &P, int64_t c, bool active,
                                             uint64_t &best_ck, int64_t &best_idx) {
   if (!s.head0) s.reasons |= ACESO_R_HEAD0;
   if (s.nheads != s.p) s.reasons |= ACESO_R_NSTAGE;

@@ -1,0 +1,481 @@
+// event_kernel.cuh — event-driven evaluation of Aceso's performance/memory model (sm_100a).
+//
+// Same contract and outputs as eval_kernel.cuh (thread = candidate, warp = tile of 32,
+// codes streamed through a per-warp cp.async.bulk ring), different arithmetic schedule:
+//
+// A stage's sums are sums over its RUNS (maximal op ranges of one (tp, dp) inside one
+// stage). Within a run every op uses the same record key (b = mbs/dp, tp), so the run's
+// contribution is a difference of position-prefix sums, PX[run][end] - PX[run][start],
+// and its transient-memory term e is a range maximum (sparse table ST, two lookups).
+// Recomputation only changes some ops of a run; its effect is the sum of per-op deltas
+// (dS = fwd, dA = act - keep, dC = fwd_comp; e1 = peak + act - keep >= e0 = peak), looked
+// up per 4-op quad and rc pattern from QR[signature][run][pattern].
+//
+// Phase A (lockstep over the code stream, 4 ops per step): per lane, one LOP3 finds the
+// "events" of a quad (stage head, tp/dp change); a quad without events or recompute
+// costs a handful of instructions and no table access. Events are appended to a per-lane
+// list in shared memory; recompute deltas are accumulated in registers and, at a stage
+// head, moved to a per-lane snapshot list (they belong to the stage the head closes).
+// Phase B (drain, lockstep over list entries): every lane processes its k-th event at
+// step k — the warp runs max_lane(#events) steps instead of one step per op position at
+// which ANY lane has an event. An event closes the current run (prefix difference, range
+// max; at a head also p2p_fwd, the snapshot, and the stage: Eq. 1/2, OOM, Heuristic-1)
+// and opens the next (validity, p2p_bwd or reshard, prefix base). The lists drain when
+// one could overflow and at the end of each tile.
+//
+// Paper: configuration (§3.1), Heuristic-1, memory Eq. 1
+// (P:L225-234), time Eq. 2; readings R1-R13 in DESIGN.md §3.
+#pragma once
+#include "eval_kernel.cuh"
+
+namespace aceso {
+
+constexpr int kEvCap = 24;      // events per lane between drains (a chunk adds <= 16)
+constexpr int kSnCap = 4;       // recompute snapshots per lane between drains (a quad adds <= 4)
+constexpr int kEvRingSlots = 3; // per-warp ring depth (1 KB slots)
+
+__host__ __device__ constexpr uint32_t ev_ring_bytes() { return (uint32_t)kWarps * kEvRingSlots * kSlotBytes; }
+__host__ __device__ constexpr uint32_t ev_list_bytes() { return (uint32_t)kWarps * kEvCap * 32 * 4; }
+__host__ __device__ constexpr uint32_t ev_snap_bytes(bool full) {
+  return (uint32_t)kWarps * kSnCap * 32 * (full ? 28u : 20u);
+}
+
+__device__ __forceinline__ uint64_t u64of(uint32_t lo, uint32_t hi) {
+  return ((uint64_t)hi << 32) | lo;
+}
+__device__ __forceinline__ void sts32(uint32_t a, uint32_t v) {
+  asm volatile("st.shared.u32 [%0], %1;" ::"r"(a), "r"(v) : "memory");
+}
+__device__ __forceinline__ void sts64(uint32_t a, uint64_t v) {
+  asm volatile("st.shared.u64 [%0], %1;" ::"r"(a), "l"(v) : "memory");
+}
+__device__ __forceinline__ uint64_t lds64u(uint32_t a) {
+  uint64_t v;
+  asm volatile("ld.shared.u64 %0, [%1];" : "=l"(v) : "r"(a));
+  return v;
+}
+
+struct EvCand {
+  // phase B: the open stage (prefix-difference form: -PX[start] + PX[end] per run)
+  uint64_t S, A, W, D, comp;
+  uint32_t E;
+  uint32_t rr, dd, a;  // open run: (b, tp) index, (tp, dp) index, first op
+  // phase A: recompute deltas since the last stage head
+  uint64_t rS, rA, rC;
+  uint32_t rE, rany;
+  uint32_t rrA;        // phase A's current run (b, tp) index
+  uint32_t ec, sc, sp; // events listed, snapshots pushed, snapshots popped
+  // candidate-level aggregates (names shared with Cand: stage_commit / finish_cand)
+  uint64_t sumS, bestT, bestM;
+  uint32_t bt, bm, oom, i, gsum, reasons, nheads, head0, gst;
+  uint32_t mbs, p, N;
+};
+
+// per-lane shared-memory addresses of the lists
+struct EvLists {
+  uint32_t ev;          // event k at ev + 128 k (u32: op | code << 16 | snapshot << 24)
+  uint32_t sS, sA, sC;  // snapshot k at +256 k (u64)
+  uint32_t sE;          // snapshot k at +128 k (u32)
+};
+
+__device__ __forceinline__ void ev_init(EvCand &s, const EvalParams &P, uint64_t h) {
+  s.mbs = (uint32_t)(h & 0xff);
+  s.p = (uint32_t)((h >> 8) & 0xff);
+  s.reasons = (h >> 16) ? ACESO_R_HDR : 0u;
+  s.N = 0;
+  if (s.mbs >= 62 || (1ull << s.mbs) > P.Bg || (P.Bg & ((1ull << s.mbs) - 1)) != 0)
+    s.reasons |= ACESO_R_MBS;
+  else
+    s.N = (uint32_t)(P.Bg >> s.mbs);
+  if (s.p == 0 || s.p > (uint32_t)P.G) s.reasons |= ACESO_R_PRANGE;
+  s.S = s.A = s.W = s.D = s.comp = 0;
+  s.E = 0;
+  s.rr = s.dd = s.a = 0;
+  s.rS = s.rA = s.rC = 0;
+  s.rE = s.rany = 0;
+  s.rrA = 0;
+  s.ec = s.sc = s.sp = 0;
+  s.sumS = s.bestT = s.bestM = 0;
+  s.bt = s.bm = 0;
+  s.oom = s.gsum = s.nheads = s.head0 = s.gst = 0;
+  s.i = 0;
+}
+
+// (b, tp) run index of an op code under the candidate's mbs (clamped: invalid encodings
+// still index inside the tables; their reasons are set when the run opens)
+__device__ __forceinline__ uint32_t ev_run(uint32_t c, uint32_t mbs, const EvalParams &P) {
+  const uint32_t tpl = (c >> 1) & 7u, dpl = c >> 5;
+  const uint32_t b = min(dpl <= mbs ? mbs - dpl : 0u, (uint32_t)P.n_b - 1);
+  return b * (uint32_t)P.n_tp + min(tpl, (uint32_t)P.n_tp - 1);
+}
+
+// recompute deltas of the ops of quad pattern pat (bit k = op 4q+k) under run rr
+template <uint32_t MODE>
+__device__ __forceinline__ void ev_rc_add(EvCand &s, const EvalParams &P, uint32_t qsb, uint32_t rr,
+                                          uint32_t pat) {
+  const uint32_t idx = qsb + rr * 16u + pat;
+  const uint4 v0 = __ldg(P.qr + 2 * (size_t)idx);
+  const uint4 v1 = __ldg(P.qr + 2 * (size_t)idx + 1);
+  s.rS += u64of(v0.x, v0.y);
+  s.rA += u64of(v0.z, v0.w);
+  s.rE = max(s.rE, v1.x);
+  if (MODE & kFull) s.rC += u64of(v1.z, v1.w);
+  s.rany = 1u;
+}
+
+// 4-bit pattern of the bytes of a quad word whose bit `bit` is set (bits 0..3 = ops 0..3)
+__device__ __forceinline__ uint32_t quad_bits(uint32_t v, int bit) {
+  return ((((v >> bit) & 0x01010101u) * 0x01020408u) >> 24) & 0xfu;
+}
+// 4-bit pattern of the non-zero bytes of a quad word
+__device__ __forceinline__ uint32_t quad_nonzero(uint32_t v) {
+  const uint32_t y = (((v & 0x7f7f7f7fu) + 0x7f7f7f7fu) | v) & 0x80808080u;
+  return quad_bits(y, 7);
+}
+
+// phase A, a quad of this lane with events and/or recompute flags (x = events, m = rc
+// flags): recompute deltas are added per segment (ops between consecutive events share
+// one run); each event is listed, a stage head first moving the deltas accumulated so
+// far to a snapshot
+template <uint32_t MODE>
+__device__ __forceinline__ void ev_quad(EvCand &s, const EvalParams &P, const EvLists &l,
+                                        uint32_t w, uint32_t x, uint32_t m, uint32_t qg,
+                                        uint32_t qsb) {
+  if (x == 0u) {  // recompute flags only: one pattern lookup under the current run
+    ev_rc_add<MODE>(s, P, qsb, s.rrA, quad_bits(m, 4));
+    return;
+  }
+  uint32_t evb = quad_nonzero(x);
+  if (m == 0u && !(s.rany && (x & 0x01010101u))) {  // events only, no snapshot needed
+    uint32_t c = 0;
+#pragma unroll 1
+    do {
+      const uint32_t k = __ffs(evb) - 1u;
+      evb &= evb - 1u;
+      c = (w >> (8u * k)) & 0xffu;
+      sts32(l.ev + 128u * s.ec, (qg * 4u + k) | (c << 16));
+      s.ec += 1;
+    } while (evb);
+    s.rrA = ev_run(c, s.mbs, P);
+    return;
+  }
+  const uint32_t pat = quad_bits(m, 4);
+  evb |= 0x10u;  // + a virtual end of the quad at op 4
+  uint32_t start = 0, rrs = s.rrA;
+#pragma unroll 1
+  while (true) {
+    const uint32_t k = __ffs(evb) - 1u;
+    evb &= evb - 1u;
+    const uint32_t segp = pat & ((1u << k) - 1u) & ~((1u << start) - 1u);  // ops [start, k)
+    if (segp) ev_rc_add<MODE>(s, P, qsb, rrs, segp);
+    if (k == 4u) break;
+    const uint32_t c = (w >> (8u * k)) & 0xffu;
+    uint32_t flag = 0;
+    if ((c & 1u) && s.rany) {  // head: recompute deltas of the stage it closes
+      sts64(l.sS + 256u * s.sc, s.rS);
+      sts64(l.sA + 256u * s.sc, s.rA);
+      sts32(l.sE + 128u * s.sc, s.rE);
+      if (MODE & kFull) sts64(l.sC + 256u * s.sc, s.rC);
+      s.sc += 1;
+      s.rS = s.rA = s.rC = 0;
+      s.rE = 0;
+      s.rany = 0;
+      flag = 1u << 24;
+    }
+    sts32(l.ev + 128u * s.ec, (qg * 4u + k) | (c << 16) | flag);
+    s.ec += 1;
+    rrs = ev_run(c, s.mbs, P);
+    start = k;
+  }
+  s.rrA = rrs;
+}
+
+// activity word of a quad: bit 4 of a byte = recompute flag, other bits = event (head or
+// tp/dp change against the previous op; p = the previous quad's word)
+__device__ __forceinline__ uint32_t quad_activity(uint32_t w, uint32_t p) {
+  const uint32_t sh = __funnelshift_l(p, w, 8);  // previous op's byte under each byte
+  uint32_t d, f;
+  asm("lop3.b32 %0, %1, %2, %3, 0xB4;" : "=r"(d) : "r"(w), "r"(sh), "r"(0x01010101u));  // c ? w : w^sh
+  asm("lop3.b32 %0, %1, %2, %3, 0xD8;" : "=r"(f) : "r"(d), "r"(w), "r"(0x10101010u));   // c ? w : d
+  return f;
+}
+
+// closes the open run [s.a, j) under s.rr (prefix difference, range max)
+template <uint32_t MODE>
+__device__ __forceinline__ void ev_close_run(EvCand &s, const EvalParams &P, uint32_t j) {
+  const uint32_t Lp1 = (uint32_t)P.L + 1u;
+  const size_t o = (size_t)s.rr * Lp1 + j;
+  const uint4 x0 = __ldg(P.px + 2 * o);
+  const uint4 x1 = __ldg(P.px + 2 * o + 1);
+  const uint64_t dsum = __ldg(P.pd + (size_t)s.dd * Lp1 + j);
+  const uint32_t k = 31u - __clz(j - s.a);
+  const uint32_t *stk = P.st + ((size_t)k * P.runs + s.rr) * (uint32_t)P.L;
+  const uint32_t e = max(__ldg(stk + s.a), __ldg(stk + j - (1u << k)));
+  s.S += u64of(x0.x, x0.y);
+  s.A += u64of(x0.z, x0.w);
+  s.W += u64of(x1.x, x1.y);
+  if (MODE & kFull) s.comp += u64of(x1.z, x1.w);
+  s.D += dsum;
+  s.E = max(s.E, e);
+}
+
+// phase B: one event (op j with code c opens a run; a head also closes a stage)
+template <uint32_t MODE>
+__device__ __forceinline__ void ev_handle(EvCand &s, const EvalParams &P, const EvLists &l,
+                                          uint32_t ent, int64_t cand, bool active) {
+  const uint32_t j = ent & 0xffffu, c = (ent >> 16) & 0xffu;
+  const uint32_t head = c & 1u;
+  const uint32_t Lp1 = (uint32_t)P.L + 1u;
+  const uint32_t *kx = reinterpret_cast<const uint32_t *>(P.kx);
+  if (j > 0) {
+    ev_close_run<MODE>(s, P, j);
+    if (head) {
+      s.S += __ldg(kx + 4 * ((size_t)s.rr * Lp1 + j) + 2);  // R5: p2p_fwd of the stage's last op
+      if (ent >> 24) {                                       // recompute deltas of this stage
+        s.S += lds64u(l.sS + 256u * s.sp);
+        s.A -= lds64u(l.sA + 256u * s.sp);
+        s.E = max(s.E, lds32(l.sE + 128u * s.sp));
+        if (MODE & kFull) s.comp += lds64u(l.sC + 256u * s.sp);
+        s.sp += 1;
+      }
+      stage_commit<MODE>(s, P, cand, active, false);
+      s.i += 1;
+    }
+  }
+  // open the run of op j: validity, table keys, p2p_bwd / reshard, prefix base
+  const uint32_t tpl = (c >> 1) & 7u, dpl = c >> 5;
+  if (dpl > s.mbs) s.reasons |= ACESO_R_DPMBS;
+  if (tpl >= (uint32_t)P.n_tp || dpl >= (uint32_t)P.n_dp || (dpl <= s.mbs && s.mbs - dpl >= (uint32_t)P.n_b))
+    s.reasons |= ACESO_R_TABLE;
+  const uint32_t b = min(dpl <= s.mbs ? s.mbs - dpl : 0u, (uint32_t)P.n_b - 1);
+  const uint32_t tplc = min(tpl, (uint32_t)P.n_tp - 1), dplc = min(dpl, (uint32_t)P.n_dp - 1);
+  s.rr = b * (uint32_t)P.n_tp + tplc;
+  s.dd = tplc * (uint32_t)P.n_dp + dplc;
+  const size_t o = (size_t)s.rr * Lp1 + j;
+  const uint32_t g = tpl + dpl;
+  if (head || j == 0) {
+    s.gst = g;
+    s.gsum += 1u << g;  // R9
+    s.nheads += head;
+    if (head && j > 0) s.S += __ldg(kx + 4 * o + 1);  // R5: p2p_bwd of the first op
+  } else {
+    if (g != s.gst) s.reasons |= ACESO_R_GSTAGE;  // P:L151 in-stage symmetry
+    s.S += __ldg(kx + 4 * o);                     // R13: reshard into this op
+  }
+  const uint4 y0 = __ldg(P.px + 2 * o);
+  const uint4 y1 = __ldg(P.px + 2 * o + 1);
+  s.S -= u64of(y0.x, y0.y);
+  s.A -= u64of(y0.z, y0.w);
+  s.W -= u64of(y1.x, y1.y);
+  if (MODE & kFull) s.comp -= u64of(y1.z, y1.w);
+  s.D -= __ldg(P.pd + (size_t)s.dd * Lp1 + j);
+  s.a = j;
+}
+
+// phase B over every lane's list (warp-uniform call)
+template <uint32_t MODE>
+__device__ __forceinline__ void ev_drain(EvCand &s, const EvalParams &P, const EvLists &l,
+                                         int64_t cand, bool active) {
+  const uint32_t mx = __reduce_max_sync(0xffffffffu, s.ec);
+#pragma unroll 1
+  for (uint32_t k = 0; k < mx; ++k) {
+    if (k < s.ec) ev_handle<MODE>(s, P, l, lds32(l.ev + 128u * k), cand, active);
+  }
+  s.ec = s.sc = s.sp = 0;
+}
+
+// phase A over the quads `now` (bit q = quad q) of one 16-op chunk of this lane (w4 =
+// its 16 code bytes, pw = the previous word): activity words of the quads; quads with
+// activity in any lane are visited
+template <uint32_t MODE>
+__device__ __forceinline__ void ev_chunk(EvCand &s, const EvalParams &P, const EvLists &l,
+                                         uint4 w4, uint32_t pw, uint32_t ch, uint32_t qo,
+                                         uint32_t now) {
+  const uint32_t f0 = quad_activity(w4.x, pw), f1 = quad_activity(w4.y, w4.x);
+  const uint32_t f2 = quad_activity(w4.z, w4.y), f3 = quad_activity(w4.w, w4.z);
+  const uint32_t lm = (f0 ? 1u : 0u) | (f1 ? 2u : 0u) | (f2 ? 4u : 0u) | (f3 ? 8u : 0u);
+  const uint32_t slow = __reduce_or_sync(0xffffffffu, lm) & now;  // quads with activity in any lane
+  if (slow == 0u) return;
+  const uint32_t qg = ch * 4u;
+  if (slow & 1u) if (f0) ev_quad<MODE>(s, P, l, w4.x, f0 & 0xefefefefu, f0 & 0x10101010u, qg, lds32(qo + 4u * qg));
+  if (slow & 2u) if (f1) ev_quad<MODE>(s, P, l, w4.y, f1 & 0xefefefefu, f1 & 0x10101010u, qg + 1u, lds32(qo + 4u * qg + 4u));
+  if (slow & 4u) if (f2) ev_quad<MODE>(s, P, l, w4.z, f2 & 0xefefefefu, f2 & 0x10101010u, qg + 2u, lds32(qo + 4u * qg + 8u));
+  if (slow & 8u) if (f3) ev_quad<MODE>(s, P, l, w4.w, f3 & 0xefefefefu, f3 & 0x10101010u, qg + 3u, lds32(qo + 4u * qg + 12u));
+}
+
+// heads in a chunk (upper bound of the snapshots it can push)
+__device__ __forceinline__ uint32_t chunk_heads(uint4 w4) {
+  uint32_t h;
+  asm("lop3.b32 %0, %1, %2, %3, 0xFE;" : "=r"(h) : "r"(w4.x & 0x01010101u), "r"((w4.y & 0x01010101u) << 1),
+      "r"((w4.z & 0x01010101u) << 2));
+  return __popc(h | ((w4.w & 0x01010101u) << 3));
+}
+
+// ops >= L of the last chunk (zero padding) take the last op's tp/dp without head or
+// recompute: no events, no deltas (nvl = valid ops of the chunk, 1..15)
+__device__ __forceinline__ uint4 pad_tail(uint4 w4, uint32_t nvl) {
+  const uint32_t i = (nvl - 1u) >> 2;
+  const uint32_t lw = i == 0u ? w4.x : i == 1u ? w4.y : i == 2u ? w4.z : w4.w;
+  const uint32_t f = ((lw >> (8u * ((nvl - 1u) & 3u))) & 0xeeu) * 0x01010101u;
+  auto keep = [&](uint32_t k) {  // valid-byte mask of word k
+    return nvl >= 4u * k + 4u ? 0xffffffffu : nvl <= 4u * k ? 0u : (1u << (8u * (nvl - 4u * k))) - 1u;
+  };
+  uint32_t m;
+  m = keep(0); w4.x = (w4.x & m) | (f & ~m);
+  m = keep(1); w4.y = (w4.y & m) | (f & ~m);
+  m = keep(2); w4.z = (w4.z & m) | (f & ~m);
+  m = keep(3); w4.w = (w4.w & m) | (f & ~m);
+  return w4;
+}
+
+template <uint32_t MODE, int MINB>
+__global__ void __launch_bounds__(kThreads, MINB) event_kernel(const __grid_constant__ EvalParams P) {
+  extern __shared__ __align__(128) unsigned char sm_raw[];
+  __shared__ __align__(8) uint64_t s_tbar;
+  __shared__ __align__(8) uint64_t s_ring_bar[kWarps][kEvRingSlots];
+  __shared__ uint64_t s_ck[kWarps];
+  __shared__ int64_t s_idx[kWarps];
+
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const uint32_t sb = smem_addr(sm_raw);
+  // layout: [qo][ring][event lists][snapshots S, A, (C), E]
+  const uint32_t qo = sb;
+  const uint32_t ring = sb + P.qo_bytes + (uint32_t)warp * kEvRingSlots * kSlotBytes;
+  const uint32_t lists = sb + P.qo_bytes + ev_ring_bytes();
+  EvLists l;
+  l.ev = lists + (uint32_t)warp * kEvCap * 128u + lane * 4u;
+  const uint32_t snap = lists + ev_list_bytes();
+  const uint32_t blk64 = (uint32_t)kWarps * kSnCap * 256u;  // one u64 snapshot field, all warps
+  l.sS = snap + (uint32_t)warp * kSnCap * 256u + lane * 8u;
+  l.sA = l.sS + blk64;
+  l.sC = l.sA + blk64;
+  l.sE = snap + ((MODE & kFull) ? 3u : 2u) * blk64 + (uint32_t)warp * kSnCap * 128u + lane * 4u;
+
+  if (threadIdx.x == 0) {
+    mbar_init(smem_addr(&s_tbar), 1);
+    fence_barrier_init();
+  }
+  if (lane == 0) {
+    for (int k = 0; k < kEvRingSlots; ++k) mbar_init(smem_addr(&s_ring_bar[warp][k]), 1);
+    fence_barrier_init();
+  }
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    const uint32_t bar = smem_addr(&s_tbar);
+    mbar_expect_tx(bar, P.qo_bytes);
+    bulk_g2s(qo, P.evblob + P.qo_off, P.qo_bytes, bar);
+  }
+
+  const uint32_t nch = (uint32_t)P.nch;
+  const uint32_t ngroups = (nch + kSlotChunks - 1) / kSlotChunks;
+  const int64_t first_tile = (int64_t)blockIdx.x * kWarps + warp;
+  const int64_t tile_stride = (int64_t)gridDim.x * kWarps;
+  const int64_t my_tiles =
+      first_tile < P.n_tiles ? (P.n_tiles - first_tile + tile_stride - 1) / tile_stride : 0;
+  const int64_t units = my_tiles * ngroups;
+  const unsigned char *codes = reinterpret_cast<const unsigned char *>(P.codes);
+
+  int64_t it_tile = first_tile;
+  uint32_t it_g = 0;
+  auto issue_next = [&](int slot) {
+    const uint32_t a = kSlotChunks * it_g, b = min(a + kSlotChunks, nch);
+    const uint32_t bar = smem_addr(&s_ring_bar[warp][slot]);
+    mbar_expect_tx(bar, (b - a) * 512u);
+    bulk_g2s(ring + slot * kSlotBytes, codes + ((size_t)it_tile * nch + a) * 512, (b - a) * 512u, bar);
+    if (++it_g == ngroups) {
+      it_g = 0;
+      it_tile += tile_stride;
+    }
+  };
+  if (lane == 0) {
+    for (int64_t u = 0; u < units && u < kEvRingSlots; ++u) issue_next((int)u);
+  }
+  __syncwarp();
+  mbar_wait(smem_addr(&s_tbar), 0);
+
+  const uint32_t nvl = (uint32_t)P.L - 16u * (nch - 1u);  // valid ops of the last chunk
+  const uint32_t ring_lane = ring + lane * 16u;
+
+  uint64_t best_ck = ~0ull;
+  int64_t best_idx = INT64_MAX;
+  EvCand s;
+  uint32_t pw = 0;
+  int64_t tile = first_tile;
+  uint32_t g = 0;
+  int slot = 0;
+  uint32_t phase = 0;
+  int64_t cand = 0;
+  bool active = false;
+  for (int64_t u = 0; u < units; ++u) {
+    if (g == 0) {
+      cand = tile * 32 + lane;
+      active = cand < P.n;
+      ev_init(s, P, active ? __ldg(P.hdr + cand) : 0ull);
+    }
+    mbar_wait(smem_addr(&s_ring_bar[warp][slot]), phase);
+    const uint32_t ch0 = kSlotChunks * g, nc = min((uint32_t)kSlotChunks, nch - ch0);
+    uint32_t addr = ring_lane + slot * kSlotBytes;
+    if (g == 0) {
+      // seed the previous word so that op 0 always shows a tp difference (an event)
+      const uint32_t w0 = lds32(addr);
+      pw = ((w0 & 0xffu) ^ 0x02u) << 24;
+      s.head0 = w0 & 1u;
+    }
+#pragma unroll 1
+    for (uint32_t c = 0; c < nc; ++c, addr += 512u) {
+      const uint32_t ch = ch0 + c;
+      uint4 w4 = lds128(addr);
+      if (ch == nch - 1u && nvl < 16u) w4 = pad_tail(w4, nvl);
+      // The lists must hold what a step adds: a whole chunk (<= 16 events, <= its heads
+      // snapshots), or — when a chunk has more heads than snapshot slots in some lane —
+      // one quad per step (<= 4 events, <= 4 snapshots).
+      const bool careful = __any_sync(0xffffffffu, chunk_heads(w4) > (uint32_t)kSnCap);
+      uint32_t todo = 0xfu;
+#pragma unroll 1
+      do {
+        const uint32_t now = careful ? (todo & (0u - todo)) : todo;
+        uint32_t heads, evmax;
+        if (careful) {
+          const uint32_t wq = now == 1u ? w4.x : now == 2u ? w4.y : now == 4u ? w4.z : w4.w;
+          heads = __popc(wq & 0x01010101u);
+          evmax = 4u;
+        } else {
+          heads = chunk_heads(w4);
+          evmax = 16u;
+        }
+        const bool full_soon = s.ec + evmax > (uint32_t)kEvCap || s.sc + heads > (uint32_t)kSnCap;
+        if (__any_sync(0xffffffffu, full_soon)) ev_drain<MODE>(s, P, l, cand, active);
+        ev_chunk<MODE>(s, P, l, w4, pw, ch, qo, now);
+        todo &= ~now;
+      } while (todo);
+      pw = w4.w;
+    }
+    __syncwarp();
+    if (lane == 0 && u + kEvRingSlots < units) {
+      fence_proxy_async();
+      issue_next(slot);
+    }
+    if (++slot == kEvRingSlots) {
+      slot = 0;
+      phase ^= 1u;
+    }
+    if (++g == ngroups) {
+      // ---- tile epilogue: drain, close the last run and stage (no p2p_fwd) ----
+      ev_drain<MODE>(s, P, l, cand, active);
+      ev_close_run<MODE>(s, P, (uint32_t)P.L);
+      s.S += s.rS;
+      s.A -= s.rA;
+      s.E = max(s.E, s.rE);
+      if (MODE & kFull) s.comp += s.rC;
+      stage_commit<MODE>(s, P, cand, active, false);
+      finish_cand<MODE>(s, P, cand, active, best_ck, best_idx);
+      g = 0;
+      tile += tile_stride;
+    }
+  }
+
+  if (MODE & kSelect)
+    block_select_finish(best_ck, best_idx, P.sel, P.n_total, P.ib, s_ck, s_idx);
+}
+
+}  // namespace aceso

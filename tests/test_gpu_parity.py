@@ -234,12 +234,14 @@ def test_random_bytes_never_crash_and_match():
 
 
 # ---------------------------------------------------------------------------
-# both work decompositions (one warp per tile / forward+reverse warp pair)
+# every kernel variant: event kernel (default), quad kernel with one warp per tile or a
+# forward+reverse warp pair; 2 or 3 resident CTAs per SM
 # ---------------------------------------------------------------------------
 @pytest.mark.parametrize("minb", ["2", "3"])
-@pytest.mark.parametrize("split", ["1", "2"])
-@pytest.mark.parametrize("name", ["gpt3-1.3b", "t5", "wrn", "gpt3-13b"])
-def test_split_modes_parity(split, minb, name, monkeypatch):
+@pytest.mark.parametrize("kernel,split", [("events", "1"), ("quad", "1"), ("quad", "2")])
+@pytest.mark.parametrize("name", ["gpt3-1.3b", "t5", "wrn", "gpt3-13b", "toy-a"])
+def test_kernel_variants_parity(kernel, split, minb, name, monkeypatch):
+    monkeypatch.setenv("ACESO_KERNEL", kernel)
     monkeypatch.setenv("ACESO_SPLIT", split)
     monkeypatch.setenv("ACESO_MINB", minb)
     prof = P.WORKLOADS[name]()
