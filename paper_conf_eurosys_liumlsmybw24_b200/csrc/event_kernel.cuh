@@ -30,12 +30,14 @@
 
 namespace aceso {
 
-constexpr int kEvCap = 24;      // events per lane between drains (a chunk adds <= 16)
-constexpr int kSnCap = 4;       // recompute snapshots per lane between drains (a quad adds <= 4)
-constexpr int kEvRingSlots = 3; // per-warp ring depth (1 KB slots)
+constexpr int kEvCap = 32;        // events per lane between drains (a chunk adds <= 16)
+constexpr int kSnCap = 4;         // recompute snapshots per lane between drains (a quad adds <= 4)
+constexpr int kEvRingSlots = 2;   // per-warp ring depth
+constexpr int kEvSlotChunks = 4;  // 16-op chunks per ring slot (2 KB)
+constexpr int kEvSlotBytes = kEvSlotChunks * 512;
 
-__host__ __device__ constexpr uint32_t ev_ring_bytes() { return (uint32_t)kWarps * kEvRingSlots * kSlotBytes; }
-__host__ __device__ constexpr uint32_t ev_list_bytes() { return (uint32_t)kWarps * kEvCap * 32 * 4; }
+__host__ __device__ constexpr uint32_t ev_ring_bytes() { return (uint32_t)kWarps * kEvRingSlots * kEvSlotBytes; }
+__host__ __device__ constexpr uint32_t ev_list_bytes() { return (uint32_t)kWarps * kEvCap * 32 * 2; }
 __host__ __device__ constexpr uint32_t ev_snap_bytes(bool full) {
   return (uint32_t)kWarps * kSnCap * 32 * (full ? 28u : 20u);
 }
@@ -48,6 +50,9 @@ __device__ __forceinline__ void sts32(uint32_t a, uint32_t v) {
 }
 __device__ __forceinline__ void sts64(uint32_t a, uint64_t v) {
   asm volatile("st.shared.u64 [%0], %1;" ::"r"(a), "l"(v) : "memory");
+}
+__device__ __forceinline__ void sts16(uint32_t a, uint32_t v) {
+  asm volatile("st.shared.u16 [%0], %1;" ::"r"(a), "h"((uint16_t)v) : "memory");
 }
 __device__ __forceinline__ uint64_t lds64u(uint32_t a) {
   uint64_t v;
@@ -73,7 +78,7 @@ struct EvCand {
 
 // per-lane shared-memory addresses of the lists
 struct EvLists {
-  uint32_t ev;          // event k at ev + 128 k (u32: op | code << 16 | snapshot << 24)
+  uint32_t ev;          // event k at ev + 64 k (u16: op | snapshot << 15)
   uint32_t sS, sA, sC;  // snapshot k at +256 k (u64)
   uint32_t sE;          // snapshot k at +128 k (u32)
 };
@@ -153,7 +158,7 @@ __device__ __forceinline__ void ev_quad(EvCand &s, const EvalParams &P, const Ev
       const uint32_t k = __ffs(evb) - 1u;
       evb &= evb - 1u;
       c = (w >> (8u * k)) & 0xffu;
-      sts32(l.ev + 128u * s.ec, (qg * 4u + k) | (c << 16));
+      sts16(l.ev + 64u * s.ec, qg * 4u + k);
       s.ec += 1;
     } while (evb);
     s.rrA = ev_run(c, s.mbs, P);
@@ -180,9 +185,9 @@ __device__ __forceinline__ void ev_quad(EvCand &s, const EvalParams &P, const Ev
       s.rS = s.rA = s.rC = 0;
       s.rE = 0;
       s.rany = 0;
-      flag = 1u << 24;
+      flag = 1u << 15;
     }
-    sts32(l.ev + 128u * s.ec, (qg * 4u + k) | (c << 16) | flag);
+    sts16(l.ev + 64u * s.ec, (qg * 4u + k) | flag);
     s.ec += 1;
     rrs = ev_run(c, s.mbs, P);
     start = k;
@@ -222,8 +227,10 @@ __device__ __forceinline__ void ev_close_run(EvCand &s, const EvalParams &P, uin
 // phase B: one event (op j with code c opens a run; a head also closes a stage)
 template <uint32_t MODE>
 __device__ __forceinline__ void ev_handle(EvCand &s, const EvalParams &P, const EvLists &l,
-                                          uint32_t ent, int64_t cand, bool active) {
-  const uint32_t j = ent & 0xffffu, c = (ent >> 16) & 0xffu;
+                                          uint32_t ent, const unsigned char *cb, int64_t cand,
+                                          bool active) {
+  const uint32_t j = ent & 0x7fffu;
+  const uint32_t c = __ldg(cb + (j >> 4) * 512u + (j & 15u));  // the op's code (L2: just streamed)
   const uint32_t head = c & 1u;
   const uint32_t Lp1 = (uint32_t)P.L + 1u;
   const uint32_t *kx = reinterpret_cast<const uint32_t *>(P.kx);
@@ -231,7 +238,7 @@ __device__ __forceinline__ void ev_handle(EvCand &s, const EvalParams &P, const 
     ev_close_run<MODE>(s, P, j);
     if (head) {
       s.S += __ldg(kx + 4 * ((size_t)s.rr * Lp1 + j) + 2);  // R5: p2p_fwd of the stage's last op
-      if (ent >> 24) {                                       // recompute deltas of this stage
+      if (ent >> 15) {                                       // recompute deltas of this stage
         s.S += lds64u(l.sS + 256u * s.sp);
         s.A -= lds64u(l.sA + 256u * s.sp);
         s.E = max(s.E, lds32(l.sE + 128u * s.sp));
@@ -275,32 +282,28 @@ __device__ __forceinline__ void ev_handle(EvCand &s, const EvalParams &P, const 
 // phase B over every lane's list (warp-uniform call)
 template <uint32_t MODE>
 __device__ __forceinline__ void ev_drain(EvCand &s, const EvalParams &P, const EvLists &l,
-                                         int64_t cand, bool active) {
+                                         const unsigned char *cb, int64_t cand, bool active) {
   const uint32_t mx = __reduce_max_sync(0xffffffffu, s.ec);
 #pragma unroll 1
   for (uint32_t k = 0; k < mx; ++k) {
-    if (k < s.ec) ev_handle<MODE>(s, P, l, lds32(l.ev + 128u * k), cand, active);
+    if (k < s.ec) ev_handle<MODE>(s, P, l, lds16(l.ev + 64u * k), cb, cand, active);
   }
   s.ec = s.sc = s.sp = 0;
 }
 
-// phase A over the quads `now` (bit q = quad q) of one 16-op chunk of this lane (w4 =
-// its 16 code bytes, pw = the previous word): activity words of the quads; quads with
-// activity in any lane are visited
-template <uint32_t MODE>
-__device__ __forceinline__ void ev_chunk(EvCand &s, const EvalParams &P, const EvLists &l,
-                                         uint4 w4, uint32_t pw, uint32_t ch, uint32_t qo,
-                                         uint32_t now) {
-  const uint32_t f0 = quad_activity(w4.x, pw), f1 = quad_activity(w4.y, w4.x);
-  const uint32_t f2 = quad_activity(w4.z, w4.y), f3 = quad_activity(w4.w, w4.z);
-  const uint32_t lm = (f0 ? 1u : 0u) | (f1 ? 2u : 0u) | (f2 ? 4u : 0u) | (f3 ? 8u : 0u);
-  const uint32_t slow = __reduce_or_sync(0xffffffffu, lm) & now;  // quads with activity in any lane
-  if (slow == 0u) return;
-  const uint32_t qg = ch * 4u;
-  if (slow & 1u) if (f0) ev_quad<MODE>(s, P, l, w4.x, f0 & 0xefefefefu, f0 & 0x10101010u, qg, lds32(qo + 4u * qg));
-  if (slow & 2u) if (f1) ev_quad<MODE>(s, P, l, w4.y, f1 & 0xefefefefu, f1 & 0x10101010u, qg + 1u, lds32(qo + 4u * qg + 4u));
-  if (slow & 4u) if (f2) ev_quad<MODE>(s, P, l, w4.z, f2 & 0xefefefefu, f2 & 0x10101010u, qg + 2u, lds32(qo + 4u * qg + 8u));
-  if (slow & 8u) if (f3) ev_quad<MODE>(s, P, l, w4.w, f3 & 0xefefefefu, f3 & 0x10101010u, qg + 3u, lds32(qo + 4u * qg + 12u));
+// activity words of a chunk's 4 quads (w4 = its 16 code bytes, pw = the previous word)
+struct ChunkAct {
+  uint32_t f0, f1, f2, f3;
+  __device__ __forceinline__ uint32_t get(uint32_t q) const {
+    return q == 0u ? f0 : q == 1u ? f1 : q == 2u ? f2 : f3;
+  }
+};
+__device__ __forceinline__ ChunkAct chunk_activity(uint4 w4, uint32_t pw) {
+  return {quad_activity(w4.x, pw), quad_activity(w4.y, w4.x), quad_activity(w4.z, w4.y),
+          quad_activity(w4.w, w4.z)};
+}
+__device__ __forceinline__ uint32_t word_of(uint4 w4, uint32_t q) {
+  return q == 0u ? w4.x : q == 1u ? w4.y : q == 2u ? w4.z : w4.w;
 }
 
 // heads in a chunk (upper bound of the snapshots it can push)
@@ -340,10 +343,10 @@ __global__ void __launch_bounds__(kThreads, MINB) event_kernel(const __grid_cons
   const uint32_t sb = smem_addr(sm_raw);
   // layout: [qo][ring][event lists][snapshots S, A, (C), E]
   const uint32_t qo = sb;
-  const uint32_t ring = sb + P.qo_bytes + (uint32_t)warp * kEvRingSlots * kSlotBytes;
+  const uint32_t ring = sb + P.qo_bytes + (uint32_t)warp * kEvRingSlots * kEvSlotBytes;
   const uint32_t lists = sb + P.qo_bytes + ev_ring_bytes();
   EvLists l;
-  l.ev = lists + (uint32_t)warp * kEvCap * 128u + lane * 4u;
+  l.ev = lists + (uint32_t)warp * kEvCap * 64u + lane * 2u;
   const uint32_t snap = lists + ev_list_bytes();
   const uint32_t blk64 = (uint32_t)kWarps * kSnCap * 256u;  // one u64 snapshot field, all warps
   l.sS = snap + (uint32_t)warp * kSnCap * 256u + lane * 8u;
@@ -367,7 +370,7 @@ __global__ void __launch_bounds__(kThreads, MINB) event_kernel(const __grid_cons
   }
 
   const uint32_t nch = (uint32_t)P.nch;
-  const uint32_t ngroups = (nch + kSlotChunks - 1) / kSlotChunks;
+  const uint32_t ngroups = (nch + kEvSlotChunks - 1) / kEvSlotChunks;
   const int64_t first_tile = (int64_t)blockIdx.x * kWarps + warp;
   const int64_t tile_stride = (int64_t)gridDim.x * kWarps;
   const int64_t my_tiles =
@@ -378,10 +381,10 @@ __global__ void __launch_bounds__(kThreads, MINB) event_kernel(const __grid_cons
   int64_t it_tile = first_tile;
   uint32_t it_g = 0;
   auto issue_next = [&](int slot) {
-    const uint32_t a = kSlotChunks * it_g, b = min(a + kSlotChunks, nch);
+    const uint32_t a = kEvSlotChunks * it_g, b = min(a + kEvSlotChunks, nch);
     const uint32_t bar = smem_addr(&s_ring_bar[warp][slot]);
     mbar_expect_tx(bar, (b - a) * 512u);
-    bulk_g2s(ring + slot * kSlotBytes, codes + ((size_t)it_tile * nch + a) * 512, (b - a) * 512u, bar);
+    bulk_g2s(ring + slot * kEvSlotBytes, codes + ((size_t)it_tile * nch + a) * 512, (b - a) * 512u, bar);
     if (++it_g == ngroups) {
       it_g = 0;
       it_tile += tile_stride;
@@ -395,83 +398,107 @@ __global__ void __launch_bounds__(kThreads, MINB) event_kernel(const __grid_cons
 
   const uint32_t nvl = (uint32_t)P.L - 16u * (nch - 1u);  // valid ops of the last chunk
   const uint32_t ring_lane = ring + lane * 16u;
+  const uint32_t bar0 = smem_addr(&s_ring_bar[warp][0]);
 
   uint64_t best_ck = ~0ull;
   int64_t best_idx = INT64_MAX;
   EvCand s;
-  uint32_t pw = 0;
-  int64_t tile = first_tile;
-  uint32_t g = 0;
   int slot = 0;
   uint32_t phase = 0;
-  int64_t cand = 0;
-  bool active = false;
-  for (int64_t u = 0; u < units; ++u) {
-    if (g == 0) {
-      cand = tile * 32 + lane;
-      active = cand < P.n;
-      ev_init(s, P, active ? __ldg(P.hdr + cand) : 0ull);
-    }
-    mbar_wait(smem_addr(&s_ring_bar[warp][slot]), phase);
-    const uint32_t ch0 = kSlotChunks * g, nc = min((uint32_t)kSlotChunks, nch - ch0);
-    uint32_t addr = ring_lane + slot * kSlotBytes;
-    if (g == 0) {
-      // seed the previous word so that op 0 always shows a tp difference (an event)
-      const uint32_t w0 = lds32(addr);
-      pw = ((w0 & 0xffu) ^ 0x02u) << 24;
-      s.head0 = w0 & 1u;
-    }
+  int64_t issued = kEvRingSlots;  // units issued so far (lane 0)
 #pragma unroll 1
-    for (uint32_t c = 0; c < nc; ++c, addr += 512u) {
-      const uint32_t ch = ch0 + c;
-      uint4 w4 = lds128(addr);
-      if (ch == nch - 1u && nvl < 16u) w4 = pad_tail(w4, nvl);
-      // The lists must hold what a step adds: a whole chunk (<= 16 events, <= its heads
-      // snapshots), or — when a chunk has more heads than snapshot slots in some lane —
-      // one quad per step (<= 4 events, <= 4 snapshots).
-      const bool careful = __any_sync(0xffffffffu, chunk_heads(w4) > (uint32_t)kSnCap);
-      uint32_t todo = 0xfu;
+  for (int64_t tile = first_tile; tile < P.n_tiles; tile += tile_stride) {
+    const int64_t cand = tile * 32 + lane;
+    const bool active = cand < P.n;
+    const unsigned char *cb = codes + (size_t)tile * nch * 512 + lane * 16;  // this lane's codes
+    ev_init(s, P, active ? __ldg(P.hdr + cand) : 0ull);
+    uint32_t pw = 0;
 #pragma unroll 1
-      do {
-        const uint32_t now = careful ? (todo & (0u - todo)) : todo;
-        uint32_t heads, evmax;
-        if (careful) {
-          const uint32_t wq = now == 1u ? w4.x : now == 2u ? w4.y : now == 4u ? w4.z : w4.w;
-          heads = __popc(wq & 0x01010101u);
-          evmax = 4u;
-        } else {
-          heads = chunk_heads(w4);
-          evmax = 16u;
+    for (uint32_t g = 0; g < ngroups; ++g) {
+      mbar_wait(bar0 + 8u * slot, phase);
+      const uint32_t ch0 = kEvSlotChunks * g, nc = min((uint32_t)kEvSlotChunks, nch - ch0);
+      uint32_t addr = ring_lane + slot * kEvSlotBytes;
+      if (g == 0) {
+        // seed the previous word so that op 0 always shows a tp difference (an event)
+        const uint32_t w0 = lds32(addr);
+        pw = ((w0 & 0xffu) ^ 0x02u) << 24;
+        s.head0 = w0 & 1u;
+      }
+      if (g == ngroups - 1u && nvl < 16u) {
+        // ops >= L of the last chunk (zero padding) take the last op's tp/dp without head
+        // or recompute: no events, no deltas (patched in this lane's ring copy)
+        const uint32_t la = addr + (nc - 1u) * 512u;
+        const uint4 t = pad_tail(lds128(la), nvl);
+        asm volatile("st.shared.v4.u32 [%0], {%1, %2, %3, %4};" ::"r"(la), "r"(t.x), "r"(t.y), "r"(t.z),
+                     "r"(t.w) : "memory");
+      }
+#pragma unroll 1
+      for (uint32_t c = 0; c < nc; ++c, addr += 512u) {
+        const uint32_t qg = (ch0 + c) * 4u;
+        const uint4 w4 = lds128(addr);
+        const ChunkAct fa = chunk_activity(w4, pw);
+        pw = w4.w;
+        const uint32_t lm = (fa.f0 ? 1u : 0u) | (fa.f1 ? 2u : 0u) | (fa.f2 ? 4u : 0u) | (fa.f3 ? 8u : 0u);
+        // The lists must hold what the chunk adds (<= 16 events, <= its heads snapshots);
+        // a chunk with more heads than snapshot slots in some lane goes quad by quad.
+        const uint32_t h = chunk_heads(w4);
+        const uint32_t rare = (h > (uint32_t)kSnCap ? 0x20u : 0u) |
+                              ((s.ec + 16u > (uint32_t)kEvCap || s.sc + h > (uint32_t)kSnCap) ? 0x10u : 0u);
+        const uint32_t v = __reduce_or_sync(0xffffffffu, lm | rare);
+        if (v & 0x30u) {
+          // rare path: drain first; quad by quad when careful
+          uint32_t todo = v & 0xfu;
+          const bool careful = (v & 0x20u) != 0u;
+#pragma unroll 1
+          do {
+            const bool one = careful && todo != 0u;
+            const uint32_t q = one ? __ffs(todo) - 1u : 0u;
+            const uint32_t heads = one ? __popc(word_of(w4, q) & 0x01010101u) : h;
+            const uint32_t evmax = one ? 4u : 16u;
+            const bool full_soon = s.ec + evmax > (uint32_t)kEvCap || s.sc + heads > (uint32_t)kSnCap;
+            if (__any_sync(0xffffffffu, full_soon)) ev_drain<MODE>(s, P, l, cb, cand, active);
+            const uint32_t now = one ? (1u << q) : todo;
+#pragma unroll 1
+            for (uint32_t t = now; t; t &= t - 1u) {
+              const uint32_t qq = __ffs(t) - 1u;
+              const uint32_t f = fa.get(qq);
+              if (f)
+                ev_quad<MODE>(s, P, l, word_of(w4, qq), f & 0xefefefefu, f & 0x10101010u, qg + qq,
+                              lds32(qo + 4u * (qg + qq)));
+            }
+            todo &= ~now;
+          } while (todo);
+        } else if (v) {
+          if ((v & 1u) && fa.f0)
+            ev_quad<MODE>(s, P, l, w4.x, fa.f0 & 0xefefefefu, fa.f0 & 0x10101010u, qg, lds32(qo + 4u * qg));
+          if ((v & 2u) && fa.f1)
+            ev_quad<MODE>(s, P, l, w4.y, fa.f1 & 0xefefefefu, fa.f1 & 0x10101010u, qg + 1u, lds32(qo + 4u * qg + 4u));
+          if ((v & 4u) && fa.f2)
+            ev_quad<MODE>(s, P, l, w4.z, fa.f2 & 0xefefefefu, fa.f2 & 0x10101010u, qg + 2u, lds32(qo + 4u * qg + 8u));
+          if ((v & 8u) && fa.f3)
+            ev_quad<MODE>(s, P, l, w4.w, fa.f3 & 0xefefefefu, fa.f3 & 0x10101010u, qg + 3u, lds32(qo + 4u * qg + 12u));
         }
-        const bool full_soon = s.ec + evmax > (uint32_t)kEvCap || s.sc + heads > (uint32_t)kSnCap;
-        if (__any_sync(0xffffffffu, full_soon)) ev_drain<MODE>(s, P, l, cand, active);
-        ev_chunk<MODE>(s, P, l, w4, pw, ch, qo, now);
-        todo &= ~now;
-      } while (todo);
-      pw = w4.w;
+      }
+      __syncwarp();
+      if (lane == 0 && issued < units) {
+        fence_proxy_async();
+        issue_next(slot);
+        issued += 1;
+      }
+      if (++slot == kEvRingSlots) {
+        slot = 0;
+        phase ^= 1u;
+      }
     }
-    __syncwarp();
-    if (lane == 0 && u + kEvRingSlots < units) {
-      fence_proxy_async();
-      issue_next(slot);
-    }
-    if (++slot == kEvRingSlots) {
-      slot = 0;
-      phase ^= 1u;
-    }
-    if (++g == ngroups) {
-      // ---- tile epilogue: drain, close the last run and stage (no p2p_fwd) ----
-      ev_drain<MODE>(s, P, l, cand, active);
-      ev_close_run<MODE>(s, P, (uint32_t)P.L);
-      s.S += s.rS;
-      s.A -= s.rA;
-      s.E = max(s.E, s.rE);
-      if (MODE & kFull) s.comp += s.rC;
-      stage_commit<MODE>(s, P, cand, active, false);
-      finish_cand<MODE>(s, P, cand, active, best_ck, best_idx);
-      g = 0;
-      tile += tile_stride;
-    }
+    // ---- tile epilogue: drain, close the last run and stage (no p2p_fwd) ----
+    ev_drain<MODE>(s, P, l, cb, cand, active);
+    ev_close_run<MODE>(s, P, (uint32_t)P.L);
+    s.S += s.rS;
+    s.A -= s.rA;
+    s.E = max(s.E, s.rE);
+    if (MODE & kFull) s.comp += s.rC;
+    stage_commit<MODE>(s, P, cand, active, false);
+    finish_cand<MODE>(s, P, cand, active, best_ck, best_idx);
   }
 
   if (MODE & kSelect)
