@@ -520,7 +520,7 @@ size_t aceso_select_buf_bytes(const aceso_ctx *ctx, int64_t n) {
   if (!ctx) return 0;
   int m = 0;
   for (int k = 1; k < 8; ++k) m = std::max(m, ctx->max_ctas[k]);
-  m = std::max(m, 4 * ctx->sms);  // select kernel grid
+  m = std::max(m, 4 * ctx->sms);  // per-CTA partials of the eval kernels; select kernel grid
   return (size_t)kSelPartialOff + 16 * (size_t)m;
 }
 

@@ -170,4 +170,78 @@ __device__ __forceinline__ void block_select_finish(uint64_t ck, int64_t idx, un
   }
 }
 
+// Argmin with grid-level completion and no CTA barrier: every warp leaves its partial in
+// shared memory; the last warp of a CTA to finish (shared counter, zeroed at kernel start)
+// reduces the CTA's partials and publishes the CTA partial; the last CTA to publish
+// (global counter) reduces all CTA partials and writes the final result. Warps that
+// finish early exit without waiting for the rest of their CTA. Called by all 32 lanes of
+// every warp of the grid.
+__device__ __forceinline__ void warp_select_finish(uint64_t ck, int64_t idx, unsigned char *sel,
+                                                   int64_t n_total, uint32_t ib, uint64_t *s_ck,
+                                                   int64_t *s_idx, unsigned int *s_cnt) {
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const uint32_t wpb = blockDim.x >> 5;
+  warp_argmin(ck, idx);
+  uint32_t last = 0;
+  if (lane == 0) {
+    s_ck[warp] = ck;
+    s_idx[warp] = idx;
+    __threadfence_block();
+    last = atomicAdd(s_cnt, 1u) == wpb - 1 ? 1u : 0u;
+  }
+  if (!__shfl_sync(0xffffffffu, last, 0)) return;
+  __threadfence_block();
+  ck = lane < (int)wpb ? ((volatile uint64_t *)s_ck)[lane] : ~0ull;
+  idx = lane < (int)wpb ? ((volatile int64_t *)s_idx)[lane] : INT64_MAX;
+  warp_argmin(ck, idx);
+  last = 0;
+  if (lane == 0) {
+    uint64_t *part = reinterpret_cast<uint64_t *>(sel + kSelPartialOff) + 2 * blockIdx.x;
+    part[0] = ck;
+    part[1] = (uint64_t)idx;
+    __threadfence();
+    unsigned int *cnt = reinterpret_cast<unsigned int *>(sel + kSelCounterOff);
+    last = atomicAdd(cnt, 1u) == gridDim.x - 1 ? 1u : 0u;
+  }
+  if (!__shfl_sync(0xffffffffu, last, 0)) return;
+  __threadfence();
+  const uint64_t *parts = reinterpret_cast<const uint64_t *>(sel + kSelPartialOff);
+  ck = ~0ull;
+  idx = INT64_MAX;
+  for (uint32_t b0 = 0; b0 < gridDim.x; b0 += 32 * 8) {
+    uint64_t c2[8];
+    int64_t i2[8];
+#pragma unroll
+    for (int k = 0; k < 8; ++k) {  // 8 independent loads in flight per lane
+      const uint32_t b = b0 + k * 32 + lane;
+      c2[k] = b < gridDim.x ? __ldcg(parts + 2 * b) : ~0ull;
+      i2[k] = b < gridDim.x ? (int64_t)__ldcg(parts + 2 * b + 1) : INT64_MAX;
+    }
+#pragma unroll
+    for (int k = 0; k < 8; ++k)
+      if (key_less(c2[k], i2[k], ck, idx)) {
+        ck = c2[k];
+        idx = i2[k];
+      }
+  }
+  warp_argmin(ck, idx);
+  if (lane == 0) {
+    aceso_select_result *res = reinterpret_cast<aceso_select_result *>(sel);
+    if (ck == ~0ull) {
+      res->key = INT64_MAX;
+      res->cls_cost = ~0ull;
+      res->index = -1;
+    } else {
+      const uint64_t cls = ck >> 62, cost = ck & ((1ull << 62) - 1);
+      const uint64_t cmax = (1ull << (62 - ib)) - 1;
+      const uint64_t c = cost < cmax ? cost : cmax;
+      res->key = (int64_t)((cls << 62) | (c << ib) | (uint64_t)idx);
+      res->cls_cost = ck;
+      res->index = idx;
+    }
+    res->reserved = 0;
+    *reinterpret_cast<unsigned int *>(sel + kSelCounterOff) = 0;  // reusable
+  }
+}
+
 }  // namespace aceso

@@ -68,20 +68,36 @@ struct EvCand {
   // phase A: recompute deltas since the last stage head
   uint64_t rS, rA, rC;
   uint32_t rE, rany;
-  uint32_t rrA;        // phase A's current run (b, tp) index
-  uint32_t ec, sc, sp; // events listed, snapshots pushed, snapshots popped
+  uint32_t cA;         // phase A: code of the last listed event (its run is the current one)
+  uint32_t ec, sc, sp; // list entries, snapshots pushed, snapshots popped
+  uint32_t sfl;        // bit k: list entry k (a single event, a head) takes the next snapshot
   // candidate-level aggregates (names shared with Cand: stage_commit / finish_cand)
   uint64_t sumS, bestT, bestM;
   uint32_t bt, bm, oom, i, gsum, reasons, nheads, head0, gst;
   uint32_t mbs, p, N;
 };
 
-// per-lane shared-memory addresses of the lists
-struct EvLists {
-  uint32_t ev;          // event k at ev + 64 k (u16: op | snapshot << 15)
-  uint32_t sS, sA, sC;  // snapshot k at +256 k (u64)
-  uint32_t sE;          // snapshot k at +128 k (u32)
+// Dynamic shared memory: [qo][ring][event lists][snapshots S, A, (C), E]. The event list
+// of a lane holds u16 entries (quad << 4 | mask of its events) at ev_base + 64 k; snapshot k of a lane
+// is in per-field arrays (u64 S/A/C at +256 k, u32 E at +128 k).
+struct EvSnap {
+  uint32_t S, A, C, E;
 };
+// shared-memory address of the snapshot block (set once per CTA; read on the rare
+// snapshot paths only, so the address does not occupy a register in the main loop)
+__shared__ uint32_t ev_snap_base;
+template <uint32_t MODE>
+__device__ __forceinline__ EvSnap ev_snap_addr(uint32_t k) {
+  const uint32_t lane = threadIdx.x & 31u, warp = threadIdx.x >> 5;
+  const uint32_t snap = *(volatile uint32_t *)&ev_snap_base;
+  const uint32_t blk64 = (uint32_t)kWarps * kSnCap * 256u;
+  EvSnap a;
+  a.S = snap + warp * kSnCap * 256u + lane * 8u + 256u * k;
+  a.A = a.S + blk64;
+  a.C = a.A + blk64;
+  a.E = snap + ((MODE & kFull) ? 3u : 2u) * blk64 + warp * kSnCap * 128u + lane * 4u + 128u * k;
+  return a;
+}
 
 __device__ __forceinline__ void ev_init(EvCand &s, const EvalParams &P, uint64_t h) {
   s.mbs = (uint32_t)(h & 0xff);
@@ -98,8 +114,9 @@ __device__ __forceinline__ void ev_init(EvCand &s, const EvalParams &P, uint64_t
   s.rr = s.dd = s.a = 0;
   s.rS = s.rA = s.rC = 0;
   s.rE = s.rany = 0;
-  s.rrA = 0;
+  s.cA = 0;
   s.ec = s.sc = s.sp = 0;
+  s.sfl = 0;
   s.sumS = s.bestT = s.bestM = 0;
   s.bt = s.bm = 0;
   s.oom = s.gsum = s.nheads = s.head0 = s.gst = 0;
@@ -143,56 +160,49 @@ __device__ __forceinline__ uint32_t quad_nonzero(uint32_t v) {
 // one run); each event is listed, a stage head first moving the deltas accumulated so
 // far to a snapshot
 template <uint32_t MODE>
-__device__ __forceinline__ void ev_quad(EvCand &s, const EvalParams &P, const EvLists &l,
+__device__ __forceinline__ void ev_quad(EvCand &s, const EvalParams &P, uint32_t lev,
                                         uint32_t w, uint32_t x, uint32_t m, uint32_t qg,
                                         uint32_t qsb) {
   if (x == 0u) {  // recompute flags only: one pattern lookup under the current run
-    ev_rc_add<MODE>(s, P, qsb, s.rrA, quad_bits(m, 4));
+    ev_rc_add<MODE>(s, P, qsb, ev_run(s.cA, s.mbs, P), quad_bits(m, 4));
     return;
   }
   uint32_t evb = quad_nonzero(x);
   if (m == 0u && !(s.rany && (x & 0x01010101u))) {  // events only, no snapshot needed
-    uint32_t c = 0;
-#pragma unroll 1
-    do {
-      const uint32_t k = __ffs(evb) - 1u;
-      evb &= evb - 1u;
-      c = (w >> (8u * k)) & 0xffu;
-      sts16(l.ev + 64u * s.ec, qg * 4u + k);
-      s.ec += 1;
-    } while (evb);
-    s.rrA = ev_run(c, s.mbs, P);
+    sts16(lev + 64u * s.ec, (qg << 4) | evb);  // one entry: the quad and its events
+    s.ec += 1;
+    s.cA = (w >> (8u * (31u - __clz(evb)))) & 0xffu;
     return;
   }
   const uint32_t pat = quad_bits(m, 4);
   evb |= 0x10u;  // + a virtual end of the quad at op 4
-  uint32_t start = 0, rrs = s.rrA;
+  uint32_t start = 0, cs = s.cA;
 #pragma unroll 1
   while (true) {
     const uint32_t k = __ffs(evb) - 1u;
     evb &= evb - 1u;
     const uint32_t segp = pat & ((1u << k) - 1u) & ~((1u << start) - 1u);  // ops [start, k)
-    if (segp) ev_rc_add<MODE>(s, P, qsb, rrs, segp);
+    if (segp) ev_rc_add<MODE>(s, P, qsb, ev_run(cs, s.mbs, P), segp);
     if (k == 4u) break;
     const uint32_t c = (w >> (8u * k)) & 0xffu;
-    uint32_t flag = 0;
     if ((c & 1u) && s.rany) {  // head: recompute deltas of the stage it closes
-      sts64(l.sS + 256u * s.sc, s.rS);
-      sts64(l.sA + 256u * s.sc, s.rA);
-      sts32(l.sE + 128u * s.sc, s.rE);
-      if (MODE & kFull) sts64(l.sC + 256u * s.sc, s.rC);
+      const EvSnap a = ev_snap_addr<MODE>(s.sc);
+      sts64(a.S, s.rS);
+      sts64(a.A, s.rA);
+      sts32(a.E, s.rE);
+      if (MODE & kFull) sts64(a.C, s.rC);
       s.sc += 1;
       s.rS = s.rA = s.rC = 0;
       s.rE = 0;
       s.rany = 0;
-      flag = 1u << 15;
+      s.sfl |= 1u << s.ec;
     }
-    sts16(l.ev + 64u * s.ec, (qg * 4u + k) | flag);
+    sts16(lev + 64u * s.ec, (qg << 4) | (1u << k));
     s.ec += 1;
-    rrs = ev_run(c, s.mbs, P);
+    cs = c;
     start = k;
   }
-  s.rrA = rrs;
+  s.cA = cs;
 }
 
 // activity word of a quad: bit 4 of a byte = recompute flag, other bits = event (head or
@@ -226,10 +236,9 @@ __device__ __forceinline__ void ev_close_run(EvCand &s, const EvalParams &P, uin
 
 // phase B: one event (op j with code c opens a run; a head also closes a stage)
 template <uint32_t MODE>
-__device__ __forceinline__ void ev_handle(EvCand &s, const EvalParams &P, const EvLists &l,
-                                          uint32_t ent, const unsigned char *cb, int64_t cand,
+__device__ __forceinline__ void ev_handle(EvCand &s, const EvalParams &P, uint32_t j,
+                                          uint32_t snapf, const unsigned char *cb, int64_t cand,
                                           bool active) {
-  const uint32_t j = ent & 0x7fffu;
   const uint32_t c = __ldg(cb + (j >> 4) * 512u + (j & 15u));  // the op's code (L2: just streamed)
   const uint32_t head = c & 1u;
   const uint32_t Lp1 = (uint32_t)P.L + 1u;
@@ -238,11 +247,12 @@ __device__ __forceinline__ void ev_handle(EvCand &s, const EvalParams &P, const 
     ev_close_run<MODE>(s, P, j);
     if (head) {
       s.S += __ldg(kx + 4 * ((size_t)s.rr * Lp1 + j) + 2);  // R5: p2p_fwd of the stage's last op
-      if (ent >> 15) {                                       // recompute deltas of this stage
-        s.S += lds64u(l.sS + 256u * s.sp);
-        s.A -= lds64u(l.sA + 256u * s.sp);
-        s.E = max(s.E, lds32(l.sE + 128u * s.sp));
-        if (MODE & kFull) s.comp += lds64u(l.sC + 256u * s.sp);
+      if (snapf) {                                           // recompute deltas of this stage
+        const EvSnap a = ev_snap_addr<MODE>(s.sp);
+        s.S += lds64u(a.S);
+        s.A -= lds64u(a.A);
+        s.E = max(s.E, lds32(a.E));
+        if (MODE & kFull) s.comp += lds64u(a.C);
         s.sp += 1;
       }
       stage_commit<MODE>(s, P, cand, active, false);
@@ -281,14 +291,25 @@ __device__ __forceinline__ void ev_handle(EvCand &s, const EvalParams &P, const 
 
 // phase B over every lane's list (warp-uniform call)
 template <uint32_t MODE>
-__device__ __forceinline__ void ev_drain(EvCand &s, const EvalParams &P, const EvLists &l,
+__device__ __forceinline__ void ev_drain(EvCand &s, const EvalParams &P, uint32_t lev,
                                          const unsigned char *cb, int64_t cand, bool active) {
   const uint32_t mx = __reduce_max_sync(0xffffffffu, s.ec);
 #pragma unroll 1
   for (uint32_t k = 0; k < mx; ++k) {
-    if (k < s.ec) ev_handle<MODE>(s, P, l, lds16(l.ev + 64u * k), cb, cand, active);
+    if (k < s.ec) {
+      const uint32_t ent = lds16(lev + 64u * k);  // quad << 4 | event mask
+      const uint32_t snapf = (s.sfl >> k) & 1u;
+      uint32_t m = ent & 0xfu;
+#pragma unroll 1
+      do {
+        const uint32_t b = __ffs(m) - 1u;
+        m &= m - 1u;
+        ev_handle<MODE>(s, P, (ent >> 4) * 4u + b, snapf, cb, cand, active);
+      } while (m);
+    }
   }
   s.ec = s.sc = s.sp = 0;
+  s.sfl = 0;
 }
 
 // activity words of a chunk's 4 quads (w4 = its 16 code bytes, pw = the previous word)
@@ -338,6 +359,7 @@ __global__ void __launch_bounds__(kThreads, MINB) event_kernel(const __grid_cons
   __shared__ __align__(8) uint64_t s_ring_bar[kWarps][kEvRingSlots];
   __shared__ uint64_t s_ck[kWarps];
   __shared__ int64_t s_idx[kWarps];
+  __shared__ unsigned int s_done;  // warps of this CTA past the tile loop
 
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   const uint32_t sb = smem_addr(sm_raw);
@@ -345,18 +367,13 @@ __global__ void __launch_bounds__(kThreads, MINB) event_kernel(const __grid_cons
   const uint32_t qo = sb;
   const uint32_t ring = sb + P.qo_bytes + (uint32_t)warp * kEvRingSlots * kEvSlotBytes;
   const uint32_t lists = sb + P.qo_bytes + ev_ring_bytes();
-  EvLists l;
-  l.ev = lists + (uint32_t)warp * kEvCap * 64u + lane * 2u;
-  const uint32_t snap = lists + ev_list_bytes();
-  const uint32_t blk64 = (uint32_t)kWarps * kSnCap * 256u;  // one u64 snapshot field, all warps
-  l.sS = snap + (uint32_t)warp * kSnCap * 256u + lane * 8u;
-  l.sA = l.sS + blk64;
-  l.sC = l.sA + blk64;
-  l.sE = snap + ((MODE & kFull) ? 3u : 2u) * blk64 + (uint32_t)warp * kSnCap * 128u + lane * 4u;
+  const uint32_t lev = lists + (uint32_t)warp * kEvCap * 64u + lane * 2u;  // this lane's event list
+  if (threadIdx.x == 0) ev_snap_base = lists + ev_list_bytes();
 
   if (threadIdx.x == 0) {
     mbar_init(smem_addr(&s_tbar), 1);
     fence_barrier_init();
+    s_done = 0;
   }
   if (lane == 0) {
     for (int k = 0; k < kEvRingSlots; ++k) mbar_init(smem_addr(&s_ring_bar[warp][k]), 1);
@@ -456,27 +473,27 @@ __global__ void __launch_bounds__(kThreads, MINB) event_kernel(const __grid_cons
             const uint32_t heads = one ? __popc(word_of(w4, q) & 0x01010101u) : h;
             const uint32_t evmax = one ? 4u : 16u;
             const bool full_soon = s.ec + evmax > (uint32_t)kEvCap || s.sc + heads > (uint32_t)kSnCap;
-            if (__any_sync(0xffffffffu, full_soon)) ev_drain<MODE>(s, P, l, cb, cand, active);
+            if (__any_sync(0xffffffffu, full_soon)) ev_drain<MODE>(s, P, lev, cb, cand, active);
             const uint32_t now = one ? (1u << q) : todo;
 #pragma unroll 1
             for (uint32_t t = now; t; t &= t - 1u) {
               const uint32_t qq = __ffs(t) - 1u;
               const uint32_t f = fa.get(qq);
               if (f)
-                ev_quad<MODE>(s, P, l, word_of(w4, qq), f & 0xefefefefu, f & 0x10101010u, qg + qq,
+                ev_quad<MODE>(s, P, lev, word_of(w4, qq), f & 0xefefefefu, f & 0x10101010u, qg + qq,
                               lds32(qo + 4u * (qg + qq)));
             }
             todo &= ~now;
           } while (todo);
         } else if (v) {
           if ((v & 1u) && fa.f0)
-            ev_quad<MODE>(s, P, l, w4.x, fa.f0 & 0xefefefefu, fa.f0 & 0x10101010u, qg, lds32(qo + 4u * qg));
+            ev_quad<MODE>(s, P, lev, w4.x, fa.f0 & 0xefefefefu, fa.f0 & 0x10101010u, qg, lds32(qo + 4u * qg));
           if ((v & 2u) && fa.f1)
-            ev_quad<MODE>(s, P, l, w4.y, fa.f1 & 0xefefefefu, fa.f1 & 0x10101010u, qg + 1u, lds32(qo + 4u * qg + 4u));
+            ev_quad<MODE>(s, P, lev, w4.y, fa.f1 & 0xefefefefu, fa.f1 & 0x10101010u, qg + 1u, lds32(qo + 4u * qg + 4u));
           if ((v & 4u) && fa.f2)
-            ev_quad<MODE>(s, P, l, w4.z, fa.f2 & 0xefefefefu, fa.f2 & 0x10101010u, qg + 2u, lds32(qo + 4u * qg + 8u));
+            ev_quad<MODE>(s, P, lev, w4.z, fa.f2 & 0xefefefefu, fa.f2 & 0x10101010u, qg + 2u, lds32(qo + 4u * qg + 8u));
           if ((v & 8u) && fa.f3)
-            ev_quad<MODE>(s, P, l, w4.w, fa.f3 & 0xefefefefu, fa.f3 & 0x10101010u, qg + 3u, lds32(qo + 4u * qg + 12u));
+            ev_quad<MODE>(s, P, lev, w4.w, fa.f3 & 0xefefefefu, fa.f3 & 0x10101010u, qg + 3u, lds32(qo + 4u * qg + 12u));
         }
       }
       __syncwarp();
@@ -491,7 +508,7 @@ __global__ void __launch_bounds__(kThreads, MINB) event_kernel(const __grid_cons
       }
     }
     // ---- tile epilogue: drain, close the last run and stage (no p2p_fwd) ----
-    ev_drain<MODE>(s, P, l, cb, cand, active);
+    ev_drain<MODE>(s, P, lev, cb, cand, active);
     ev_close_run<MODE>(s, P, (uint32_t)P.L);
     s.S += s.rS;
     s.A -= s.rA;
@@ -501,8 +518,7 @@ __global__ void __launch_bounds__(kThreads, MINB) event_kernel(const __grid_cons
     finish_cand<MODE>(s, P, cand, active, best_ck, best_idx);
   }
 
-  if (MODE & kSelect)
-    block_select_finish(best_ck, best_idx, P.sel, P.n_total, P.ib, s_ck, s_idx);
+  if (MODE & kSelect) warp_select_finish(best_ck, best_idx, P.sel, P.n_total, P.ib, s_ck, s_idx, &s_done);
 }
 
 }  // namespace aceso
