@@ -38,6 +38,8 @@ def parse():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--config", default="gpt3-1.3b")
     ap.add_argument("--dist", default="search", choices=["search", "dense"])
+    ap.add_argument("--no-hint", action="store_true",
+                    help="do not pass ACESO_HINT_DENSE for --dist dense (time the default schedule)")
     ap.add_argument("--batch", type=int, default=65536)
     ap.add_argument("--group", type=int, default=1024, help="candidates sharing a base config")
     ap.add_argument("--no-e2e", action="store_true")
@@ -196,6 +198,9 @@ def run_reference(args):
     return 0
 
 
+HINT = False  # ACESO_HINT_DENSE for every aceso_eval of the run (set in main)
+
+
 def main():
     args = parse()
     if args.impl == "reference":
@@ -223,6 +228,11 @@ def main():
     L = prof.n_ops
     n = args.batch
     ctx = A.Context(prof, local)
+    global HINT
+    HINT = args.dist == "dense" and not args.no_hint
+    env_k = os.environ.get("ACESO_KERNEL")
+    schedule = ("per-op kernel (ACESO_HINT_DENSE)" if HINT else
+                "per-op kernel" if env_k == "quad" or (env_k != "events" and L <= 64) else "event kernel")
 
     # distinct device-resident batches, rotating, together larger than L2
     per_batch = A.tiled_bytes(n, L) + 8 * n
@@ -244,7 +254,7 @@ def main():
         codes_d, hdr_d = dev_batches[b]
         gofs = rank * n
         ctx.eval(codes_d, hdr_d, n=n, global_offset=gofs, n_total=n_total, summary=True, full=False,
-                 select=True, out=out, sel=sels[b], stream=stream)
+                 select=True, out=out, sel=sels[b], stream=stream, dense_hint=HINT)
         if world > 1:
             key = sels[b][0:8].view(torch.int64)
             dist.all_reduce(key, op=dist.ReduceOp.MIN)
@@ -283,7 +293,7 @@ def main():
                 st.wait_event(comm_done.pop(s - nbuf))
             ev_s[s].record(st)
             ctx.eval(codes_d, hdr_d, n=n, global_offset=rank * n, n_total=n_total, summary=True,
-                     select=True, out=outs[s % nstr], sel=sels[b], stream=st)
+                     select=True, out=outs[s % nstr], sel=sels[b], stream=st, dense_hint=HINT)
             ev_k[s].record(st)
             if world > 1:
                 done = torch.cuda.Event()
@@ -339,7 +349,7 @@ def main():
             codes_d, hdr_d = dev_batches[b]
             evs[s].record(cs)
             ctx.eval(codes_d, hdr_d, n=n, global_offset=rank * n, n_total=n_total, summary=True,
-                     select=True, out=out, sel=sels[b], stream=cs)
+                     select=True, out=out, sel=sels[b], stream=cs, dense_hint=HINT)
             eve[s].record(cs)
     g_ser.replay()
     torch.cuda.synchronize()
@@ -367,7 +377,7 @@ def main():
             dc.copy_(c, non_blocking=True)
             dh.copy_(h, non_blocking=True)
             ctx.eval(dc, dh, n=n, global_offset=rank * n, n_total=n_total, summary=True, select=True,
-                     out=out, sel=sel_e, stream=stream)
+                     out=out, sel=sel_e, stream=stream, dense_hint=HINT)
             if world > 1:
                 dist.all_reduce(sel_e[0:8].view(torch.int64), op=dist.ReduceOp.MIN)
             res_host.copy_(sel_e[:32], non_blocking=True)
@@ -412,7 +422,7 @@ def main():
             "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True,
             "scaling": "weak", "vs_baseline": None, "dtype": "u64", "data": "synthetic",
             "config": {"workload": prof.name, "batch_per_gpu": n, "n_ops": L,
-                       "distribution": args.dist, "group_size": args.group,
+                       "distribution": args.dist, "group_size": args.group, "schedule": schedule,
                        "l2": f"{nbuf} distinct device-resident batches rotated "
                              f"({nbuf * per_batch / 2**20:.0f} MiB > 126 MiB L2)",
                        "parallelism": f"dp{world} (candidate shards) + NCCL all-reduce MIN"},

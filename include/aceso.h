@@ -179,6 +179,10 @@ typedef struct {
 #define ACESO_OUT_SUMMARY  1u /* write iter_ns, max_mem, info                   */
 #define ACESO_OUT_FULL     2u /* also write the per-stage arrays                 */
 #define ACESO_FUSED_SELECT 4u /* reduce the batch argmin into d_sel (fused K2)   */
+#define ACESO_HINT_DENSE   8u /* schedule hint: candidates change tp/dp or
+                                 recompute at most ops (e.g. uniformly random
+                                 encodings); selects the per-op kernel instead
+                                 of the event kernel. Results are identical.  */
 
 /* ------------------------------------------------------------------------- */
 /* Selection (Alg. 1 GetBestOf P:L543, Alg. 2 `perf < init_perf` P:L576).     */
@@ -204,7 +208,13 @@ size_t aceso_select_buf_bytes(const aceso_ctx *ctx, int64_t n);
 /* Evaluates candidates [0, n) of a batch whose first candidate has global index
  * `global_offset` in a job of `n_total` candidates (sharding, §8e).
  *   d_codes : tiled op codes (device)        d_hdr : [n] headers (device)
- *   flags   : OR of ACESO_OUT_SUMMARY / ACESO_OUT_FULL / ACESO_FUSED_SELECT
+ *   flags   : OR of ACESO_OUT_SUMMARY / ACESO_OUT_FULL / ACESO_FUSED_SELECT, plus
+ *             optionally ACESO_HINT_DENSE. Schedules (results are bit-identical):
+ *             the event kernel (default for n_ops > 64) walks each candidate's
+ *             stage heads and tp/dp changes and takes run sums from position-prefix
+ *             tables; the per-op kernel (default for n_ops <= 64, or with the hint)
+ *             accumulates every op. The environment variable ACESO_KERNEL=quad|events,
+ *             read by aceso_load_profile, overrides the default.
  *   out     : host struct of device pointers (may be null if no OUT_* flag)
  *   d_sel   : select buffer (device), required with ACESO_FUSED_SELECT
  *   stream  : cudaStream_t

@@ -98,7 +98,7 @@ struct aceso_ctx {
   uint32_t mem_shift;
   Tables tab;
   void *d_blob;
-  int kernel;       // 0: quad kernel, 1: event kernel (default; ACESO_KERNEL=quad|events)
+  int kernel;       // default schedule: 0 per-op (quad) kernel, 1 event kernel (ACESO_KERNEL=quad|events)
   void *d_ev;       // event-kernel tables
   uint32_t qo_off, qo_bytes;
   const uint4 *px, *kx, *qr;
@@ -106,8 +106,8 @@ struct aceso_ctx {
   const uint32_t *st;
   int split;        // warps per tile (1 or 2)
   int minb;         // register target: 2 or 3 resident CTAs per SM
-  int max_ctas[8];  // per mode: resident CTAs (occupancy x SMs)
-  size_t smem[8];
+  int max_ctas[2][8];  // per kernel and mode: resident CTAs (occupancy x SMs)
+  size_t smem[2][8];
 };
 
 extern "C" {
@@ -440,7 +440,7 @@ int aceso_load_profile(const aceso_profile_desc *d, int cuda_device, aceso_ctx *
   ctx->mem_shift = ms;
   ctx->d_blob = nullptr;
   ctx->d_ev = nullptr;
-  ctx->kernel = 1;
+  ctx->kernel = L > 64 ? 1 : 0;  // short models: per-tile event overheads outweigh the per-op work
   if (const char *env = getenv("ACESO_KERNEL")) {
     if (!strcmp(env, "quad")) ctx->kernel = 0;
     else if (!strcmp(env, "events")) ctx->kernel = 1;
@@ -477,21 +477,24 @@ int aceso_load_profile(const aceso_profile_desc *d, int cuda_device, aceso_ctx *
       ctx->st = reinterpret_cast<const uint32_t *>(eb + ev_st);
       ctx->qr = reinterpret_cast<const uint4 *>(eb + ev_qr);
     }
-    if (ctx->kernel == 1) ctx->split = 1;
-    for (uint32_t mode = 1; mode < 8; ++mode) {
-      const size_t smem =
-          ctx->kernel == 1
-              ? (size_t)qo_bytes + ev_ring_bytes() + ev_list_bytes() + ev_snap_bytes(mode & ACESO_OUT_FULL)
-              : ((mode & ACESO_OUT_FULL) ? tab.bytes_full : tab.bytes) + (tab.k_smem ? bytesK : 0u) +
-                    kRingBytesPerCta + (ctx->split == 2 ? (size_t)(kWarps / 2) * 32 * sizeof(Xchg) : 0);
-      ctx->smem[mode] = smem;
-      void *k = eval_kernel_for(mode, ctx->split, ctx->minb, ctx->kernel);
-      e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-      int occ = 0;
-      if (e == cudaSuccess) e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k, kThreads, smem);
-      if (e != cudaSuccess || occ < 1) { rc = fail(ACESO_ECUDA, "kernel setup (mode %u, %zu B smem): %s", mode, smem, cudaGetErrorString(e)); break; }
-      ctx->max_ctas[mode] = occ * ctx->sms;
-    }
+    for (int kern = 0; kern < 2 && rc == ACESO_OK; ++kern)
+      for (uint32_t mode = 1; mode < 8; ++mode) {
+        const size_t smem =
+            kern == 1
+                ? (size_t)qo_bytes + ev_ring_bytes() + ev_list_bytes() + ev_snap_bytes(mode & ACESO_OUT_FULL)
+                : ((mode & ACESO_OUT_FULL) ? tab.bytes_full : tab.bytes) + (tab.k_smem ? bytesK : 0u) +
+                      kRingBytesPerCta + (ctx->split == 2 ? (size_t)(kWarps / 2) * 32 * sizeof(Xchg) : 0);
+        ctx->smem[kern][mode] = smem;
+        void *k = eval_kernel_for(mode, ctx->split, ctx->minb, kern);
+        e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        int occ = 0;
+        if (e == cudaSuccess) e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k, kThreads, smem);
+        if (e != cudaSuccess || occ < 1) {
+          rc = fail(ACESO_ECUDA, "kernel setup (kernel %d, mode %u, %zu B smem): %s", kern, mode, smem, cudaGetErrorString(e));
+          break;
+        }
+        ctx->max_ctas[kern][mode] = occ * ctx->sms;
+      }
   } while (0);
   cudaSetDevice(prev_dev);
   if (rc != ACESO_OK) {
@@ -519,7 +522,8 @@ size_t aceso_select_buf_bytes(const aceso_ctx *ctx, int64_t n) {
   (void)n;
   if (!ctx) return 0;
   int m = 0;
-  for (int k = 1; k < 8; ++k) m = std::max(m, ctx->max_ctas[k]);
+  for (int kern = 0; kern < 2; ++kern)
+    for (int k = 1; k < 8; ++k) m = std::max(m, ctx->max_ctas[kern][k]);
   m = std::max(m, 4 * ctx->sms);  // per-CTA partials of the eval kernels; select kernel grid
   return (size_t)kSelPartialOff + 16 * (size_t)m;
 }
@@ -531,7 +535,8 @@ int aceso_eval(aceso_ctx *ctx, const uint8_t *d_codes, const uint64_t *d_hdr, in
   if (n < 0 || global_offset < 0 || n_total < global_offset + n) return fail(ACESO_EINVAL, "bad n / global_offset / n_total");
   if (n_total >= (1ll << 40)) return fail(ACESO_EINVAL, "n_total >= 2^40");
   const uint32_t mode = flags & 7u;
-  if (mode == 0 || (flags & ~7u)) return fail(ACESO_EINVAL, "bad flags 0x%x", flags);
+  if (mode == 0 || (flags & ~(7u | ACESO_HINT_DENSE))) return fail(ACESO_EINVAL, "bad flags 0x%x", flags);
+  const int kern = (flags & ACESO_HINT_DENSE) ? 0 : ctx->kernel;
   if (n > 0 && (!d_codes || !d_hdr)) return fail(ACESO_EINVAL, "null codes/headers");
   if ((mode & (ACESO_OUT_SUMMARY | ACESO_OUT_FULL)) && !out) return fail(ACESO_EINVAL, "null outputs");
   if ((mode & ACESO_OUT_SUMMARY) && n > 0 && (!out->iter_ns || !out->max_mem || !out->info)) return fail(ACESO_EINVAL, "null summary array");
@@ -584,14 +589,14 @@ int aceso_eval(aceso_ctx *ctx, const uint8_t *d_codes, const uint64_t *d_hdr, in
   P.qo_off = ctx->qo_off;
   P.evblob = reinterpret_cast<const unsigned char *>(ctx->d_ev);
 
-  const int tiles_per_cta = kWarps / ctx->split;
+  const int tiles_per_cta = kern == 1 ? kWarps : kWarps / ctx->split;
   const int64_t need = (P.n_tiles + tiles_per_cta - 1) / tiles_per_cta;
-  int grid = (int)std::max<int64_t>(1, std::min<int64_t>(need, ctx->max_ctas[mode]));
+  int grid = (int)std::max<int64_t>(1, std::min<int64_t>(need, ctx->max_ctas[kern][mode]));
   int prev = 0;
   CUDA_TRY(cudaGetDevice(&prev));
   if (prev != ctx->device) CUDA_TRY(cudaSetDevice(ctx->device));
   void *args[] = {&P};
-  cudaError_t e = cudaLaunchKernel(eval_kernel_for(mode, ctx->split, ctx->minb, ctx->kernel), dim3(grid), dim3(kThreads), args, ctx->smem[mode],
+  cudaError_t e = cudaLaunchKernel(eval_kernel_for(mode, ctx->split, ctx->minb, kern), dim3(grid), dim3(kThreads), args, ctx->smem[kern][mode],
                                    reinterpret_cast<cudaStream_t>(stream));
   if (prev != ctx->device) cudaSetDevice(prev);
   if (e != cudaSuccess) return fail(ACESO_ECUDA, "eval launch: %s", cudaGetErrorString(e));

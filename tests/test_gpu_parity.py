@@ -35,7 +35,8 @@ def ctx_for(prof):
     return _ctx_cache[key][1]
 
 
-def run_gpu(prof, codes, hdr, full=False, gofs=0, n_total=None, pack_on_device=False, select=True):
+def run_gpu(prof, codes, hdr, full=False, gofs=0, n_total=None, pack_on_device=False, select=True,
+            dense_hint=False):
     ctx = ctx_for(prof)
     n = len(hdr)
     if pack_on_device:
@@ -43,7 +44,8 @@ def run_gpu(prof, codes, hdr, full=False, gofs=0, n_total=None, pack_on_device=F
     else:
         tiled = torch.from_numpy(ai.tile(codes)).cuda()
     hd = torch.from_numpy(np.ascontiguousarray(hdr, np.uint64).view(np.int64)).cuda()
-    out, sel = ctx.eval(tiled, hd, n=n, global_offset=gofs, n_total=n_total, full=full, select=select)
+    out, sel = ctx.eval(tiled, hd, n=n, global_offset=gofs, n_total=n_total, full=full, select=select,
+                        dense_hint=dense_hint)
     torch.cuda.synchronize()
     g = dict(iter=as_u64(out.iter_ns), max_mem=as_u64(out.max_mem), info=as_u32(out.info))
     if full:
@@ -52,8 +54,8 @@ def run_gpu(prof, codes, hdr, full=False, gofs=0, n_total=None, pack_on_device=F
     return g, (Selection.from_buffer(sel) if select else None), out, ctx
 
 
-def compare(prof, codes, hdr, full=False, gofs=0, n_total=None, pack_on_device=False):
-    g, sel, out, ctx = run_gpu(prof, codes, hdr, full, gofs, n_total, pack_on_device)
+def compare(prof, codes, hdr, full=False, gofs=0, n_total=None, pack_on_device=False, dense_hint=False):
+    g, sel, out, ctx = run_gpu(prof, codes, hdr, full, gofs, n_total, pack_on_device, dense_hint=dense_hint)
     o = oracle.evaluate(prof, codes, hdr, full=full, threads=8)
     for k in ["iter", "max_mem", "info"]:
         bad = np.nonzero(g[k] != o[k])[0]
@@ -118,6 +120,16 @@ def test_full_mode_parity(name):
     compare(prof, codes, hdr, full=True)
     codes, hdr = ai.dense_random(prof, SEED + 4, 0, 500)
     compare(prof, codes, hdr, full=True)
+
+
+@pytest.mark.parametrize("name", WL)
+def test_dense_hint_schedule_parity(name):
+    """ACESO_HINT_DENSE selects the per-op kernel: identical results on both distributions."""
+    prof = P.WORKLOADS[name]()
+    codes, hdr = ai.dense_random(prof, SEED + 12, 0, 1500)
+    compare(prof, codes, hdr, full=True, dense_hint=True)
+    codes, hdr = ai.search_shaped(prof, SEED + 13, 0, 1500, group_size=64)
+    compare(prof, codes, hdr, dense_hint=True)
 
 
 def test_gpt_1k_layers_parity():
