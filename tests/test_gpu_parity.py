@@ -132,6 +132,48 @@ def test_dense_hint_schedule_parity(name):
     compare(prof, codes, hdr, dense_hint=True)
 
 
+def _crowded_candidates(prof, n, seed, pair_stages):
+    """Valid candidates that stress the event kernel's rare paths: many one-op stages at the
+    start (more heads in a 16-op chunk than snapshot slots -> quad-by-quad mode), random
+    recompute bits (a snapshot at almost every head), and, with pair_stages, two-device stages
+    whose ops alternate tp/dp (an event at every op -> list drains mid-tile)."""
+    rng = np.random.default_rng(seed)
+    L, G = prof.n_ops, prof.n_devices
+    rows, hdrs = [], []
+    for _ in range(n):
+        dev = 2 if pair_stages else 1
+        p = G // dev
+        n_small = int(rng.integers(p // 2, p))               # leading stages of 1-2 ops
+        starts = list(np.cumsum(rng.integers(1, 3, size=n_small)))
+        rest = sorted(rng.choice(np.arange(starts[-1] + 1, L), size=p - 1 - n_small, replace=False))
+        starts = [0] + starts[:-1] + [starts[-1]] + list(rest)
+        starts = sorted(set(starts))[:p]
+        while len(starts) < p:                               # keep exactly p stages
+            cand = int(rng.integers(1, L))
+            if cand not in starts:
+                starts = sorted(starts + [cand])
+        mbs = int(rng.integers(1 if pair_stages else 0, 5))
+        row = np.zeros(L, np.uint8)
+        heads = set(starts)
+        for j in range(L):
+            tpl, dpl = (0, 0)
+            if pair_stages:
+                tpl, dpl = ((1, 0) if (j + int(rng.integers(0, 2))) % 2 else (0, 1))
+            row[j] = ai.code(1 if j in heads else 0, tpl, dpl, int(rng.random() < 0.35))
+        rows.append(row)
+        hdrs.append(ai.header(mbs, p))
+    return np.array(rows, np.uint8), np.array(hdrs, np.uint64)
+
+
+@pytest.mark.parametrize("pair_stages", [False, True])
+def test_event_kernel_rare_paths_parity(pair_stages):
+    prof = P.WORKLOADS["gpt3-13b"]()
+    codes, hdr = _crowded_candidates(prof, 700, SEED + 14 + int(pair_stages), pair_stages)
+    g, o, sel, _, _ = compare(prof, codes, hdr, full=True)
+    assert ((o["info"] & oracle.INFO_INVALID) == 0).mean() > 0.9  # the sums are really compared
+    compare(prof, codes, hdr, full=True, dense_hint=True)
+
+
 def test_gpt_1k_layers_parity():
     prof = P.WORKLOADS["gpt-1k"]()
     codes, hdr = ai.search_shaped(prof, SEED + 5, 0, 257, group_size=8)
