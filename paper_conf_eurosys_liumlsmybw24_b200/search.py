@@ -111,9 +111,10 @@ def perf_of(info, it, mem):
 # ---------------------------------------------------------------------------
 # reconfiguration primitives (Table 1) applied to one configuration
 # ---------------------------------------------------------------------------
-def _move_front(codes, s, k):
-    """dec-op# of stage s / inc-op# of s-1: first k ops of stage s join stage s-1."""
-    heads, ends = stages_of(codes)
+def _move_front(codes, s, k, st=None):
+    """dec-op# of stage s / inc-op# of s-1: first k ops of stage s join stage s-1.
+    st = stages_of(codes) when the caller has it."""
+    heads, ends = stages_of(codes) if st is None else st
     a, e = heads[s], ends[s]
     if s == 0 or k < 1 or k >= e - a:
         return None
@@ -124,9 +125,9 @@ def _move_front(codes, s, k):
     return c
 
 
-def _move_back(codes, s, k):
+def _move_back(codes, s, k, st=None):
     """dec-op# of stage s / inc-op# of s+1: last k ops of stage s join stage s+1."""
-    heads, ends = stages_of(codes)
+    heads, ends = stages_of(codes) if st is None else st
     p = len(heads)
     a, e = heads[s], ends[s]
     if s >= p - 1 or k < 1 or k >= e - a:
@@ -139,8 +140,8 @@ def _move_back(codes, s, k):
     return c
 
 
-def _recode_stage(codes, s, dt, dd, from_op=None):
-    heads, ends = stages_of(codes)
+def _recode_stage(codes, s, dt, dd, from_op=None, st=None):
+    heads, ends = stages_of(codes) if st is None else st
     a, e = heads[s], ends[s]
     lo = a if from_op is None else from_op
     c = codes.copy()
@@ -152,9 +153,9 @@ def _recode_stage(codes, s, dt, dd, from_op=None):
     return c
 
 
-def _rc_order(prof, codes, s, mbs):
+def _rc_order(prof, codes, s, mbs, st=None):
     """Ops of stage s by activation size at their partition, largest first."""
-    heads, ends = stages_of(codes)
+    heads, ends = stages_of(codes) if st is None else st
     a, e = heads[s], ends[s]
     j = np.arange(a, e)
     tpl = (codes[a:e] >> 1) & 7
@@ -194,19 +195,27 @@ class Primitives:
         # inc/dec-op#: move ops out of the bottleneck at either edge (every resource),
         # with a relay toward the idlest stage
         idle = int(np.argmin(stage_time[:p])) if p > 1 else bn
+        st = (heads, ends)
         for k in range(1, kmax + 1):
-            c = _move_front(codes, bn, k)
+            c = _move_front(codes, bn, k, st)
             if c is not None:
                 out.append((c, mbs))
                 if idle < bn - 1:
-                    c2 = _move_front(c, bn - 1, k)
+                    # stage bn-1 of c: heads unchanged below bn, its end moved by k
+                    h2, e2 = heads.copy(), ends.copy()
+                    h2[bn] += k
+                    e2[bn - 1] += k
+                    c2 = _move_front(c, bn - 1, k, (h2, e2))
                     if c2 is not None:
                         out.append((c2, mbs))
-            c = _move_back(codes, bn, k)
+            c = _move_back(codes, bn, k, st)
             if c is not None:
                 out.append((c, mbs))
                 if idle > bn + 1:
-                    c2 = _move_back(c, bn + 1, k)
+                    h2, e2 = heads.copy(), ends.copy()
+                    h2[bn + 1] -= k
+                    e2[bn] -= k
+                    c2 = _move_back(c, bn + 1, k, (h2, e2))
                     if c2 is not None:
                         out.append((c2, mbs))
         log2bg = int(math.log2(prof.global_batch & -prof.global_batch))
@@ -218,7 +227,7 @@ class Primitives:
             out.append((codes, mbs + 1))
         # tp <-> dp inside the stage (same devices): inc-tp/dec-dp and dec-tp/inc-dp
         for dt in (1, -1):
-            c = _recode_stage(codes, bn, dt, -dt)
+            c = _recode_stage(codes, bn, dt, -dt, st=st)
             if c is not None:
                 out.append((c, max(mbs, int(((c >> 5) & 7).max()))))
         # inc-dp / inc-tp with a partner stage holding twice the devices
@@ -230,19 +239,19 @@ class Primitives:
             if kq == kb + 1 and ("comp" in want or "mem" in want):
                 for dtb, ddb in ((1, 0), (0, 1)):
                     for dtq, ddq in ((-1, 0), (0, -1)):
-                        c = _recode_stage(codes, bn, dtb, ddb)
-                        c = _recode_stage(c, q, dtq, ddq) if c is not None else None
+                        c = _recode_stage(codes, bn, dtb, ddb, st=st)
+                        c = _recode_stage(c, q, dtq, ddq, st=st) if c is not None else None
                         if c is not None:
                             out.append((c, max(mbs, int(((c >> 5) & 7).max()))))
             if kq + 1 == kb and "comm" in want:  # give devices away (dec-dp/tp on the bottleneck)
                 for dtb, ddb in ((-1, 0), (0, -1)):
                     for dtq, ddq in ((1, 0), (0, 1)):
-                        c = _recode_stage(codes, bn, dtb, ddb)
-                        c = _recode_stage(c, q, dtq, ddq) if c is not None else None
+                        c = _recode_stage(codes, bn, dtb, ddb, st=st)
+                        c = _recode_stage(c, q, dtq, ddq, st=st) if c is not None else None
                         if c is not None:
                             out.append((c, max(mbs, int(((c >> 5) & 7).max()))))
         # greedy inc-rc (memory) / dec-rc (computation) on the largest-activation ops
-        order = _rc_order(prof, codes, bn, mbs)
+        order = _rc_order(prof, codes, bn, mbs, st)
         rc = (codes[order] >> 4) & 1
         if "mem" in want:
             todo = order[rc == 0]
@@ -257,11 +266,27 @@ class Primitives:
                 c[have[:k]] &= 0xEF
                 out.append((c, mbs))
         # op-level fine-tune: tp/dp change from op k to the end of the stage
-        for j in range(heads[bn] + 1, ends[bn]):
-            for dt in (1, -1):
-                c = _recode_stage(codes, bn, dt, -dt, from_op=j)
-                if c is not None:
-                    out.append((c, max(mbs, int(((c >> 5) & 7).max()))))
+        a, e = int(heads[bn]), int(ends[bn])
+        if e - a > 1:
+            # suffix extrema of the stage's tp/dp fields decide which shifts stay in range
+            tp = ((codes[a:e] >> 1) & 7).astype(np.int16)
+            dp = ((codes[a:e] >> 5) & 7).astype(np.int16)
+            tmin, tmax = np.minimum.accumulate(tp[::-1])[::-1], np.maximum.accumulate(tp[::-1])[::-1]
+            dmin, dmax_s = np.minimum.accumulate(dp[::-1])[::-1], np.maximum.accumulate(dp[::-1])[::-1]
+            dmax_pre = int(((codes[:a] >> 5) & 7).max()) if a > 0 else 0
+            dmax_post = int(((codes[e:] >> 5) & 7).max()) if e < len(codes) else 0
+            dmax_out = max(dmax_pre, dmax_post)
+            for j in range(a + 1, e):
+                r = j - a
+                for dt in (1, -1):
+                    if tmin[r] + dt < 0 or tmax[r] + dt > 7 or dmin[r] - dt < 0 or dmax_s[r] - dt > 7:
+                        continue
+                    c = codes.copy()
+                    seg = c[j:e]
+                    c[j:e] = (seg & 0x11) | (((tp[r:] + dt).astype(np.uint8) & 7) << 1) | \
+                        (((dp[r:] - dt).astype(np.uint8) & 7) << 5)
+                    dnew = max(dmax_out, int(((codes[a:j] >> 5) & 7).max()), int(dmax_s[r] - dt))
+                    out.append((c, max(mbs, dnew)))
         return out
 
 

@@ -82,3 +82,36 @@ def test_search_on_toy_reaches_a_feasible_near_optimum():
     r, st = S.search(prof, OracleEvaluator(prof), budget_s=30, max_hops=7, beam=4)
     assert r.perf[0] == 0
     assert r.perf[1] <= best[1] * 1.10
+
+
+@pytest.mark.parametrize("name", ["gpt3-1.3b", "t5", "wrn", "toy-b"])
+def test_optimised_primitives_match_reference(name):
+    """The generator (stage structure computed once per node, vectorised fine-tune checks)
+    yields exactly the candidates of the first, one-pass-per-candidate version."""
+    import importlib.util
+    import os
+    spec = importlib.util.spec_from_file_location(
+        "_search_reference", os.path.join(os.path.dirname(__file__), "_search_reference.py"))
+    R = importlib.util.module_from_spec(spec)
+    spec.loader.exec_module(R)
+    prof = P.WORKLOADS[name]()
+    codes, hdr = ai.search_shaped(prof, 99, 0, 60, group_size=8)
+    o = oracle.evaluate(prof, codes, hdr)
+    rng = np.random.default_rng(3)
+    checked = 0
+    for i in np.nonzero((o["info"] & oracle.INFO_INVALID) == 0)[0][:25]:
+        c, mbs = codes[i], int(hdr[i] & 0xFF)
+        p = int((c & 1).sum())
+        G = prof.n_devices
+        for h2, oom, mk in [(True, False, None), (True, True, 6), (False, False, 3)]:
+            info = int(rng.integers(0, p)) | (S.INFO_OOM if oom else 0)
+            comp = rng.integers(1, 1000, size=G).astype(np.uint64)
+            comm = rng.integers(1, 1000, size=G).astype(np.uint64)
+            stt = rng.integers(1, 1000, size=G).astype(np.uint64)
+            a = S.Primitives(prof, heuristic2=h2, max_k=mk).apply_all(c, mbs, info, comp, comm, stt)
+            b = R.PrimitivesReference(prof, heuristic2=h2, max_k=mk).apply_all(c, mbs, info, comp, comm, stt)
+            assert len(a) == len(b)
+            for (ca, ma), (cb, mb) in zip(a, b):
+                assert ma == mb and np.array_equal(ca, cb)
+            checked += len(a)
+    assert checked > 500
