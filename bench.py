@@ -278,7 +278,8 @@ def main():
     outs = [out] + [ctx.alloc_outputs(n) for _ in range(nstr - 1)]
     side = [torch.cuda.Stream() for _ in range(nstr)]
     comm = torch.cuda.Stream()  # all-reduces in step order on one stream (same on every rank)
-    with torch.cuda.graph(graph):
+    def issue_steps():
+        """The K steps on the side streams (+ all-reduces in step order on `comm`)."""
         cs = torch.cuda.current_stream()
         fork = torch.cuda.Event()
         fork.record(cs)
@@ -308,9 +309,22 @@ def main():
             j = torch.cuda.Event()
             j.record(st)
             cs.wait_event(j)
-    torch.cuda.synchronize()
-    graph.replay()  # one untimed replay (graph upload)
-    torch.cuda.synchronize()
+
+    timing_mode = "graph"
+    try:
+        with torch.cuda.graph(graph):
+            issue_steps()
+        torch.cuda.synchronize()
+        graph.replay()  # one untimed replay (graph upload)
+        torch.cuda.synchronize()
+    except Exception as e:  # e.g. a collective that cannot be captured: time eager issue
+        timing_mode = f"eager ({type(e).__name__} during graph capture)"
+        print(f"[bench] graph capture failed ({e}); timing eagerly issued steps", file=sys.stderr)
+        torch.cuda.synchronize()
+        ev_s = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps)]
+        ev_k = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps)]
+        issue_steps()  # untimed pass
+        torch.cuda.synchronize()
 
     clocks = ClockSampler(local)
     t_start = torch.cuda.Event(enable_timing=True)
@@ -320,7 +334,10 @@ def main():
     torch.cuda.synchronize()
     clocks.start()
     t_start.record(stream)
-    graph.replay()
+    if timing_mode == "graph":
+        graph.replay()
+    else:
+        issue_steps()
     t_end.record(stream)
     torch.cuda.synchronize()
     if world > 1:
@@ -440,8 +457,9 @@ def main():
                                  "on streams); *_serial = same kernel launched back to back "
                                  "on one stream"},
             "gpu_launches": args.steps,
-            "timing": f"K steps captured in one CUDA graph ({nstr} streams, independent batches "
-                      f"round-robin), replayed once between CUDA events",
+            "timing": (f"K steps captured in one CUDA graph ({nstr} streams, independent batches "
+                       f"round-robin), replayed once between CUDA events") if timing_mode == "graph" else
+                      (f"K steps issued eagerly ({nstr} streams) between CUDA events: {timing_mode}"),
             "clocks": clk,
             "result": {"cls": best.cls, "cost": best.cost, "index": best.index},
         }
