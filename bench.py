@@ -44,6 +44,7 @@ def parse():
     ap.add_argument("--group", type=int, default=1024, help="candidates sharing a base config")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--no-dedup", action="store_true", help="skip the hash / visited-set measurement")
     ap.add_argument("--search-budget", type=float, default=20.0,
                     help="seconds for the search-time measurement (0: skip)")
     ap.add_argument("--streams", type=int, default=4,
@@ -155,6 +156,54 @@ def cpu_baseline(prof, batches_rowmajor, max_cands, min_core_seconds=10.0):
     return {"value": done / dt, "unit": "configs/s", "cores": threads, "kind": "oracle",
             "sample": f"{len(hdr)} candidates of the timed workload (same seed) x {passes} passes "
                       f"= {done} evaluations, {dt:.2f} s wall on {threads} threads"}
+
+
+def measure_dedup(A, dev_batches, n, L, hbm, reps=200):
+    """NEXT(3) kernels on the bench batches: aceso_hash (streaming: reads the tiled codes and
+    headers, writes 8 B per candidate) and aceso_dedup (visited-set insert + flag)."""
+    import torch
+    hs = [torch.empty(n, dtype=torch.int64, device=dev_batches[0][0].device) for _ in dev_batches]
+    for (c, h), o in zip(dev_batches, hs):
+        A.hash_candidates(c, h, L, out=o)
+    torch.cuda.synchronize()
+    ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    g = torch.cuda.CUDAGraph()  # launches captured: host call overhead must not pace the GPU
+    with torch.cuda.graph(g):
+        for r in range(reps):
+            c, h = dev_batches[r % len(dev_batches)]
+            A.hash_candidates(c, h, L, out=hs[r % len(hs)])
+    g.replay()
+    torch.cuda.synchronize()
+    ev0.record()
+    g.replay()
+    ev1.record()
+    torch.cuda.synchronize()
+    ms = ev0.elapsed_time(ev1) / reps
+    hbytes = n * (L + 8 + 8)  # codes + header read, hash written
+    # visited set sized for every batch's hashes at <= 50% load
+    slots = 1 << int(np.ceil(np.log2(2 * n * len(hs))))
+    vs = A.VisitedSet(slots, device=hs[0].device.index)
+    dup = torch.empty(n, dtype=torch.uint8, device=hs[0].device)
+    vs.insert(hs[0][:1], dup=dup)  # warm-up (epoch 1)
+    torch.cuda.synchronize()
+    gv = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(gv):
+        for o in hs:  # distinct batches (later epochs): duplicates are the generator's own
+            vs.insert(o, dup=dup)
+    ev0.record()
+    gv.replay()
+    ev1.record()
+    torch.cuda.synchronize()
+    dms = ev0.elapsed_time(ev1) / len(hs)
+    return {"hash": {"ms_per_batch": ms, "configs_per_s": n / (ms * 1e-3),
+                     "roofline": {"bound": "hbm", "achieved": hbytes / (ms * 1e-3) / 1e9, "peak": hbm,
+                                  "unit": "GB/s", "frac": hbytes / (ms * 1e-3) / 1e9 / hbm,
+                                  "bytes_per_launch": hbytes}},
+            "visited_set": {"ms_per_batch": dms, "hashes_per_s": n / (dms * 1e-3), "slots": slots,
+                            "duplicates_in_last_batch": int(dup.sum().item()),
+                            "overflow": vs.overflowed()},
+            "note": "SURVEY 8(f) NEXT(3): configuration hash (aceso_hash) and first-occurrence "
+                    "visited set (aceso_dedup) on the bench batches; not part of the timed step"}
 
 
 def run_reference(args):
@@ -465,6 +514,8 @@ def main():
         }
         if e2e is not None:
             line["e2e"] = e2e
+        if not args.no_dedup:
+            line["dedup"] = measure_dedup(A, dev_batches, n, L, hbm)
         if args.search_budget > 0 and world == 1:
             from paper_conf_eurosys_liumlsmybw24_b200 import search as S
             ev = S.GPUEvaluator(ctx)

@@ -235,6 +235,36 @@ int aceso_select(aceso_ctx *ctx, const aceso_eval_out *out, int64_t n, int64_t g
 int aceso_decode_key(int64_t key, int64_t n_total, int *cls, uint64_t *cost, int64_t *index,
                      int *saturated);
 
+/* ------------------------------------------------------------------------- */
+/* Configuration dedup ("skip configurations     */
+/* already explored"). The encoding above is canonical (one byte per op plus   */
+/* the header), so equal configurations have equal bytes and hash equal.       */
+/* ------------------------------------------------------------------------- */
+/* 64-bit hash of every candidate: the row-major byte string (L code bytes, then
+ * the 8 header bytes little-endian, zero-padded to a multiple of 8) read as
+ * little-endian u64 words w_0..w_{m-1}; with mix(x) = splitmix64's finalizer
+ *   (x ^= x >> 30; x *= 0xBF58476D1CE4E5B9; x ^= x >> 27; x *= 0x94D049BB133111EB;
+ *    x ^= x >> 31),
+ *   h = mix(0x243F6A8885A308D3 + sum_i mix(w_i ^ (i + 1) * 0x9E3779B97F4A7C15))  (mod 2^64),
+ *   h = 1 if h == 0 (0 marks an empty visited-set slot). Words mix independently
+ *   (position-tagged), so the kernel streams them with full instruction parallelism.
+ *   d_codes : tiled codes (device, 16-byte aligned)   d_hdr : [n] headers
+ *   d_hash  : [n] u64 output (device). Async on `stream`. */
+int aceso_hash(const uint8_t *d_codes, const uint64_t *d_hdr, int64_t n, int32_t n_ops,
+               uint64_t *d_hash, void *stream);
+
+/* Visited set: open addressing over `slots` (a power of two >= 2) entries of 16
+ * bytes {hash, tag} in caller-owned device memory, zero-filled once. A call with
+ * epoch e (1 <= e < 2^23, increasing across calls) inserts the n hashes and
+ * writes d_dup[i] = 1 if hash i was inserted by an earlier call or by a lower
+ * index of this call, else 0 (deterministic first occurrence). A full table is
+ * reported asynchronously: *d_status = 1 (device u32, zeroed by the call) and
+ * d_dup is unspecified. Entries: {hash, ~(epoch << 40 | index) max-reduced}.
+ * Two launches on `stream` (insert, then flag). n < 2^40. */
+size_t aceso_visited_bytes(int64_t slots);
+int aceso_dedup(const uint64_t *d_hash, int64_t n, uint32_t epoch, void *d_table, int64_t slots,
+                uint8_t *d_dup, uint32_t *d_status, void *stream);
+
 /* Message of the last failing call on this thread ("" if none). */
 const char *aceso_last_error(void);
 

@@ -2,9 +2,10 @@
 
 Public API (names follow include/aceso.h): Context (aceso_load_profile/aceso_free),
 Context.eval (aceso_eval), Context.select (aceso_select), Context.pack_rowmajor
-(aceso_pack_rowmajor), decode_key (aceso_decode_key), dist.global_select (NCCL
-all-reduce MIN of the packed key).
+(aceso_pack_rowmajor), decode_key (aceso_decode_key), hash_candidates (aceso_hash),
+VisitedSet (aceso_visited_bytes/aceso_dedup), dist.global_select (NCCL all-reduce MIN of the
+packed key).
 """
-from .api import AcesoError, Context, Outputs, Selection, as_u32, as_u64, decode_key, tiled_bytes, \
-    upload_candidates, version  # noqa: F401
+from .api import AcesoError, Context, Outputs, Selection, VisitedSet, as_u32, as_u64, decode_key, \
+    hash_candidates, tiled_bytes, upload_candidates, version  # noqa: F401
 from .buildlib import LIB, build  # noqa: F401

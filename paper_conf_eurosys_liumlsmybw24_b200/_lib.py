@@ -14,7 +14,7 @@ INFO_INVALID = 1 << 17
 
 SYMBOLS = ["aceso_load_profile", "aceso_free", "aceso_tiled_bytes", "aceso_pack_rowmajor",
            "aceso_select_buf_bytes", "aceso_eval", "aceso_select", "aceso_decode_key",
-           "aceso_last_error", "aceso_version"]
+           "aceso_last_error", "aceso_version", "aceso_hash", "aceso_visited_bytes", "aceso_dedup"]
 
 
 class ProfileDesc(ctypes.Structure):
@@ -65,5 +65,11 @@ def load():
     lib.aceso_last_error.restype = ctypes.c_char_p
     lib.aceso_version.argtypes = []
     lib.aceso_version.restype = ctypes.c_char_p
+    lib.aceso_hash.argtypes = [P, P, c_i64, c_i32, P, P]
+    lib.aceso_hash.restype = ctypes.c_int
+    lib.aceso_visited_bytes.argtypes = [c_i64]
+    lib.aceso_visited_bytes.restype = c_sz
+    lib.aceso_dedup.argtypes = [P, c_i64, c_u32, P, c_i64, P, P, P]
+    lib.aceso_dedup.restype = ctypes.c_int
     _lib = lib
     return lib

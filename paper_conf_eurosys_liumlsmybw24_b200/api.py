@@ -194,6 +194,43 @@ class Context:
         return sel
 
 
+def hash_candidates(codes: torch.Tensor, hdr: torch.Tensor, n_ops: int, n: int | None = None,
+                    out: torch.Tensor | None = None, stream=None) -> torch.Tensor:
+    """aceso_hash: 64-bit configuration hash of every candidate of a tiled batch (int64 view)."""
+    n = int(hdr.shape[0]) if n is None else int(n)
+    if out is None:
+        out = torch.empty(n, dtype=torch.int64, device=hdr.device)
+    _check(L.load().aceso_hash(_ptr(codes), _ptr(hdr), n, int(n_ops), _ptr(out), _stream(stream)),
+           "aceso_hash")
+    return out
+
+
+class VisitedSet:
+    """Device visited set of configuration hashes (aceso_dedup): first occurrence across calls."""
+
+    def __init__(self, slots: int, device: int = 0):
+        nb = int(L.load().aceso_visited_bytes(int(slots)))
+        if nb == 0:
+            raise AcesoError("slots must be a power of two >= 2")
+        self.slots = int(slots)
+        self.table = torch.zeros(nb, dtype=torch.uint8, device=torch.device("cuda", device))
+        self.status = torch.zeros(1, dtype=torch.int32, device=self.table.device)
+        self.epoch = 0
+
+    def insert(self, hashes: torch.Tensor, dup: torch.Tensor | None = None, stream=None) -> torch.Tensor:
+        """Marks dup[i] = 1 for hashes seen in an earlier call or at a lower index of this one."""
+        n = int(hashes.shape[0])
+        if dup is None:
+            dup = torch.empty(n, dtype=torch.uint8, device=hashes.device)
+        self.epoch += 1
+        _check(L.load().aceso_dedup(_ptr(hashes), n, self.epoch, _ptr(self.table), self.slots, _ptr(dup),
+                                    _ptr(self.status), _stream(stream)), "aceso_dedup")
+        return dup
+
+    def overflowed(self) -> bool:
+        return bool(self.status.item())
+
+
 def decode_key(key: int, n_total: int):
     """aceso_decode_key -> (cls, cost, index, saturated)."""
     cls = ctypes.c_int()

@@ -16,6 +16,7 @@
 
 #include "aux_kernels.cuh"
 #include "common.cuh"
+#include "dedup_kernels.cuh"
 #include "eval_kernel.cuh"
 #include "event_kernel.cuh"
 
@@ -649,6 +650,44 @@ int aceso_pack_rowmajor(const uint8_t *d_rowmajor, int64_t n, int32_t n_ops, uin
   pack_kernel<<<grid, 256, 0, reinterpret_cast<cudaStream_t>(stream)>>>(d_rowmajor, n, n_ops, reinterpret_cast<uint4 *>(d_tiled), total_vec);
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return fail(ACESO_ECUDA, "pack launch: %s", cudaGetErrorString(e));
+  return ACESO_OK;
+}
+
+int aceso_hash(const uint8_t *d_codes, const uint64_t *d_hdr, int64_t n, int32_t n_ops,
+               uint64_t *d_hash, void *stream) {
+  if (n < 0 || n_ops < 1 || n_ops > kMaxOps || (n > 0 && (!d_codes || !d_hdr || !d_hash)))
+    return fail(ACESO_EINVAL, "bad argument");
+  if (((uintptr_t)d_codes & 15) != 0) return fail(ACESO_EINVAL, "codes not 16-byte aligned");
+  if (n == 0) return ACESO_OK;
+  const int64_t tiles = (n + 31) / 32;
+  const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(tiles, 148 * 32));
+  hash_kernel<<<grid, kHashWarps * 32, 0, reinterpret_cast<cudaStream_t>(stream)>>>(
+      reinterpret_cast<const uint4 *>(d_codes), d_hdr, n, n_ops, d_hash);
+  cudaError_t e = cudaGetLastError();
+  if (e != cudaSuccess) return fail(ACESO_ECUDA, "hash launch: %s", cudaGetErrorString(e));
+  return ACESO_OK;
+}
+
+size_t aceso_visited_bytes(int64_t slots) {
+  if (slots < 2 || (slots & (slots - 1)) != 0) return 0;
+  return (size_t)slots * sizeof(VisitedEntry);
+}
+
+int aceso_dedup(const uint64_t *d_hash, int64_t n, uint32_t epoch, void *d_table, int64_t slots,
+                uint8_t *d_dup, uint32_t *d_status, void *stream) {
+  if (n < 0 || n >= (1ll << 40)) return fail(ACESO_EINVAL, "n outside [0, 2^40)");
+  if (epoch < 1 || epoch >= (1u << 23)) return fail(ACESO_EINVAL, "epoch outside [1, 2^23)");
+  if (slots < 2 || (slots & (slots - 1)) != 0) return fail(ACESO_EINVAL, "slots must be a power of two >= 2");
+  if (!d_table || !d_status || (n > 0 && (!d_hash || !d_dup))) return fail(ACESO_EINVAL, "null argument");
+  cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
+  CUDA_TRY(cudaMemsetAsync(d_status, 0, sizeof(uint32_t), st));
+  if (n == 0) return ACESO_OK;
+  const int grid = (int)std::max<int64_t>(1, std::min<int64_t>((n + 255) / 256, 148 * 16));
+  VisitedEntry *t = reinterpret_cast<VisitedEntry *>(d_table);
+  visit_insert_kernel<<<grid, 256, 0, st>>>(d_hash, n, epoch, t, (uint64_t)slots - 1, d_status);
+  visit_flag_kernel<<<grid, 256, 0, st>>>(d_hash, n, epoch, t, (uint64_t)slots - 1, d_dup);
+  cudaError_t e = cudaGetLastError();
+  if (e != cudaSuccess) return fail(ACESO_ECUDA, "dedup launch: %s", cudaGetErrorString(e));
   return ACESO_OK;
 }
 

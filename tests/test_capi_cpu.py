@@ -117,3 +117,29 @@ def test_every_workload_profile_is_accepted_by_validation():
     for name, fn in P.WORKLOADS.items():
         rc, msg = _load(fn())
         assert rc == 0 or (not torch.cuda.is_available() and rc in (L.ACESO_ENODEV, L.ACESO_ECUDA)), (name, msg)
+
+
+def test_dedup_rejects_bad_arguments():
+    lib = L.load()
+    assert lib.aceso_visited_bytes(1000) == 0 and lib.aceso_visited_bytes(1024) == 16 * 1024
+    st = ctypes.c_uint32()
+    # slots not a power of two / epoch 0 / epoch too large: rejected before any device call
+    assert lib.aceso_dedup(None, 0, 1, ctypes.addressof(st), 1000, None, ctypes.addressof(st), None) == L.ACESO_EINVAL
+    assert lib.aceso_dedup(None, 0, 0, ctypes.addressof(st), 1024, None, ctypes.addressof(st), None) == L.ACESO_EINVAL
+    assert lib.aceso_dedup(None, 0, 1 << 23, ctypes.addressof(st), 1024, None, ctypes.addressof(st), None) == L.ACESO_EINVAL
+    assert lib.aceso_hash(None, None, -1, 10, None, None) == L.ACESO_EINVAL
+
+
+def test_hash_reference_is_order_and_header_sensitive():
+    import sys
+    sys.path.insert(0, os.path.dirname(__file__))
+    from hash_reference import config_hash
+    rng = np.random.default_rng(0)
+    c = rng.integers(0, 256, size=(50, 37), dtype=np.uint8)
+    h = rng.integers(0, 1 << 60, size=50, dtype=np.uint64)
+    base = config_hash(c, h)
+    assert len(set(base.tolist())) == 50
+    c2 = c.copy()
+    c2[:, [3, 4]] = c2[:, [4, 3]]
+    assert (config_hash(c2, h) != base)[c[:, 3] != c[:, 4]].all()
+    assert (config_hash(c, h ^ np.uint64(1 << 8)) != base).all()
