@@ -213,7 +213,9 @@ size_t aceso_select_buf_bytes(const aceso_ctx *ctx, int64_t n);
  *             the event kernel (default for n_ops > 64) walks each candidate's
  *             stage heads and tp/dp changes and takes run sums from position-prefix
  *             tables; the per-op kernel (default for n_ops <= 64, or with the hint)
- *             accumulates every op. The environment variable ACESO_KERNEL=quad|events,
+ *             accumulates every op; it stages its tables in shared memory, so for
+ *             profiles whose tables exceed ~200 KB only the event kernel is used (the
+ *             hint is then ignored). The environment variable ACESO_KERNEL=quad|events,
  *             read by aceso_load_profile, overrides the default.
  *   out     : host struct of device pointers (may be null if no OUT_* flag)
  *   d_sel   : select buffer (device), required with ACESO_FUSED_SELECT

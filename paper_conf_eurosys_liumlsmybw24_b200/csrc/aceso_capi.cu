@@ -100,6 +100,7 @@ struct aceso_ctx {
   Tables tab;
   void *d_blob;
   int kernel;       // default schedule: 0 per-op (quad) kernel, 1 event kernel (ACESO_KERNEL=quad|events)
+  int quad_ok;      // the per-op kernel's tables fit in shared memory
   void *d_ev;       // event-kernel tables
   uint32_t qo_off, qo_bytes;
   const uint4 *px, *kx, *qr;
@@ -242,8 +243,9 @@ int aceso_load_profile(const aceso_profile_desc *d, int cuda_device, aceso_ctx *
   tab.bytesK = bytesK;
   // stage the cold table too when shared memory allows ~2 CTAs per SM
   tab.k_smem = (tab.bytes_full + bytesK + kRingBytesPerCta + 16384u <= 100u * 1024u) ? 1u : 0u;
-  if (tab.bytes_full + kRingBytesPerCta + 16384u > 220u * 1024u)
-    return fail(ACESO_EINVAL, "packed tables of %u bytes exceed shared memory", tab.bytes_full);
+  // the per-op kernel stages its tables in shared memory; larger profiles use the event
+  // kernel only (its tables are in global memory)
+  const bool quad_ok = tab.bytes_full + kRingBytesPerCta + 16384u <= 220u * 1024u;
   const uint32_t blob_bytes = tab.offK + bytesK;
   std::vector<uint32_t> blob(blob_bytes / 4, 0u);
   auto rec_S = [&](int t, int tp, int b, int rc) -> uint64_t {
@@ -441,9 +443,10 @@ int aceso_load_profile(const aceso_profile_desc *d, int cuda_device, aceso_ctx *
   ctx->mem_shift = ms;
   ctx->d_blob = nullptr;
   ctx->d_ev = nullptr;
-  ctx->kernel = L > 64 ? 1 : 0;  // short models: per-tile event overheads outweigh the per-op work
+  ctx->quad_ok = quad_ok ? 1 : 0;
+  ctx->kernel = (L > 64 || !quad_ok) ? 1 : 0;  // short models: per-tile event overheads outweigh the per-op work
   if (const char *env = getenv("ACESO_KERNEL")) {
-    if (!strcmp(env, "quad")) ctx->kernel = 0;
+    if (!strcmp(env, "quad") && quad_ok) ctx->kernel = 0;
     else if (!strcmp(env, "events")) ctx->kernel = 1;
   }
   ctx->qo_off = (uint32_t)ev_qo;
@@ -480,6 +483,11 @@ int aceso_load_profile(const aceso_profile_desc *d, int cuda_device, aceso_ctx *
     }
     for (int kern = 0; kern < 2 && rc == ACESO_OK; ++kern)
       for (uint32_t mode = 1; mode < 8; ++mode) {
+        if (kern == 0 && !quad_ok) {
+          ctx->smem[0][mode] = 0;
+          ctx->max_ctas[0][mode] = 0;
+          continue;
+        }
         const size_t smem =
             kern == 1
                 ? (size_t)qo_bytes + ev_ring_bytes() + ev_list_bytes() + ev_snap_bytes(mode & ACESO_OUT_FULL)
@@ -537,7 +545,7 @@ int aceso_eval(aceso_ctx *ctx, const uint8_t *d_codes, const uint64_t *d_hdr, in
   if (n_total >= (1ll << 40)) return fail(ACESO_EINVAL, "n_total >= 2^40");
   const uint32_t mode = flags & 7u;
   if (mode == 0 || (flags & ~(7u | ACESO_HINT_DENSE))) return fail(ACESO_EINVAL, "bad flags 0x%x", flags);
-  const int kern = (flags & ACESO_HINT_DENSE) ? 0 : ctx->kernel;
+  const int kern = ((flags & ACESO_HINT_DENSE) && ctx->quad_ok) ? 0 : ctx->kernel;
   if (n > 0 && (!d_codes || !d_hdr)) return fail(ACESO_EINVAL, "null codes/headers");
   if ((mode & (ACESO_OUT_SUMMARY | ACESO_OUT_FULL)) && !out) return fail(ACESO_EINVAL, "null outputs");
   if ((mode & ACESO_OUT_SUMMARY) && n > 0 && (!out->iter_ns || !out->max_mem || !out->info)) return fail(ACESO_EINVAL, "null summary array");

@@ -174,6 +174,36 @@ def test_event_kernel_rare_paths_parity(pair_stages):
     compare(prof, codes, hdr, full=True, dense_hint=True)
 
 
+def _limit_profile(seed=0):
+    """Random profile at the API limits: 16,384 ops, 8 tp and 8 dp choices, 16 per-GPU
+    batch sizes, 128 devices (RUNS = 128: the largest event-kernel tables)."""
+    rng = np.random.default_rng(seed)
+    L, T, NT, NB, ND, G = 16384, 300, 8, 16, 8, 128
+    rec = np.zeros((T, NT, NB, P.NF), np.int64)
+    rec[..., 0:4] = rng.integers(0, 1 << 20, size=(T, NT, NB, 4))
+    act = rng.integers(0, 1 << 20, size=(T, NT, NB)) * 512
+    rec[..., 4] = act
+    rec[..., 5] = (rng.random((T, NT, NB)) * act).astype(np.int64) // 512 * 512
+    rec[..., 6] = rng.integers(0, 1 << 18, size=(T, NT, NB)) * 512
+    rec[..., 7:10] = rng.integers(0, 1 << 20, size=(T, NT, NB, 3))
+    wmem = rng.integers(0, 1 << 16, size=(T, NT, 2)).astype(np.int64) * 512
+    dps = rng.integers(0, 1 << 20, size=(T, NT, ND)).astype(np.int64)
+    op_type = rng.integers(0, T, size=L).astype(np.uint16)
+    return P.Profile("limits", op_type, [f"t{i}" for i in range(T)], rec, wmem, dps, G,
+                     1 << 45, 1 << 16)
+
+
+def test_api_limits_parity():
+    """Tables too large for the per-op kernel's shared memory: the event kernel serves every
+    call (also with the dense hint)."""
+    prof = _limit_profile()
+    codes, hdr = ai.search_shaped(prof, SEED + 15, 0, 130, group_size=8)
+    compare(prof, codes, hdr, full=True)
+    codes, hdr = ai.dense_random(prof, SEED + 16, 0, 65)
+    compare(prof, codes, hdr)
+    compare(prof, codes, hdr, dense_hint=True)
+
+
 def test_gpt_1k_layers_parity():
     prof = P.WORKLOADS["gpt-1k"]()
     codes, hdr = ai.search_shaped(prof, SEED + 5, 0, 257, group_size=8)
