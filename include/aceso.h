@@ -238,6 +238,48 @@ int aceso_decode_key(int64_t key, int64_t n_total, int *cls, uint64_t *cost, int
                      int *saturated);
 
 /* ------------------------------------------------------------------------- */
+/* On-device candidate generation (Table 1): */
+/* a candidate is a base configuration plus up to 6 byte-range patches, the   */
+/* form every reconfiguration primitive of the search driver takes; the      */
+/* kernel writes the expanded candidates directly in the tiled layout.       */
+/* ------------------------------------------------------------------------- */
+enum {
+  ACESO_PATCH_NONE = 0,
+  ACESO_PATCH_MASK = 1,    /* ops [a, b): c = (c & v0) | v1                          */
+  ACESO_PATCH_ADD = 2,     /* ops [a, b): tp field += (int8)v0, dp field += (int8)v1;
+                              the caller keeps every field inside [0, 7]           */
+  ACESO_PATCH_RANK_RC = 3  /* ops j in [a, b) with rank[v2 & 1][j] < (v0 | v1 << 8):
+                              recompute bit set (v2 bit 1 = 0) or cleared (= 1)      */
+};
+typedef struct {
+  uint16_t a, b;     /* op range [a, b), b <= n_ops                                */
+  uint8_t kind;      /* ACESO_PATCH_*                                             */
+  uint8_t v0, v1, v2;
+} aceso_patch;       /* 8 bytes                                                    */
+typedef struct {
+  uint32_t base;     /* row of the bases array                                    */
+  uint8_t mbs_log2;  /* header byte 0 of the candidate                            */
+  uint8_t p;         /* header byte 1 (stage count)                               */
+  uint8_t n_patch;   /* patches applied in order, <= 6                             */
+  uint8_t reserved;
+  aceso_patch patch[6];
+} aceso_cand;        /* 56 bytes                                                   */
+
+/* Expands n candidates.
+ *   d_bases : [n_bases][stride] u8 row-major base encodings, stride = 16 *
+ *             ceil(n_ops / 16), bytes >= n_ops zero (device)
+ *   d_ranks : [n_bases][2][stride] u16 ranks for ACESO_PATCH_RANK_RC (device; may
+ *             be null when no candidate uses that patch)
+ *   d_cands : [n] aceso_cand (device)
+ *   d_tiled : tiled output, aceso_tiled_bytes(n, n_ops) bytes (device, 16-byte
+ *             aligned); d_hdr : [n] u64 headers out (mbs_log2 | p << 8)
+ * Out-of-range base indices or patch ranges are clamped away (no access outside
+ * the arrays); the result is then unspecified. Async on `stream`. */
+int aceso_expand(const uint8_t *d_bases, const uint16_t *d_ranks, int32_t n_bases, int32_t n_ops,
+                 const aceso_cand *d_cands, int64_t n, uint8_t *d_tiled, uint64_t *d_hdr,
+                 void *stream);
+
+/* ------------------------------------------------------------------------- */
 /* Configuration dedup ("skip configurations     */
 /* already explored"). The encoding above is canonical (one byte per op plus   */
 /* the header), so equal configurations have equal bytes and hash equal.       */

@@ -14,7 +14,7 @@ INFO_INVALID = 1 << 17
 
 SYMBOLS = ["aceso_load_profile", "aceso_free", "aceso_tiled_bytes", "aceso_pack_rowmajor",
            "aceso_select_buf_bytes", "aceso_eval", "aceso_select", "aceso_decode_key",
-           "aceso_last_error", "aceso_version", "aceso_hash", "aceso_visited_bytes", "aceso_dedup"]
+           "aceso_last_error", "aceso_version", "aceso_hash", "aceso_visited_bytes", "aceso_dedup", "aceso_expand"]
 
 
 class ProfileDesc(ctypes.Structure):
@@ -71,5 +71,7 @@ def load():
     lib.aceso_visited_bytes.restype = c_sz
     lib.aceso_dedup.argtypes = [P, c_i64, c_u32, P, c_i64, P, P, P]
     lib.aceso_dedup.restype = ctypes.c_int
+    lib.aceso_expand.argtypes = [P, P, c_i32, c_i32, P, c_i64, P, P, P]
+    lib.aceso_expand.restype = ctypes.c_int
     _lib = lib
     return lib

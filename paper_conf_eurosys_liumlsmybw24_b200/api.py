@@ -181,6 +181,22 @@ class Context:
         _check(rc, "aceso_eval")
         return out, sel
 
+    def expand(self, bases: torch.Tensor, cands: torch.Tensor, ranks: torch.Tensor | None = None,
+               n: int | None = None, tiled: torch.Tensor | None = None, hdr: torch.Tensor | None = None,
+               stream=None):
+        """aceso_expand: device candidates (base + patches, uint8 view of aceso_cand rows) ->
+        (tiled codes, int64 headers)."""
+        n = int(cands.numel() // 56) if n is None else int(n)
+        if tiled is None:
+            tiled = self.alloc_tiled(max(n, 1))
+        if hdr is None:
+            hdr = torch.empty(max(n, 1), dtype=torch.int64, device=self._dev)
+        nb = int(bases.shape[0])
+        _check(L.load().aceso_expand(_ptr(bases), _ptr(ranks) if ranks is not None else None, nb,
+                                     self.n_ops, _ptr(cands), n, _ptr(tiled), _ptr(hdr), _stream(stream)),
+               "aceso_expand")
+        return tiled, hdr[:n]
+
     def select(self, out: Outputs, n: int | None = None, global_offset: int = 0,
                n_total: int | None = None, sel: torch.Tensor | None = None, stream=None):
         """aceso_select: argmin over an already written summary."""

@@ -17,6 +17,7 @@
 #include "aux_kernels.cuh"
 #include "common.cuh"
 #include "dedup_kernels.cuh"
+#include "expand_kernel.cuh"
 #include "eval_kernel.cuh"
 #include "event_kernel.cuh"
 
@@ -658,6 +659,23 @@ int aceso_pack_rowmajor(const uint8_t *d_rowmajor, int64_t n, int32_t n_ops, uin
   pack_kernel<<<grid, 256, 0, reinterpret_cast<cudaStream_t>(stream)>>>(d_rowmajor, n, n_ops, reinterpret_cast<uint4 *>(d_tiled), total_vec);
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return fail(ACESO_ECUDA, "pack launch: %s", cudaGetErrorString(e));
+  return ACESO_OK;
+}
+
+int aceso_expand(const uint8_t *d_bases, const uint16_t *d_ranks, int32_t n_bases, int32_t n_ops,
+                 const aceso_cand *d_cands, int64_t n, uint8_t *d_tiled, uint64_t *d_hdr,
+                 void *stream) {
+  static_assert(sizeof(aceso_patch) == 8 && sizeof(aceso_cand) == 56, "aceso_cand layout");
+  if (n < 0 || n_ops < 1 || n_ops > kMaxOps || n_bases < 1) return fail(ACESO_EINVAL, "bad sizes");
+  if (n > 0 && (!d_bases || !d_cands || !d_tiled || !d_hdr)) return fail(ACESO_EINVAL, "null argument");
+  if (((uintptr_t)d_tiled & 15) != 0 || ((uintptr_t)d_bases & 15) != 0)
+    return fail(ACESO_EINVAL, "bases / tiled output not 16-byte aligned");
+  if (n == 0) return ACESO_OK;
+  const int grid = (int)std::max<int64_t>(1, std::min<int64_t>((n + 255) / 256, 148 * 16));
+  expand_kernel<<<grid, 256, 0, reinterpret_cast<cudaStream_t>(stream)>>>(
+      d_bases, d_ranks, n_bases, n_ops, d_cands, n, reinterpret_cast<uint4 *>(d_tiled), d_hdr);
+  cudaError_t e = cudaGetLastError();
+  if (e != cudaSuccess) return fail(ACESO_ECUDA, "expand launch: %s", cudaGetErrorString(e));
   return ACESO_OK;
 }
 
