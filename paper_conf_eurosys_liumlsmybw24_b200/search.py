@@ -290,6 +290,126 @@ class Primitives:
         return out
 
 
+    def describe_all(self, codes, mbs, info, comp, comm, stage_time):
+        """The candidates of apply_all, in the same order, as base + patches
+        (candidates.CAND_DTYPE rows with base = 0) plus the two rank rows of this base
+        used by the recompute patches. Nothing is materialised on the host."""
+        from . import candidates as C
+        prof = self.prof
+        L = len(codes)
+        heads, ends = stages_of(codes)
+        p = len(heads)
+        bn = int(info & 0xFF)
+        if bn >= p:
+            bn = 0
+        oom = bool(info & INFO_OOM)
+        if oom:
+            want = {"mem"}
+        else:
+            cs, ms = max(int(comp[:p].sum()), 1), max(int(comm[:p].sum()), 1)
+            want = {"comp"} if comp[bn] / cs >= comm[bn] / ms else {"comm"}
+        if not self.heuristic2:
+            want = {"mem", "comp", "comm"}
+        out = []
+
+        def emit(m, patches):
+            out.append((int(m), patches))
+        a, e = int(heads[bn]), int(ends[bn])
+        size = e - a
+        kmax = size - 1 if self.max_k is None else min(size - 1, self.max_k)
+        idle = int(np.argmin(stage_time[:p])) if p > 1 else bn
+        for k in range(1, kmax + 1):
+            if bn > 0 and k < size:  # _move_front(codes, bn, k)
+                pf = [C.mask(a, a + k, 0x10, int(codes[a - 1]) & 0xEE), C.mask(a + k, a + k + 1, 0xFE, 1)]
+                emit(mbs, pf)
+                if idle < bn - 1:  # relay: stage bn-1 = [heads[bn-1], a + k) after the move
+                    a2 = int(heads[bn - 1])
+                    emit(mbs, pf + [C.mask(a2, a2 + k, 0x10, int(codes[a2 - 1]) & 0xEE),
+                                    C.mask(a2 + k, a2 + k + 1, 0xFE, 1)])
+            if bn < p - 1 and k < size:  # _move_back(codes, bn, k)
+                pb = [C.mask(e, e + 1, 0xFE, 0), C.mask(e - k, e, 0x10, int(codes[e]) & 0xEE),
+                      C.mask(e - k, e - k + 1, 0xFF, 1)]
+                emit(mbs, pb)
+                if idle > bn + 1:  # relay: stage bn+1 = [heads[bn+1] - k, ends[bn+1])
+                    e2 = int(ends[bn + 1])
+                    emit(mbs, pb + [C.mask(e2, e2 + 1, 0xFE, 0), C.mask(e2 - k, e2, 0x10, int(codes[e2]) & 0xEE),
+                                    C.mask(e2 - k, e2 - k + 1, 0xFF, 1)])
+        log2bg = int(math.log2(prof.global_batch & -prof.global_batch))
+        dpl_all = ((codes >> 5) & 7).astype(np.int16)
+        tpl_all = ((codes >> 1) & 7).astype(np.int16)
+        dmax = int(dpl_all.max())
+        if ("mem" in want or "comm" in want) and mbs - 1 >= dmax:
+            emit(mbs - 1, [])
+        if ("comp" in want) and mbs + 1 <= log2bg:
+            emit(mbs + 1, [])
+
+        def stage_ok(sg, dt, dd):
+            x, y = int(heads[sg]), int(ends[sg])
+            t, d = tpl_all[x:y], dpl_all[x:y]
+            return t.min() + dt >= 0 and t.max() + dt <= 7 and d.min() + dd >= 0 and d.max() + dd <= 7
+
+        def dmax_after(changes):  # max dp field after per-stage shifts {stage: dd}
+            m = 0
+            for sg in range(p):
+                x, y = int(heads[sg]), int(ends[sg])
+                m = max(m, int(dpl_all[x:y].max()) + changes.get(sg, 0))
+            return m
+        for dt in (1, -1):
+            if stage_ok(bn, dt, -dt):
+                emit(max(mbs, dmax_after({bn: -dt})), [C.add(a, e, dt, -dt)])
+        kb = ((int(codes[heads[bn]]) >> 1) & 7) + ((int(codes[heads[bn]]) >> 5) & 7)
+        for q in range(p):
+            if q == bn:
+                continue
+            kq = ((int(codes[heads[q]]) >> 1) & 7) + ((int(codes[heads[q]]) >> 5) & 7)
+            trades = []
+            if kq == kb + 1 and ("comp" in want or "mem" in want):
+                trades = [(dtb, ddb, dtq, ddq) for dtb, ddb in ((1, 0), (0, 1)) for dtq, ddq in ((-1, 0), (0, -1))]
+            if kq + 1 == kb and "comm" in want:
+                trades += [(dtb, ddb, dtq, ddq) for dtb, ddb in ((-1, 0), (0, -1)) for dtq, ddq in ((1, 0), (0, 1))]
+            for dtb, ddb, dtq, ddq in trades:
+                if stage_ok(bn, dtb, ddb) and stage_ok(q, dtq, ddq):
+                    qa, qe = int(heads[q]), int(ends[q])
+                    emit(max(mbs, dmax_after({bn: ddb, q: ddq})), [C.add(a, e, dtb, ddb), C.add(qa, qe, dtq, ddq)])
+        stride = C.stride_of(L)
+        ranks = np.full((2, stride), 0xFFFF, np.uint16)
+        order = _rc_order(prof, codes, bn, mbs, (heads, ends))
+        rc = (codes[order] >> 4) & 1
+        if "mem" in want:
+            todo = order[rc == 0]
+            ranks[0, todo] = np.arange(len(todo), dtype=np.uint16)
+            for k in range(1, len(todo) + 1):
+                emit(mbs, [C.rank_rc(a, e, k, 0, False)])
+        if "comp" in want:
+            have = order[rc == 1][::-1]
+            ranks[1, have] = np.arange(len(have), dtype=np.uint16)
+            for k in range(1, len(have) + 1):
+                emit(mbs, [C.rank_rc(a, e, k, 1, True)])
+        if e - a > 1:
+            tp, dp = tpl_all[a:e], dpl_all[a:e]
+            tmin, tmax = np.minimum.accumulate(tp[::-1])[::-1], np.maximum.accumulate(tp[::-1])[::-1]
+            dmin, dmax_s = np.minimum.accumulate(dp[::-1])[::-1], np.maximum.accumulate(dp[::-1])[::-1]
+            dmax_pre = int(dpl_all[:a].max()) if a > 0 else 0
+            dmax_post = int(dpl_all[e:].max()) if e < L else 0
+            dmax_out = max(dmax_pre, dmax_post)
+            for j in range(a + 1, e):
+                r = j - a
+                for dt in (1, -1):
+                    if tmin[r] + dt < 0 or tmax[r] + dt > 7 or dmin[r] - dt < 0 or dmax_s[r] - dt > 7:
+                        continue
+                    dnew = max(dmax_out, int(dpl_all[a:j].max()), int(dmax_s[r] - dt))
+                    emit(max(mbs, dnew), [C.add(j, e, dt, -dt)])
+        cands = np.zeros(len(out), C.CAND_DTYPE)
+        cands["mbs"] = [m for m, _ in out]
+        cands["p"] = p
+        cands["n_patch"] = [len(pts) for _, pts in out]
+        pa = cands["patch"]
+        for i, (_, pts) in enumerate(out):
+            for j, pt in enumerate(pts):
+                pa[i, j] = pt
+        return cands, ranks
+
+
 # ---------------------------------------------------------------------------
 # evaluators
 # ---------------------------------------------------------------------------
@@ -316,13 +436,33 @@ class GPUEvaluator:
             res[k] = as_u64(getattr(out, k)).reshape(out.p_max, n).T
         return res
 
+    def evaluate_cands(self, bases, ranks, cands):
+        """Candidates as base + patches: aceso_expand -> aceso_eval (FULL) -> aceso_hash on the
+        device; only the descriptors go up (56 B each) and the results come back."""
+        from .api import as_u32, as_u64, hash_candidates
+        n = int(len(cands))
+        self.calls += 1
+        self.evaluated += n
+        dev = torch.device("cuda", self.ctx.device)
+        tb = torch.from_numpy(np.ascontiguousarray(bases)).to(dev)
+        rk = torch.from_numpy(np.ascontiguousarray(ranks).view(np.int16)).to(dev)
+        cd = torch.from_numpy(np.ascontiguousarray(cands).view(np.uint8)).to(dev)
+        tiled, hdr = self.ctx.expand(tb, cd, rk, n=n)
+        out, _ = self.ctx.eval(tiled, hdr, n=n, full=True, select=False)
+        hs = hash_candidates(tiled, hdr, self.ctx.n_ops, n=n)
+        res = dict(iter=as_u64(out.iter_ns), max_mem=as_u64(out.max_mem), info=as_u32(out.info),
+                   hash=hs.cpu().numpy().view(np.uint64))
+        for k in ["stage_T", "stage_mem", "stage_comp", "stage_comm"]:
+            res[k] = as_u64(getattr(out, k)).reshape(out.p_max, n).T
+        return res
+
 
 # ---------------------------------------------------------------------------
 # Alg. 1 / Alg. 2, batched
 # ---------------------------------------------------------------------------
 @dataclasses.dataclass
 class _Node:
-    codes: np.ndarray
+    key: int            # configuration hash (aceso_hash)
     mbs: int
     perf: tuple
     info: int
@@ -331,6 +471,19 @@ class _Node:
     time: np.ndarray
     iter_ns: int
     max_mem: int
+    src: tuple          # (base row, rank rows, descriptor, n_ops): materialised on demand
+    _codes: np.ndarray | None = None
+
+    @property
+    def codes(self):
+        if self._codes is None:
+            from . import candidates as C
+            base, ranks, cand, L = self.src
+            one = np.array([cand])
+            one["base"] = 0  # the single base row passed below
+            c, _ = C.expand_host(base[None], ranks[None], one, L)
+            self._codes = c[0]
+        return self._codes
 
 
 class _Search:
@@ -349,32 +502,45 @@ class _Search:
 
 def search(prof, evaluator, p_values=None, budget_s=10.0, max_hops=7, beam=4, heuristic2=True,
            max_batch=200000, max_k=None, patience=None):
-    """Runs the batched Aceso search. Returns (best Result, stats dict)."""
+    """Runs the batched Aceso search. Returns (best Result, stats dict).
+
+    Every hop's candidates are generated as base + patches (Primitives.describe_all) and
+    evaluated by `evaluator.evaluate_cands(bases, ranks, cands)`, which also returns each
+    candidate's configuration hash; configurations are deduplicated by hash in
+    generation order, and only the ones the search keeps are materialised on the host."""
+    from . import candidates as C
     t0 = time.perf_counter()
+    L = prof.n_ops
+    stride = C.stride_of(L)
     prims = Primitives(prof, heuristic2=heuristic2, max_k=max_k)
     if p_values is None:
         p_values = [p for p in (1, 2, 3, 4, 6, 8, 12, 16, 24, 32, 48, 64) if p <= min(prof.n_devices, prof.n_ops)]
     visited = set()
-    # initial configurations, one search per stage count (P:L276)
     init = []
     for p in p_values:
         r = initial_config(prof, p)
         if r is not None:
             init.append(r)
-    codes = np.stack([c for c, _ in init])
-    mbs = np.array([m for _, m in init])
-    res = evaluator.evaluate(codes, np.array([header(int(m), int((c & 1).sum())) for c, m in init], np.uint64))
+    bases = np.zeros((len(init), stride), np.uint8)
+    ranks = np.full((len(init), 2, stride), 0xFFFF, np.uint16)
+    cands = np.zeros(len(init), C.CAND_DTYPE)
+    for i, (c, m) in enumerate(init):
+        bases[i, :L] = c
+        cands[i]["base"], cands[i]["mbs"], cands[i]["p"] = i, m, int((c & 1).sum())
+    res = evaluator.evaluate_cands(bases, ranks, cands)
 
-    def node(i, cds, mb, r):
+    def node(i, r, base_row, rank_rows, cand):
         info = int(r["info"][i])
-        return _Node(cds, int(mb), perf_of(info, r["iter"][i], r["max_mem"][i]), info,
-                     r["stage_comp"][i], r["stage_comm"][i], r["stage_T"][i], int(r["iter"][i]),
-                     int(r["max_mem"][i]))
+        nd = _Node(int(r["hash"][i]), int(cand["mbs"]), perf_of(info, r["iter"][i], r["max_mem"][i]), info,
+                   r["stage_comp"][i], r["stage_comm"][i], r["stage_T"][i], int(r["iter"][i]),
+                   int(r["max_mem"][i]), (base_row, rank_rows, cand, L))
+        return nd
 
     searches = []
     for i in range(len(init)):
-        n0 = node(i, codes[i], mbs[i], res)
-        visited.add((codes[i].tobytes(), int(mbs[i])))
+        n0 = node(i, res, bases[i], ranks[i], cands[i])
+        n0._codes = init[i][0]
+        visited.add(n0.key)
         searches.append(_Search(n0))
     best = min((s.best for s in searches), key=lambda n: n.perf)
     t_best = time.perf_counter() - t0
@@ -383,36 +549,45 @@ def search(prof, evaluator, p_values=None, budget_s=10.0, max_hops=7, beam=4, he
     history = [(t_best, best.perf)]
     stale = 0
     while time.perf_counter() - t0 < budget_s and any(not s.done for s in searches):
-        # one hop of every active search, generated into one batch
-        owners, cand_codes, cand_mbs = [], [], []
+        # one hop of every active search, generated into one batch of descriptors
+        owners, chunks, base_rows, rank_rows = [], [], [], []
+        total = 0
         for si, s in enumerate(searches):
             if s.done:
                 continue
             for nd in s.frontier:
-                if nd.perf[0] == 2:
+                if nd.perf[0] == 2 or total >= max_batch:
                     continue
-                for c, m in prims.apply_all(nd.codes, nd.mbs, nd.info, nd.comp, nd.comm, nd.time):
-                    key = (c.tobytes(), int(m))
-                    if key in visited:
-                        continue
-                    visited.add(key)
-                    owners.append(si)
-                    cand_codes.append(c)
-                    cand_mbs.append(m)
-                    if len(cand_codes) >= max_batch:
-                        break
-        if not cand_codes:
+                cd, rk = prims.describe_all(nd.codes, nd.mbs, nd.info, nd.comp, nd.comm, nd.time)
+                if len(cd) == 0:
+                    continue
+                cd = cd[: max_batch - total]
+                cd["base"] = len(base_rows)
+                row = np.zeros(stride, np.uint8)
+                row[:L] = nd.codes
+                base_rows.append(row)
+                rank_rows.append(rk)
+                chunks.append(cd)
+                owners.extend([si] * len(cd))
+                total += len(cd)
+        if not chunks:
             for s in searches:
                 s.done = True
             break
-        cc = np.stack(cand_codes)
-        hdr = np.array([header(int(m), int((c & 1).sum())) for c, m in zip(cand_codes, cand_mbs)], np.uint64)
-        r = evaluator.evaluate(cc, hdr)
+        bases = np.stack(base_rows)
+        ranks = np.stack(rank_rows)
+        cands = np.concatenate(chunks)
+        r = evaluator.evaluate_cands(bases, ranks, cands)
         batches += 1
-        evaluated += len(cand_codes)
+        evaluated += len(cands)
         per = {}
         for i, si in enumerate(owners):
-            per.setdefault(si, []).append(node(i, cc[i], cand_mbs[i], r))
+            h = int(r["hash"][i])
+            if h in visited:  # an explored configuration (or an earlier one of this batch)
+                continue
+            visited.add(h)
+            b = int(cands[i]["base"])
+            per.setdefault(si, []).append(node(i, r, bases[b], ranks[b], cands[i]))
         improved_any = False
         for si, s in enumerate(searches):
             if s.done:
@@ -420,7 +595,7 @@ def search(prof, evaluator, p_values=None, budget_s=10.0, max_hops=7, beam=4, he
             new = per.get(si, [])
             new.sort(key=lambda n: n.perf)  # Heuristic-2: best estimated performance first
             for nd in new:
-                s.unexplored[(nd.codes.tobytes(), nd.mbs)] = nd
+                s.unexplored[nd.key] = nd
             if new and new[0].perf < s.init_perf:
                 # Alg. 2 returns the improved configuration; Alg. 1 restarts from it
                 s.cur = new[0]
@@ -430,7 +605,7 @@ def search(prof, evaluator, p_values=None, budget_s=10.0, max_hops=7, beam=4, he
                 s.frontier = [new[0]]
                 s.hop = 0
                 s.improvements += 1
-                s.unexplored.pop((new[0].codes.tobytes(), new[0].mbs), None)
+                s.unexplored.pop(new[0].key, None)
                 improved_any = True
                 continue
             s.hop += 1
@@ -457,8 +632,8 @@ def search(prof, evaluator, p_values=None, budget_s=10.0, max_hops=7, beam=4, he
             stale += 1
         if patience is not None and stale >= patience:
             break
-    total = time.perf_counter() - t0
-    stats = dict(time_s=total, time_to_best_s=t_best, batches=batches, evaluated=evaluated,
+    total_t = time.perf_counter() - t0
+    stats = dict(time_s=total_t, time_to_best_s=t_best, batches=batches, evaluated=evaluated,
                  searches=len(searches), history=history,
                  improvements=sum(s.improvements for s in searches))
     return Result(best.codes, best.mbs, best.perf, best.iter_ns, best.max_mem, best.info), stats

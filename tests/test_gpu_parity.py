@@ -372,15 +372,15 @@ def test_nccl_allreduce_min_single_rank():
 def test_search_driver_gpu_matches_oracle_trajectory():
     """The batched search (Alg. 1/2) driven by aceso_eval follows exactly the trajectory
     of the same search driven by the oracle (bit-exact evaluations)."""
+    import os
+    import sys
     from paper_conf_eurosys_liumlsmybw24_b200 import search as S
-
-    class OracleEvaluator:
-        def evaluate(self, codes, hdr):
-            return oracle.evaluate(prof, codes, hdr, full=True, threads=8)
+    sys.path.insert(0, os.path.dirname(__file__))
+    from oracle_evaluator import OracleEvaluator
 
     prof = P.WORKLOADS["gpt3-1.3b"]()
     kw = dict(p_values=[2, 4, 8], budget_s=120, max_hops=3, beam=2, max_k=8, patience=3)
     rg, sg = S.search(prof, S.GPUEvaluator(ctx_for(prof)), **kw)
-    ro, so = S.search(prof, OracleEvaluator(), **kw)
+    ro, so = S.search(prof, OracleEvaluator(prof), **kw)
     assert rg.perf == ro.perf and rg.mbs == ro.mbs and np.array_equal(rg.codes, ro.codes)
     assert sg["evaluated"] == so["evaluated"] and sg["batches"] == so["batches"]

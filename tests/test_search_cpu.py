@@ -9,14 +9,11 @@ from aceso_inputs import profiles as P
 from paper_conf_eurosys_liumlsmybw24_b200 import search as S
 
 
-class OracleEvaluator:
-    def __init__(self, prof):
-        self.prof = prof
-        self.evaluated = 0
+import os  # noqa: E402
+import sys  # noqa: E402
 
-    def evaluate(self, codes, hdr):
-        self.evaluated += len(hdr)
-        return oracle.evaluate(self.prof, codes, hdr, full=True, threads=8)
+sys.path.insert(0, os.path.dirname(__file__))
+from oracle_evaluator import OracleEvaluator  # noqa: E402
 
 
 def perf_tuple(out, i):
@@ -114,4 +111,43 @@ def test_optimised_primitives_match_reference(name):
             for (ca, ma), (cb, mb) in zip(a, b):
                 assert ma == mb and np.array_equal(ca, cb)
             checked += len(a)
+    assert checked > 500
+
+
+@pytest.mark.parametrize("name", ["gpt3-1.3b", "t5", "wrn", "toy-b"])
+def test_descriptors_expand_to_the_reference_candidates(name):
+    """Primitives.describe_all (base + patches, evaluated after aceso_expand) expands to
+    exactly the candidates of the reference generator, in the same order."""
+    import importlib.util
+    import os
+    from paper_conf_eurosys_liumlsmybw24_b200 import candidates as C
+    spec = importlib.util.spec_from_file_location(
+        "_search_reference", os.path.join(os.path.dirname(__file__), "_search_reference.py"))
+    R = importlib.util.module_from_spec(spec)
+    spec.loader.exec_module(R)
+    prof = P.WORKLOADS[name]()
+    codes, hdr = ai.search_shaped(prof, 98, 0, 60, group_size=8)
+    o = oracle.evaluate(prof, codes, hdr)
+    rng = np.random.default_rng(5)
+    checked = 0
+    L = prof.n_ops
+    for i in np.nonzero((o["info"] & oracle.INFO_INVALID) == 0)[0][:20]:
+        c, mbs = codes[i], int(hdr[i] & 0xFF)
+        p = int((c & 1).sum())
+        G = prof.n_devices
+        for h2, oom, mk in [(True, False, None), (True, True, 5), (False, False, 3)]:
+            info = int(rng.integers(0, p)) | (S.INFO_OOM if oom else 0)
+            comp = rng.integers(1, 1000, size=G).astype(np.uint64)
+            comm = rng.integers(1, 1000, size=G).astype(np.uint64)
+            stt = rng.integers(1, 1000, size=G).astype(np.uint64)
+            ref = R.PrimitivesReference(prof, heuristic2=h2, max_k=mk).apply_all(c, mbs, info, comp, comm, stt)
+            cands, ranks = S.Primitives(prof, heuristic2=h2, max_k=mk).describe_all(c, mbs, info, comp, comm, stt)
+            assert len(cands) == len(ref)
+            bases = np.zeros((1, C.stride_of(L)), np.uint8)
+            bases[0, :L] = c
+            got, ghdr = C.expand_host(bases, ranks[None], cands, L)
+            for k, (cr, mr) in enumerate(ref):
+                assert np.array_equal(got[k], cr), (k, cands[k])
+                assert int(ghdr[k] & np.uint64(0xFF)) == mr and int(ghdr[k] >> np.uint64(8)) == p
+            checked += len(ref)
     assert checked > 500
