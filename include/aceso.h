@@ -279,6 +279,21 @@ int aceso_expand(const uint8_t *d_bases, const uint16_t *d_ranks, int32_t n_base
                  const aceso_cand *d_cands, int64_t n, uint8_t *d_tiled, uint64_t *d_hdr,
                  void *stream);
 
+/* Incremental evaluation ("re-reduce only the touched
+ * stages"): same outputs, flags and select semantics as aceso_eval for the
+ * candidates of aceso_expand, without expanding them. d_base_hdr: [n_bases]
+ * headers of the bases. The bases are evaluated once into d_work (per-stage
+ * sums, an op -> stage map); each candidate then re-walks only the ops of the
+ * stages its patch ranges [a-1, b) touch and takes every other stage from the
+ * cache. Candidates whose microbatch or stage count differ from their base's,
+ * or whose base is invalid or has more than 64 stages, are walked over all ops.
+ * ACESO_HINT_DENSE is ignored. Two launches on `stream`. */
+size_t aceso_incr_work_bytes(const aceso_ctx *ctx, int32_t n_bases);
+int aceso_eval_incr(aceso_ctx *ctx, const uint8_t *d_bases, const uint64_t *d_base_hdr,
+                    const uint16_t *d_ranks, int32_t n_bases, const aceso_cand *d_cands, int64_t n,
+                    int64_t global_offset, int64_t n_total, uint32_t flags,
+                    const aceso_eval_out *out, void *d_sel, void *d_work, void *stream);
+
 /* ------------------------------------------------------------------------- */
 /* Configuration dedup ("skip configurations     */
 /* already explored"). The encoding above is canonical (one byte per op plus   */

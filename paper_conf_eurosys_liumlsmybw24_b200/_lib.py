@@ -14,7 +14,7 @@ INFO_INVALID = 1 << 17
 
 SYMBOLS = ["aceso_load_profile", "aceso_free", "aceso_tiled_bytes", "aceso_pack_rowmajor",
            "aceso_select_buf_bytes", "aceso_eval", "aceso_select", "aceso_decode_key",
-           "aceso_last_error", "aceso_version", "aceso_hash", "aceso_visited_bytes", "aceso_dedup", "aceso_expand"]
+           "aceso_last_error", "aceso_version", "aceso_hash", "aceso_visited_bytes", "aceso_dedup", "aceso_expand", "aceso_incr_work_bytes", "aceso_eval_incr"]
 
 
 class ProfileDesc(ctypes.Structure):
@@ -73,5 +73,10 @@ def load():
     lib.aceso_dedup.restype = ctypes.c_int
     lib.aceso_expand.argtypes = [P, P, c_i32, c_i32, P, c_i64, P, P, P]
     lib.aceso_expand.restype = ctypes.c_int
+    lib.aceso_incr_work_bytes.argtypes = [P, c_i32]
+    lib.aceso_incr_work_bytes.restype = c_sz
+    lib.aceso_eval_incr.argtypes = [P, P, P, P, c_i32, P, c_i64, c_i64, c_i64, c_u32, ctypes.POINTER(EvalOut),
+                                    P, P, P]
+    lib.aceso_eval_incr.restype = ctypes.c_int
     _lib = lib
     return lib

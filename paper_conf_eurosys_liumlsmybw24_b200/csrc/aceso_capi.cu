@@ -18,6 +18,7 @@
 #include "common.cuh"
 #include "dedup_kernels.cuh"
 #include "expand_kernel.cuh"
+#include "incr_kernel.cuh"
 #include "eval_kernel.cuh"
 #include "event_kernel.cuh"
 
@@ -112,6 +113,56 @@ struct aceso_ctx {
   int max_ctas[2][8];  // per kernel and mode: resident CTAs (occupancy x SMs)
   size_t smem[2][8];
 };
+
+namespace {
+template <uint32_t M>
+void *incr_kernel_ptr() { return reinterpret_cast<void *>(&incr_kernel<M>); }
+
+// kernel parameter block of a call (tables, outputs, selection); codes/hdr set by the caller
+EvalParams make_params(const aceso_ctx *ctx, int64_t n, int64_t global_offset, int64_t n_total,
+                       const aceso_eval_out *out, void *d_sel) {
+  EvalParams P;
+  memset(&P, 0, sizeof(P));
+  P.n = n;
+  P.gofs = global_offset;
+  P.n_tiles = (n + 31) / 32;
+  P.L = ctx->L;
+  P.nch = (ctx->L + 15) / 16;
+  P.T = ctx->T;
+  P.n_tp = ctx->n_tp;
+  P.n_dp = ctx->n_dp;
+  P.n_b = ctx->n_b;
+  P.G = ctx->G;
+  P.Bg = ctx->Bg;
+  P.C = ctx->C;
+  P.mem_shift = ctx->mem_shift;
+  P.blob = reinterpret_cast<const uint4 *>(ctx->d_blob);
+  P.tab = ctx->tab;
+  if (out) {
+    P.iter_ns = out->iter_ns;
+    P.max_mem = out->max_mem;
+    P.info = out->info;
+    P.stage_T = out->stage_T;
+    P.stage_mem = out->stage_mem;
+    P.stage_comp = out->stage_comp;
+    P.stage_comm = out->stage_comm;
+    P.p_max = out->p_max;
+  }
+  P.sel = reinterpret_cast<unsigned char *>(d_sel);
+  P.n_total = n_total;
+  P.ib = std::max(1u, bitlen((uint64_t)n_total));
+  P.px = ctx->px;
+  P.kx = ctx->kx;
+  P.pd = ctx->pd;
+  P.st = ctx->st;
+  P.qr = ctx->qr;
+  P.runs = (uint32_t)(ctx->n_b * ctx->n_tp);
+  P.qo_bytes = ctx->qo_bytes;
+  P.qo_off = ctx->qo_off;
+  P.evblob = reinterpret_cast<const unsigned char *>(ctx->d_ev);
+  return P;
+}
+}  // namespace
 
 extern "C" {
 
@@ -557,47 +608,9 @@ int aceso_eval(aceso_ctx *ctx, const uint8_t *d_codes, const uint64_t *d_hdr, in
   if ((mode & ACESO_FUSED_SELECT) && !d_sel) return fail(ACESO_EINVAL, "null select buffer");
   if (((uintptr_t)d_codes & 15) != 0) return fail(ACESO_EINVAL, "codes not 16-byte aligned");
 
-  EvalParams P;
-  memset(&P, 0, sizeof(P));
+  EvalParams P = make_params(ctx, n, global_offset, n_total, out, d_sel);
   P.codes = reinterpret_cast<const uint4 *>(d_codes);
   P.hdr = d_hdr;
-  P.n = n;
-  P.gofs = global_offset;
-  P.n_tiles = (n + 31) / 32;
-  P.L = ctx->L;
-  P.nch = (ctx->L + 15) / 16;
-  P.T = ctx->T;
-  P.n_tp = ctx->n_tp;
-  P.n_dp = ctx->n_dp;
-  P.n_b = ctx->n_b;
-  P.G = ctx->G;
-  P.Bg = ctx->Bg;
-  P.C = ctx->C;
-  P.mem_shift = ctx->mem_shift;
-  P.blob = reinterpret_cast<const uint4 *>(ctx->d_blob);
-  P.tab = ctx->tab;
-  if (out) {
-    P.iter_ns = out->iter_ns;
-    P.max_mem = out->max_mem;
-    P.info = out->info;
-    P.stage_T = out->stage_T;
-    P.stage_mem = out->stage_mem;
-    P.stage_comp = out->stage_comp;
-    P.stage_comm = out->stage_comm;
-    P.p_max = out->p_max;
-  }
-  P.sel = reinterpret_cast<unsigned char *>(d_sel);
-  P.n_total = n_total;
-  P.ib = std::max(1u, bitlen((uint64_t)n_total));
-  P.px = ctx->px;
-  P.kx = ctx->kx;
-  P.pd = ctx->pd;
-  P.st = ctx->st;
-  P.qr = ctx->qr;
-  P.runs = (uint32_t)(ctx->n_b * ctx->n_tp);
-  P.qo_bytes = ctx->qo_bytes;
-  P.qo_off = ctx->qo_off;
-  P.evblob = reinterpret_cast<const unsigned char *>(ctx->d_ev);
 
   const int tiles_per_cta = kern == 1 ? kWarps : kWarps / ctx->split;
   const int64_t need = (P.n_tiles + tiles_per_cta - 1) / tiles_per_cta;
@@ -659,6 +672,65 @@ int aceso_pack_rowmajor(const uint8_t *d_rowmajor, int64_t n, int32_t n_ops, uin
   pack_kernel<<<grid, 256, 0, reinterpret_cast<cudaStream_t>(stream)>>>(d_rowmajor, n, n_ops, reinterpret_cast<uint4 *>(d_tiled), total_vec);
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return fail(ACESO_ECUDA, "pack launch: %s", cudaGetErrorString(e));
+  return ACESO_OK;
+}
+
+size_t aceso_incr_work_bytes(const aceso_ctx *ctx, int32_t n_bases) {
+  if (!ctx || n_bases < 1) return 0;
+  auto al = [](size_t v) { return (v + 255) & ~(size_t)255; };
+  return al((size_t)n_bases * sizeof(IncrBaseHdr)) + al((size_t)n_bases * ctx->G * sizeof(IncrBaseStage)) +
+         al((size_t)n_bases * ctx->L);
+}
+
+int aceso_eval_incr(aceso_ctx *ctx, const uint8_t *d_bases, const uint64_t *d_base_hdr,
+                    const uint16_t *d_ranks, int32_t n_bases, const aceso_cand *d_cands, int64_t n,
+                    int64_t global_offset, int64_t n_total, uint32_t flags,
+                    const aceso_eval_out *out, void *d_sel, void *d_work, void *stream) {
+  if (!ctx) return fail(ACESO_EINVAL, "null context");
+  if (n < 0 || global_offset < 0 || n_total < global_offset + n) return fail(ACESO_EINVAL, "bad n / global_offset / n_total");
+  if (n_total >= (1ll << 40)) return fail(ACESO_EINVAL, "n_total >= 2^40");
+  const uint32_t mode = flags & 7u;
+  if (mode == 0 || (flags & ~(7u | ACESO_HINT_DENSE))) return fail(ACESO_EINVAL, "bad flags 0x%x", flags);
+  if (n_bases < 1 || !d_bases || !d_base_hdr || !d_work || (n > 0 && !d_cands)) return fail(ACESO_EINVAL, "null argument");
+  if ((mode & (ACESO_OUT_SUMMARY | ACESO_OUT_FULL)) && !out) return fail(ACESO_EINVAL, "null outputs");
+  if ((mode & ACESO_OUT_SUMMARY) && n > 0 && (!out->iter_ns || !out->max_mem || !out->info)) return fail(ACESO_EINVAL, "null summary array");
+  if (mode & ACESO_OUT_FULL) {
+    if (out->p_max < ctx->G) return fail(ACESO_EINVAL, "p_max %d < n_devices %d", out->p_max, ctx->G);
+    if (n > 0 && (!out->stage_T || !out->stage_mem || !out->stage_comp || !out->stage_comm)) return fail(ACESO_EINVAL, "null stage array");
+  }
+  if ((mode & ACESO_FUSED_SELECT) && !d_sel) return fail(ACESO_EINVAL, "null select buffer");
+  EvalParams P = make_params(ctx, n, global_offset, n_total, out, d_sel);
+  auto al = [](size_t v) { return (v + 255) & ~(size_t)255; };
+  unsigned char *w = reinterpret_cast<unsigned char *>(d_work);
+  IncrBaseHdr *hdrs = reinterpret_cast<IncrBaseHdr *>(w);
+  IncrBaseStage *stages = reinterpret_cast<IncrBaseStage *>(w + al((size_t)n_bases * sizeof(IncrBaseHdr)));
+  uint8_t *smap = w + al((size_t)n_bases * sizeof(IncrBaseHdr)) + al((size_t)n_bases * ctx->G * sizeof(IncrBaseStage));
+  int prev = 0;
+  CUDA_TRY(cudaGetDevice(&prev));
+  if (prev != ctx->device) CUDA_TRY(cudaSetDevice(ctx->device));
+  cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
+  base_cache_kernel<<<(n_bases + 127) / 128, 128, 0, st>>>(P, d_bases, d_base_hdr, n_bases, hdrs, stages, smap);
+  void *k = nullptr;
+  switch (mode) {
+    case 1: k = incr_kernel_ptr<1>(); break;
+    case 2: k = incr_kernel_ptr<2>(); break;
+    case 3: k = incr_kernel_ptr<3>(); break;
+    case 4: k = incr_kernel_ptr<4>(); break;
+    case 5: k = incr_kernel_ptr<5>(); break;
+    case 6: k = incr_kernel_ptr<6>(); break;
+    default: k = incr_kernel_ptr<7>(); break;
+  }
+  const int grid = (int)std::max<int64_t>(1, std::min<int64_t>((n + 255) / 256, (int64_t)ctx->sms * 8));
+  const uint8_t *b = d_bases;
+  const uint16_t *r = d_ranks;
+  const IncrBaseHdr *ch = hdrs;
+  const IncrBaseStage *cs = stages;
+  const uint8_t *cm = smap;
+  void *args[] = {&P, &b, &r, &n_bases, &d_cands, &ch, &cs, &cm};
+  cudaError_t e = cudaLaunchKernel(k, dim3(grid), dim3(256), args, 0, st);
+  if (e == cudaSuccess) e = cudaGetLastError();
+  if (prev != ctx->device) cudaSetDevice(prev);
+  if (e != cudaSuccess) return fail(ACESO_ECUDA, "incremental eval launch: %s", cudaGetErrorString(e));
   return ACESO_OK;
 }
 
