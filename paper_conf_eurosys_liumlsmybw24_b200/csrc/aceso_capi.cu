@@ -542,7 +542,7 @@ int aceso_load_profile(const aceso_profile_desc *d, int cuda_device, aceso_ctx *
         }
         const size_t smem =
             kern == 1
-                ? (size_t)qo_bytes + ev_ring_bytes() + ev_list_bytes() + ev_snap_bytes(mode & ACESO_OUT_FULL)
+                ? (size_t)qo_bytes + ev_ring_bytes() + ev_list_bytes((mode & ACESO_OUT_FULL) != 0)
                 : ((mode & ACESO_OUT_FULL) ? tab.bytes_full : tab.bytes) + (tab.k_smem ? bytesK : 0u) +
                       kRingBytesPerCta + (ctx->split == 2 ? (size_t)(kWarps / 2) * 32 * sizeof(Xchg) : 0);
         ctx->smem[kern][mode] = smem;
