@@ -221,7 +221,8 @@ size_t aceso_select_buf_bytes(const aceso_ctx *ctx, int64_t n);
  *   d_sel   : select buffer (device), required with ACESO_FUSED_SELECT
  *   stream  : cudaStream_t
  * Asynchronous; no allocation, no host synchronisation. n == 0 is valid (the
- * select result becomes "nothing valid"). */
+ * select result becomes "nothing valid"). ACESO_EINVAL if n >= 2^37 or
+ * n_total >= 2^40 (far beyond device memory at one byte per op). */
 int aceso_eval(aceso_ctx *ctx, const uint8_t *d_codes, const uint64_t *d_hdr, int64_t n,
                int64_t global_offset, int64_t n_total, uint32_t flags,
                const aceso_eval_out *out, void *d_sel, void *stream);

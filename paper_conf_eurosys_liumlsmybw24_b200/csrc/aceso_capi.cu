@@ -595,6 +595,7 @@ int aceso_eval(aceso_ctx *ctx, const uint8_t *d_codes, const uint64_t *d_hdr, in
   if (!ctx) return fail(ACESO_EINVAL, "null context");
   if (n < 0 || global_offset < 0 || n_total < global_offset + n) return fail(ACESO_EINVAL, "bad n / global_offset / n_total");
   if (n_total >= (1ll << 40)) return fail(ACESO_EINVAL, "n_total >= 2^40");
+  if (n >= (1ll << 37)) return fail(ACESO_EINVAL, "n >= 2^37");
   const uint32_t mode = flags & 7u;
   if (mode == 0 || (flags & ~(7u | ACESO_HINT_DENSE))) return fail(ACESO_EINVAL, "bad flags 0x%x", flags);
   const int kern = ((flags & ACESO_HINT_DENSE) && ctx->quad_ok) ? 0 : ctx->kernel;

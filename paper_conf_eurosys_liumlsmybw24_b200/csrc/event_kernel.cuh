@@ -359,12 +359,14 @@ __global__ void __launch_bounds__(kThreads, MINB) event_kernel(const __grid_cons
 
   const uint32_t nch = (uint32_t)P.nch;
   const uint32_t ngroups = (nch + kEvSlotChunks - 1) / kEvSlotChunks;
-  const int64_t first_tile = (int64_t)blockIdx.x * kWarps + warp;
-  const int64_t tile_stride = (int64_t)gridDim.x * kWarps;
+  // tile indices fit 32 bits (aceso_eval rejects n >= 2^37)
+  const uint32_t n_tiles = (uint32_t)P.n_tiles;
+  const uint32_t first_tile = blockIdx.x * kWarps + warp;
+  const uint32_t tile_stride = gridDim.x * kWarps;
   const unsigned char *codes = reinterpret_cast<const unsigned char *>(P.codes);
 
   // producer state (lane 0): the next (tile, slot group) to copy; done when it_tile >= n_tiles
-  int64_t it_tile = first_tile;
+  uint32_t it_tile = first_tile;
   uint32_t it_g = 0;
   auto issue_next = [&](uint32_t slot) {
     const uint32_t a = kEvSlotChunks * it_g, b = min(a + kEvSlotChunks, nch);
@@ -377,7 +379,7 @@ __global__ void __launch_bounds__(kThreads, MINB) event_kernel(const __grid_cons
     }
   };
   if (lane == 0) {
-    for (uint32_t u = 0; u < (uint32_t)kEvRingSlots && it_tile < P.n_tiles; ++u) issue_next(u);
+    for (uint32_t u = 0; u < (uint32_t)kEvRingSlots && it_tile < n_tiles; ++u) issue_next(u);
   }
   __syncwarp();
   mbar_wait(smem_addr(&s_tbar), 0);
@@ -389,8 +391,8 @@ __global__ void __launch_bounds__(kThreads, MINB) event_kernel(const __grid_cons
   uint32_t rE;          // phase A: their recompute peak since the last list entry
   uint32_t slot = 0, phase = 0;
 #pragma unroll 1
-  for (int64_t tile = first_tile; tile < P.n_tiles; tile += tile_stride) {
-    const int64_t cand = tile * 32 + lane;
+  for (uint32_t tile = first_tile; tile < n_tiles; tile += tile_stride) {
+    const int64_t cand = (int64_t)tile * 32 + lane;
     const bool active = cand < P.n;
     ev_init(s, P, active ? __ldg(P.hdr + cand) : 0ull);
     cS = cA = cC = 0;
@@ -462,7 +464,7 @@ __global__ void __launch_bounds__(kThreads, MINB) event_kernel(const __grid_cons
         }
       }
       __syncwarp();
-      if (lane == 0 && it_tile < P.n_tiles) {
+      if (lane == 0 && it_tile < n_tiles) {
         fence_proxy_async();
         issue_next(slot);
       }
