@@ -80,38 +80,115 @@ __device__ __forceinline__ void sts128(uint32_t a, uint4 v) {
                : "memory");
 }
 
+// Per-candidate state. Small fields are packed (registers are the occupancy limit):
+//   run = rr | dd << 8 | cc << 16   open run: (b, tp) index (< 128), (tp, dp) index (< 64),
+//                                   code of its first op (tp/dp bits = every op of the run)
+//   fl  = bt | bm << 8 | oom << 16 | head0 << 17 | gst << 20
+//         Heuristic-1 argmax stages (low 8 bits of the index; only valid candidates, whose
+//         p <= 64, report them), any stage OOM, op 0 has a head, 2^gst devices in the open stage
+//   hd  = mbs | p << 8              header: log2 microbatch, stage count
 struct EvCand {
-  // phase B: the open stage (prefix-difference form: -PX[start] + PX[end] per run)
+  // the open stage (prefix-difference form: -PX[start] + PX[end] per run)
   uint64_t S, A, W, D, comp;
   uint32_t E;
-  uint32_t rr, dd, a;  // open run: (b, tp) index, (tp, dp) index, first op
-  uint32_t cc;         // open run: code of its first op (tp/dp bits = every op of the run)
-  uint32_t ec;         // phase A: list entries
-  // candidate-level aggregates (names shared with Cand: stage_commit / finish_cand)
+  uint32_t a;   // open run: first op
+  uint32_t run;
+  uint32_t ec;  // phase A: list entries
+  // candidate-level aggregates
   uint64_t sumS, bestT, bestM;
-  uint32_t bt, bm, oom, i, gsum, reasons, nheads, head0, gst;
-  uint32_t mbs, p, N;
+  uint32_t i;   // stages closed so far (= heads at ops > 0)
+  uint32_t gsum, reasons, N, fl, hd;
+  __device__ __forceinline__ uint32_t rr() const { return run & 0xffu; }
+  __device__ __forceinline__ uint32_t dd() const { return (run >> 8) & 0xffu; }
+  __device__ __forceinline__ uint32_t cc() const { return run >> 16; }
+  __device__ __forceinline__ uint32_t mbs() const { return hd & 0xffu; }
+  __device__ __forceinline__ uint32_t p() const { return hd >> 8; }
 };
 
 __device__ __forceinline__ void ev_init(EvCand &s, const EvalParams &P, uint64_t h) {
-  s.mbs = (uint32_t)(h & 0xff);
-  s.p = (uint32_t)((h >> 8) & 0xff);
+  const uint32_t mbs = (uint32_t)(h & 0xff), p = (uint32_t)((h >> 8) & 0xff);
+  s.hd = mbs | (p << 8);
   s.reasons = (h >> 16) ? ACESO_R_HDR : 0u;
   s.N = 0;
-  if (s.mbs >= 62 || (1ull << s.mbs) > P.Bg || (P.Bg & ((1ull << s.mbs) - 1)) != 0)
+  if (mbs >= 62 || (1ull << mbs) > P.Bg || (P.Bg & ((1ull << mbs) - 1)) != 0)
     s.reasons |= ACESO_R_MBS;
   else
-    s.N = (uint32_t)(P.Bg >> s.mbs);
-  if (s.p == 0 || s.p > (uint32_t)P.G) s.reasons |= ACESO_R_PRANGE;
+    s.N = (uint32_t)(P.Bg >> mbs);
+  if (p == 0 || p > (uint32_t)P.G) s.reasons |= ACESO_R_PRANGE;
   s.S = s.A = s.W = s.D = s.comp = 0;
   s.E = 0;
-  s.rr = s.dd = s.a = 0;
-  s.cc = 0;
+  s.a = 0;
+  s.run = 0;
   s.ec = 0;
   s.sumS = s.bestT = s.bestM = 0;
-  s.bt = s.bm = 0;
-  s.oom = s.gsum = s.nheads = s.head0 = s.gst = 0;
+  s.fl = 0;
+  s.gsum = 0;
   s.i = 0;
+}
+
+// Closes stage s.i: Eq. 2 key, Eq. 1 memory, OOM, Heuristic-1 maxima (ascending stage
+// order, strict > keeps the lowest index on ties, R11), FULL per-stage outputs.
+template <uint32_t MODE>
+__device__ __forceinline__ void ev_commit(EvCand &s, const EvalParams &P, int64_t c, bool active) {
+  s.sumS += s.S;
+  const uint64_t tk = (uint64_t)(s.N - 1) * s.S + s.D;  // T_i - sum_k S_k (Eq. 2, R1, R6)
+  const uint32_t p = s.p();
+  const uint64_t infl = p > s.i ? (uint64_t)min(p - s.i, s.N) : 0ull;  // R2
+  const uint64_t M = (s.W + infl * s.A + s.E) << P.mem_shift;         // Eq. 1 (R3, R4)
+  const uint32_t i8 = s.i & 0xffu;
+  if (tk > s.bestT) { s.bestT = tk; s.fl = (s.fl & ~0xffu) | i8; }
+  if (M > s.bestM) { s.bestM = M; s.fl = (s.fl & ~0xff00u) | (i8 << 8); }
+  if (M > P.C) s.fl |= 1u << 16;  // R10
+  if (MODE & kFull) {
+    if (active && s.i < (uint32_t)P.p_max) {
+      const int64_t o = (int64_t)s.i * P.n + c;
+      P.stage_T[o] = tk;  // + sum_k S_k in the epilogue
+      P.stage_mem[o] = M;
+      P.stage_comp[o] = (uint64_t)s.N * s.comp;
+      P.stage_comm[o] = (uint64_t)s.N * (s.S - s.comp) + s.D;
+    }
+  }
+  s.S = s.A = s.W = s.D = s.comp = 0;
+  s.E = 0;
+}
+
+// Candidate epilogue: validity, summary outputs, fused argmin (same contract as
+// finish_cand of eval_kernel.cuh).
+template <uint32_t MODE>
+__device__ __forceinline__ void ev_finish(EvCand &s, const EvalParams &P, int64_t c, bool active,
+                                          uint64_t &best_ck, int64_t &best_idx) {
+  const uint32_t head0 = (s.fl >> 17) & 1u, p = s.p();
+  uint32_t reasons = s.reasons;
+  if (!head0) reasons |= ACESO_R_HEAD0;
+  if (s.i + head0 != p) reasons |= ACESO_R_NSTAGE;  // heads = heads at ops > 0 + op 0's
+  if (s.gsum != (uint32_t)P.G) reasons |= ACESO_R_GSUM;
+  const bool invalid = reasons != 0;
+  const bool oom = (s.fl >> 16) & 1u;
+  const uint64_t iter = invalid ? 0ull : s.sumS + s.bestT;  // max_i T_i (Eq. 2)
+  const uint64_t mem = invalid ? 0ull : s.bestM;
+  uint32_t info = (p << 8);
+  if (invalid) info |= ACESO_INFO_INVALID | (reasons << 18);
+  else info |= (oom ? (((s.fl >> 8) & 0xffu) | ACESO_INFO_OOM) : (s.fl & 0xffu));  // Heuristic-1
+  if (active) {
+    if (MODE & kSummary) {
+      P.iter_ns[c] = iter;
+      P.max_mem[c] = mem;
+      P.info[c] = info;
+    }
+    if ((MODE & kFull) && !invalid) {
+      const uint32_t ns = min(p, (uint32_t)P.p_max);
+      for (uint32_t k = 0; k < ns; ++k) P.stage_T[(int64_t)k * P.n + c] += s.sumS;
+    }
+    if ((MODE & kSelect) && !invalid) {
+      // class 0 feasible (cost = iteration time), class 1 OOM (cost = max memory), R12
+      const uint64_t ck = oom ? ((1ull << 62) | mem) : iter;
+      const int64_t g = P.gofs + c;
+      if (key_less(ck, g, best_ck, best_idx)) {
+        best_ck = ck;
+        best_idx = g;
+      }
+    }
+  }
 }
 
 // recompute deltas of the ops of quad pattern pat (bit k = op 4q+k) under run rr
@@ -132,7 +209,7 @@ template <uint32_t MODE>
 __device__ __forceinline__ void ev_rc_add(EvCand &s, const EvalParams &P, uint32_t qsb, uint32_t pat) {
   uint64_t dS = 0, dA = 0, dC = 0;
   uint32_t e1 = 0;
-  ev_rc_lookup<MODE>(P, qsb, s.rr, pat, dS, dA, e1, dC);
+  ev_rc_lookup<MODE>(P, qsb, s.rr(), pat, dS, dA, e1, dC);
   s.S += dS;
   s.A -= dA;
   s.E = max(s.E, e1);
@@ -165,12 +242,13 @@ __device__ __forceinline__ uint32_t quad_activity(uint32_t w, uint32_t p) {
 template <uint32_t MODE>
 __device__ __forceinline__ void ev_close_run(EvCand &s, const EvalParams &P, uint32_t j) {
   const uint32_t Lp1 = (uint32_t)P.L + 1u;
-  const uint32_t o = s.rr * Lp1 + j;
+  const uint32_t rr = s.rr();
+  const uint32_t o = rr * Lp1 + j;
   const uint4 x0 = __ldg(P.px + 2u * o);
   const uint4 x1 = __ldg(P.px + 2u * o + 1u);
-  const uint64_t dsum = __ldg(P.pd + (s.dd * Lp1 + j));
+  const uint64_t dsum = __ldg(P.pd + (s.dd() * Lp1 + j));
   const uint32_t k = 31u - __clz(j - s.a);
-  const uint32_t *stk = P.st + ((k * (uint32_t)P.runs + s.rr) * (uint32_t)P.L);
+  const uint32_t *stk = P.st + ((k * (uint32_t)P.runs + rr) * (uint32_t)P.L);
   const uint32_t e = max(__ldg(stk + s.a), __ldg(stk + (j - (1u << k))));
   s.S += u64of(x0.x, x0.y);
   s.A += u64of(x0.z, x0.w);
@@ -201,10 +279,10 @@ __device__ __forceinline__ void ev_handle(EvCand &s, const EvalParams &P, uint32
         const uint2 x = lds64x2(xad);
         cC = u64of(x.x, x.y);
       }
-      s.S += __ldg(kx + (4u * (s.rr * Lp1 + j) + 2u)) + cS;  // R5: p2p_fwd of the stage's last op
+      s.S += __ldg(kx + (4u * (s.rr() * Lp1 + j) + 2u)) + cS;  // R5: p2p_fwd of the stage's last op
       s.A -= cA;
       if (MODE & kFull) s.comp += cC;
-      stage_commit<MODE>(s, P, cand, active, false);
+      ev_commit<MODE>(s, P, cand, active);
       s.i += 1;
       s.S -= cS;
       s.A += cA;
@@ -213,24 +291,23 @@ __device__ __forceinline__ void ev_handle(EvCand &s, const EvalParams &P, uint32
   }
   // open the run of op j: validity, table keys, p2p_bwd / reshard, prefix base
   const uint32_t tpl = (c >> 1) & 7u, dpl = c >> 5;
-  if (dpl > s.mbs) s.reasons |= ACESO_R_DPMBS;
-  if (tpl >= (uint32_t)P.n_tp || dpl >= (uint32_t)P.n_dp || (dpl <= s.mbs && s.mbs - dpl >= (uint32_t)P.n_b))
+  const uint32_t mbs = s.mbs();
+  if (dpl > mbs) s.reasons |= ACESO_R_DPMBS;
+  if (tpl >= (uint32_t)P.n_tp || dpl >= (uint32_t)P.n_dp || (dpl <= mbs && mbs - dpl >= (uint32_t)P.n_b))
     s.reasons |= ACESO_R_TABLE;
   // clamped indices keep every gather inside the tables for invalid encodings
-  const uint32_t b = min(dpl <= s.mbs ? s.mbs - dpl : 0u, (uint32_t)P.n_b - 1);
+  const uint32_t b = min(dpl <= mbs ? mbs - dpl : 0u, (uint32_t)P.n_b - 1);
   const uint32_t tplc = min(tpl, (uint32_t)P.n_tp - 1), dplc = min(dpl, (uint32_t)P.n_dp - 1);
-  s.rr = b * (uint32_t)P.n_tp + tplc;
-  s.dd = tplc * (uint32_t)P.n_dp + dplc;
-  s.cc = c;
-  const uint32_t o = s.rr * Lp1 + j;
+  const uint32_t rr = b * (uint32_t)P.n_tp + tplc;
+  s.run = rr | ((tplc * (uint32_t)P.n_dp + dplc) << 8) | (c << 16);
+  const uint32_t o = rr * Lp1 + j;
   const uint32_t g = tpl + dpl;
   if (head || j == 0) {
-    s.gst = g;
+    s.fl = (s.fl & 0xfffffu) | (g << 20);
     s.gsum += 1u << g;  // R9
-    s.nheads += head;
     if (head && j > 0) s.S += __ldg(kx + (4u * o + 1u));  // R5: p2p_bwd of the first op
   } else {
-    if (g != s.gst) s.reasons |= ACESO_R_GSTAGE;  // P:L151 in-stage symmetry
+    if (g != (s.fl >> 20)) s.reasons |= ACESO_R_GSTAGE;  // P:L151 in-stage symmetry
     s.S += __ldg(kx + 4u * o);                     // R13: reshard into this op
   }
   const uint4 y0 = __ldg(P.px + 2u * o);
@@ -239,7 +316,7 @@ __device__ __forceinline__ void ev_handle(EvCand &s, const EvalParams &P, uint32
   s.A -= u64of(y0.z, y0.w);
   s.W -= u64of(y1.x, y1.y);
   if (MODE & kFull) s.comp -= u64of(y1.z, y1.w);
-  s.D -= __ldg(P.pd + (s.dd * Lp1 + j));
+  s.D -= __ldg(P.pd + (s.dd() * Lp1 + j));
   s.a = j;
 }
 
@@ -289,7 +366,7 @@ __device__ __forceinline__ void ev_drain(EvCand &s, const EvalParams &P, uint32_
       const uint32_t j = __ffs(all) - 1u;
       if ((em >> j) & 1u) {
         // the op's code: head and rc bits as stored, tp/dp = previous op's (the open run's) ^ change
-        const uint32_t c = lds8(ent + kEvF + j) ^ (s.cc & 0xeeu);
+        const uint32_t c = lds8(ent + kEvF + j) ^ (s.cc() & 0xeeu);
         ev_handle<MODE>(s, P, 4u * q0 + j, c, ent + kEvC, xe + 8u, cand, active);
         em &= em - 1u;
       } else {
@@ -407,8 +484,8 @@ __global__ void __launch_bounds__(kThreads, MINB) event_kernel(const __grid_cons
         // seed the previous word so that op 0 always shows a tp difference (an event)
         const uint32_t w0 = lds32(addr);
         pw = ((w0 & 0xffu) ^ 0x02u) << 24;
-        s.cc = (w0 & 0xffu) ^ 0x02u;  // phase B rebuilds op 0's code against the same seed
-        s.head0 = w0 & 1u;
+        s.run = ((w0 & 0xffu) ^ 0x02u) << 16;  // phase B rebuilds op 0's code against the same seed
+        s.fl = (w0 & 1u) << 17;                 // head0
       }
       if (g == ngroups - 1u) {
         const uint32_t nvl = (uint32_t)P.L - 16u * (nch - 1u);  // valid ops of the last chunk
@@ -439,7 +516,7 @@ __global__ void __launch_bounds__(kThreads, MINB) event_kernel(const __grid_cons
             if (rcc) {
               // recompute flags in an event-free chunk: every op is in the open run, whose
               // (tp, dp) is that of op 0 of the chunk
-              const uint32_t rr = ev_run(w4.x & 0xffu, s.mbs, P);
+              const uint32_t rr = ev_run(w4.x & 0xffu, s.mbs(), P);
               const uint4 qs = lds128(qo + 16u * (ch0 + c));
               uint32_t pat;
               if ((pat = quad_rc(f.x))) ev_rc_lookup<MODE>(P, qs.x, rr, pat, cS, cA, rE, cC);
@@ -478,8 +555,8 @@ __global__ void __launch_bounds__(kThreads, MINB) event_kernel(const __grid_cons
     s.E = max(s.E, rE);
     if (MODE & kFull) s.comp += cC;
     ev_close_run<MODE>(s, P, (uint32_t)P.L);
-    stage_commit<MODE>(s, P, cand, active, false);
-    finish_cand<MODE>(s, P, cand, active, best_ck, best_idx);
+    ev_commit<MODE>(s, P, cand, active);
+    ev_finish<MODE>(s, P, cand, active, best_ck, best_idx);
   }
 
   if (MODE & kSelect) warp_select_finish(best_ck, best_idx, P.sel, P.n_total, P.ib, s_ck, s_idx, &s_done);
