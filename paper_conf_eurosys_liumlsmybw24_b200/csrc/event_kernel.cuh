@@ -464,17 +464,63 @@ __global__ void __launch_bounds__(kThreads, MINB) event_kernel(const __grid_cons
   uint64_t best_ck = ~0ull;
   int64_t best_idx = INT64_MAX;
   EvCand s;
-  uint64_t cS, cA, cC;  // phase A: cumulative recompute deltas of the tile's event-free chunks
-  uint32_t rE;          // phase A: their recompute peak since the last list entry
+  ev_init(s, P, 0ull);
+  uint64_t cS = 0, cA = 0, cC = 0;  // phase A: cumulative recompute deltas of the tile's event-free chunks
+  uint32_t rE = 0;                  // phase A: their recompute peak since the last list entry
   uint32_t slot = 0, phase = 0;
+  uint32_t pw = 0;       // phase A: the previous code word (its top byte = the previous op)
+  int64_t cand = 0;
+  bool active = false;
+  // the lists must hold what the next 2 chunks add
+  auto drain_check = [&]() {
+    if (__any_sync(0xffffffffu, s.ec + 2u > (uint32_t)kEvCap)) ev_drain<MODE>(s, P, qo, lb, lx, cand, active);
+  };
+  // phase A, one 16-op chunk (ring address a, chunk index ci)
+  auto chunk = [&](uint32_t a, uint32_t ci) {
+    const uint4 w4 = lds128(a);
+    uint4 f;
+    f.x = quad_activity(w4.x, pw);
+    f.y = quad_activity(w4.y, w4.x);
+    f.z = quad_activity(w4.z, w4.y);
+    f.w = quad_activity(w4.w, w4.z);
+    pw = w4.w;
+    const uint32_t orw = f.x | f.y | f.z | f.w;
+    const bool evc = (orw & 0xefefefefu) != 0u;
+    const bool rcc = !evc && (orw & 0x10101010u) != 0u;
+    const uint32_t k = s.ec;
+    const uint32_t e = lb + 512u * k;
+    sts128(e + kEvF, f);
+    sts128(e + kEvC, make_uint4((uint32_t)cS, (uint32_t)(cS >> 32), (uint32_t)cA, (uint32_t)(cA >> 32)));
+    if (FULL)
+      sts128(lx + 32u * XR * k, make_uint4(rE, ci, (uint32_t)cC, (uint32_t)(cC >> 32)));
+    else
+      sts64x2(lx + 32u * XR * k, rE, ci);
+    if (evc) {
+      rE = 0;
+      s.ec = k + 1u;
+    }
+    if (__any_sync(0xffffffffu, rcc)) {
+      if (rcc) {
+        // recompute flags in an event-free chunk: every op is in the open run, whose
+        // (tp, dp) is that of op 0 of the chunk
+        const uint32_t rr = ev_run(w4.x & 0xffu, s.mbs(), P);
+        const uint4 qs = lds128(qo + 16u * ci);
+        uint32_t pat;
+        if ((pat = quad_rc(f.x))) ev_rc_lookup<MODE>(P, qs.x, rr, pat, cS, cA, rE, cC);
+        if ((pat = quad_rc(f.y))) ev_rc_lookup<MODE>(P, qs.y, rr, pat, cS, cA, rE, cC);
+        if ((pat = quad_rc(f.z))) ev_rc_lookup<MODE>(P, qs.z, rr, pat, cS, cA, rE, cC);
+        if ((pat = quad_rc(f.w))) ev_rc_lookup<MODE>(P, qs.w, rr, pat, cS, cA, rE, cC);
+      }
+    }
+  };
 #pragma unroll 1
   for (uint32_t tile = first_tile; tile < n_tiles; tile += tile_stride) {
-    const int64_t cand = (int64_t)tile * 32 + lane;
-    const bool active = cand < P.n;
+    cand = (int64_t)tile * 32 + lane;
+    active = cand < P.n;
     ev_init(s, P, active ? __ldg(P.hdr + cand) : 0ull);
     cS = cA = cC = 0;
     rE = 0;
-    uint32_t pw = 0;
+    pw = 0;
 #pragma unroll 1
     for (uint32_t g = 0; g < ngroups; ++g) {
       const uint32_t ch0 = kEvSlotChunks * g, nc = min((uint32_t)kEvSlotChunks, nch - ch0);
@@ -496,48 +542,18 @@ __global__ void __launch_bounds__(kThreads, MINB) event_kernel(const __grid_cons
           sts128(la, pad_tail(lds128(la), nvl));
         }
       }
-#pragma unroll
-      for (uint32_t c = 0; c < (uint32_t)kEvSlotChunks; ++c) {
-        if (c < nc) {
-          if ((c & 1u) == 0u) {  // the lists must hold what the next 2 chunks add
-            if (__any_sync(0xffffffffu, s.ec + 2u > (uint32_t)kEvCap)) ev_drain<MODE>(s, P, qo, lb, lx, cand, active);
-          }
-          const uint4 w4 = lds128(addr + 512u * c);
-          uint4 f;
-          f.x = quad_activity(w4.x, pw);
-          f.y = quad_activity(w4.y, w4.x);
-          f.z = quad_activity(w4.z, w4.y);
-          f.w = quad_activity(w4.w, w4.z);
-          pw = w4.w;
-          const uint32_t orw = f.x | f.y | f.z | f.w;
-          const bool evc = (orw & 0xefefefefu) != 0u;
-          const bool rcc = !evc && (orw & 0x10101010u) != 0u;
-          if (__any_sync(0xffffffffu, rcc)) {
-            if (rcc) {
-              // recompute flags in an event-free chunk: every op is in the open run, whose
-              // (tp, dp) is that of op 0 of the chunk
-              const uint32_t rr = ev_run(w4.x & 0xffu, s.mbs(), P);
-              const uint4 qs = lds128(qo + 16u * (ch0 + c));
-              uint32_t pat;
-              if ((pat = quad_rc(f.x))) ev_rc_lookup<MODE>(P, qs.x, rr, pat, cS, cA, rE, cC);
-              if ((pat = quad_rc(f.y))) ev_rc_lookup<MODE>(P, qs.y, rr, pat, cS, cA, rE, cC);
-              if ((pat = quad_rc(f.z))) ev_rc_lookup<MODE>(P, qs.z, rr, pat, cS, cA, rE, cC);
-              if ((pat = quad_rc(f.w))) ev_rc_lookup<MODE>(P, qs.w, rr, pat, cS, cA, rE, cC);
-            }
-          }
-          // unconditional store to the next entry; the count advances iff the chunk has events
-          const uint32_t k = s.ec;
-          const uint32_t e = lb + 512u * k;
-          sts128(e + kEvF, f);
-          sts128(e + kEvC, make_uint4((uint32_t)cS, (uint32_t)(cS >> 32), (uint32_t)cA, (uint32_t)(cA >> 32)));
-          if (FULL)
-            sts128(lx + 32u * XR * k, make_uint4(rE, ch0 + c, (uint32_t)cC, (uint32_t)(cC >> 32)));
-          else
-            sts64x2(lx + 32u * XR * k, rE, ch0 + c);
-          if (evc) {
-            rE = 0;
-            s.ec = k + 1u;
-          }
+      if (nc == (uint32_t)kEvSlotChunks) {
+        drain_check();
+        chunk(addr, ch0);
+        chunk(addr + 512u, ch0 + 1u);
+        drain_check();
+        chunk(addr + 1024u, ch0 + 2u);
+        chunk(addr + 1536u, ch0 + 3u);
+      } else {
+#pragma unroll 1
+        for (uint32_t c = 0; c < nc; ++c) {
+          if ((c & 1u) == 0u) drain_check();
+          chunk(addr + 512u * c, ch0 + c);
         }
       }
       __syncwarp();
