@@ -45,6 +45,7 @@ def parse():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--no-dedup", action="store_true", help="skip the hash / visited-set measurement")
+    ap.add_argument("--no-incr", action="store_true", help="skip the incremental-evaluation measurement")
     ap.add_argument("--search-budget", type=float, default=20.0,
                     help="seconds for the search-time measurement (0: skip)")
     ap.add_argument("--streams", type=int, default=4,
@@ -204,6 +205,73 @@ def measure_dedup(A, dev_batches, n, L, hbm, reps=200):
                             "overflow": vs.overflowed()},
             "note": "SURVEY 8(f) NEXT(3): configuration hash (aceso_hash) and first-occurrence "
                     "visited set (aceso_dedup) on the bench batches; not part of the timed step"}
+
+
+def measure_incr(A, ctx, prof, n, hbm, seed=SEED, reps=100):
+    """NEXT(2): the same metric for candidates given as base + patches (the search driver's
+    Table-1 primitives, 56-byte descriptors) evaluated by aceso_eval_incr against per-base
+    stage caches. Bases: valid search-shaped configurations; every base gets the driver's
+    primitives for a bottleneck taken from its own evaluation (FULL outputs from aceso_eval,
+    so no oracle on this path); descriptors are tiled to n candidates."""
+    import torch
+    from paper_conf_eurosys_liumlsmybw24_b200 import candidates as C
+    from paper_conf_eurosys_liumlsmybw24_b200 import search as S
+    from paper_conf_eurosys_liumlsmybw24_b200.api import as_u32, as_u64
+    dev = torch.device("cuda", torch.cuda.current_device())
+    L, stride = prof.n_ops, C.stride_of(prof.n_ops)
+    codes, hdr = gen_batch(prof, "search", 0, 4096, 64, tiled=False)
+    out, _ = ctx.eval(ctx.pack_rowmajor(torch.from_numpy(codes).to(dev)), torch.from_numpy(hdr.view(np.int64)).to(dev),
+                      full=True, select=False)
+    torch.cuda.synchronize()
+    info = as_u32(out.info)
+    pm = out.p_max
+    st_T, st_c, st_m = (as_u64(getattr(out, k)).reshape(pm, -1).T for k in ("stage_T", "stage_comp", "stage_comm"))
+    ok = np.nonzero((info & (1 << 17)) == 0)[0][:64]
+    prim = S.Primitives(prof)
+    bases = np.zeros((len(ok), stride), np.uint8)
+    bhdr = np.zeros(len(ok), np.uint64)
+    ranks = np.zeros((len(ok), 2, stride), np.uint16)
+    chunks = []
+    for bi, i in enumerate(ok):
+        bases[bi, :L] = codes[i]
+        bhdr[bi] = hdr[i]
+        cd, rk = prim.describe_all(codes[i], int(hdr[i] & 0xFF), int(info[i]), st_c[i], st_m[i], st_T[i])
+        cd["base"] = bi
+        ranks[bi] = rk
+        chunks.append(cd)
+    allc = np.concatenate(chunks)
+    cands = allc[np.arange(n) % len(allc)]
+    tb = torch.from_numpy(bases).to(dev)
+    th = torch.from_numpy(bhdr.view(np.int64)).to(dev)
+    tr = torch.from_numpy(ranks.view(np.int16)).to(dev)
+    tc = torch.from_numpy(cands.view(np.uint8)).to(dev)
+    o2 = ctx.alloc_outputs(n)
+    sel = ctx.alloc_select(n)
+    from paper_conf_eurosys_liumlsmybw24_b200 import _lib
+    work = torch.empty(int(_lib.load().aceso_incr_work_bytes(ctx._h, len(ok))), dtype=torch.uint8, device=dev)
+    for _ in range(3):
+        ctx.eval_incr(tb, th, tc, tr, n=n, out=o2, sel=sel, work=work)
+    torch.cuda.synchronize()
+    g = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(g):
+        for _ in range(reps):
+            ctx.eval_incr(tb, th, tc, tr, n=n, out=o2, sel=sel, work=work)
+    g.replay()
+    torch.cuda.synchronize()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record()
+    g.replay()
+    e1.record()
+    torch.cuda.synchronize()
+    ms = e0.elapsed_time(e1) / reps
+    b = n * (56 + 20)
+    return {"configs_per_s": n / (ms * 1e-3), "ms_per_batch": ms, "batch": n, "bases": int(len(ok)),
+            "distinct_descriptors": int(len(allc)),
+            "roofline": {"bound": "hbm", "achieved": b / (ms * 1e-3) / 1e9, "peak": hbm, "unit": "GB/s",
+                         "frac": b / (ms * 1e-3) / 1e9 / hbm, "bytes_per_candidate": 76},
+            "note": "SURVEY 8(f) NEXT(2): candidates as base + patches (56 B descriptor + 20 B "
+                    "summary), aceso_eval_incr with fused select, one stream, CUDA graph; not part "
+                    "of the timed step"}
 
 
 def run_reference(args):
@@ -516,6 +584,8 @@ def main():
             line["e2e"] = e2e
         if not args.no_dedup:
             line["dedup"] = measure_dedup(A, dev_batches, n, L, hbm)
+        if not args.no_incr:
+            line["incremental"] = measure_incr(A, ctx, prof, n, hbm)
         if args.search_budget > 0 and world == 1:
             from paper_conf_eurosys_liumlsmybw24_b200 import search as S
             ev = S.GPUEvaluator(ctx)

@@ -12,10 +12,18 @@
 // microbatch or stage count differs from its base, or whose base is invalid or has more than
 // 64 stages, is walked over all ops (same code, every stage touched).
 //
+// The candidate walk (walk_events) is event-driven like event_kernel.cuh: it patches the
+// base's codes 16 ops at a time, finds the chunk's events (stage heads, tp/dp changes) and
+// recompute flags with the activity words, and takes every run's sums from the position-
+// prefix tables (PX, PD, sparse-table range max ST, recompute deltas QR per quad pattern),
+// so a touched stage costs O(its chunks + its events), not a table walk per op.
+//
 // Paper: Eq. 1, Eq. 2, Heuristic-1, readings R1-R13, R18-R20.
 #pragma once
 #include "common.cuh"
-#include "eval_kernel.cuh"  // kSummary / kFull / kSelect
+#include "eval_kernel.cuh"    // kSummary / kFull / kSelect
+#include "event_kernel.cuh"   // activity words, event / recompute masks, event tables
+#include "expand_kernel.cuh"  // patched_chunk
 
 namespace aceso {
 
@@ -28,76 +36,125 @@ struct IncrBaseStage {  // 48 bytes
   uint32_t g, head;
 };
 
-struct IncrTabs {
-  const uint32_t *R, *D, *F, *K;  // packed per-op tables of the blob (eval_kernel.cuh layout)
-  const uint16_t *T;              // op types
-  uint32_t nT;
-};
-
-__device__ __forceinline__ IncrTabs incr_tabs(const EvalParams &P) {
-  const unsigned char *blob = reinterpret_cast<const unsigned char *>(P.blob);
-  IncrTabs t;
-  t.R = reinterpret_cast<const uint32_t *>(blob + P.tab.offR);
-  t.D = reinterpret_cast<const uint32_t *>(blob + P.tab.offD);
-  t.F = reinterpret_cast<const uint32_t *>(blob + P.tab.offF);
-  t.K = reinterpret_cast<const uint32_t *>(blob + P.tab.offK);
-  t.T = reinterpret_cast<const uint16_t *>(blob + P.tab.offT);
-  t.nT = (uint32_t)P.T;
-  return t;
-}
-
 // one stage being accumulated by the walk
 struct WalkStage {
   uint64_t S, A, W, D, comp;
   uint32_t E, g, head;
 };
 
-// Walks ops [A, B) (A is a stage start, B = L or a head) of the configuration code_at(j),
-// calling emit(stage) for every stage it closes, in order. Per-op validity goes to *reasons;
-// returns the number of head bits walked.
-template <bool FULL, class CodeAt, class Emit>
-__device__ __forceinline__ uint32_t walk_ops(const EvalParams &P, const IncrTabs &t, uint32_t mbs,
-                                             uint32_t A, uint32_t B, CodeAt code_at, Emit emit,
-                                             uint32_t *reasons) {
-  const uint32_t NT = (uint32_t)P.n_tp, NB = (uint32_t)P.n_b;
+// Event-driven walk of ops [A, B) of a candidate (A is a segment start: a stage starts at A
+// whatever its head bit, R19; B = L or a head): same stages, same emit order and same
+// per-op validity as a walk over every op would give, from the event tables. Sums are kept in prefix-difference
+// form (exact mod 2^64). Returns the number of head bits walked.
+template <bool FULL, class Emit>
+__device__ __forceinline__ uint32_t walk_events(const EvalParams &P, const uint4 *__restrict__ brow,
+                                                const uint16_t *__restrict__ ranks, uint32_t base,
+                                                const aceso_cand &cd, int np, uint32_t mbs, uint32_t A,
+                                                uint32_t B, Emit emit, uint32_t *reasons) {
+  const uint32_t L = (uint32_t)P.L, Lp1 = L + 1u, NT = (uint32_t)P.n_tp, NB = (uint32_t)P.n_b;
+  const int32_t stride = 16 * (int32_t)((L + 15u) / 16u);
+  const uint32_t *qo = reinterpret_cast<const uint32_t *>(P.evblob + P.qo_off);
   WalkStage st;
-  uint32_t nst = 0, pc = 0, prt = 0;  // previous op's code and (run, type) index
-  for (uint32_t j = A; j < B; ++j) {
-    const uint32_t c = code_at(j);
-    const uint32_t head = c & 1u, tpl = (c >> 1) & 7u, rc = (c >> 4) & 1u, dpl = c >> 5;
-    if (dpl > mbs) *reasons |= ACESO_R_DPMBS;
-    if (tpl >= NT || dpl >= (uint32_t)P.n_dp || (dpl <= mbs && mbs - dpl >= NB)) *reasons |= ACESO_R_TABLE;
-    const uint32_t b = min(dpl <= mbs ? mbs - dpl : 0u, NB - 1);
-    const uint32_t tplc = min(tpl, NT - 1);
-    const uint32_t type = __ldg(t.T + j);
-    const uint32_t rt = (b * NT + tplc) * t.nT + type;  // (run, type) record index
-    if (j == A || head) {
-      if (j > A) {  // close the previous stage: p2p_fwd of its last op (R5)
-        st.S += __ldg(t.K + prt * 4 + 1);
-        emit(st);
+  st.S = st.A = st.W = st.D = st.comp = 0;
+  st.E = 0;
+  st.g = 0;
+  st.head = A;
+  uint32_t rr = 0, dd = 0, ra = A, nst = 0;
+  // closes the open run [ra, j) (prefix differences, range max R4)
+  auto close_run = [&](uint32_t j) {
+    const uint32_t o = rr * Lp1 + j;
+    const uint4 x0 = __ldg(P.px + 2u * o);
+    const uint4 x1 = __ldg(P.px + 2u * o + 1u);
+    const uint32_t k = 31u - __clz(j - ra);
+    const uint32_t *stk = P.st + ((k * (uint32_t)P.runs + rr) * L);
+    st.S += u64of(x0.x, x0.y);
+    st.A += u64of(x0.z, x0.w);
+    st.W += u64of(x1.x, x1.y);
+    if (FULL) st.comp += u64of(x1.z, x1.w);
+    st.D += __ldg(P.pd + (dd * Lp1 + j));
+    st.E = max(st.E, max(__ldg(stk + ra), __ldg(stk + (j - (1u << k)))));
+  };
+  const uint32_t *kx = reinterpret_cast<const uint32_t *>(P.kx);
+  uint32_t pw = 0;
+  const uint32_t c0 = A >> 4, c1 = (B - 1u) >> 4;
+  if (c0 > 0) pw = patched_chunk(brow, ranks, base, stride, (int32_t)L, cd, np, (int32_t)c0 - 1).w;
+  for (uint32_t ch = c0; ch <= c1; ++ch) {
+    const uint4 w4 = patched_chunk(brow, ranks, base, stride, (int32_t)L, cd, np, (int32_t)ch);
+    uint4 f;
+    f.x = quad_activity(w4.x, pw);
+    f.y = quad_activity(w4.y, w4.x);
+    f.z = quad_activity(w4.z, w4.y);
+    f.w = quad_activity(w4.w, w4.z);
+    pw = w4.w;
+    // ops of the chunk inside [A, B); op A is always an event (segment start)
+    const uint32_t lo = ch == c0 ? (A & 15u) : 0u, hi = ch == c1 ? ((B - 1u) & 15u) + 1u : 16u;
+    const uint32_t in = (hi >= 16u ? 0xffffu : ((1u << hi) - 1u)) & ~((1u << lo) - 1u);
+    uint32_t em = (ev_event_mask(f) | (ch == c0 ? (1u << lo) : 0u)) & in;
+    uint32_t rm = ev_rc_mask(f) & in;
+    while (em | rm) {
+      const uint32_t j = __ffs(em | rm) - 1u;
+      const uint32_t op = 16u * ch + j;
+      if ((em >> j) & 1u) {
+        const uint32_t wq = (j >> 2) == 0u ? w4.x : (j >> 2) == 1u ? w4.y : (j >> 2) == 2u ? w4.z : w4.w;
+        const uint32_t c = (wq >> (8u * (j & 3u))) & 0xffu;
+        const uint32_t head = c & 1u, tpl = (c >> 1) & 7u, dpl = c >> 5;
+        if (dpl > mbs) *reasons |= ACESO_R_DPMBS;
+        if (tpl >= NT || dpl >= (uint32_t)P.n_dp || (dpl <= mbs && mbs - dpl >= NB)) *reasons |= ACESO_R_TABLE;
+        // clamped indices keep every gather inside the tables for invalid encodings
+        const uint32_t b = min(dpl <= mbs ? mbs - dpl : 0u, NB - 1);
+        const uint32_t tplc = min(tpl, NT - 1), dplc = min(dpl, (uint32_t)P.n_dp - 1);
+        const uint32_t rn = b * NT + tplc;
+        const uint32_t on = rn * Lp1 + op;
+        if (op == A || head) {
+          if (op > A) {  // close the stage: its last run, p2p_fwd of its last op (R5)
+            close_run(op);
+            st.S += __ldg(kx + (4u * (rr * Lp1 + op) + 2u));
+            emit(st);
+          }
+          st.S = st.A = st.W = st.D = st.comp = 0;
+          st.E = 0;
+          st.g = tpl + dpl;
+          st.head = op;
+          nst += head;
+          if (op > 0 && head) st.S += __ldg(kx + (4u * on + 1u));  // p2p_bwd of the first op (R5)
+        } else {
+          close_run(op);
+          if (tpl + dpl != st.g) *reasons |= ACESO_R_GSTAGE;
+          st.S += __ldg(kx + 4u * on);                        // reshard into this op (R13)
+        }
+        // open the run of op `op`
+        const uint4 y0 = __ldg(P.px + 2u * on);
+        const uint4 y1 = __ldg(P.px + 2u * on + 1u);
+        st.S -= u64of(y0.x, y0.y);
+        st.A -= u64of(y0.z, y0.w);
+        st.W -= u64of(y1.x, y1.y);
+        if (FULL) st.comp -= u64of(y1.z, y1.w);
+        rr = rn;
+        dd = tplc * (uint32_t)P.n_dp + dplc;
+        st.D -= __ldg(P.pd + (dd * Lp1 + op));
+        ra = op;
+        em &= em - 1u;
+      } else {
+        // recompute flags of quad j/4 from op j up to the quad's next event, under the open
+        // run (R3, R4, R7)
+        const uint32_t qb = j & ~3u;
+        const uint32_t nxt = em & (0xfu << qb);
+        const uint32_t lim = nxt ? __ffs(nxt) - 1u : qb + 4u;
+        const uint32_t seg = rm & ((1u << lim) - 1u);
+        uint64_t dS = 0, dA = 0, dC = 0;
+        uint32_t e1 = 0;
+        ev_rc_lookup<FULL ? kFull : 0u>(P, __ldg(qo + 4u * ch + (j >> 2)), rr, seg >> qb, dS, dA, e1, dC);
+        st.S += dS;
+        st.A -= dA;
+        st.E = max(st.E, e1);
+        if (FULL) st.comp += dC;
+        rm &= ~seg;
       }
-      st.S = st.A = st.W = st.D = st.comp = 0;
-      st.E = 0;
-      st.g = tpl + dpl;
-      st.head = j;
-      nst += head;  // NSTAGE counts head bits (op 0 starts a segment even without one, R19)
-      if (j > 0 && head) st.S += __ldg(t.K + rt * 4 + 2);  // p2p_bwd of the stage's first op (R5)
-    } else {
-      if (tpl + dpl != st.g) *reasons |= ACESO_R_GSTAGE;
-      if (((c ^ pc) & 0xEEu) != 0u) st.S += __ldg(t.K + rt * 4);  // reshard into this op (R13)
     }
-    const uint4 r = __ldg(reinterpret_cast<const uint4 *>(t.R + rt * 8 + rc * 4));
-    st.S += r.x;
-    st.A += r.y;
-    st.E = max(st.E, r.z);
-    st.W += r.w;
-    st.D += __ldg(t.D + (tplc * t.nT + type) * 8 + dpl);
-    if (FULL) st.comp += __ldg(t.F + rt * 2 + rc);
-    pc = c;
-    prt = rt;
   }
-  if (B < (uint32_t)P.L) st.S += __ldg(t.K + prt * 4 + 1);  // followed by a stage (R5, R20)
-  if (B > A) emit(st);
+  close_run(B);
+  if (B < L) st.S += __ldg(kx + (4u * (rr * Lp1 + B) + 2u));  // followed by a stage (R5, R20)
+  emit(st);
   return nst;
 }
 
@@ -119,7 +176,6 @@ __global__ void __launch_bounds__(128) base_cache_kernel(const __grid_constant__
                                                          IncrBaseStage *stages, uint8_t *smap) {
   const int32_t b = blockIdx.x * blockDim.x + threadIdx.x;
   if (b >= nb) return;
-  const IncrTabs t = incr_tabs(P);
   const uint32_t L = (uint32_t)P.L, stride = 16u * (((uint32_t)P.L + 15u) / 16u);
   const uint8_t *row = bases + (size_t)b * stride;
   const uint64_t hb = base_hdr[b];
@@ -129,7 +185,6 @@ __global__ void __launch_bounds__(128) base_cache_kernel(const __grid_constant__
   IncrBaseStage *out = stages + (size_t)b * P.G;
   uint64_t sumS = 0;
   uint32_t i = 0, gsum = 0;
-  auto code_at = [&](uint32_t j) { return (uint32_t)__ldg(row + j); };
   auto emit = [&](const WalkStage &s) {
     if (i < (uint32_t)P.G) {
       const uint64_t infl = p > i ? (uint64_t)min(p - i, N) : 0ull;
@@ -148,7 +203,10 @@ __global__ void __launch_bounds__(128) base_cache_kernel(const __grid_constant__
     gsum += 1u << s.g;
     i += 1;
   };
-  const uint32_t nst = walk_ops<true>(P, t, mbs, 0, L, code_at, emit, &reasons);
+  aceso_cand cd0;
+  memset(&cd0, 0, sizeof(cd0));  // no patches: the base itself
+  const uint32_t nst = walk_events<true>(P, reinterpret_cast<const uint4 *>(row), nullptr, (uint32_t)b, cd0, 0, mbs,
+                                         0, L, emit, &reasons);
   if (!(row[0] & 1u)) reasons |= ACESO_R_HEAD0;
   if (nst != p) reasons |= ACESO_R_NSTAGE;
   if (gsum != (uint32_t)P.G) reasons |= ACESO_R_GSUM;
@@ -176,7 +234,6 @@ __global__ void __launch_bounds__(256) incr_kernel(const __grid_constant__ EvalP
   __shared__ unsigned int s_done;
   if (threadIdx.x == 0) s_done = 0;
   __syncthreads();
-  const IncrTabs t = incr_tabs(P);
   const uint32_t L = (uint32_t)P.L, stride = 16u * ((L + 15u) / 16u);
   uint64_t best_ck = ~0ull;
   int64_t best_idx = INT64_MAX;
@@ -190,24 +247,8 @@ __global__ void __launch_bounds__(256) incr_kernel(const __grid_constant__ EvalP
     uint32_t N = 0;
     uint32_t reasons = header_reasons((uint64_t)mbs | ((uint64_t)p << 8), P, &N);
     const int np = min((int)cd.n_patch, 6);
-    // the candidate's code at op j: the base's byte with the patches applied in order
-    auto code_at = [&](uint32_t j) {
-      uint32_t v = __ldg(row + j);
-      for (int k = 0; k < np; ++k) {
-        const aceso_patch pt = cd.patch[k];
-        if (j < pt.a || j >= pt.b) continue;
-        if (pt.kind == ACESO_PATCH_MASK) {
-          v = (v & pt.v0) | pt.v1;
-        } else if (pt.kind == ACESO_PATCH_ADD) {
-          v = (v + (uint32_t)(((int)(int8_t)pt.v0 << 1) + ((int)(int8_t)pt.v1 << 5))) & 0xffu;
-        } else if (pt.kind == ACESO_PATCH_RANK_RC && ranks != nullptr) {
-          const uint32_t kk = (uint32_t)pt.v0 | ((uint32_t)pt.v1 << 8);
-          if ((uint32_t)__ldg(ranks + ((size_t)base * 2 + (pt.v2 & 1u)) * stride + j) < kk)
-            v = (pt.v2 & 2u) ? (v & 0xefu) : (v | 0x10u);
-        }
-      }
-      return v;
-    };
+    const uint4 *brow = reinterpret_cast<const uint4 *>(row);
+    const int32_t stride_i = (int32_t)stride;
     const IncrBaseHdr bh = hdrs[base];
     const bool full = bh.reasons != 0u || bh.mbs != mbs || bh.p != p || p > 64u;
     uint64_t touched = ~0ull;  // stages to re-walk (bit i)
@@ -244,9 +285,9 @@ __global__ void __launch_bounds__(256) incr_kernel(const __grid_constant__ EvalP
       const uint64_t infl = p > i ? (uint64_t)min(p - i, N) : 0ull;
       fold(s.S, s.D, s.comp, (uint64_t)(N - 1) * s.S + s.D, (s.W + infl * s.A + s.E) << P.mem_shift, s.g);
     };
-    uint32_t op0 = code_at(0);
+    const uint32_t op0 = patched_chunk(brow, ranks, base, stride_i, (int32_t)L, cd, np, 0).x & 0xffu;
     if (full) {
-      nst = walk_ops<(MODE & kFull) != 0>(P, t, mbs, 0, L, code_at, emit, &reasons);
+      nst = walk_events<(MODE & kFull) != 0>(P, brow, ranks, base, cd, np, mbs, 0, L, emit, &reasons);
     } else {
       const IncrBaseStage *bs = stages + (size_t)base * P.G;
       uint32_t s = 0;
@@ -261,7 +302,7 @@ __global__ void __launch_bounds__(256) incr_kernel(const __grid_constant__ EvalP
         uint32_t e = s;
         while (e + 1 < bh.p && ((touched >> (e + 1)) & 1ull)) e += 1;
         const uint32_t A = bs[s].head, B = e + 1 < bh.p ? bs[e + 1].head : L;
-        nst += walk_ops<(MODE & kFull) != 0>(P, t, mbs, A, B, code_at, emit, &reasons);
+        nst += walk_events<(MODE & kFull) != 0>(P, brow, ranks, base, cd, np, mbs, A, B, emit, &reasons);
         s = e + 1;
       }
     }
