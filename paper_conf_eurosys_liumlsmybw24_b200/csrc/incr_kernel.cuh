@@ -86,11 +86,16 @@ __device__ __forceinline__ uint32_t walk_events(const EvalParams &P, const uint4
     f.z = quad_activity(w4.z, w4.y);
     f.w = quad_activity(w4.w, w4.z);
     pw = w4.w;
-    // ops of the chunk inside [A, B); op A is always an event (segment start)
-    const uint32_t lo = ch == c0 ? (A & 15u) : 0u, hi = ch == c1 ? ((B - 1u) & 15u) + 1u : 16u;
-    const uint32_t in = (hi >= 16u ? 0xffffu : ((1u << hi) - 1u)) & ~((1u << lo) - 1u);
-    uint32_t em = (ev_event_mask(f) | (ch == c0 ? (1u << lo) : 0u)) & in;
-    uint32_t rm = ev_rc_mask(f) & in;
+    const bool edge = ch == c0 || ch == c1;
+    if (!edge && (f.x | f.y | f.z | f.w) == 0u) continue;  // no event, no recompute flag
+    uint32_t em = ev_event_mask(f), rm = ev_rc_mask(f);
+    if (edge) {
+      // ops of the chunk inside [A, B); op A is always an event (segment start)
+      const uint32_t lo = ch == c0 ? (A & 15u) : 0u, hi = ch == c1 ? ((B - 1u) & 15u) + 1u : 16u;
+      const uint32_t in = (hi >= 16u ? 0xffffu : ((1u << hi) - 1u)) & ~((1u << lo) - 1u);
+      em = (em | (ch == c0 ? (1u << lo) : 0u)) & in;
+      rm &= in;
+    }
     while (em | rm) {
       const uint32_t j = __ffs(em | rm) - 1u;
       const uint32_t op = 16u * ch + j;
