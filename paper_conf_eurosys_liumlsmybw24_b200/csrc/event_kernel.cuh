@@ -345,6 +345,10 @@ __device__ __forceinline__ uint32_t ev_rc_mask(uint4 f) {
 template <uint32_t MODE>
 __device__ __forceinline__ void ev_drain(EvCand &s, const EvalParams &P, uint32_t qo, uint32_t lb,
                                          uint32_t lx, int64_t cand, bool active) {
+#ifdef ACESO_EXPERIMENT_NO_PHASEB
+  s.ec = 0;
+  return;
+#endif
   constexpr uint32_t XS = 32u * ev_xrec(MODE & kFull);  // X stride per entry
   uint32_t k = 0, em = 0, rm = 0, ent = 0, xe = 0, q0 = 0;
 #pragma unroll 1
@@ -499,7 +503,11 @@ __global__ void __launch_bounds__(kThreads, MINB) event_kernel(const __grid_cons
       rE = 0;
       s.ec = k + 1u;
     }
+#ifdef ACESO_EXPERIMENT_NO_RC
+    if (false) {
+#else
     if (__any_sync(0xffffffffu, rcc)) {
+#endif
       if (rcc) {
         // recompute flags in an event-free chunk: every op is in the open run, whose
         // (tp, dp) is that of op 0 of the chunk
