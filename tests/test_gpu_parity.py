@@ -384,3 +384,48 @@ def test_search_driver_gpu_matches_oracle_trajectory():
     ro, so = S.search(prof, OracleEvaluator(prof), **kw)
     assert rg.perf == ro.perf and rg.mbs == ro.mbs and np.array_equal(rg.codes, ro.codes)
     assert sg["evaluated"] == so["evaluated"] and sg["batches"] == so["batches"]
+
+
+def _attribution_candidates(prof, n, seed):
+    """Valid candidates aimed at the event kernel v2's bookkeeping: stage heads at chunk edges
+    (ops 16k-1, 16k, 16k+1) and inside chunks, in-stage tp/dp trades (same device count) in some
+    chunks, and recompute flags in sparse runs of chunks, some of them event-free (phase-A
+    lookups attributed through the list entries' cumulative sums), some next to heads."""
+    rng = np.random.default_rng(seed)
+    L, G = prof.n_ops, prof.n_devices
+    kmax = prof.n_tp - 1
+    rows, hdrs = [], []
+    for _ in range(n):
+        p = int(rng.choice([q for q in (1, 2, 4, 8) if q <= G]))
+        cuts = set()
+        while len(cuts) < p - 1:
+            k = int(rng.integers(1, L // 16 + 1)) * 16 + int(rng.choice([-1, 0, 1, 5]))
+            if 0 < k < L:
+                cuts.add(k)
+        starts = [0] + sorted(cuts)
+        g = int(np.log2(G // p))
+        mbs = int(rng.integers(g, g + 3))
+        row = np.zeros(L, np.uint8)
+        for si, a in enumerate(starts):
+            b = starts[si + 1] if si + 1 < len(starts) else L
+            tpl = int(rng.integers(0, min(g, kmax) + 1))
+            dpl = g - tpl
+            for j in range(a, b):
+                t, d = tpl, dpl
+                if (j // 16) % 3 == 1 and rng.random() < 0.5 and g > 0:  # in-stage trade
+                    t = int(rng.integers(0, min(g, kmax) + 1))
+                    d = g - t
+                rc = 1 if ((j // 16) % 4 in (0, 3) and rng.random() < 0.3) else 0
+                row[j] = ai.code(1 if j == a else 0, t, d, rc)
+        rows.append(row)
+        hdrs.append(ai.header(mbs, p))
+    return np.array(rows, np.uint8), np.array(hdrs, np.uint64)
+
+
+@pytest.mark.parametrize("name", ["gpt3-1.3b", "t5", "wrn"])
+def test_event_kernel_recompute_attribution_parity(name):
+    prof = P.WORKLOADS[name]()
+    codes, hdr = _attribution_candidates(prof, 900, SEED + 21)
+    g, o, sel, _, _ = compare(prof, codes, hdr, full=True)
+    assert ((o["info"] & oracle.INFO_INVALID) == 0).mean() > 0.5  # the sums are really compared
+    compare(prof, codes, hdr)
