@@ -48,6 +48,8 @@ def parse():
     ap.add_argument("--no-incr", action="store_true", help="skip the incremental-evaluation measurement")
     ap.add_argument("--search-budget", type=float, default=20.0,
                     help="seconds for the search-time measurement (0: skip)")
+    ap.add_argument("--keys-per-allreduce", type=int, default=16,
+                    help="N > 1: packed keys of this many steps per all-reduce MIN")
     ap.add_argument("--streams", type=int, default=4,
                     help="independent batches in flight (steps round-robin over streams)")
     return ap.parse_args()
@@ -395,6 +397,8 @@ def main():
     outs = [out] + [ctx.alloc_outputs(n) for _ in range(nstr - 1)]
     side = [torch.cuda.Stream() for _ in range(nstr)]
     comm = torch.cuda.Stream()  # all-reduces in step order on one stream (same on every rank)
+    keyvec = torch.empty(args.steps, dtype=torch.int64, device=dev)  # per-step global keys
+    kpa = max(1, args.keys_per_allreduce)
     def issue_steps():
         """The K steps on the side streams (+ all-reduces in step order on `comm`)."""
         cs = torch.cuda.current_stream()
@@ -414,11 +418,16 @@ def main():
                      select=True, out=outs[s % nstr], sel=sels[b], stream=st, dense_hint=HINT)
             ev_k[s].record(st)
             if world > 1:
+                # the step's packed key joins a vector of keys; one all-reduce MIN per
+                # `keys_per_allreduce` steps (8*K bytes for K batches)
                 done = torch.cuda.Event()
                 done.record(st)
                 comm.wait_event(done)
                 with torch.cuda.stream(comm):
-                    dist.all_reduce(sels[b][0:8].view(torch.int64), op=dist.ReduceOp.MIN)
+                    keyvec[s:s + 1].copy_(sels[b][0:8].view(torch.int64))
+                    if (s + 1) % kpa == 0 or s == args.steps - 1:
+                        s0 = (s // kpa) * kpa
+                        dist.all_reduce(keyvec[s0:s + 1], op=dist.ReduceOp.MIN)
                 cd = torch.cuda.Event()
                 cd.record(comm)
                 comm_done[s] = cd
@@ -494,6 +503,10 @@ def main():
     # correctness of the timed result of the last step (global select over ranks)
     last = (args.steps - 1) % nbuf
     best = Selection.from_buffer(sels[last])
+    if world > 1:  # the global key of the last step (vector all-reduce); exact fallback if saturated
+        kl = int(keyvec[args.steps - 1].item())
+        gc, gcost, gidx, sat = A.decode_key(kl, n_total)
+        best = adist.global_select(sels[last], n_total) if sat else Selection(gc, gcost, gidx, kl)
 
     # ---- end to end through the public API: host (pinned) -> device -> result -> host
     e2e = None
