@@ -170,31 +170,26 @@ __device__ __forceinline__ void block_select_finish(uint64_t ck, int64_t idx, un
   }
 }
 
-// Argmin with grid-level completion and no CTA barrier: every warp leaves its partial in
-// shared memory; the last warp of a CTA to finish (shared counter, zeroed at kernel start)
-// reduces the CTA's partials and publishes the CTA partial; the last CTA to publish
-// (global counter) reduces all CTA partials and writes the final result. Warps that
-// finish early exit without waiting for the rest of their CTA. Called by all 32 lanes of
-// every warp of the grid.
+// Argmin with grid-level completion: every warp leaves its partial in shared memory, one
+// CTA barrier, warp 0 reduces the CTA's partials and publishes the CTA partial; the last
+// CTA to publish (global counter) reduces all CTA partials and writes the final result.
+// Called by all 32 lanes of every warp of the grid.
 __device__ __forceinline__ void warp_select_finish(uint64_t ck, int64_t idx, unsigned char *sel,
                                                    int64_t n_total, uint32_t ib, uint64_t *s_ck,
-                                                   int64_t *s_idx, unsigned int *s_cnt) {
+                                                   int64_t *s_idx) {
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   const uint32_t wpb = blockDim.x >> 5;
   warp_argmin(ck, idx);
-  uint32_t last = 0;
   if (lane == 0) {
     s_ck[warp] = ck;
     s_idx[warp] = idx;
-    __threadfence_block();
-    last = atomicAdd(s_cnt, 1u) == wpb - 1 ? 1u : 0u;
   }
-  if (!__shfl_sync(0xffffffffu, last, 0)) return;
-  __threadfence_block();
-  ck = lane < (int)wpb ? ((volatile uint64_t *)s_ck)[lane] : ~0ull;
-  idx = lane < (int)wpb ? ((volatile int64_t *)s_idx)[lane] : INT64_MAX;
+  __syncthreads();
+  if (warp != 0) return;
+  ck = lane < (int)wpb ? s_ck[lane] : ~0ull;
+  idx = lane < (int)wpb ? s_idx[lane] : INT64_MAX;
   warp_argmin(ck, idx);
-  last = 0;
+  uint32_t last = 0;
   if (lane == 0) {
     uint64_t *part = reinterpret_cast<uint64_t *>(sel + kSelPartialOff) + 2 * blockIdx.x;
     part[0] = ck;

@@ -412,7 +412,6 @@ __global__ void __launch_bounds__(kThreads, MINB) event_kernel(const __grid_cons
   __shared__ __align__(8) uint64_t s_ring_bar[kEvRingSlots][kWarps];
   __shared__ uint64_t s_ck[kWarps];
   __shared__ int64_t s_idx[kWarps];
-  __shared__ unsigned int s_done;  // warps of this CTA past the tile loop
   constexpr bool FULL = (MODE & kFull) != 0;
   constexpr uint32_t XR = ev_xrec(FULL);
 
@@ -425,7 +424,6 @@ __global__ void __launch_bounds__(kThreads, MINB) event_kernel(const __grid_cons
   if (threadIdx.x == 0) {
     mbar_init(smem_addr(&s_tbar), 1);
     fence_barrier_init();
-    s_done = 0;
   }
   if (lane == 0) {
     for (int k = 0; k < kEvRingSlots; ++k) mbar_init(smem_addr(&s_ring_bar[k][warp]), 1);
@@ -583,7 +581,7 @@ __global__ void __launch_bounds__(kThreads, MINB) event_kernel(const __grid_cons
     ev_finish<MODE>(s, P, cand, active, best_ck, best_idx);
   }
 
-  if (MODE & kSelect) warp_select_finish(best_ck, best_idx, P.sel, P.n_total, P.ib, s_ck, s_idx, &s_done);
+  if (MODE & kSelect) warp_select_finish(best_ck, best_idx, P.sel, P.n_total, P.ib, s_ck, s_idx);
 }
 
 }  // namespace aceso

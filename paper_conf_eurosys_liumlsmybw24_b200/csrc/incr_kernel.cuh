@@ -236,9 +236,6 @@ __global__ void __launch_bounds__(256) incr_kernel(const __grid_constant__ EvalP
                                                    const uint8_t *__restrict__ smap) {
   __shared__ uint64_t s_ck[kWarps];
   __shared__ int64_t s_idx[kWarps];
-  __shared__ unsigned int s_done;
-  if (threadIdx.x == 0) s_done = 0;
-  __syncthreads();
   const uint32_t L = (uint32_t)P.L, stride = 16u * ((L + 15u) / 16u);
   uint64_t best_ck = ~0ull;
   int64_t best_idx = INT64_MAX;
@@ -339,7 +336,7 @@ __global__ void __launch_bounds__(256) incr_kernel(const __grid_constant__ EvalP
       }
     }
   }
-  if (MODE & kSelect) warp_select_finish(best_ck, best_idx, P.sel, P.n_total, P.ib, s_ck, s_idx, &s_done);
+  if (MODE & kSelect) warp_select_finish(best_ck, best_idx, P.sel, P.n_total, P.ib, s_ck, s_idx);
 }
 
 }  // namespace aceso
