@@ -296,6 +296,27 @@ int aceso_eval_incr(aceso_ctx *ctx, const uint8_t *d_bases, const uint64_t *d_ba
                     const aceso_eval_out *out, void *d_sel, void *d_work, void *stream);
 
 /* ------------------------------------------------------------------------- */
+/* Exhaustive stage-partition enumeration (the Exp#4     */
+/* mathematical-programming baseline explores a pruned configuration space    */
+/* with the same performance model).                               */
+/* ------------------------------------------------------------------------- */
+/* Number of candidates of a family: C(n_ops - 1, p - 1) (the (p-1)-subsets of the
+ * cut positions 1 .. n_ops-1). -1 if 1 <= p <= min(8, n_ops) does not hold or the
+ * count is >= 2^62. Host only, no device access. */
+int64_t aceso_enum_cuts_count(int32_t n_ops, int32_t p);
+/* Writes candidates [first, first + n) of the family (p, code, hdr) in the tiled
+ * layout: candidate r has stage heads at op 0 and at the cuts of the r-th
+ * (p-1)-subset of {1, ..., n_ops-1} in colex order (r = sum_i C(cut_i - 1, i),
+ * cuts ascending, i = 1..p-1); every op carries `code` with its head bit cleared
+ * (tp, dp and recompute bits: a stage-uniform configuration); headers = hdr.
+ *   d_tiled : aceso_tiled_bytes(n, n_ops) bytes (device, 16-byte aligned)
+ *   d_hdr   : [n] u64 (device)
+ * ACESO_ERANGE for a bad family, ACESO_EINVAL for a range outside the family.
+ * Async on `stream`. */
+int aceso_enum_cuts(int32_t n_ops, int32_t p, uint8_t code, uint64_t hdr, int64_t first, int64_t n,
+                    uint8_t *d_tiled, uint64_t *d_hdr, void *stream);
+
+/* ------------------------------------------------------------------------- */
 /* Configuration dedup ("skip configurations     */
 /* already explored"). The encoding above is canonical (one byte per op plus   */
 /* the header), so equal configurations have equal bytes and hash equal.       */

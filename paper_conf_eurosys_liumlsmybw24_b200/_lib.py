@@ -14,7 +14,8 @@ INFO_INVALID = 1 << 17
 
 SYMBOLS = ["aceso_load_profile", "aceso_free", "aceso_tiled_bytes", "aceso_pack_rowmajor",
            "aceso_select_buf_bytes", "aceso_eval", "aceso_select", "aceso_decode_key",
-           "aceso_last_error", "aceso_version", "aceso_hash", "aceso_visited_bytes", "aceso_dedup", "aceso_expand", "aceso_incr_work_bytes", "aceso_eval_incr"]
+           "aceso_last_error", "aceso_version", "aceso_hash", "aceso_visited_bytes", "aceso_dedup", "aceso_expand", "aceso_incr_work_bytes", "aceso_eval_incr",
+           "aceso_enum_cuts_count", "aceso_enum_cuts"]
 
 
 class ProfileDesc(ctypes.Structure):
@@ -73,6 +74,10 @@ def load():
     lib.aceso_dedup.restype = ctypes.c_int
     lib.aceso_expand.argtypes = [P, P, c_i32, c_i32, P, c_i64, P, P, P]
     lib.aceso_expand.restype = ctypes.c_int
+    lib.aceso_enum_cuts_count.argtypes = [c_i32, c_i32]
+    lib.aceso_enum_cuts_count.restype = c_i64
+    lib.aceso_enum_cuts.argtypes = [c_i32, c_i32, ctypes.c_uint8, ctypes.c_uint64, c_i64, c_i64, P, P, P]
+    lib.aceso_enum_cuts.restype = ctypes.c_int
     lib.aceso_incr_work_bytes.argtypes = [P, c_i32]
     lib.aceso_incr_work_bytes.restype = c_sz
     lib.aceso_eval_incr.argtypes = [P, P, P, P, c_i32, P, c_i64, c_i64, c_i64, c_u32, ctypes.POINTER(EvalOut),

@@ -282,6 +282,19 @@ def decode_key(key: int, n_total: int):
     return cls.value, cost.value, idx.value, bool(sat.value)
 
 
+def enum_cuts_count(n_ops: int, p: int) -> int:
+    """aceso_enum_cuts_count: C(n_ops - 1, p - 1), or -1 outside the supported range."""
+    return int(L.load().aceso_enum_cuts_count(int(n_ops), int(p)))
+
+
+def enum_cuts(n_ops: int, p: int, code: int, hdr: int, first: int, n: int, tiled: torch.Tensor,
+              hdr_out: torch.Tensor, stream=None):
+    """aceso_enum_cuts: candidates [first, first + n) of the stage-partition family (p, code,
+    hdr) written to device `tiled` (uint8, tiled layout) and `hdr_out` (int64)."""
+    _check(L.load().aceso_enum_cuts(int(n_ops), int(p), int(code) & 0xFF, int(hdr), int(first), int(n),
+                                    _ptr(tiled), _ptr(hdr_out), _stream(stream)), "aceso_enum_cuts")
+
+
 def upload_candidates(codes_tiled: np.ndarray, hdr: np.ndarray, device=0, pin=False):
     """Host tiled codes + uint64 headers -> device tensors (tiled uint8, int64 headers)."""
     c = torch.from_numpy(np.ascontiguousarray(codes_tiled, dtype=np.uint8))

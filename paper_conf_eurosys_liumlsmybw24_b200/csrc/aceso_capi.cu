@@ -21,6 +21,7 @@
 #include "incr_kernel.cuh"
 #include "eval_kernel.cuh"
 #include "event_kernel.cuh"
+#include "enum_kernel.cuh"
 
 using namespace aceso;
 
@@ -749,6 +750,28 @@ int aceso_expand(const uint8_t *d_bases, const uint16_t *d_ranks, int32_t n_base
       d_bases, d_ranks, n_bases, n_ops, d_cands, n, reinterpret_cast<uint4 *>(d_tiled), d_hdr);
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return fail(ACESO_ECUDA, "expand launch: %s", cudaGetErrorString(e));
+  return ACESO_OK;
+}
+
+int64_t aceso_enum_cuts_count(int32_t n_ops, int32_t p) {
+  if (n_ops < 1 || n_ops > kMaxOps || p < 1 || p > 8 || p > n_ops) return -1;
+  const uint64_t c = binom_sat((uint64_t)n_ops - 1, (uint32_t)p - 1);
+  return c >= (1ull << 62) ? -1 : (int64_t)c;
+}
+
+int aceso_enum_cuts(int32_t n_ops, int32_t p, uint8_t code, uint64_t hdr, int64_t first, int64_t n,
+                    uint8_t *d_tiled, uint64_t *d_hdr, void *stream) {
+  const int64_t cnt = aceso_enum_cuts_count(n_ops, p);
+  if (cnt < 0) return fail(ACESO_ERANGE, "C(n_ops - 1, p - 1) outside [0, 2^62) or bad n_ops / p");
+  if (first < 0 || n < 0 || first + n > cnt) return fail(ACESO_EINVAL, "range [first, first + n) outside [0, %lld)", (long long)cnt);
+  if (n > 0 && (!d_tiled || !d_hdr)) return fail(ACESO_EINVAL, "null argument");
+  if (((uintptr_t)d_tiled & 15) != 0) return fail(ACESO_EINVAL, "tiled output not 16-byte aligned");
+  if (n == 0) return ACESO_OK;
+  const int grid = (int)std::max<int64_t>(1, std::min<int64_t>((n + 255) / 256, 148 * 16));
+  enum_cuts_kernel<<<grid, 256, 0, reinterpret_cast<cudaStream_t>(stream)>>>(
+      n_ops, (uint32_t)(p - 1), code, hdr, first, n, reinterpret_cast<uint4 *>(d_tiled), d_hdr);
+  cudaError_t e = cudaGetLastError();
+  if (e != cudaSuccess) return fail(ACESO_ECUDA, "enumeration launch: %s", cudaGetErrorString(e));
   return ACESO_OK;
 }
 

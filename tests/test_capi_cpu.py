@@ -143,3 +143,14 @@ def test_hash_reference_is_order_and_header_sensitive():
     c2[:, [3, 4]] = c2[:, [4, 3]]
     assert (config_hash(c2, h) != base)[c[:, 3] != c[:, 4]].all()
     assert (config_hash(c, h ^ np.uint64(1 << 8)) != base).all()
+
+
+def test_enum_cuts_count_is_the_binomial():
+    import math
+    from paper_conf_eurosys_liumlsmybw24_b200 import enum_cuts_count
+    for L in (1, 6, 10, 315, 821, 13003, 16384):
+        for p in range(1, 9):
+            want = math.comb(L - 1, p - 1) if p <= L else -1
+            got = enum_cuts_count(L, p)
+            assert got == (want if 0 <= want < (1 << 62) else -1), (L, p, got, want)
+    assert enum_cuts_count(315, 9) == -1 and enum_cuts_count(0, 1) == -1 and enum_cuts_count(315, 0) == -1
