@@ -501,8 +501,12 @@ class _Search:
 
 
 def search(prof, evaluator, p_values=None, budget_s=10.0, max_hops=7, beam=4, heuristic2=True,
-           max_batch=200000, max_k=None, patience=None):
+           max_batch=200000, max_k=None, patience=None, starts=None):
     """Runs the batched Aceso search. Returns (best Result, stats dict).
+
+    starts: optional extra initial configurations [(codes, mbs_log2)], each searched like the
+    paper's initial configurations (e.g. the optimum of the exhaustive stage-uniform space,
+    exhaustive.py, for the hybrid of §9b of DESIGN.md).
 
     Every hop's candidates are generated as base + patches (Primitives.describe_all) and
     evaluated by `evaluator.evaluate_cands(bases, ranks, cands)`, which also returns each
@@ -521,6 +525,8 @@ def search(prof, evaluator, p_values=None, budget_s=10.0, max_hops=7, beam=4, he
         r = initial_config(prof, p)
         if r is not None:
             init.append(r)
+    for c, m in (starts or []):
+        init.append((np.asarray(c, np.uint8), int(m)))
     bases = np.zeros((len(init), stride), np.uint8)
     ranks = np.full((len(init), 2, stride), 0xFFFF, np.uint16)
     cands = np.zeros(len(init), C.CAND_DTYPE)

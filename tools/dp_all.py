@@ -19,13 +19,16 @@ for name in ["toy-a", "toy-b", "gpt3-1.3b", "gpt3-13b", "t5", "wrn", "gpt-1k"]:
     ctx = A.Context(prof, 0)
     X.exhaustive_best(prof, ctx, max_per_family=1 << 10)  # warm-up
     dp = X.exhaustive_best(prof, ctx)
-    dp.pop("codes", None)
-    dp.pop("hdr", None)
+    codes, hdr = dp.pop("codes", None), dp.pop("hdr", None)
     kw = dict(budget_s=budget, patience=8)
     if name == "gpt-1k":
         kw.update(max_k=64, beam=2)
     res, st = S.search(prof, S.GPUEvaluator(ctx), **kw)
-    print(json.dumps({"workload": prof.name, "exhaustive": dp,
-                      "search": {"best": [res.perf[0], res.perf[1]], "explored": st["evaluated"],
-                                 "time_s": st["time_s"]}}), flush=True)
+    line = {"workload": prof.name, "exhaustive": dp,
+            "search": {"best": [res.perf[0], res.perf[1]], "explored": st["evaluated"], "time_s": st["time_s"]}}
+    if codes is not None:  # hybrid: the search also starts from the exhaustive optimum
+        hres, hst = S.search(prof, S.GPUEvaluator(ctx), starts=[(codes, int(hdr & 0xFF))], **kw)
+        line["hybrid"] = {"best": [hres.perf[0], hres.perf[1]], "explored": hst["evaluated"] + dp["explored"],
+                          "time_s": hst["time_s"] + dp["time_s"]}
+    print(json.dumps(line), flush=True)
     ctx.close()
