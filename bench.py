@@ -51,7 +51,9 @@ def parse():
                     help="seconds for the search-time measurement (0: skip)")
     ap.add_argument("--keys-per-allreduce", type=int, default=16,
                     help="N > 1: packed keys of this many steps per all-reduce MIN")
-    ap.add_argument("--streams", type=int, default=4,
+    ap.add_argument("--no-overlap-hint", action="store_true",
+                    help="do not pass ACESO_HINT_OVERLAP when several streams are in flight")
+    ap.add_argument("--streams", type=int, default=8,
                     help="independent batches in flight (steps round-robin over streams)")
     return ap.parse_args()
 
@@ -427,6 +429,7 @@ def main():
         dist.barrier()
     torch.cuda.synchronize()
     nstr = max(1, min(args.streams, nbuf))
+    OVERLAP = nstr > 1 and not args.no_overlap_hint  # ACESO_HINT_OVERLAP: batches overlap on streams
     outs = [out] + [ctx.alloc_outputs(n) for _ in range(nstr - 1)]
     side = [torch.cuda.Stream() for _ in range(nstr)]
     comm = torch.cuda.Stream()  # all-reduces in step order on one stream (same on every rank)
@@ -448,7 +451,8 @@ def main():
                 st.wait_event(comm_done.pop(s - nbuf))
             ev_s[s].record(st)
             ctx.eval(codes_d, hdr_d, n=n, global_offset=rank * n, n_total=n_total, summary=True,
-                     select=True, out=outs[s % nstr], sel=sels[b], stream=st, dense_hint=HINT)
+                     select=True, out=outs[s % nstr], sel=sels[b], stream=st, dense_hint=HINT,
+                     overlap_hint=OVERLAP)
             ev_k[s].record(st)
             if world > 1:
                 # the step's packed key joins a vector of keys; one all-reduce MIN per
@@ -603,6 +607,7 @@ def main():
             "scaling": "weak", "vs_baseline": None, "dtype": "u64", "data": "synthetic",
             "config": {"workload": prof.name, "batch_per_gpu": n, "n_ops": L,
                        "distribution": args.dist, "group_size": args.group, "schedule": schedule,
+                       "streams": nstr, "overlap_hint": OVERLAP,
                        "l2": f"{nbuf} distinct device-resident batches rotated "
                              f"({nbuf * per_batch / 2**20:.0f} MiB > 126 MiB L2)",
                        "parallelism": f"dp{world} (candidate shards) + NCCL all-reduce MIN"},

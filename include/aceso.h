@@ -183,6 +183,13 @@ typedef struct {
                                  recompute at most ops (e.g. uniformly random
                                  encodings); selects the per-op kernel instead
                                  of the event kernel. Results are identical.  */
+#define ACESO_HINT_OVERLAP 16u /* schedule hint: the caller keeps several
+                                 independent batches in flight on different
+                                 streams; the event kernel then launches half the
+                                 CTAs and each warp walks two tiles (per-launch
+                                 prologue/epilogue amortised; higher throughput,
+                                 longer single-launch latency). Results are
+                                 identical.                                    */
 
 /* ------------------------------------------------------------------------- */
 /* Selection (Alg. 1 GetBestOf P:L543, Alg. 2 `perf < init_perf` P:L576).     */
@@ -209,7 +216,8 @@ size_t aceso_select_buf_bytes(const aceso_ctx *ctx, int64_t n);
  * `global_offset` in a job of `n_total` candidates (sharding, §8e).
  *   d_codes : tiled op codes (device)        d_hdr : [n] headers (device)
  *   flags   : OR of ACESO_OUT_SUMMARY / ACESO_OUT_FULL / ACESO_FUSED_SELECT, plus
- *             optionally ACESO_HINT_DENSE. Schedules (results are bit-identical):
+ *             optionally ACESO_HINT_DENSE / ACESO_HINT_OVERLAP. Schedules (results
+ *             are bit-identical):
  *             the event kernel (default for n_ops > 64) walks each candidate's
  *             stage heads and tp/dp changes and takes run sums from position-prefix
  *             tables; the per-op kernel (default for n_ops <= 64, or with the hint)

@@ -161,16 +161,20 @@ class Context:
     def eval(self, codes: torch.Tensor, hdr: torch.Tensor, n: int | None = None, global_offset: int = 0,
              n_total: int | None = None, summary: bool = True, full: bool = False, select: bool = True,
              out: Outputs | None = None, sel: torch.Tensor | None = None, stream=None,
-             dense_hint: bool = False):
+             dense_hint: bool = False, overlap_hint: bool = False):
         """aceso_eval on tiled device codes and int64 device headers.
 
         dense_hint sets ACESO_HINT_DENSE (per-op kernel; identical results).
+        overlap_hint sets ACESO_HINT_OVERLAP (the caller overlaps independent batches on
+        several streams: throughput launch geometry; identical results).
         Returns (out, sel): the output arrays (or None) and the select buffer (or None)."""
         n = int(hdr.shape[0]) if n is None else int(n)
         n_total = global_offset + n if n_total is None else int(n_total)
         flags = (L.OUT_SUMMARY if summary else 0) | (L.OUT_FULL if full else 0) | (L.FUSED_SELECT if select else 0)
         if dense_hint:
             flags |= L.HINT_DENSE
+        if overlap_hint:
+            flags |= L.HINT_OVERLAP
         if (summary or full) and out is None:
             out = self.alloc_outputs(n, full=full)
         if select and sel is None:

@@ -111,6 +111,7 @@ struct aceso_ctx {
   const uint32_t *st;
   int split;        // warps per tile (1 or 2)
   int minb;         // register target: 2 or 3 resident CTAs per SM
+  int tiles_per_warp;  // ACESO_TILES_PER_WARP (measurement knob): tiles each warp walks per launch (default 1)
   int max_ctas[2][8];  // per kernel and mode: resident CTAs (occupancy x SMs)
   size_t smem[2][8];
 };
@@ -522,6 +523,11 @@ int aceso_load_profile(const aceso_profile_desc *d, int cuda_device, aceso_ctx *
       if (v == 1 || (v == 2 && nch >= 2)) ctx->split = v;
     }
     ctx->minb = 3;  // ACESO_MINB=2 selects the ~96-register variant (lower single-launch latency)
+    ctx->tiles_per_warp = 1;
+    if (const char *env = getenv("ACESO_TILES_PER_WARP")) {
+      int v = atoi(env);
+      if (v >= 1 && v <= 64) ctx->tiles_per_warp = v;
+    }
     if (const char *env = getenv("ACESO_MINB")) {
       int v = atoi(env);
       if (v == 2 || v == 3) ctx->minb = v;
@@ -598,7 +604,7 @@ int aceso_eval(aceso_ctx *ctx, const uint8_t *d_codes, const uint64_t *d_hdr, in
   if (n_total >= (1ll << 40)) return fail(ACESO_EINVAL, "n_total >= 2^40");
   if (n >= (1ll << 37)) return fail(ACESO_EINVAL, "n >= 2^37");
   const uint32_t mode = flags & 7u;
-  if (mode == 0 || (flags & ~(7u | ACESO_HINT_DENSE))) return fail(ACESO_EINVAL, "bad flags 0x%x", flags);
+  if (mode == 0 || (flags & ~(7u | ACESO_HINT_DENSE | ACESO_HINT_OVERLAP))) return fail(ACESO_EINVAL, "bad flags 0x%x", flags);
   const int kern = ((flags & ACESO_HINT_DENSE) && ctx->quad_ok) ? 0 : ctx->kernel;
   if (n > 0 && (!d_codes || !d_hdr)) return fail(ACESO_EINVAL, "null codes/headers");
   if ((mode & (ACESO_OUT_SUMMARY | ACESO_OUT_FULL)) && !out) return fail(ACESO_EINVAL, "null outputs");
@@ -614,7 +620,9 @@ int aceso_eval(aceso_ctx *ctx, const uint8_t *d_codes, const uint64_t *d_hdr, in
   P.codes = reinterpret_cast<const uint4 *>(d_codes);
   P.hdr = d_hdr;
 
-  const int tiles_per_cta = kern == 1 ? kWarps : kWarps / ctx->split;
+  // tiles per warp: 1 (latency), 2 with ACESO_HINT_OVERLAP on the event kernel (throughput)
+  const int tpw = (kern == 1 && (flags & ACESO_HINT_OVERLAP)) ? std::max(2, ctx->tiles_per_warp) : ctx->tiles_per_warp;
+  const int tiles_per_cta = (kern == 1 ? kWarps : kWarps / ctx->split) * tpw;
   const int64_t need = (P.n_tiles + tiles_per_cta - 1) / tiles_per_cta;
   int grid = (int)std::max<int64_t>(1, std::min<int64_t>(need, ctx->max_ctas[kern][mode]));
   int prev = 0;

@@ -36,7 +36,7 @@ def ctx_for(prof):
 
 
 def run_gpu(prof, codes, hdr, full=False, gofs=0, n_total=None, pack_on_device=False, select=True,
-            dense_hint=False):
+            dense_hint=False, overlap_hint=False):
     ctx = ctx_for(prof)
     n = len(hdr)
     if pack_on_device:
@@ -45,7 +45,7 @@ def run_gpu(prof, codes, hdr, full=False, gofs=0, n_total=None, pack_on_device=F
         tiled = torch.from_numpy(ai.tile(codes)).cuda()
     hd = torch.from_numpy(np.ascontiguousarray(hdr, np.uint64).view(np.int64)).cuda()
     out, sel = ctx.eval(tiled, hd, n=n, global_offset=gofs, n_total=n_total, full=full, select=select,
-                        dense_hint=dense_hint)
+                        dense_hint=dense_hint, overlap_hint=overlap_hint)
     torch.cuda.synchronize()
     g = dict(iter=as_u64(out.iter_ns), max_mem=as_u64(out.max_mem), info=as_u32(out.info))
     if full:
@@ -54,8 +54,10 @@ def run_gpu(prof, codes, hdr, full=False, gofs=0, n_total=None, pack_on_device=F
     return g, (Selection.from_buffer(sel) if select else None), out, ctx
 
 
-def compare(prof, codes, hdr, full=False, gofs=0, n_total=None, pack_on_device=False, dense_hint=False):
-    g, sel, out, ctx = run_gpu(prof, codes, hdr, full, gofs, n_total, pack_on_device, dense_hint=dense_hint)
+def compare(prof, codes, hdr, full=False, gofs=0, n_total=None, pack_on_device=False, dense_hint=False,
+            overlap_hint=False):
+    g, sel, out, ctx = run_gpu(prof, codes, hdr, full, gofs, n_total, pack_on_device, dense_hint=dense_hint,
+                               overlap_hint=overlap_hint)
     o = oracle.evaluate(prof, codes, hdr, full=full, threads=8)
     for k in ["iter", "max_mem", "info"]:
         bad = np.nonzero(g[k] != o[k])[0]
@@ -130,6 +132,18 @@ def test_dense_hint_schedule_parity(name):
     compare(prof, codes, hdr, full=True, dense_hint=True)
     codes, hdr = ai.search_shaped(prof, SEED + 13, 0, 1500, group_size=64)
     compare(prof, codes, hdr, dense_hint=True)
+
+
+@pytest.mark.parametrize("name", WL)
+def test_overlap_hint_schedule_parity(name):
+    """ACESO_HINT_OVERLAP (half the CTAs, two tiles per warp): identical results, including
+    ragged batches whose last warps walk one tile and a 64K batch (the bench launch)."""
+    prof = P.WORKLOADS[name]()
+    for n, seed in [(4099, SEED + 14), (33, SEED + 15), (65536, SEED + 16)]:
+        codes, hdr = ai.search_shaped(prof, seed, 0, n, group_size=64)
+        compare(prof, codes, hdr, overlap_hint=True)
+    codes, hdr = ai.dense_random(prof, SEED + 17, 0, 1025)
+    compare(prof, codes, hdr, full=True, overlap_hint=True)
 
 
 def _crowded_candidates(prof, n, seed, pair_stages):
