@@ -185,11 +185,12 @@ typedef struct {
                                  of the event kernel. Results are identical.  */
 #define ACESO_HINT_OVERLAP 16u /* schedule hint: the caller keeps several
                                  independent batches in flight on different
-                                 streams; the event kernel then launches half the
-                                 CTAs and each warp walks two tiles (per-launch
-                                 prologue/epilogue amortised; higher throughput,
-                                 longer single-launch latency). Results are
-                                 identical.                                    */
+                                 streams; for models of at most 384 ops the event
+                                 kernel then launches half the CTAs and each warp
+                                 walks two tiles (per-launch prologue/epilogue
+                                 amortised; higher throughput, longer single-
+                                 launch latency); longer models are unaffected.
+                                 Results are identical.                         */
 
 /* ------------------------------------------------------------------------- */
 /* Selection (Alg. 1 GetBestOf P:L543, Alg. 2 `perf < init_perf` P:L576).     */

@@ -227,10 +227,31 @@ def test_gpt_1k_layers_parity():
 
 
 def test_bench_config_full_size_parity():
-    """The bench workload (GPT-3 1.3B, 8 devices, 65,536 candidates, bench seed) at full size."""
+    """The bench workload (GPT-3 1.3B, 8 devices, 65,536 candidates, bench seed) at full size,
+    in both launch geometries (bench.py times the overlap hint)."""
     prof = P.WORKLOADS["gpt3-1.3b"]()
     codes, hdr = ai.search_shaped(prof, SEED, 0, 65536, group_size=1024)
     compare(prof, codes, hdr)
+    compare(prof, codes, hdr, overlap_hint=True)
+
+
+def test_gpt3_13b_full_batch_parity():
+    """BASELINE configs[2]: GPT-3 13B on 32 devices, a 262,144-candidate batch,
+    overlap-hint launch, every output and the selection against the oracle."""
+    prof = P.WORKLOADS["gpt3-13b"]()
+    codes, hdr = ai.search_shaped(prof, SEED + 20, 0, 262144, group_size=1024)
+    compare(prof, codes, hdr, overlap_hint=True)
+
+
+def test_gpt_1k_one_gpu_share_parity():
+    """BASELINE configs[4]: 1K-layer GPT on 64 devices, 1M candidates across 8 GPUs; one GPU's
+    share (131,072 candidates, rank 3's global offsets in n_total = 1,048,576) as bench.py
+    --config gpt-1k --gpus 8 launches it, every output and the shard's selection against the
+    oracle."""
+    prof = P.WORKLOADS["gpt-1k"]()
+    n, rank = 131072, 3
+    codes, hdr = ai.search_shaped(prof, SEED + 21, rank * n, n, group_size=1024)
+    compare(prof, codes, hdr, gofs=rank * n, n_total=8 * n, overlap_hint=True)
 
 
 # ---------------------------------------------------------------------------
