@@ -24,9 +24,11 @@
  * Pins (tests/test_oracle_pins.py): 1F1B discrete-event simulation of uniform
  * pipelines (makespan and in-flight activations), closed forms for p = 1 and
  * recomputation, zero-cost-op invariance, Fig. 3 scenarios, record-lookup
- * fingerprints, brute-force enumeration of the toy spaces. The placement of the
- * p2p, reshard and DP-sync terms (R5, R6, R13) is "parity unpinned" beyond the
- * worked examples derived from the readings.
+ * fingerprints, brute-force enumeration of the toy spaces, and the inter-stage
+ * sends (R5) against the 1F1B simulation with sender-side sends on pipelines
+ * made uniform by compensating compute. The reshard term (R13) and the DP sync
+ * of stages other than stage 0 (R6) are "parity unpinned" beyond the worked
+ * examples derived from the readings.
  */
 #include <stdint.h>
 #include <stdlib.h>

@@ -262,6 +262,49 @@ def test_memory_terms_special_cases():
 
 
 # --------------------------------------------------------------------------
+# R5 (inter-stage sends) against the 1F1B simulation: a send occupies its sender
+# after the compute and the receiver waits for its end, i.e. the simulation runs with
+# F'_i = F_i + [i < p-1] c_fwd and B'_i = B_i + [i > 0] c_bwd. The edge stage that sends
+# nothing in one direction gets the same amount of extra compute instead, so the pipeline
+# is uniform and Eq. 2 (R1) is exact -- but only if the oracle charges p2p_fwd of each
+# non-last stage's LAST op and p2p_bwd of each non-first stage's FIRST op, per microbatch.
+# The other ops carry different p2p values that must not be charged.
+# --------------------------------------------------------------------------
+@pytest.mark.parametrize("p", [2, 3, 4, 5])
+@pytest.mark.parametrize("mbs_log2", [0, 1, 3])
+def test_p2p_forward_sends_match_1f1b_simulation(p, mbs_log2):
+    k, f, b, c = 3, 7, 13, 5
+    recs = {0: lambda tpl, bb: [f, 0, b, 0, 0, 0, 0, 0, 1000, 0],     # inner op: p2p_fwd never charged
+            1: lambda tpl, bb: [f, 0, b, 0, 0, 0, 0, 0, c, 0],        # last op of stages 0..p-2
+            2: lambda tpl, bb: [f + c, 0, b, 0, 0, 0, 0, 0, 3000, 0]}  # last op of the last stage
+    types = ([0] * (k - 1) + [1]) * (p - 1) + [0] * (k - 1) + [2]
+    prof = mkprof(recs, types, G=p, Bg=8)
+    N = 8 >> mbs_log2
+    out = ev(prof, [cand([k] * p)], [ai.header(mbs_log2, p)])
+    assert out["info"][0] & oracle.INFO_INVALID == 0
+    mk, _ = simulate([k * f + c] * p, [k * b] * p, N)
+    assert int(out["iter"][0]) == mk == (N + p - 1) * (k * (f + b) + c)
+    assert len(set(int(x) for x in out["stage_T"][0, :p])) == 1
+
+
+@pytest.mark.parametrize("p", [2, 3, 4, 5])
+@pytest.mark.parametrize("mbs_log2", [0, 1, 3])
+def test_p2p_backward_sends_match_1f1b_simulation(p, mbs_log2):
+    k, f, b, c = 3, 7, 13, 5
+    recs = {0: lambda tpl, bb: [f, 0, b, 0, 0, 0, 0, 0, 0, 1000],     # inner op: p2p_bwd never charged
+            1: lambda tpl, bb: [f, 0, b, 0, 0, 0, 0, 0, 0, c],        # first op of stages 1..p-1
+            2: lambda tpl, bb: [f, 0, b + c, 0, 0, 0, 0, 0, 0, 3000]}  # first op of stage 0
+    types = [2] + [0] * (k - 1) + ([1] + [0] * (k - 1)) * (p - 1)
+    prof = mkprof(recs, types, G=p, Bg=8)
+    N = 8 >> mbs_log2
+    out = ev(prof, [cand([k] * p)], [ai.header(mbs_log2, p)])
+    assert out["info"][0] & oracle.INFO_INVALID == 0
+    mk, _ = simulate([k * f] * p, [k * b + c] * p, N)
+    assert int(out["iter"][0]) == mk == (N + p - 1) * (k * (f + b) + c)
+    assert len(set(int(x) for x in out["stage_T"][0, :p])) == 1
+
+
+# --------------------------------------------------------------------------
 # readings without an independent pin: worked examples (parity unpinned beyond these)
 # --------------------------------------------------------------------------
 def test_p2p_and_reshard_worked_example():
