@@ -112,6 +112,28 @@ def test_dp_sync_on_first_stage_matches_simulation():
     assert int(out["iter"][0]) == mk
 
 
+def test_dp_sync_on_any_stage_with_free_backward_matches_simulation():
+    """R6 on every stage: with a zero-time backward the 1F1B backward cascade is instant,
+    every stage ends its last backward at the same time, and the iteration ends with the
+    slowest stage's own DP sync: makespan = (N+p-1)F + max_i D_i. Eq. 2 gives the same only
+    if D_i is added to stage i's own T_i (not summed over stages, not added to others)."""
+    rng = np.random.default_rng(11)
+    for _ in range(30):
+        p = int(rng.integers(2, 6))
+        k = int(rng.integers(1, 4))
+        d = [int(x) for x in rng.integers(0, 400, size=p)]
+        recs = {i: (lambda tpl, bb: [5, 0, 0, 0, 0, 0, 0, 0, 0, 0]) for i in range(p)}
+        types = [i for i in range(p) for _ in range(k)]
+        dps = [[[d[i]]] for i in range(p)]
+        prof = mkprof(recs, types, G=p, Bg=8, dps=dps)
+        mbs_log2 = int(rng.integers(0, 4))
+        N = 8 >> mbs_log2
+        out = ev(prof, [cand([k] * p)], [ai.header(mbs_log2, p)])
+        assert out["info"][0] & oracle.INFO_INVALID == 0
+        mk, _ = simulate([5 * k] * p, [0] * p, N, sync=[k * x for x in d])
+        assert int(out["iter"][0]) == mk == (N + p - 1) * 5 * k + k * max(d)
+
+
 # --------------------------------------------------------------------------
 # recomputation (P:L241, R3, R7)
 # --------------------------------------------------------------------------
