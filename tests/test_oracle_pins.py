@@ -132,6 +132,10 @@ def test_dp_sync_on_any_stage_with_free_backward_matches_simulation():
         assert out["info"][0] & oracle.INFO_INVALID == 0
         mk, _ = simulate([5 * k] * p, [0] * p, N, sync=[k * x for x in d])
         assert int(out["iter"][0]) == mk == (N + p - 1) * 5 * k + k * max(d)
+        # per stage: T_i = the makespan when only stage i synchronises (attribution of D_i)
+        for i in range(p):
+            mk_i, _ = simulate([5 * k] * p, [0] * p, N, sync=[k * d[i] if s == i else 0 for s in range(p)])
+            assert int(out["stage_T"][0, i]) == mk_i
 
 
 # --------------------------------------------------------------------------
