@@ -26,9 +26,10 @@
  * recomputation, zero-cost-op invariance, Fig. 3 scenarios, record-lookup
  * fingerprints, brute-force enumeration of the toy spaces, and the inter-stage
  * sends (R5) against the 1F1B simulation with sender-side sends on pipelines
- * made uniform by compensating compute. The reshard term (R13) and the DP sync
- * of stages other than stage 0 (R6) are "parity unpinned" beyond the worked
- * examples derived from the readings.
+ * made uniform by compensating compute, and the DP sync of every stage (R6)
+ * against the simulation with a zero-time backward (instant cascade). The
+ * reshard term (R13) is "parity unpinned" beyond the worked example derived from
+ * its reading.
  */
 #include <stdint.h>
 #include <stdlib.h>
