@@ -21,6 +21,7 @@
 #include "incr_kernel.cuh"
 #include "eval_kernel.cuh"
 #include "event_kernel.cuh"
+#include "dense_kernel.cuh"
 #include "enum_kernel.cuh"
 
 using namespace aceso;
@@ -79,9 +80,25 @@ void *event_kernel_for(uint32_t mode) {
   }
 }
 
-// kernel 0: per-op/quad kernel (eval_kernel.cuh); kernel 1: event kernel (event_kernel.cuh)
+template <int B>
+void *dense_kernel_for(uint32_t mode) {
+  switch (mode) {
+    case 1: return reinterpret_cast<void *>(&dense_kernel<1, B>);
+    case 2: return reinterpret_cast<void *>(&dense_kernel<2, B>);
+    case 3: return reinterpret_cast<void *>(&dense_kernel<3, B>);
+    case 4: return reinterpret_cast<void *>(&dense_kernel<4, B>);
+    case 5: return reinterpret_cast<void *>(&dense_kernel<5, B>);
+    case 6: return reinterpret_cast<void *>(&dense_kernel<6, B>);
+    case 7: return reinterpret_cast<void *>(&dense_kernel<7, B>);
+    default: return nullptr;
+  }
+}
+
+// kernel 0: per-op/quad kernel (eval_kernel.cuh); kernel 1: event kernel (event_kernel.cuh);
+// kernel 2: dense kernel (dense_kernel.cuh, ACESO_HINT_DENSE)
 void *eval_kernel_for(uint32_t mode, int split, int minb, int kernel) {
   if (kernel == 1) return minb == 2 ? event_kernel_for<2>(mode) : event_kernel_for<3>(mode);
+  if (kernel == 2) return minb == 2 ? dense_kernel_for<2>(mode) : dense_kernel_for<3>(mode);
   if (minb == 2) return split == 2 ? eval_kernel_split<2, 2>(mode) : eval_kernel_split<1, 2>(mode);
   return split == 2 ? eval_kernel_split<2, 3>(mode) : eval_kernel_split<1, 3>(mode);
 }
@@ -112,8 +129,9 @@ struct aceso_ctx {
   int split;        // warps per tile (1 or 2)
   int minb;         // register target: 2 or 3 resident CTAs per SM
   int tiles_per_warp;  // ACESO_TILES_PER_WARP (measurement knob): tiles each warp walks per launch (default 1)
-  int max_ctas[2][8];  // per kernel and mode: resident CTAs (occupancy x SMs)
-  size_t smem[2][8];
+  int max_ctas[3][8];  // per kernel and mode: resident CTAs (occupancy x SMs)
+  int dense_kernel;    // schedule of ACESO_HINT_DENSE: 2 dense kernel (default), 0 per-op kernel (ACESO_DENSE_KERNEL=quad)
+  size_t smem[3][8];
 };
 
 namespace {
@@ -540,18 +558,21 @@ int aceso_load_profile(const aceso_profile_desc *d, int cuda_device, aceso_ctx *
       ctx->st = reinterpret_cast<const uint32_t *>(eb + ev_st);
       ctx->qr = reinterpret_cast<const uint4 *>(eb + ev_qr);
     }
-    for (int kern = 0; kern < 2 && rc == ACESO_OK; ++kern)
+    ctx->dense_kernel = 2;
+    if (const char *env = getenv("ACESO_DENSE_KERNEL"))
+      if (!strcmp(env, "quad")) ctx->dense_kernel = 0;
+    for (int kern = 0; kern < 3 && rc == ACESO_OK; ++kern)
       for (uint32_t mode = 1; mode < 8; ++mode) {
-        if (kern == 0 && !quad_ok) {
-          ctx->smem[0][mode] = 0;
-          ctx->max_ctas[0][mode] = 0;
+        if (kern != 1 && !quad_ok) {
+          ctx->smem[kern][mode] = 0;
+          ctx->max_ctas[kern][mode] = 0;
           continue;
         }
+        const size_t tabs = ((mode & ACESO_OUT_FULL) ? tab.bytes_full : tab.bytes) + (tab.k_smem ? bytesK : 0u);
         const size_t smem =
-            kern == 1
-                ? (size_t)qo_bytes + ev_ring_bytes() + ev_list_bytes((mode & ACESO_OUT_FULL) != 0)
-                : ((mode & ACESO_OUT_FULL) ? tab.bytes_full : tab.bytes) + (tab.k_smem ? bytesK : 0u) +
-                      kRingBytesPerCta + (ctx->split == 2 ? (size_t)(kWarps / 2) * 32 * sizeof(Xchg) : 0);
+            kern == 1   ? (size_t)qo_bytes + ev_ring_bytes() + ev_list_bytes((mode & ACESO_OUT_FULL) != 0)
+            : kern == 2 ? tabs + kRingBytesPerCta
+                        : tabs + kRingBytesPerCta + (ctx->split == 2 ? (size_t)(kWarps / 2) * 32 * sizeof(Xchg) : 0);
         ctx->smem[kern][mode] = smem;
         void *k = eval_kernel_for(mode, ctx->split, ctx->minb, kern);
         e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
@@ -590,7 +611,7 @@ size_t aceso_select_buf_bytes(const aceso_ctx *ctx, int64_t n) {
   (void)n;
   if (!ctx) return 0;
   int m = 0;
-  for (int kern = 0; kern < 2; ++kern)
+  for (int kern = 0; kern < 3; ++kern)
     for (int k = 1; k < 8; ++k) m = std::max(m, ctx->max_ctas[kern][k]);
   m = std::max(m, 4 * ctx->sms);  // per-CTA partials of the eval kernels; select kernel grid
   return (size_t)kSelPartialOff + 16 * (size_t)m;
@@ -605,7 +626,7 @@ int aceso_eval(aceso_ctx *ctx, const uint8_t *d_codes, const uint64_t *d_hdr, in
   if (n >= (1ll << 37)) return fail(ACESO_EINVAL, "n >= 2^37");
   const uint32_t mode = flags & 7u;
   if (mode == 0 || (flags & ~(7u | ACESO_HINT_DENSE | ACESO_HINT_OVERLAP))) return fail(ACESO_EINVAL, "bad flags 0x%x", flags);
-  const int kern = ((flags & ACESO_HINT_DENSE) && ctx->quad_ok) ? 0 : ctx->kernel;
+  const int kern = ((flags & ACESO_HINT_DENSE) && ctx->quad_ok) ? ctx->dense_kernel : ctx->kernel;
   if (n > 0 && (!d_codes || !d_hdr)) return fail(ACESO_EINVAL, "null codes/headers");
   if ((mode & (ACESO_OUT_SUMMARY | ACESO_OUT_FULL)) && !out) return fail(ACESO_EINVAL, "null outputs");
   if ((mode & ACESO_OUT_SUMMARY) && n > 0 && (!out->iter_ns || !out->max_mem || !out->info)) return fail(ACESO_EINVAL, "null summary array");
@@ -625,7 +646,7 @@ int aceso_eval(aceso_ctx *ctx, const uint8_t *d_codes, const uint64_t *d_hdr, in
   // epilogue (measured: GPT-3 1.3B +7%, Wide-ResNet +7%; GPT-3 13B, T5 and 1K layers lose with 2)
   const int tpw = (kern == 1 && (flags & ACESO_HINT_OVERLAP) && P.nch <= 24) ? std::max(2, ctx->tiles_per_warp)
                                                                             : ctx->tiles_per_warp;
-  const int tiles_per_cta = (kern == 1 ? kWarps : kWarps / ctx->split) * tpw;
+  const int tiles_per_cta = (kern != 0 ? kWarps : kWarps / ctx->split) * tpw;
   const int64_t need = (P.n_tiles + tiles_per_cta - 1) / tiles_per_cta;
   int grid = (int)std::max<int64_t>(1, std::min<int64_t>(need, ctx->max_ctas[kern][mode]));
   int prev = 0;

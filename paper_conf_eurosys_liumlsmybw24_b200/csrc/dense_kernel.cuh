@@ -1,0 +1,182 @@
+// dense_kernel.cuh — per-op evaluation for candidates whose tp/dp changes at most ops
+// (ACESO_HINT_DENSE; e.g. uniformly random encodings), sm_100a.
+//
+// Same contract, tables and outputs as eval_kernel.cuh (thread = candidate, warp = tile of
+// 32 candidates streamed through a per-warp cp.async.bulk ring, profile tables staged in
+// shared memory), but no event handler: every op is accumulated by the same branch-free
+// sequence under its OWN (b, tp) record — so an in-stage tp/dp change costs one predicated
+// reshard lookup instead of a run switch, and lanes stay converged except at stage heads
+// (at most p per candidate).
+//
+// Per op j with code c (head, log2 tp, recompute, log2 dp):
+//   head at j > 0 : the open stage takes p2p_fwd of op j-1 (R5) and closes (Eq. 1/2, OOM,
+//                   Heuristic-1: stage_commit); the new stage takes p2p_bwd of op j (R5)
+//   otherwise     : reshard of op j if its (tp, dp) differs from op j-1's (R13);
+//                   tp*dp must equal the stage's (R9)
+//   every op      : S += fwd+bwd (+fwd if rc, R7), A += act or keep (R3),
+//                   E = max(E, peak (+act-keep if rc)) (R4), W += param+opt, D += DP sync (R6)
+// Readings R1-R13, R18-R20 in DESIGN.md §3.
+#pragma once
+#include "eval_kernel.cuh"
+
+namespace aceso {
+
+template <uint32_t MODE, int MINB>
+__global__ void __launch_bounds__(kThreads, MINB) dense_kernel(const __grid_constant__ EvalParams P) {
+  extern __shared__ __align__(128) unsigned char sm_raw[];
+  __shared__ __align__(8) uint64_t s_tbar;
+  __shared__ __align__(8) uint64_t s_ring_bar[kWarps][kRingSlots];
+  __shared__ uint64_t s_ck[kWarps];
+  __shared__ int64_t s_idx[kWarps];
+
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const uint32_t tab_bytes = (MODE & kFull) ? P.tab.bytes_full : P.tab.bytes;
+  const uint32_t sb = smem_addr(sm_raw);
+  Smem sm;
+  sm.R = sb + P.tab.offR;
+  sm.D = sb + P.tab.offD;
+  sm.T = sb + P.tab.offT;
+  sm.F = sb + P.tab.offF;
+  sm.K = sb + tab_bytes;  // cold table staged after the other tables when k_smem
+  sm.Kg = reinterpret_cast<const unsigned char *>(P.blob) + P.tab.offK;
+  sm.k_smem = P.tab.k_smem;
+  sm.TS = (uint32_t)P.T * kTypeStride;
+  const uint32_t stage_bytes = tab_bytes + (P.tab.k_smem ? P.tab.bytesK : 0u);
+  const uint32_t ring = sb + stage_bytes + (uint32_t)warp * kRingSlots * kSlotBytes;
+
+  if (threadIdx.x == 0) {
+    mbar_init(smem_addr(&s_tbar), 1);
+    fence_barrier_init();
+  }
+  if (lane == 0) {
+    for (int k = 0; k < kRingSlots; ++k) mbar_init(smem_addr(&s_ring_bar[warp][k]), 1);
+    fence_barrier_init();
+  }
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    const uint32_t bar = smem_addr(&s_tbar);
+    mbar_expect_tx(bar, stage_bytes);
+    bulk_g2s(sb, P.blob, tab_bytes, bar);
+    if (P.tab.k_smem) bulk_g2s(sb + tab_bytes, sm.Kg, P.tab.bytesK, bar);
+  }
+
+  const uint32_t nch = (uint32_t)P.nch;
+  const uint32_t L = (uint32_t)P.L;
+  const uint32_t ngroups = (nch + kSlotChunks - 1) / kSlotChunks;
+  const int64_t first_tile = (int64_t)blockIdx.x * kWarps + warp;
+  const int64_t tile_stride = (int64_t)gridDim.x * kWarps;
+  const int64_t my_tiles = first_tile < P.n_tiles ? (P.n_tiles - first_tile + tile_stride - 1) / tile_stride : 0;
+  const int64_t units = my_tiles * ngroups;
+  const unsigned char *codes = reinterpret_cast<const unsigned char *>(P.codes);
+
+  int64_t it_tile = first_tile;
+  uint32_t it_g = 0;
+  auto issue_next = [&](int slot) {
+    const uint32_t a = kSlotChunks * it_g, b = min(a + kSlotChunks, nch);
+    const uint32_t bar = smem_addr(&s_ring_bar[warp][slot]);
+    mbar_expect_tx(bar, (b - a) * 512u);
+    bulk_g2s(ring + slot * kSlotBytes, codes + ((size_t)it_tile * nch + a) * 512, (b - a) * 512u, bar);
+    if (++it_g == ngroups) {
+      it_g = 0;
+      it_tile += tile_stride;
+    }
+  };
+  if (lane == 0) {
+    for (int64_t u = 0; u < units && u < kRingSlots; ++u) issue_next((int)u);
+  }
+  __syncwarp();
+  mbar_wait(smem_addr(&s_tbar), 0);  // tables resident
+
+  const uint32_t n_tp = (uint32_t)P.n_tp, n_dp = (uint32_t)P.n_dp, n_b = (uint32_t)P.n_b;
+  uint64_t best_ck = ~0ull;
+  int64_t best_idx = INT64_MAX;
+  Cand s;
+  uint32_t prev = 0;   // code of op j-1
+  uint32_t pk = 0;     // K-table byte offset of op j-1 (its run and type)
+  int64_t tile = first_tile;
+  uint32_t g = 0;
+  int slot = 0;
+  uint32_t phase = 0;
+  int64_t cand = 0;
+  bool active = false;
+  for (int64_t u = 0; u < units; ++u) {
+    if (g == 0) {
+      cand = tile * 32 + lane;
+      active = cand < P.n;
+      init_cand(s, sm, P, active ? __ldg(P.hdr + cand) : 0ull, false);
+    }
+    mbar_wait(smem_addr(&s_ring_bar[warp][slot]), phase);
+    const uint32_t a = kSlotChunks * g, b = min(a + kSlotChunks, nch);
+    const uint32_t slot_a = ring + slot * kSlotBytes + lane * 16;
+    if (g == 0) s.head0 = lds32(slot_a) & 1u;
+#pragma unroll 1
+    for (uint32_t ch = a; ch < b; ++ch) {
+      const uint4 w4 = lds128(slot_a + (ch - a) * 512u);
+      const uint32_t nq = min(4u, (L - ch * 16u + 3u) >> 2);  // quads inside L
+#pragma unroll 1
+      for (uint32_t q = 0; q < nq; ++q) {
+        const uint32_t w = q == 0 ? w4.x : q == 1 ? w4.y : q == 2 ? w4.z : w4.w;
+        const uint32_t j0 = ch * 16u + q * 4u;
+        const uint2 tt = lds64(sm.T + 2u * j0);  // the quad's 4 u16 types
+        const uint32_t nv = min(4u, L - j0);
+#pragma unroll
+        for (uint32_t k = 0; k < 4; ++k) {
+          if (k < nv) {
+            const uint32_t j = j0 + k;
+            const uint32_t c = (w >> (8u * k)) & 0xffu;
+            const uint32_t toff = ((k < 2 ? tt.x >> (16u * k) : tt.y >> (16u * (k - 2))) & 0xffffu) << 5;
+            const uint32_t tpl = (c >> 1) & 7u, dpl = c >> 5, rc = (c >> 4) & 1u;
+            const uint32_t gg = tpl + dpl;
+            if (dpl > s.mbs) s.reasons |= ACESO_R_DPMBS;
+            if (tpl >= n_tp || dpl >= n_dp || (dpl <= s.mbs && s.mbs - dpl >= n_b)) s.reasons |= ACESO_R_TABLE;
+            // clamped indices keep every gather inside the tables for invalid encodings
+            const uint32_t bb = min(dpl <= s.mbs ? s.mbs - dpl : 0u, n_b - 1u);
+            const uint32_t tplc = min(tpl, n_tp - 1u);
+            const uint32_t run = bb * n_tp + tplc;
+            const uint32_t kofs = run * (sm.TS >> 1) + (toff >> 1);
+            if ((c & 1u) || j == 0) {
+              if ((c & 1u) && j > 0) {
+                s.S += ldk(sm, pk + 4u);  // R5: p2p_fwd of the stage's last op (j-1)
+                stage_commit<MODE>(s, P, cand, active, false);
+                s.i += 1;
+                s.S += ldk(sm, kofs + 8u);  // R5: p2p_bwd of the stage's first op
+              }
+              s.gst = gg;
+              s.gsum += 1u << gg;  // R9
+              s.nheads += c & 1u;
+            } else {
+              if (gg != s.gst) s.reasons |= ACESO_R_GSTAGE;     // P:L151 in-stage symmetry
+              if ((c ^ prev) & 0xeeu) s.S += ldk(sm, kofs);      // R13: reshard into op j
+            }
+            const uint4 r = lds128(sm.R + run * sm.TS + toff + rc * 16u);
+            s.S += r.x;
+            s.A += r.y;
+            s.E = max(s.E, r.z);
+            s.W += r.w;
+            s.D += lds32(sm.D + tplc * sm.TS + toff + dpl * 4u);
+            if (MODE & kFull) s.comp += lds32(sm.F + run * (sm.TS >> 2) + (toff >> 2) + rc * 4u);
+            prev = c;
+            pk = kofs;
+          }
+        }
+      }
+    }
+    __syncwarp();
+    if (lane == 0 && u + kRingSlots < units) {
+      fence_proxy_async();
+      issue_next(slot);
+    }
+    slot = (slot + 1) % kRingSlots;
+    if (slot == 0) phase ^= 1u;
+    if (++g == ngroups) {
+      stage_commit<MODE>(s, P, cand, active, false);  // last stage: no p2p_fwd
+      finish_cand<MODE>(s, P, cand, active, best_ck, best_idx);
+      g = 0;
+      tile += tile_stride;
+    }
+  }
+
+  if (MODE & kSelect) block_select_finish(best_ck, best_idx, P.sel, P.n_total, P.ib, s_ck, s_idx);
+}
+
+}  // namespace aceso

@@ -380,6 +380,33 @@ def test_kernel_variants_parity(kernel, split, minb, name, monkeypatch):
         ctx.close()
 
 
+@pytest.mark.parametrize("minb", ["2", "3"])
+@pytest.mark.parametrize("dense_kernel", ["dense", "quad"])
+@pytest.mark.parametrize("name", ["gpt3-1.3b", "t5", "wrn", "gpt3-13b", "toy-a", "toy-b"])
+def test_dense_hint_kernels_parity(dense_kernel, minb, name, monkeypatch):
+    """ACESO_HINT_DENSE runs the dense kernel (default) or the per-op kernel
+    (ACESO_DENSE_KERNEL=quad): every output bit-exact on dense, search-shaped and random-byte
+    batches, all modes, ragged sizes."""
+    monkeypatch.setenv("ACESO_DENSE_KERNEL", dense_kernel)
+    monkeypatch.setenv("ACESO_MINB", minb)
+    prof = P.WORKLOADS[name]()
+    ctx = A.Context(prof, 0)
+    _ctx_cache[id(prof)] = (prof, ctx)
+    try:
+        codes, hdr = ai.dense_random(prof, SEED + 40, 0, 1031)
+        compare(prof, codes, hdr, full=True, dense_hint=True)
+        compare(prof, codes[:77], hdr[:77], dense_hint=True)
+        codes, hdr = ai.search_shaped(prof, SEED + 41, 0, 999, group_size=16)
+        compare(prof, codes, hdr, full=True, dense_hint=True)
+        rng = np.random.default_rng(6)
+        codes = rng.integers(0, 256, size=(300, prof.n_ops), dtype=np.uint8)
+        hdr = rng.integers(0, 1 << 16, size=300, dtype=np.uint64)
+        compare(prof, codes, hdr, full=True, dense_hint=True)
+    finally:
+        _ctx_cache.pop(id(prof), None)
+        ctx.close()
+
+
 def test_nccl_allreduce_min_single_rank():
     """dist.global_select over a one-rank NCCL group on the device select buffer."""
     import socket
