@@ -318,7 +318,16 @@ int aceso_load_profile(const aceso_profile_desc *d, int cuda_device, aceso_ctx *
   // the per-op kernel stages its tables in shared memory; larger profiles use the event
   // kernel only (its tables are in global memory)
   const bool quad_ok = tab.bytes_full + kRingBytesPerCta + 16384u <= 220u * 1024u;
-  const uint32_t blob_bytes = tab.offK + bytesK;
+  tab.dOff = a16(tab.offK + bytesK);
+  tab.dR = 0;
+  tab.dD = tab.dR + bytesR;
+  tab.dK = tab.dD + bytesD;
+  tab.dT = tab.dK + bytesK;
+  tab.dbytes = tab.dT + bytesT;
+  tab.dF = tab.dbytes;
+  tab.dbytes_full = tab.dF + bytesF;
+  const bool dense_ok = tab.dbytes_full + kRingBytesPerCta + 16384u <= 220u * 1024u;
+  const uint32_t blob_bytes = tab.dOff + tab.dbytes_full;
   std::vector<uint32_t> blob(blob_bytes / 4, 0u);
   auto rec_S = [&](int t, int tp, int b, int rc) -> uint64_t {
     uint64_t F = (uint64_t)R(t, tp, b, 0) + R(t, tp, b, 1);
@@ -351,14 +360,32 @@ int aceso_load_profile(const aceso_profile_desc *d, int cuda_device, aceso_ctx *
         k[0] = (uint32_t)R(t, tp, b, 7);
         k[1] = (uint32_t)R(t, tp, b, 8);
         k[2] = (uint32_t)R(t, tp, b, 9);
+        // dense-kernel copies, type-major
+        const uint32_t tr = (uint32_t)t * RUNS + (uint32_t)(b * NT + tp);  // (type, run) index
+        for (int rc = 0; rc < 2; ++rc) {
+          uint32_t *r = &blob[(tab.dOff + tab.dR) / 4 + tr * 8 + rc * 4];
+          r[0] = (uint32_t)rec_S(t, tp, b, rc);
+          r[1] = (uint32_t)rec_A(t, tp, b, rc);
+          r[2] = (uint32_t)rec_e(t, tp, b, rc);
+          r[3] = (uint32_t)rec_W(t, tp);
+          blob[(tab.dOff + tab.dF) / 4 + tr * 2 + rc] = (uint32_t)rec_C(t, tp, b, rc);
+        }
+        uint32_t *dk = &blob[(tab.dOff + tab.dK) / 4 + tr * 4];
+        dk[0] = k[0];
+        dk[1] = k[1];
+        dk[2] = k[2];
       }
   for (int tp = 0; tp < NT; ++tp)
     for (int t = 0; t < T; ++t)
       for (int dp = 0; dp < ND; ++dp)
+      {
         blob[(tab.offD + ((uint32_t)tp * T + t) * S) / 4 + dp] = (uint32_t)dps_of(t, tp, dp);
+        blob[(tab.dOff + tab.dD) / 4 + ((uint32_t)t * NT + tp) * 8 + dp] = (uint32_t)dps_of(t, tp, dp);
+      }
   {
     uint16_t *tt = reinterpret_cast<uint16_t *>(&blob[tab.offT / 4]);
-    for (int j = 0; j < L; ++j) tt[j] = d->op_type[j];
+    uint16_t *dt = reinterpret_cast<uint16_t *>(&blob[(tab.dOff + tab.dT) / 4]);
+    for (int j = 0; j < L; ++j) tt[j] = dt[j] = d->op_type[j];
   }
   // quad sums; a signature whose sums do not fit 32 bits is not used (per-op path)
   std::vector<char> sig_ok(NS, 1);
@@ -558,12 +585,12 @@ int aceso_load_profile(const aceso_profile_desc *d, int cuda_device, aceso_ctx *
       ctx->st = reinterpret_cast<const uint32_t *>(eb + ev_st);
       ctx->qr = reinterpret_cast<const uint4 *>(eb + ev_qr);
     }
-    ctx->dense_kernel = 2;
+    ctx->dense_kernel = dense_ok ? 2 : 0;  // its tables must fit in shared memory
     if (const char *env = getenv("ACESO_DENSE_KERNEL"))
       if (!strcmp(env, "quad")) ctx->dense_kernel = 0;
     for (int kern = 0; kern < 3 && rc == ACESO_OK; ++kern)
       for (uint32_t mode = 1; mode < 8; ++mode) {
-        if (kern != 1 && !quad_ok) {
+        if ((kern == 0 && !quad_ok) || (kern == 2 && !dense_ok)) {
           ctx->smem[kern][mode] = 0;
           ctx->max_ctas[kern][mode] = 0;
           continue;
@@ -571,7 +598,7 @@ int aceso_load_profile(const aceso_profile_desc *d, int cuda_device, aceso_ctx *
         const size_t tabs = ((mode & ACESO_OUT_FULL) ? tab.bytes_full : tab.bytes) + (tab.k_smem ? bytesK : 0u);
         const size_t smem =
             kern == 1   ? (size_t)qo_bytes + ev_ring_bytes() + ev_list_bytes((mode & ACESO_OUT_FULL) != 0)
-            : kern == 2 ? tabs + kRingBytesPerCta
+            : kern == 2 ? ((mode & ACESO_OUT_FULL) ? tab.dbytes_full : tab.dbytes) + kRingBytesPerCta
                         : tabs + kRingBytesPerCta + (ctx->split == 2 ? (size_t)(kWarps / 2) * 32 * sizeof(Xchg) : 0);
         ctx->smem[kern][mode] = smem;
         void *k = eval_kernel_for(mode, ctx->split, ctx->minb, kern);

@@ -41,6 +41,11 @@ struct Tables {
   uint32_t offK;                    // byte offset of the cold table in the global blob
   uint32_t bytesK;                  // bytes of the cold table
   uint32_t k_smem;                  // 1: the cold table is staged to shared memory too
+  // dense-kernel tables (dense_kernel.cuh): the same records TYPE-major, so that the lanes of
+  // a warp (same op, same type, different runs) read neighbouring records, not one bank
+  //   DR[type][run][rc] 16 B, DD[type][tpl][dpl] u32 (8 slots), DK[type][run] 16 B,
+  //   DT[j] u16, DF[type][run][rc] u32 (FULL) — at dOff in the blob, offsets relative to it
+  uint32_t dOff, dR, dD, dK, dT, dF, dbytes, dbytes_full;
 };
 
 struct EvalParams {

@@ -1,9 +1,11 @@
 // dense_kernel.cuh — per-op evaluation for candidates whose tp/dp changes at most ops
 // (ACESO_HINT_DENSE; e.g. uniformly random encodings), sm_100a.
 //
-// Same contract, tables and outputs as eval_kernel.cuh (thread = candidate, warp = tile of
+// Same contract, records and outputs as eval_kernel.cuh (thread = candidate, warp = tile of
 // 32 candidates streamed through a per-warp cp.async.bulk ring, profile tables staged in
-// shared memory), but no event handler: every op is accumulated by the same branch-free
+// shared memory, here TYPE-major: the 32 lanes evaluate the same op, so they read one type's
+// records of different runs — neighbouring 32-byte records instead of one bank every
+// T x 32 bytes), but no event handler: every op is accumulated by the same branch-free
 // sequence under its OWN (b, tp) record — so an in-stage tp/dp change costs one predicated
 // reshard lookup instead of a run switch, and lanes stay converged except at stage heads
 // (at most p per candidate).
@@ -30,19 +32,14 @@ __global__ void __launch_bounds__(kThreads, MINB) dense_kernel(const __grid_cons
   __shared__ int64_t s_idx[kWarps];
 
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-  const uint32_t tab_bytes = (MODE & kFull) ? P.tab.bytes_full : P.tab.bytes;
+  const uint32_t stage_bytes = (MODE & kFull) ? P.tab.dbytes_full : P.tab.dbytes;
   const uint32_t sb = smem_addr(sm_raw);
-  Smem sm;
-  sm.R = sb + P.tab.offR;
-  sm.D = sb + P.tab.offD;
-  sm.T = sb + P.tab.offT;
-  sm.F = sb + P.tab.offF;
-  sm.K = sb + tab_bytes;  // cold table staged after the other tables when k_smem
-  sm.Kg = reinterpret_cast<const unsigned char *>(P.blob) + P.tab.offK;
-  sm.k_smem = P.tab.k_smem;
-  sm.TS = (uint32_t)P.T * kTypeStride;
-  const uint32_t stage_bytes = tab_bytes + (P.tab.k_smem ? P.tab.bytesK : 0u);
+  const uint32_t DR = sb + P.tab.dR, DD = sb + P.tab.dD, DK = sb + P.tab.dK, DT = sb + P.tab.dT,
+                 DF = sb + P.tab.dF;
+  const uint32_t runs = (uint32_t)(P.n_b * P.n_tp);
   const uint32_t ring = sb + stage_bytes + (uint32_t)warp * kRingSlots * kSlotBytes;
+  Smem sm;  // init_cand's table bases (unused here)
+  sm.R = sm.D = sm.F = sm.QT = sm.QD = sm.QF = sb;
 
   if (threadIdx.x == 0) {
     mbar_init(smem_addr(&s_tbar), 1);
@@ -56,8 +53,7 @@ __global__ void __launch_bounds__(kThreads, MINB) dense_kernel(const __grid_cons
   if (threadIdx.x == 0) {
     const uint32_t bar = smem_addr(&s_tbar);
     mbar_expect_tx(bar, stage_bytes);
-    bulk_g2s(sb, P.blob, tab_bytes, bar);
-    if (P.tab.k_smem) bulk_g2s(sb + tab_bytes, sm.Kg, P.tab.bytesK, bar);
+    bulk_g2s(sb, reinterpret_cast<const unsigned char *>(P.blob) + P.tab.dOff, stage_bytes, bar);
   }
 
   const uint32_t nch = (uint32_t)P.nch;
@@ -92,7 +88,7 @@ __global__ void __launch_bounds__(kThreads, MINB) dense_kernel(const __grid_cons
   int64_t best_idx = INT64_MAX;
   Cand s;
   uint32_t prev = 0;   // code of op j-1
-  uint32_t pk = 0;     // K-table byte offset of op j-1 (its run and type)
+  uint32_t pk = 0;     // shared address of op j-1's DK record (its run and type)
   int64_t tile = first_tile;
   uint32_t g = 0;
   int slot = 0;
@@ -117,14 +113,14 @@ __global__ void __launch_bounds__(kThreads, MINB) dense_kernel(const __grid_cons
       for (uint32_t q = 0; q < nq; ++q) {
         const uint32_t w = q == 0 ? w4.x : q == 1 ? w4.y : q == 2 ? w4.z : w4.w;
         const uint32_t j0 = ch * 16u + q * 4u;
-        const uint2 tt = lds64(sm.T + 2u * j0);  // the quad's 4 u16 types
+        const uint2 tt = lds64(DT + 2u * j0);  // the quad's 4 u16 types
         const uint32_t nv = min(4u, L - j0);
 #pragma unroll
         for (uint32_t k = 0; k < 4; ++k) {
           if (k < nv) {
             const uint32_t j = j0 + k;
             const uint32_t c = (w >> (8u * k)) & 0xffu;
-            const uint32_t toff = ((k < 2 ? tt.x >> (16u * k) : tt.y >> (16u * (k - 2))) & 0xffffu) << 5;
+            const uint32_t ty = (k < 2 ? tt.x >> (16u * k) : tt.y >> (16u * (k - 2))) & 0xffffu;
             const uint32_t tpl = (c >> 1) & 7u, dpl = c >> 5, rc = (c >> 4) & 1u;
             const uint32_t gg = tpl + dpl;
             if (dpl > s.mbs) s.reasons |= ACESO_R_DPMBS;
@@ -133,28 +129,29 @@ __global__ void __launch_bounds__(kThreads, MINB) dense_kernel(const __grid_cons
             const uint32_t bb = min(dpl <= s.mbs ? s.mbs - dpl : 0u, n_b - 1u);
             const uint32_t tplc = min(tpl, n_tp - 1u);
             const uint32_t run = bb * n_tp + tplc;
-            const uint32_t kofs = run * (sm.TS >> 1) + (toff >> 1);
+            const uint32_t tr = ty * runs + run;  // (type, run) record index
+            const uint32_t kofs = DK + tr * 16u;
             if ((c & 1u) || j == 0) {
               if ((c & 1u) && j > 0) {
-                s.S += ldk(sm, pk + 4u);  // R5: p2p_fwd of the stage's last op (j-1)
+                s.S += lds32(pk + 4u);  // R5: p2p_fwd of the stage's last op (j-1)
                 stage_commit<MODE>(s, P, cand, active, false);
                 s.i += 1;
-                s.S += ldk(sm, kofs + 8u);  // R5: p2p_bwd of the stage's first op
+                s.S += lds32(kofs + 8u);  // R5: p2p_bwd of the stage's first op
               }
               s.gst = gg;
               s.gsum += 1u << gg;  // R9
               s.nheads += c & 1u;
             } else {
               if (gg != s.gst) s.reasons |= ACESO_R_GSTAGE;     // P:L151 in-stage symmetry
-              if ((c ^ prev) & 0xeeu) s.S += ldk(sm, kofs);      // R13: reshard into op j
+              if ((c ^ prev) & 0xeeu) s.S += lds32(kofs);        // R13: reshard into op j
             }
-            const uint4 r = lds128(sm.R + run * sm.TS + toff + rc * 16u);
+            const uint4 r = lds128(DR + tr * 32u + rc * 16u);
             s.S += r.x;
             s.A += r.y;
             s.E = max(s.E, r.z);
             s.W += r.w;
-            s.D += lds32(sm.D + tplc * sm.TS + toff + dpl * 4u);
-            if (MODE & kFull) s.comp += lds32(sm.F + run * (sm.TS >> 2) + (toff >> 2) + rc * 4u);
+            s.D += lds32(DD + (ty * n_tp + tplc) * 32u + dpl * 4u);
+            if (MODE & kFull) s.comp += lds32(DF + tr * 8u + rc * 4u);
             prev = c;
             pk = kofs;
           }
