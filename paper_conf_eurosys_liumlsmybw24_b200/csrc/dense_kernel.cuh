@@ -86,7 +86,7 @@ __global__ void __launch_bounds__(kThreads, MINB) dense_kernel(const __grid_cons
   const uint32_t n_tp = (uint32_t)P.n_tp, n_dp = (uint32_t)P.n_dp, n_b = (uint32_t)P.n_b;
   uint64_t best_ck = ~0ull;
   int64_t best_idx = INT64_MAX;
-  Cand s;
+  Cand s = Cand();
   uint32_t prev = 0;   // code of op j-1
   uint32_t pk = 0;     // shared address of op j-1's DK record (its run and type)
   int64_t tile = first_tile;
@@ -95,11 +95,52 @@ __global__ void __launch_bounds__(kThreads, MINB) dense_kernel(const __grid_cons
   uint32_t phase = 0;
   int64_t cand = 0;
   bool active = false;
+  // table-range validity (R18 DPMBS / TABLE) depends only on the extremes of tp and dp over
+  // the candidate's ops: tracked per op, decided once per candidate
+  uint32_t max_tpl = 0, max_dpl = 0, min_dpl = 7;
+  // one op (j, code c, type ty): the accumulation described at the top of the file
+  auto op = [&](uint32_t j, uint32_t c, uint32_t ty) {
+    const uint32_t tpl = (c >> 1) & 7u, dpl = c >> 5, rc = (c >> 4) & 1u;
+    const uint32_t gg = tpl + dpl;
+    max_tpl = max(max_tpl, tpl);
+    max_dpl = max(max_dpl, dpl);
+    min_dpl = min(min_dpl, dpl);
+    // clamped indices keep every gather inside the tables for invalid encodings
+    const uint32_t bb = min(dpl <= s.mbs ? s.mbs - dpl : 0u, n_b - 1u);
+    const uint32_t tplc = min(tpl, n_tp - 1u);
+    const uint32_t tr = ty * runs + bb * n_tp + tplc;  // (type, run) record index
+    const uint32_t kofs = DK + tr * 16u;
+    if ((c & 1u) || j == 0) {
+      if ((c & 1u) && j > 0) {
+        s.S += lds32(pk + 4u);  // R5: p2p_fwd of the stage's last op (j-1)
+        stage_commit<MODE>(s, P, cand, active, false);
+        s.i += 1;
+        s.S += lds32(kofs + 8u);  // R5: p2p_bwd of the stage's first op
+      }
+      s.gst = gg;
+      s.gsum += 1u << gg;  // R9
+      s.nheads += c & 1u;
+    } else {
+      if (gg != s.gst) s.reasons |= ACESO_R_GSTAGE;  // P:L151 in-stage symmetry
+      if ((c ^ prev) & 0xeeu) s.S += lds32(kofs);     // R13: reshard into op j
+    }
+    const uint4 r = lds128(DR + tr * 32u + rc * 16u);
+    s.S += r.x;
+    s.A += r.y;
+    s.E = max(s.E, r.z);
+    s.W += r.w;
+    s.D += lds32(DD + (ty * n_tp + tplc) * 32u + dpl * 4u);
+    if (MODE & kFull) s.comp += lds32(DF + tr * 8u + rc * 4u);
+    prev = c;
+    pk = kofs;
+  };
   for (int64_t u = 0; u < units; ++u) {
     if (g == 0) {
       cand = tile * 32 + lane;
       active = cand < P.n;
       init_cand(s, sm, P, active ? __ldg(P.hdr + cand) : 0ull, false);
+      max_tpl = max_dpl = 0;
+      min_dpl = 7;
     }
     mbar_wait(smem_addr(&s_ring_bar[warp][slot]), phase);
     const uint32_t a = kSlotChunks * g, b = min(a + kSlotChunks, nch);
@@ -114,47 +155,15 @@ __global__ void __launch_bounds__(kThreads, MINB) dense_kernel(const __grid_cons
         const uint32_t w = q == 0 ? w4.x : q == 1 ? w4.y : q == 2 ? w4.z : w4.w;
         const uint32_t j0 = ch * 16u + q * 4u;
         const uint2 tt = lds64(DT + 2u * j0);  // the quad's 4 u16 types
-        const uint32_t nv = min(4u, L - j0);
-#pragma unroll
-        for (uint32_t k = 0; k < 4; ++k) {
-          if (k < nv) {
-            const uint32_t j = j0 + k;
-            const uint32_t c = (w >> (8u * k)) & 0xffu;
-            const uint32_t ty = (k < 2 ? tt.x >> (16u * k) : tt.y >> (16u * (k - 2))) & 0xffffu;
-            const uint32_t tpl = (c >> 1) & 7u, dpl = c >> 5, rc = (c >> 4) & 1u;
-            const uint32_t gg = tpl + dpl;
-            if (dpl > s.mbs) s.reasons |= ACESO_R_DPMBS;
-            if (tpl >= n_tp || dpl >= n_dp || (dpl <= s.mbs && s.mbs - dpl >= n_b)) s.reasons |= ACESO_R_TABLE;
-            // clamped indices keep every gather inside the tables for invalid encodings
-            const uint32_t bb = min(dpl <= s.mbs ? s.mbs - dpl : 0u, n_b - 1u);
-            const uint32_t tplc = min(tpl, n_tp - 1u);
-            const uint32_t run = bb * n_tp + tplc;
-            const uint32_t tr = ty * runs + run;  // (type, run) record index
-            const uint32_t kofs = DK + tr * 16u;
-            if ((c & 1u) || j == 0) {
-              if ((c & 1u) && j > 0) {
-                s.S += lds32(pk + 4u);  // R5: p2p_fwd of the stage's last op (j-1)
-                stage_commit<MODE>(s, P, cand, active, false);
-                s.i += 1;
-                s.S += lds32(kofs + 8u);  // R5: p2p_bwd of the stage's first op
-              }
-              s.gst = gg;
-              s.gsum += 1u << gg;  // R9
-              s.nheads += c & 1u;
-            } else {
-              if (gg != s.gst) s.reasons |= ACESO_R_GSTAGE;     // P:L151 in-stage symmetry
-              if ((c ^ prev) & 0xeeu) s.S += lds32(kofs);        // R13: reshard into op j
-            }
-            const uint4 r = lds128(DR + tr * 32u + rc * 16u);
-            s.S += r.x;
-            s.A += r.y;
-            s.E = max(s.E, r.z);
-            s.W += r.w;
-            s.D += lds32(DD + (ty * n_tp + tplc) * 32u + dpl * 4u);
-            if (MODE & kFull) s.comp += lds32(DF + tr * 8u + rc * 4u);
-            prev = c;
-            pk = kofs;
-          }
+        if (j0 + 4u <= L) {  // full quad
+          op(j0, w & 0xffu, tt.x & 0xffffu);
+          op(j0 + 1u, (w >> 8) & 0xffu, tt.x >> 16);
+          op(j0 + 2u, (w >> 16) & 0xffu, tt.y & 0xffffu);
+          op(j0 + 3u, w >> 24, tt.y >> 16);
+        } else {
+#pragma unroll 1
+          for (uint32_t k = 0; j0 + k < L; ++k)
+            op(j0 + k, (w >> (8u * k)) & 0xffu, (k < 2 ? tt.x >> (16u * k) : tt.y >> (16u * (k - 2))) & 0xffffu);
         }
       }
     }
@@ -166,6 +175,9 @@ __global__ void __launch_bounds__(kThreads, MINB) dense_kernel(const __grid_cons
     slot = (slot + 1) % kRingSlots;
     if (slot == 0) phase ^= 1u;
     if (++g == ngroups) {
+      if (max_dpl > s.mbs) s.reasons |= ACESO_R_DPMBS;
+      if (max_tpl >= n_tp || max_dpl >= n_dp || (min_dpl <= s.mbs && s.mbs - min_dpl >= n_b))
+        s.reasons |= ACESO_R_TABLE;
       stage_commit<MODE>(s, P, cand, active, false);  // last stage: no p2p_fwd
       finish_cand<MODE>(s, P, cand, active, best_ck, best_idx);
       g = 0;
