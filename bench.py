@@ -392,8 +392,10 @@ def main():
     global HINT
     HINT = args.dist == "dense" and not args.no_hint
     env_k = os.environ.get("ACESO_KERNEL")
-    schedule = ("per-op kernel (ACESO_HINT_DENSE)" if HINT else
-                "per-op kernel" if env_k == "quad" or (env_k != "events" and L <= 64) else "event kernel")
+    dense_k = "per-op kernel" if os.environ.get("ACESO_DENSE_KERNEL") == "quad" else "dense kernel"
+    schedule = (f"{dense_k} (ACESO_HINT_DENSE)" if HINT else
+                "per-op kernel" if env_k == "quad" else
+                "dense kernel" if env_k == "dense" or (env_k != "events" and L <= 64) else "event kernel")
 
     # distinct device-resident batches, rotating, together larger than L2
     per_batch = A.tiled_bytes(n, L) + 8 * n

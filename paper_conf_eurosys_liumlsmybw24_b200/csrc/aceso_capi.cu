@@ -543,10 +543,14 @@ int aceso_load_profile(const aceso_profile_desc *d, int cuda_device, aceso_ctx *
   ctx->d_blob = nullptr;
   ctx->d_ev = nullptr;
   ctx->quad_ok = quad_ok ? 1 : 0;
-  ctx->kernel = (L > 64 || !quad_ok) ? 1 : 0;  // short models: per-tile event overheads outweigh the per-op work
+  // short models: per-tile event overheads outweigh the per-op work; the dense kernel's
+  // branch-free per-op accumulation beats the per-op kernel there (toy-A 25.1 vs 21.4, toy-B
+  // 20.1 vs 16.4 G configs/s, search-shaped)
+  ctx->kernel = L > 64 ? 1 : dense_ok ? 2 : quad_ok ? 0 : 1;
   if (const char *env = getenv("ACESO_KERNEL")) {
     if (!strcmp(env, "quad") && quad_ok) ctx->kernel = 0;
     else if (!strcmp(env, "events")) ctx->kernel = 1;
+    else if (!strcmp(env, "dense")) ctx->kernel = 2;  // validated against dense_ok below
   }
   ctx->qo_off = (uint32_t)ev_qo;
   ctx->qo_bytes = qo_bytes;
@@ -586,6 +590,7 @@ int aceso_load_profile(const aceso_profile_desc *d, int cuda_device, aceso_ctx *
       ctx->qr = reinterpret_cast<const uint4 *>(eb + ev_qr);
     }
     ctx->dense_kernel = dense_ok ? 2 : 0;  // its tables must fit in shared memory
+    if (ctx->kernel == 2 && !dense_ok) ctx->kernel = (L > 64 || !quad_ok) ? 1 : 0;  // ACESO_KERNEL=dense
     if (const char *env = getenv("ACESO_DENSE_KERNEL"))
       if (!strcmp(env, "quad")) ctx->dense_kernel = 0;
     for (int kern = 0; kern < 3 && rc == ACESO_OK; ++kern)
