@@ -293,7 +293,9 @@ class Primitives:
     def describe_all(self, codes, mbs, info, comp, comm, stage_time):
         """The candidates of apply_all, in the same order, as base + patches
         (candidates.CAND_DTYPE rows with base = 0) plus the two rank rows of this base
-        used by the recompute patches. Nothing is materialised on the host."""
+        used by the recompute patches. Nothing is materialised on the host; the families
+        with one candidate per op (op moves, recompute ranks, fine-tune starts) are built as
+        arrays (numpy), the few others one by one."""
         from . import candidates as C
         prof = self.prof
         L = len(codes)
@@ -310,38 +312,65 @@ class Primitives:
             want = {"comp"} if comp[bn] / cs >= comm[bn] / ms else {"comm"}
         if not self.heuristic2:
             want = {"mem", "comp", "comm"}
-        out = []
+        groups = []  # (mbs [n], patches [n][MAX_PATCH] PATCH_DTYPE, n_patch [n]) in emission order
 
-        def emit(m, patches):
-            out.append((int(m), patches))
+        def block(mbs_v, pts):
+            """n candidates sharing a patch structure: pts = list of per-slot patch columns,
+            each a tuple of arrays/scalars (a, b, kind, v0, v1, v2) broadcast to n."""
+            n = len(mbs_v)
+            pa = np.zeros((n, C.MAX_PATCH), C.PATCH_DTYPE)
+            for j, (pa_, pb_, kind, v0, v1, v2) in enumerate(pts):
+                pa["a"][:, j], pa["b"][:, j], pa["kind"][:, j] = pa_, pb_, kind
+                pa["v0"][:, j], pa["v1"][:, j], pa["v2"][:, j] = v0, v1, v2
+            groups.append((np.asarray(mbs_v, np.uint8), pa, np.full(n, len(pts), np.uint8)))
+
+        def one(m, patches):
+            block([m], [tuple(np.array([x]) for x in pt) for pt in patches])
+
         a, e = int(heads[bn]), int(ends[bn])
         size = e - a
         kmax = size - 1 if self.max_k is None else min(size - 1, self.max_k)
         idle = int(np.argmin(stage_time[:p])) if p > 1 else bn
-        for k in range(1, kmax + 1):
-            if bn > 0 and k < size:  # _move_front(codes, bn, k)
-                pf = [C.mask(a, a + k, 0x10, int(codes[a - 1]) & 0xEE), C.mask(a + k, a + k + 1, 0xFE, 1)]
-                emit(mbs, pf)
-                if idle < bn - 1:  # relay: stage bn-1 = [heads[bn-1], a + k) after the move
+        if kmax >= 1:
+            # op moves at both edges of the bottleneck (P:L253), relayed toward the idlest
+            # stage (P:L274); per k in the order front, front relay, back, back relay
+            k = np.arange(1, kmax + 1)
+            M, F = C.PATCH_MASK, 0
+            fam = []
+            if bn > 0:
+                pf = [(a, a + k, M, 0x10, int(codes[a - 1]) & 0xEE, F), (a + k, a + k + 1, M, 0xFE, 1, F)]
+                fam.append(pf)
+                if idle < bn - 1:
                     a2 = int(heads[bn - 1])
-                    emit(mbs, pf + [C.mask(a2, a2 + k, 0x10, int(codes[a2 - 1]) & 0xEE),
-                                    C.mask(a2 + k, a2 + k + 1, 0xFE, 1)])
-            if bn < p - 1 and k < size:  # _move_back(codes, bn, k)
-                pb = [C.mask(e, e + 1, 0xFE, 0), C.mask(e - k, e, 0x10, int(codes[e]) & 0xEE),
-                      C.mask(e - k, e - k + 1, 0xFF, 1)]
-                emit(mbs, pb)
-                if idle > bn + 1:  # relay: stage bn+1 = [heads[bn+1] - k, ends[bn+1])
+                    fam.append(pf + [(a2, a2 + k, M, 0x10, int(codes[a2 - 1]) & 0xEE, F),
+                                     (a2 + k, a2 + k + 1, M, 0xFE, 1, F)])
+            if bn < p - 1:
+                pb = [(e, e + 1, M, 0xFE, 0, F), (e - k, e, M, 0x10, int(codes[e]) & 0xEE, F),
+                      (e - k, e - k + 1, M, 0xFF, 1, F)]
+                fam.append(pb)
+                if idle > bn + 1:
                     e2 = int(ends[bn + 1])
-                    emit(mbs, pb + [C.mask(e2, e2 + 1, 0xFE, 0), C.mask(e2 - k, e2, 0x10, int(codes[e2]) & 0xEE),
-                                    C.mask(e2 - k, e2 - k + 1, 0xFF, 1)])
+                    fam.append(pb + [(e2, e2 + 1, M, 0xFE, 0, F), (e2 - k, e2, M, 0x10, int(codes[e2]) & 0xEE, F),
+                                     (e2 - k, e2 - k + 1, M, 0xFF, 1, F)])
+            if fam:
+                nf, nk = len(fam), len(k)
+                pa = np.zeros((nk, nf, C.MAX_PATCH), C.PATCH_DTYPE)
+                npch = np.zeros((nk, nf), np.uint8)
+                for fi, pts in enumerate(fam):
+                    npch[:, fi] = len(pts)
+                    for j, (pa_, pb_, kind, v0, v1, v2) in enumerate(pts):
+                        pa["a"][:, fi, j], pa["b"][:, fi, j], pa["kind"][:, fi, j] = pa_, pb_, kind
+                        pa["v0"][:, fi, j], pa["v1"][:, fi, j], pa["v2"][:, fi, j] = v0, v1, v2
+                groups.append((np.full(nk * nf, mbs, np.uint8), pa.reshape(nk * nf, C.MAX_PATCH),
+                               npch.reshape(-1)))
         log2bg = int(math.log2(prof.global_batch & -prof.global_batch))
         dpl_all = ((codes >> 5) & 7).astype(np.int16)
         tpl_all = ((codes >> 1) & 7).astype(np.int16)
         dmax = int(dpl_all.max())
         if ("mem" in want or "comm" in want) and mbs - 1 >= dmax:
-            emit(mbs - 1, [])
+            one(mbs - 1, [])
         if ("comp" in want) and mbs + 1 <= log2bg:
-            emit(mbs + 1, [])
+            one(mbs + 1, [])
 
         def stage_ok(sg, dt, dd):
             x, y = int(heads[sg]), int(ends[sg])
@@ -356,7 +385,7 @@ class Primitives:
             return m
         for dt in (1, -1):
             if stage_ok(bn, dt, -dt):
-                emit(max(mbs, dmax_after({bn: -dt})), [C.add(a, e, dt, -dt)])
+                one(max(mbs, dmax_after({bn: -dt})), [C.add(a, e, dt, -dt)])
         kb = ((int(codes[heads[bn]]) >> 1) & 7) + ((int(codes[heads[bn]]) >> 5) & 7)
         for q in range(p):
             if q == bn:
@@ -370,21 +399,24 @@ class Primitives:
             for dtb, ddb, dtq, ddq in trades:
                 if stage_ok(bn, dtb, ddb) and stage_ok(q, dtq, ddq):
                     qa, qe = int(heads[q]), int(ends[q])
-                    emit(max(mbs, dmax_after({bn: ddb, q: ddq})), [C.add(a, e, dtb, ddb), C.add(qa, qe, dtq, ddq)])
+                    one(max(mbs, dmax_after({bn: ddb, q: ddq})), [C.add(a, e, dtb, ddb), C.add(qa, qe, dtq, ddq)])
         stride = C.stride_of(L)
         ranks = np.full((2, stride), 0xFFFF, np.uint16)
         order = _rc_order(prof, codes, bn, mbs, (heads, ends))
         rc = (codes[order] >> 4) & 1
+        R = C.PATCH_RANK_RC
         if "mem" in want:
             todo = order[rc == 0]
             ranks[0, todo] = np.arange(len(todo), dtype=np.uint16)
-            for k in range(1, len(todo) + 1):
-                emit(mbs, [C.rank_rc(a, e, k, 0, False)])
+            if len(todo):
+                k = np.arange(1, len(todo) + 1)
+                block(np.full(len(k), mbs), [(a, e, R, k & 0xFF, (k >> 8) & 0xFF, 0)])
         if "comp" in want:
             have = order[rc == 1][::-1]
             ranks[1, have] = np.arange(len(have), dtype=np.uint16)
-            for k in range(1, len(have) + 1):
-                emit(mbs, [C.rank_rc(a, e, k, 1, True)])
+            if len(have):
+                k = np.arange(1, len(have) + 1)
+                block(np.full(len(k), mbs), [(a, e, R, k & 0xFF, (k >> 8) & 0xFF, 1 | 2)])
         if e - a > 1:
             tp, dp = tpl_all[a:e], dpl_all[a:e]
             tmin, tmax = np.minimum.accumulate(tp[::-1])[::-1], np.maximum.accumulate(tp[::-1])[::-1]
@@ -392,21 +424,30 @@ class Primitives:
             dmax_pre = int(dpl_all[:a].max()) if a > 0 else 0
             dmax_post = int(dpl_all[e:].max()) if e < L else 0
             dmax_out = max(dmax_pre, dmax_post)
-            for j in range(a + 1, e):
-                r = j - a
-                for dt in (1, -1):
-                    if tmin[r] + dt < 0 or tmax[r] + dt > 7 or dmin[r] - dt < 0 or dmax_s[r] - dt > 7:
-                        continue
-                    dnew = max(dmax_out, int(dpl_all[a:j].max()), int(dmax_s[r] - dt))
-                    emit(max(mbs, dnew), [C.add(j, e, dt, -dt)])
-        cands = np.zeros(len(out), C.CAND_DTYPE)
-        cands["mbs"] = [m for m, _ in out]
+            pmax = np.maximum.accumulate(dp)  # pmax[r - 1] = max dp over [a, a + r)
+            r = np.arange(1, e - a)
+            js, dts, ms_ = [], [], []
+            for dt in (1, -1):  # interleaved per j below: (j, +1), (j, -1)
+                ok = ~((tmin[r] + dt < 0) | (tmax[r] + dt > 7) | (dmin[r] - dt < 0) | (dmax_s[r] - dt > 7))
+                dnew = np.maximum(np.maximum(dmax_out, pmax[r - 1]), dmax_s[r] - dt)
+                js.append(np.where(ok, r, -1))
+                dts.append(np.full(len(r), dt))
+                ms_.append(np.maximum(mbs, dnew))
+            jj = np.stack(js, 1).reshape(-1)
+            dd = np.stack(dts, 1).reshape(-1)
+            mm = np.stack(ms_, 1).reshape(-1)
+            keep = jj >= 0
+            jj, dd, mm = jj[keep] + a, dd[keep], mm[keep]
+            if len(jj):
+                block(mm, [(jj, e, C.PATCH_ADD, dd & 0xFF, (-dd) & 0xFF, 0)])
+        if not groups:
+            return np.zeros(0, C.CAND_DTYPE), ranks
+        n = sum(len(g[0]) for g in groups)
+        cands = np.zeros(n, C.CAND_DTYPE)
+        cands["mbs"] = np.concatenate([g[0] for g in groups])
         cands["p"] = p
-        cands["n_patch"] = [len(pts) for _, pts in out]
-        pa = cands["patch"]
-        for i, (_, pts) in enumerate(out):
-            for j, pt in enumerate(pts):
-                pa[i, j] = pt
+        cands["n_patch"] = np.concatenate([g[2] for g in groups])
+        cands["patch"] = np.concatenate([g[1] for g in groups])
         return cands, ranks
 
 
