@@ -527,6 +527,39 @@ class _Node:
         return self._codes
 
 
+def _key(perf):
+    """(class, cost) as one integer with the same order (cost < 2^62)."""
+    return (int(perf[0]) << 62) | int(perf[1])
+
+
+class _Chunk:
+    """The configurations one hop added to a search's unexplored set, kept as arrays in
+    best-performance-first order (stable: generation order among equals). Nodes are only
+    materialised when the search takes them; they leave the set from the front (the
+    improving node, GetBestOf)."""
+
+    def __init__(self, keys, idx, r, bases, ranks, cands, L):
+        self.keys = keys[idx]
+        self.hash = r["hash"][idx]
+        self.info = r["info"][idx]
+        self.iter = r["iter"][idx]
+        self.mem = r["max_mem"][idx]
+        self.comp = r["stage_comp"][idx]
+        self.comm = r["stage_comm"][idx]
+        self.time = r["stage_T"][idx]
+        self.cands = cands[idx]
+        self.bases, self.ranks, self.L = bases, ranks, L
+        self.head = 0
+
+    def node(self, t):
+        info = int(self.info[t])
+        c = self.cands[t]
+        b = int(c["base"])
+        return _Node(int(self.hash[t]), int(c["mbs"]), perf_of(info, self.iter[t], self.mem[t]), info,
+                     self.comp[t], self.comm[t], self.time[t], int(self.iter[t]), int(self.mem[t]),
+                     (self.bases[b], self.ranks[b], c, self.L))
+
+
 class _Search:
     """One AcesoSearch (Alg. 1) for one stage count, stepped one hop at a time."""
 
@@ -536,9 +569,22 @@ class _Search:
         self.init_perf = start.perf
         self.frontier = [start]
         self.hop = 0
-        self.unexplored = {}
+        self.chunks = []  # unexplored configurations, in insertion order (_Chunk)
         self.done = False
         self.improvements = 0
+
+    def get_best_of_unexplored(self):
+        """GetBestOf(unexplored) (Alg. 1): the best remaining configuration, the
+        earliest inserted among equals; removed from the set. None if empty."""
+        best = None
+        for ch in self.chunks:
+            if ch.head < len(ch.keys) and (best is None or ch.keys[ch.head] < best.keys[best.head]):
+                best = ch
+        if best is None:
+            return None
+        nd = best.node(best.head)
+        best.head += 1
+        return nd
 
 
 def search(prof, evaluator, p_values=None, budget_s=10.0, max_hops=7, beam=4, heuristic2=True,
@@ -560,7 +606,7 @@ def search(prof, evaluator, p_values=None, budget_s=10.0, max_hops=7, beam=4, he
     prims = Primitives(prof, heuristic2=heuristic2, max_k=max_k)
     if p_values is None:
         p_values = [p for p in (1, 2, 3, 4, 6, 8, 12, 16, 24, 32, 48, 64) if p <= min(prof.n_devices, prof.n_ops)]
-    visited = set()
+    visited = np.zeros(0, np.uint64)  # sorted hashes of every configuration seen
     init = []
     for p in p_values:
         r = initial_config(prof, p)
@@ -587,7 +633,7 @@ def search(prof, evaluator, p_values=None, budget_s=10.0, max_hops=7, beam=4, he
     for i in range(len(init)):
         n0 = node(i, res, bases[i], ranks[i], cands[i])
         n0._codes = init[i][0]
-        visited.add(n0.key)
+        visited = np.union1d(visited, np.array([n0.key], np.uint64))
         searches.append(_Search(n0))
     best = min((s.best for s in searches), key=lambda n: n.perf)
     t_best = time.perf_counter() - t0
@@ -615,7 +661,7 @@ def search(prof, evaluator, p_values=None, budget_s=10.0, max_hops=7, beam=4, he
                 base_rows.append(row)
                 rank_rows.append(rk)
                 chunks.append(cd)
-                owners.extend([si] * len(cd))
+                owners.append(np.full(len(cd), si, np.int32))
                 total += len(cd)
         if not chunks:
             for s in searches:
@@ -627,44 +673,50 @@ def search(prof, evaluator, p_values=None, budget_s=10.0, max_hops=7, beam=4, he
         r = evaluator.evaluate_cands(bases, ranks, cands)
         batches += 1
         evaluated += len(cands)
-        per = {}
-        for i, si in enumerate(owners):
-            h = int(r["hash"][i])
-            if h in visited:  # an explored configuration (or an earlier one of this batch)
-                continue
-            visited.add(h)
-            b = int(cands[i]["base"])
-            per.setdefault(si, []).append(node(i, r, bases[b], ranks[b], cands[i]))
+        owner = np.concatenate(owners)
+        # configurations seen before (or earlier in this batch) are dropped
+        hs = np.asarray(r["hash"], np.uint64)
+        _, first = np.unique(hs, return_index=True)
+        keep = np.zeros(len(hs), bool)
+        keep[first] = True
+        keep &= ~np.isin(hs, visited)
+        visited = np.union1d(visited, hs[keep])
+        info = np.asarray(r["info"], np.uint64)
+        cls = np.where(info & INFO_INVALID, 2, np.where(info & INFO_OOM, 1, 0)).astype(np.uint64)
+        cost = np.where(cls == 2, 0, np.where(cls == 1, r["max_mem"], r["iter"])).astype(np.uint64)
+        keys = (cls << np.uint64(62)) | cost  # perf_of as one ordered integer
         improved_any = False
         for si, s in enumerate(searches):
             if s.done:
                 continue
-            new = per.get(si, [])
-            new.sort(key=lambda n: n.perf)  # Heuristic-2: best estimated performance first
-            for nd in new:
-                s.unexplored[nd.key] = nd
-            if new and new[0].perf < s.init_perf:
+            idx = np.nonzero(keep & (owner == si))[0]
+            # Heuristic-2: best estimated performance first (stable: generation order)
+            idx = idx[np.argsort(keys[idx], kind="stable")]
+            ch = _Chunk(keys, idx, r, bases, ranks, cands, L) if len(idx) else None
+            if ch is not None:
+                s.chunks.append(ch)
+            if ch is not None and int(ch.keys[0]) < _key(s.init_perf):
                 # Alg. 2 returns the improved configuration; Alg. 1 restarts from it
-                s.cur = new[0]
-                if new[0].perf < s.best.perf:
-                    s.best = new[0]
-                s.init_perf = new[0].perf
-                s.frontier = [new[0]]
+                nd0 = ch.node(0)
+                ch.head = 1  # leaves the unexplored set
+                s.cur = nd0
+                if nd0.perf < s.best.perf:
+                    s.best = nd0
+                s.init_perf = nd0.perf
+                s.frontier = [nd0]
                 s.hop = 0
                 s.improvements += 1
-                s.unexplored.pop(new[0].key, None)
                 improved_any = True
                 continue
             s.hop += 1
-            if s.hop < max_hops and new:
-                s.frontier = new[:beam]
+            if s.hop < max_hops and ch is not None:
+                s.frontier = [ch.node(t) for t in range(min(beam, len(ch.keys)))]
                 continue
             # MultiHop failed within MaxHops: Alg. 1 continues from GetBestOf(unexplored)
-            if not s.unexplored:
+            nd = s.get_best_of_unexplored()
+            if nd is None:
                 s.done = True
                 continue
-            k_best = min(s.unexplored, key=lambda k: s.unexplored[k].perf)
-            nd = s.unexplored.pop(k_best)
             s.cur = nd
             s.init_perf = nd.perf
             s.frontier = [nd]
