@@ -493,8 +493,10 @@ class GPUEvaluator:
         hs = hash_candidates(tiled, hdr, self.ctx.n_ops, n=n)
         res = dict(iter=as_u64(out.iter_ns), max_mem=as_u64(out.max_mem), info=as_u32(out.info),
                    hash=hs.cpu().numpy().view(np.uint64))
+        # per-stage rows stay on the device ([n][p_max] views): the search reads the few rows
+        # of the configurations it takes (Heuristic-2 needs them), not the whole batch
         for k in ["stage_T", "stage_mem", "stage_comp", "stage_comm"]:
-            res[k] = as_u64(getattr(out, k)).reshape(out.p_max, n).T
+            res[k] = getattr(out, k).view(torch.int64).reshape(out.p_max, n).T
         return res
 
 
@@ -527,6 +529,32 @@ class _Node:
         return self._codes
 
 
+def _first_new(hs, visited):
+    """Configuration dedup: mask of the candidates whose hash is neither in the
+    sorted array `visited` nor earlier in `hs` (first occurrence in generation order), and the
+    updated sorted array. Sort-based, O(n log n) per batch."""
+    keep = np.zeros(len(hs), bool)
+    if len(hs) == 0:
+        return keep, visited
+    order = np.argsort(hs, kind="stable")
+    sh = hs[order]
+    first = np.empty(len(sh), bool)
+    first[0] = True
+    first[1:] = sh[1:] != sh[:-1]
+    idx, h = order[first], sh[first]
+    if len(visited):
+        pos = np.searchsorted(visited, h)
+        seen = visited[np.minimum(pos, len(visited) - 1)] == h
+        idx, h = idx[~seen], h[~seen]
+    keep[idx] = True
+    return keep, np.insert(visited, np.searchsorted(visited, h), h)
+
+
+def _row(x, i):
+    """Row i of a per-stage array, as numpy (device tensors are copied on demand)."""
+    return x[i].cpu().numpy().view(np.uint64) if isinstance(x, torch.Tensor) else x[i]
+
+
 def _key(perf):
     """(class, cost) as one integer with the same order (cost < 2^62)."""
     return (int(perf[0]) << 62) | int(perf[1])
@@ -540,13 +568,12 @@ class _Chunk:
 
     def __init__(self, keys, idx, r, bases, ranks, cands, L):
         self.keys = keys[idx]
+        self.idx = idx
         self.hash = r["hash"][idx]
         self.info = r["info"][idx]
         self.iter = r["iter"][idx]
         self.mem = r["max_mem"][idx]
-        self.comp = r["stage_comp"][idx]
-        self.comm = r["stage_comm"][idx]
-        self.time = r["stage_T"][idx]
+        self.stage = (r["stage_comp"], r["stage_comm"], r["stage_T"])  # [n][p_max], host or device
         self.cands = cands[idx]
         self.bases, self.ranks, self.L = bases, ranks, L
         self.head = 0
@@ -555,8 +582,10 @@ class _Chunk:
         info = int(self.info[t])
         c = self.cands[t]
         b = int(c["base"])
+        i = int(self.idx[t])
+        rows = [_row(x, i) for x in self.stage]
         return _Node(int(self.hash[t]), int(c["mbs"]), perf_of(info, self.iter[t], self.mem[t]), info,
-                     self.comp[t], self.comm[t], self.time[t], int(self.iter[t]), int(self.mem[t]),
+                     rows[0], rows[1], rows[2], int(self.iter[t]), int(self.mem[t]),
                      (self.bases[b], self.ranks[b], c, self.L))
 
 
@@ -625,7 +654,7 @@ def search(prof, evaluator, p_values=None, budget_s=10.0, max_hops=7, beam=4, he
     def node(i, r, base_row, rank_rows, cand):
         info = int(r["info"][i])
         nd = _Node(int(r["hash"][i]), int(cand["mbs"]), perf_of(info, r["iter"][i], r["max_mem"][i]), info,
-                   r["stage_comp"][i], r["stage_comm"][i], r["stage_T"][i], int(r["iter"][i]),
+                   _row(r["stage_comp"], i), _row(r["stage_comm"], i), _row(r["stage_T"], i), int(r["iter"][i]),
                    int(r["max_mem"][i]), (base_row, rank_rows, cand, L))
         return nd
 
@@ -633,7 +662,7 @@ def search(prof, evaluator, p_values=None, budget_s=10.0, max_hops=7, beam=4, he
     for i in range(len(init)):
         n0 = node(i, res, bases[i], ranks[i], cands[i])
         n0._codes = init[i][0]
-        visited = np.union1d(visited, np.array([n0.key], np.uint64))
+        _, visited = _first_new(np.array([n0.key], np.uint64), visited)
         searches.append(_Search(n0))
     best = min((s.best for s in searches), key=lambda n: n.perf)
     t_best = time.perf_counter() - t0
@@ -675,12 +704,7 @@ def search(prof, evaluator, p_values=None, budget_s=10.0, max_hops=7, beam=4, he
         evaluated += len(cands)
         owner = np.concatenate(owners)
         # configurations seen before (or earlier in this batch) are dropped
-        hs = np.asarray(r["hash"], np.uint64)
-        _, first = np.unique(hs, return_index=True)
-        keep = np.zeros(len(hs), bool)
-        keep[first] = True
-        keep &= ~np.isin(hs, visited)
-        visited = np.union1d(visited, hs[keep])
+        keep, visited = _first_new(np.asarray(r["hash"], np.uint64), visited)
         info = np.asarray(r["info"], np.uint64)
         cls = np.where(info & INFO_INVALID, 2, np.where(info & INFO_OOM, 1, 0)).astype(np.uint64)
         cost = np.where(cls == 2, 0, np.where(cls == 1, r["max_mem"], r["iter"])).astype(np.uint64)

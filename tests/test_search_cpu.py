@@ -151,3 +151,21 @@ def test_descriptors_expand_to_the_reference_candidates(name):
                 assert int(ghdr[k] & np.uint64(0xFF)) == mr and int(ghdr[k] >> np.uint64(8)) == p
             checked += len(ref)
     assert checked > 500
+
+
+def test_first_new_dedup_is_first_occurrence_against_visited():
+    """_first_new (configuration dedup) equals the plain set loop: first occurrence
+    in generation order of every hash not seen before; the visited array stays sorted."""
+    rng = np.random.default_rng(3)
+    visited_set = set()
+    visited = np.zeros(0, np.uint64)
+    for _ in range(6):
+        hs = rng.integers(0, 50, size=200).astype(np.uint64)
+        want = np.zeros(len(hs), bool)
+        for i, h in enumerate(hs.tolist()):
+            if h not in visited_set:
+                visited_set.add(h)
+                want[i] = True
+        keep, visited = S._first_new(hs, visited)
+        assert np.array_equal(keep, want)
+        assert np.array_equal(visited, np.array(sorted(visited_set), np.uint64))
