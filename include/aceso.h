@@ -221,11 +221,17 @@ size_t aceso_select_buf_bytes(const aceso_ctx *ctx, int64_t n);
  *             are bit-identical):
  *             the event kernel (default for n_ops > 64) walks each candidate's
  *             stage heads and tp/dp changes and takes run sums from position-prefix
- *             tables; the per-op kernel (default for n_ops <= 64, or with the hint)
- *             accumulates every op; it stages its tables in shared memory, so for
+ *             tables; the dense kernel (default for n_ops <= 64, and with
+ *             ACESO_HINT_DENSE) accumulates every op branch-free under its own record;
+ *             the per-op kernel accumulates every op with quad-signature sums. The
+ *             dense and per-op kernels stage their tables in shared memory, so for
  *             profiles whose tables exceed ~200 KB only the event kernel is used (the
- *             hint is then ignored). The environment variable ACESO_KERNEL=quad|events,
- *             read by aceso_load_profile, overrides the default.
+ *             hint is then ignored). Environment variables read by aceso_load_profile
+ *             (measurement and test knobs; results never change):
+ *             ACESO_KERNEL=quad|events|dense (default schedule), ACESO_DENSE_KERNEL=quad
+ *             (schedule of the dense hint), ACESO_SPLIT=2 (per-op kernel: warp pair per
+ *             tile), ACESO_MINB=2|3 (register target: resident CTAs per SM),
+ *             ACESO_TILES_PER_WARP=k (event kernel: tiles per warp per launch).
  *   out     : host struct of device pointers (may be null if no OUT_* flag)
  *   d_sel   : select buffer (device), required with ACESO_FUSED_SELECT
  *   stream  : cudaStream_t
