@@ -442,6 +442,11 @@ def main():
     outs = [out] + [ctx.alloc_outputs(n) for _ in range(nstr - 1)]
     side = [torch.cuda.Stream() for _ in range(nstr)]
     comm = torch.cuda.Stream()  # all-reduces in step order on one stream (same on every rank)
+    for si, st in enumerate(side):  # untimed warm-up of every side stream (per-stream state)
+        ctx.eval(dev_batches[si % nbuf][0], dev_batches[si % nbuf][1], n=n, global_offset=rank * n,
+                 n_total=n_total, summary=True, select=True, out=outs[si], sel=sels[si % nbuf], stream=st,
+                 dense_hint=HINT, overlap_hint=OVERLAP)
+    torch.cuda.synchronize()
     keyvec = torch.empty(args.steps, dtype=torch.int64, device=dev)  # per-step global keys
     kpa = max(1, args.keys_per_allreduce)
     def issue_steps():
