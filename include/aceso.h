@@ -186,10 +186,12 @@ typedef struct {
 #define ACESO_HINT_OVERLAP 16u /* schedule hint: the caller keeps several
                                  independent batches in flight on different
                                  streams; for models of at most 384 ops the event
-                                 kernel then launches half the CTAs and each warp
-                                 walks two tiles (per-launch prologue/epilogue
-                                 amortised; higher throughput, longer single-
-                                 launch latency); longer models are unaffected.
+                                 kernel then launches a half or a third of the
+                                 CTAs and each warp walks two tiles (at most 384
+                                 ops) or three (at most 320) (per-launch prologue/
+                                 epilogue amortised; higher throughput, longer
+                                 single-launch latency); longer models are
+                                 unaffected.
                                  Results are identical.                         */
 
 /* ------------------------------------------------------------------------- */

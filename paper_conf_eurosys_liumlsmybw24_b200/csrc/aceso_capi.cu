@@ -673,11 +673,13 @@ int aceso_eval(aceso_ctx *ctx, const uint8_t *d_codes, const uint64_t *d_hdr, in
   P.codes = reinterpret_cast<const uint4 *>(d_codes);
   P.hdr = d_hdr;
 
-  // tiles per warp: 1 (latency), 2 with ACESO_HINT_OVERLAP on the event kernel for models of at
-  // most 24 chunks (384 ops), whose per-tile work does not amortise the per-launch prologue and
-  // epilogue (measured: GPT-3 1.3B +7%, Wide-ResNet +7%; GPT-3 13B, T5 and 1K layers lose with 2)
-  const int tpw = (kern == 1 && (flags & ACESO_HINT_OVERLAP) && P.nch <= 24) ? std::max(2, ctx->tiles_per_warp)
-                                                                            : ctx->tiles_per_warp;
+  // tiles per warp: 1 (latency); with ACESO_HINT_OVERLAP on the event kernel, 3 for models of at
+  // most 20 chunks (320 ops) and 2 for at most 24 (384 ops), whose per-tile work does not amortise
+  // the per-launch prologue and epilogue (measured, 8 streams: GPT-3 1.3B 5.39 / 5.83 / 5.97 G/s
+  // with 1 / 2 / 3 tiles; Wide-ResNet 4.66 / 5.04 / 4.99; GPT-3 13B 3.21 / 2.96 / 2.35)
+  const int tpw_hint = P.nch <= 20 ? 3 : P.nch <= 24 ? 2 : 1;
+  const int tpw = (kern == 1 && (flags & ACESO_HINT_OVERLAP) && tpw_hint > 1) ? std::max(tpw_hint, ctx->tiles_per_warp)
+                                                                          : ctx->tiles_per_warp;
   const int tiles_per_cta = (kern != 0 ? kWarps : kWarps / ctx->split) * tpw;
   const int64_t need = (P.n_tiles + tiles_per_cta - 1) / tiles_per_cta;
   int grid = (int)std::max<int64_t>(1, std::min<int64_t>(need, ctx->max_ctas[kern][mode]));
