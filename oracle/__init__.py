@@ -29,8 +29,13 @@ def build(force=False):
 def _load():
     global _lib
     if _lib is None:
-        build()
-        lib = ctypes.CDLL(_LIB)
+        # ACESO_ORACLE_LIB: a mutant build of aceso_oracle.c (tests/test_oracle_mutations.py
+        # checks that the pins reject every one of them)
+        path = os.environ.get("ACESO_ORACLE_LIB")
+        if not path:
+            build()
+            path = _LIB
+        lib = ctypes.CDLL(path)
         P = ctypes.c_void_p
         i32, i64 = ctypes.c_int32, ctypes.c_int64
         lib.oracle_eval.argtypes = [i32, i32, i32, i32, i32, i32, P, P, P, P, i64, i64, P, P, i64,

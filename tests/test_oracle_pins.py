@@ -435,3 +435,140 @@ def test_select_orders_classes_then_cost_then_index():
     assert oracle.select(out) == (1, 1, 1)
     out["info"][:] = oracle.INFO_INVALID
     assert oracle.select(out)[2] == -1
+
+
+# --------------------------------------------------------------------------
+# Eq. 1 weight term: parameters + gradients + optimizer state. Mixed-precision
+# Adam keeps fp16 weights (2 B) and gradients (2 B) plus fp32 master weights, momentum
+# and variance (12 B): the textbook 16 bytes per parameter (ZeRO, Rajbhandari et al.).
+# --------------------------------------------------------------------------
+def test_mixed_precision_adam_is_16_bytes_per_parameter():
+    rng = np.random.default_rng(21)
+    for _ in range(20):
+        T = int(rng.integers(1, 5))
+        L = int(rng.integers(2, 9))
+        params = [int(x) for x in rng.integers(1, 10 ** 6, size=T)]
+        op_type = [int(x) for x in rng.integers(0, T, size=L)]
+        recs = {t: (lambda tpl, b: [3, 0, 5, 0, 0, 0, 0, 0, 0, 0]) for t in range(T)}
+        wm = np.array([[[4 * params[t], 12 * params[t]]] for t in range(T)], np.int64)
+        p = int(rng.integers(1, min(L, 4) + 1))
+        cuts = sorted(int(x) for x in rng.choice(np.arange(1, L), size=p - 1, replace=False))
+        sizes = [b - a for a, b in zip([0] + cuts, cuts + [L])]
+        prof = mkprof(recs, op_type, G=p, Bg=8, wmem=wm)
+        out = ev(prof, [cand(sizes)], [ai.header(1, p)])
+        assert out["info"][0] & oracle.INFO_INVALID == 0
+        a = 0
+        for i, n in enumerate(sizes):
+            assert int(out["stage_mem"][0, i]) == 16 * sum(params[t] for t in op_type[a:a + n])
+            a += n
+
+
+# --------------------------------------------------------------------------
+# Recomputation memory (R3, R4) against the memory timeline of a 1F1B stage
+# (tests/memsim.py). Eq. 1 bounds the timeline from above, and equals it when the op with
+# the largest transient is the stage's last op: there the recomputed op's rebuilt
+# activations (act - keep) and its workspace coexist with every stashed microbatch.
+# --------------------------------------------------------------------------
+def test_recompute_transient_matches_memory_timeline():
+    from tests.memsim import stage_memory_peak
+    rng = np.random.default_rng(23)
+    checked = 0
+    for _ in range(60):
+        p = int(rng.integers(1, 5))
+        k = int(rng.integers(2, 5))
+        L = p * k
+        vals = []
+        for j in range(L):
+            act = int(rng.integers(10, 1000))
+            keep = int(rng.integers(0, act + 1))
+            peak = int(rng.integers(0, 200))
+            vals.append((act, keep, peak))
+        rc = [int(x) for x in rng.integers(0, 2, size=L)]
+        for i in range(p):  # each stage's last op: recomputed, the largest transient
+            j = i * k + k - 1
+            act = 5000 + int(rng.integers(0, 1000))
+            vals[j] = (act, int(rng.integers(0, 100)), 300 + int(rng.integers(0, 100)))
+            rc[j] = 1
+        recs = {j: (lambda v: (lambda tpl, b: [1, 0, 1, 0, v[0], v[1], v[2], 0, 0, 0]))(vals[j])
+                for j in range(L)}
+        Wt = [int(x) for x in rng.integers(0, 10 ** 4, size=L)]
+        wm = np.array([[[Wt[j], 0]] for j in range(L)], np.int64)
+        prof = mkprof(recs, list(range(L)), G=p, Bg=16, wmem=wm)
+        mbs_log2 = int(rng.integers(0, 5))
+        N = 16 >> mbs_log2
+        out = ev(prof, [cand([k] * p, rc=rc)], [ai.header(mbs_log2, p)])
+        assert out["info"][0] & oracle.INFO_INVALID == 0
+        for i in range(p):
+            ops = [vals[j] + (rc[j],) for j in range(i * k, i * k + k)]
+            sim = stage_memory_peak(ops, sum(Wt[i * k:i * k + k]), p, i, N)
+            assert int(out["stage_mem"][0, i]) == sim
+            checked += 1
+    assert checked > 100
+
+
+def test_eq1_bounds_the_memory_timeline():
+    """Any stage composition: the timeline never exceeds Eq. 1 (R3, R4: conservative)."""
+    from tests.memsim import stage_memory_peak
+    rng = np.random.default_rng(29)
+    for _ in range(60):
+        p = int(rng.integers(1, 5))
+        k = int(rng.integers(1, 5))
+        L = p * k
+        vals = []
+        for j in range(L):
+            act = int(rng.integers(0, 1000))
+            vals.append((act, int(rng.integers(0, act + 1)), int(rng.integers(0, 3000))))
+        rc = [int(x) for x in rng.integers(0, 2, size=L)]
+        recs = {j: (lambda v: (lambda tpl, b: [1, 0, 1, 0, v[0], v[1], v[2], 0, 0, 0]))(vals[j])
+                for j in range(L)}
+        prof = mkprof(recs, list(range(L)), G=p, Bg=16)
+        mbs_log2 = int(rng.integers(0, 5))
+        out = ev(prof, [cand([k] * p, rc=rc)], [ai.header(mbs_log2, p)])
+        for i in range(p):
+            ops = [vals[j] + (rc[j],) for j in range(i * k, i * k + k)]
+            assert stage_memory_peak(ops, 0, p, i, 16 >> mbs_log2) <= int(out["stage_mem"][0, i])
+
+
+# --------------------------------------------------------------------------
+# FULL outputs (Heuristic-2's per-stage resource consumption, P:L206-210) with every term
+# present: each record field is a distinct power of ten, so the per-stage totals read as
+# digit counts and a dropped or misattributed term changes a digit.
+#   fwd_comp 1, fwd_comm 10, bwd_comp 100, bwd_comm 1000, reshard 1e4, p2p_fwd 1e5,
+#   p2p_bwd 1e6; DP sync 1e7 per op with dp = 2 (0 with dp = 1, no data parallelism)
+# --------------------------------------------------------------------------
+def test_full_outputs_resource_split_fingerprint():
+    prof = mkprof({0: lambda tpl, b: [1, 10, 100, 1000, 0, 0, 0, 10 ** 4, 10 ** 5, 10 ** 6]},
+                  [0] * 5, n_tp=2, n_b=2, n_dp=2, G=4, Bg=8,
+                  dps=[[[0, 10 ** 7], [0, 10 ** 7]]])
+    # stage 0 (2 devices): op0 tp2/dp1 (head), op1 tp1/dp2 (tp/dp change: reshard), op2 tp1/dp2 rc
+    # stage 1 (2 devices): op3 tp1/dp2 (head), op4 tp1/dp2 rc
+    row = [ai.code(1, 1, 0, 0), ai.code(0, 0, 1, 0), ai.code(0, 0, 1, 1),
+           ai.code(1, 0, 1, 0), ai.code(0, 0, 1, 1)]
+    out = ev(prof, [row], [ai.header(1, 2)])  # mbs 2, N = 4
+    assert out["info"][0] & oracle.INFO_INVALID == 0
+    N = 4
+    # compute per microbatch: 3 ops x (fwd 1 + bwd 100) + 1 recomputed forward = 304 / 203
+    assert list(out["stage_comp"][0, :2]) == [N * 304, N * 203]
+    # communication per microbatch: 3 x (10 + 1000) + 10 (recomputed forward collective)
+    #   + 1e4 (reshard into op1) + 1e5 (p2p_fwd of op2: stage 0 sends forward)  = 113,040
+    #   stage 1: 2 x 1010 + 10 + 1e6 (p2p_bwd of op3: stage 1 sends backward) = 1,002,030
+    # plus the DP sync once per iteration: 2 ops with dp = 2 on each stage    = 2e7
+    assert list(out["stage_comm"][0, :2]) == [N * 113040 + 2 * 10 ** 7, N * 1002030 + 2 * 10 ** 7]
+    S0, S1 = 304 + 113040, 203 + 1002030
+    assert list(out["stage_T"][0, :2]) == [S0 + S1 + (N - 1) * S0 + 2 * 10 ** 7,
+                                           S0 + S1 + (N - 1) * S1 + 2 * 10 ** 7]
+
+
+def test_heuristic1_memory_first_when_oom():
+    """Heuristic-1 when the largest-memory stage is not the slowest one: out of
+    memory -> the largest-memory stage; feasible -> the slowest stage."""
+    # stage 0: 1 light op (memory-heavy: 3 in-flight microbatches of 40 B); stage 1: 3 slow ops
+    recs = {0: lambda tpl, b: [1, 0, 1, 0, 40, 40, 0, 0, 0, 0],
+            1: lambda tpl, b: [50, 0, 70, 0, 1, 1, 0, 0, 0, 0]}
+    for cap, oom, neck in [(60, True, 0), (1 << 20, False, 1)]:
+        prof = mkprof(recs, [0, 1, 1, 1], G=2, Bg=8, C=cap)
+        out = ev(prof, [cand([1, 3])], [ai.header(1, 2)])   # N = 4, in-flight 2 / 1
+        assert list(out["stage_mem"][0, :2]) == [80, 3]
+        assert out["stage_T"][0, 1] > out["stage_T"][0, 0]
+        assert bool(out["info"][0] & oracle.INFO_OOM) == oom
+        assert out["info"][0] & 0xFF == neck
