@@ -65,27 +65,55 @@ def _alloc(n, L, tiled):
     return np.zeros((n, L), dtype=np.uint8)
 
 
+def _parts(n, threads):
+    """Splits [0, n) into up to `threads` ranges aligned to 32 candidates (whole tiles)."""
+    k = max(1, min(threads, (n + 31) // 32))
+    tiles = (n + 31) // 32
+    cuts = [min(n, 32 * (tiles * i // k)) for i in range(k + 1)]
+    return [(a, b) for a, b in zip(cuts[:-1], cuts[1:]) if b > a]
+
+
+def _run_parts(fn, n, threads):
+    parts = _parts(n, threads)
+    if len(parts) == 1:
+        fn(*parts[0])
+        return
+    from concurrent.futures import ThreadPoolExecutor  # ctypes calls release the GIL
+    with ThreadPoolExecutor(len(parts)) as ex:
+        for f in [ex.submit(fn, a, b) for a, b in parts]:
+            f.result()
+
+
 def search_shaped(prof: Profile, seed: int, first: int, n: int, group_size: int = 1024,
-                  invalid_permille: int = 20, tiled: bool = False):
-    """Candidates [first, first+n) of the search-shaped distribution."""
+                  invalid_permille: int = 20, tiled: bool = False, threads: int = 1):
+    """Candidates [first, first+n) of the search-shaped distribution.
+    The generator is counter-based, so `threads` > 1 only splits the work (same bytes)."""
     lib = _load()
     m, keep = _model(prof)
     codes = _alloc(n, prof.n_ops, tiled)
     hdr = np.zeros(n, dtype=np.uint64)
-    rc = lib.gen_search_shaped(ctypes.byref(m), seed, first, n, group_size, invalid_permille,
-                               codes.ctypes.data, int(tiled), hdr.ctypes.data)
-    assert rc == 0
+    row = tiled_bytes(32, prof.n_ops) // 32 if tiled else prof.n_ops  # bytes per candidate
+
+    def part(a, b):
+        rc = lib.gen_search_shaped(ctypes.byref(m), seed, first + a, b - a, group_size, invalid_permille,
+                                   codes.ctypes.data + a * row, int(tiled), hdr.ctypes.data + 8 * a)
+        assert rc == 0
+    _run_parts(part, n, threads)
     return codes, hdr
 
 
-def dense_random(prof: Profile, seed: int, first: int, n: int, tiled: bool = False):
+def dense_random(prof: Profile, seed: int, first: int, n: int, tiled: bool = False, threads: int = 1):
     lib = _load()
     m, keep = _model(prof)
     codes = _alloc(n, prof.n_ops, tiled)
     hdr = np.zeros(n, dtype=np.uint64)
-    rc = lib.gen_dense_random(ctypes.byref(m), seed, first, n, codes.ctypes.data, int(tiled),
-                              hdr.ctypes.data)
-    assert rc == 0
+    row = tiled_bytes(32, prof.n_ops) // 32 if tiled else prof.n_ops
+
+    def part(a, b):
+        rc = lib.gen_dense_random(ctypes.byref(m), seed, first + a, b - a, codes.ctypes.data + a * row,
+                                  int(tiled), hdr.ctypes.data + 8 * a)
+        assert rc == 0
+    _run_parts(part, n, threads)
     return codes, hdr
 
 

@@ -1,16 +1,23 @@
 """Benchmark: candidate configurations evaluated per second (BASELINE.json metric).
 
-One step = one pass of the whole hot path over one batch
-of synthetic candidates resident in HBM: aceso_eval (decode, lookup, per-stage
-reduce, Eq. 1/2, OOM, Heuristic-1, summary outputs, fused argmin) and, for N > 1,
-the NCCL all-reduce MIN of the packed key. Weak scaling: every rank evaluates its
-own batch of `--batch` candidates per step.
+One step = one pass of the whole hot path over one batch of
+synthetic candidates resident in HBM: aceso_eval (decode, lookup, per-stage reduce, Eq. 1/2,
+OOM, Heuristic-1, summary outputs, fused argmin) and, for N > 1, the NCCL all-reduce MIN of
+the packed keys. Weak scaling: every rank evaluates its own shard of `--batch` candidates per
+step (global indices rank*batch ... (rank+1)*batch - 1 of the step's job).
+
+Headline workload (BASELINE.json configs[4], the paper's scalability case P:L339): the
+1K-layer GPT on 64 simulated devices, 131,072 candidates per GPU per step (the 1M-candidate
+batch across 8 GPUs). `all_workloads` measures every other BASELINE config in the same run
+(GPT-3 1.3B / 13B, T5, Wide-ResNet, the toy models) with its own roofline, single-stream
+roofline, oracle baseline, search time and Exp#4 exhaustive baseline.
 
   python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
-                  [--config gpt3-1.3b] [--dist search|dense] [--batch 65536]
+                  [--config gpt-1k] [--dist search|dense] [--batch 0 (= the config's)]
 
-Prints one JSON line (rank 0). `--impl reference` times the CPU oracle (this
-tier's reference arm) on the host cores with the same metric/config.
+`--gpus N` without torchrun relaunches itself under torch.distributed.run with N ranks.
+Prints one JSON line (rank 0). `--impl reference` times the CPU oracle (this tier's
+reference arm) on the host cores with the same metric/config.
 """
 import argparse
 import json
@@ -28,41 +35,54 @@ sys.path.insert(0, ROOT)
 
 SEED = 20240422
 L2_BYTES = 126 * 2 ** 20
+# candidates per GPU per step (the 1K-layer share is 1M / 8 GPUs)
+BATCH = {"gpt-1k": 131072, "gpt3-13b": 262144, "gpt3-1.3b": 65536, "t5": 65536, "wrn": 65536,
+         "toy-a": 0, "toy-b": 0}  # 0: the toy's whole exhaustively enumerable space
+ALL_WORKLOADS = ["gpt3-1.3b", "gpt3-13b", "t5", "wrn", "gpt-1k", "toy-a", "toy-b"]
 
 
 def parse():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=2000)
-    ap.add_argument("--warmup", type=int, default=20)
+    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    ap.add_argument("--config", default="gpt3-1.3b")
+    ap.add_argument("--config", default="gpt-1k", choices=sorted(BATCH))
     ap.add_argument("--dist", default="search", choices=["search", "dense"])
     ap.add_argument("--no-hint", action="store_true",
                     help="do not pass ACESO_HINT_DENSE for --dist dense (time the default schedule)")
-    ap.add_argument("--batch", type=int, default=65536)
+    ap.add_argument("--batch", type=int, default=0, help="candidates per GPU per step (0: the config's)")
     ap.add_argument("--group", type=int, default=1024, help="candidates sharing a base config")
+    ap.add_argument("--streams", type=int, default=0,
+                    help="independent batches in flight (0: 8 for batches under 64 MB, else 2)")
+    ap.add_argument("--no-overlap-hint", action="store_true",
+                    help="do not pass ACESO_HINT_OVERLAP when several streams are in flight")
+    ap.add_argument("--keys-per-allreduce", type=int, default=16,
+                    help="N > 1: packed keys of this many steps per all-reduce MIN")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--no-dedup", action="store_true", help="skip the hash / visited-set measurement")
-    ap.add_argument("--no-incr", action="store_true", help="skip the incremental-evaluation measurement")
     ap.add_argument("--no-dp", action="store_true", help="skip the Exp#4 exhaustive-baseline measurement")
+    ap.add_argument("--no-all", action="store_true", help="skip the all_workloads measurements")
+    ap.add_argument("--all-steps", type=int, default=200, help="timed steps per all_workloads entry")
     ap.add_argument("--search-budget", type=float, default=20.0,
-                    help="seconds for the search-time measurement (0: skip)")
-    ap.add_argument("--keys-per-allreduce", type=int, default=16,
-                    help="N > 1: packed keys of this many steps per all-reduce MIN")
-    ap.add_argument("--no-overlap-hint", action="store_true",
-                    help="do not pass ACESO_HINT_OVERLAP when several streams are in flight")
-    ap.add_argument("--streams", type=int, default=8,
-                    help="independent batches in flight (steps round-robin over streams)")
+                    help="seconds for each search-time measurement (0: skip)")
     return ap.parse_args()
+
+
+def relaunch(args):
+    """`--gpus N` (N > 1) without torchrun: run this command under torch.distributed.run."""
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={args.gpus}",
+           "--master-addr=127.0.0.1", f"--master-port={29500 + os.getpid() % 1000}", os.path.abspath(__file__)]
+    cmd += sys.argv[1:]
+    return subprocess.call(cmd)
 
 
 def peaks():
     try:
         with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
             d = json.load(f)
-        return float(d["hbm_gbs"]), "measured"
+        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json)"
     except Exception:
         return 6650.0, "fallback (B200_PROFILING.md)"
 
@@ -73,15 +93,17 @@ def bytes_per_cand(L, summary=True):
     return L + 8 + (20 if summary else 0)
 
 
-def workload_name(prof):
-    return prof.name
-
-
 def gen_batch(prof, dist, first, n, group, tiled=True):
     import aceso_inputs as ai
+    th = max(1, min(16, len(os.sched_getaffinity(0))))
     if dist == "search":
-        return ai.search_shaped(prof, SEED, first, n, group_size=group, tiled=tiled)
-    return ai.dense_random(prof, SEED, first, n, tiled=tiled)
+        return ai.search_shaped(prof, SEED, first, n, group_size=group, tiled=tiled, threads=th)
+    return ai.dense_random(prof, SEED, first, n, tiled=tiled, threads=th)
+
+
+def toy_space(prof):
+    import aceso_inputs as ai
+    return ai.exhaustive(prof, per_op=prof.name == "toy-a")
 
 
 class ClockSampler:
@@ -142,41 +164,330 @@ class ClockSampler:
                 "reasons": sorted(self.reasons), "samples": len(self.samples)}
 
 
-def cpu_baseline(prof, batches_rowmajor, max_cands, min_core_seconds=10.0):
-    """The oracle (as it stands) on the host cores over a bounded sample of the workload:
-    passes over the same candidates until about `min_core_seconds` of CPU work."""
+def cpu_baseline(prof, codes, hdr, target_core_s=15.0, what="candidates of the timed workload (same seed)"):
+    """The oracle (as it stands) on the host cores over a bounded sample of the workload: one
+    pass sized to about `target_core_s` seconds of CPU work (from a timed warm-up)."""
     import oracle
     threads = len(os.sched_getaffinity(0))
-    codes = np.concatenate([b[0] for b in batches_rowmajor])[:max_cands]
-    hdr = np.concatenate([b[1] for b in batches_rowmajor])[:max_cands]
-    oracle.evaluate(prof, codes[:256], hdr[:256], threads=threads)  # warm
-    done, passes = 0, 0
+    w = min(len(hdr), max(64, 4 * threads))
     t0 = time.perf_counter()
-    while True:
-        oracle.evaluate(prof, codes, hdr, threads=threads)
-        done += len(hdr)
-        passes += 1
-        dt = time.perf_counter() - t0
-        if dt * threads >= min_core_seconds or passes >= 64:
-            break
-    return {"value": done / dt, "unit": "configs/s", "cores": threads, "kind": "oracle",
-            "sample": f"{len(hdr)} candidates of the timed workload (same seed) x {passes} passes "
-                      f"= {done} evaluations, {dt:.2f} s wall on {threads} threads"}
+    oracle.evaluate(prof, codes[:w], hdr[:w], threads=threads)  # warm-up, also sizes the sample
+    per_cand_core = (time.perf_counter() - t0) * threads / w
+    m = int(min(len(hdr), max(w, target_core_s / max(per_cand_core, 1e-9))))
+    t0 = time.perf_counter()
+    oracle.evaluate(prof, codes[:m], hdr[:m], threads=threads)
+    dt = time.perf_counter() - t0
+    return {"value": m / dt, "unit": "configs/s", "cores": threads, "kind": "oracle",
+            "sample": f"{m} {what}, one pass, {dt:.2f} s wall on {threads} threads"}
 
 
-def measure_dedup(A, dev_batches, n, L, hbm, reps=200):
+class Batches:
+    """Distinct device-resident batches (together larger than L2) of this rank's shard."""
+
+    def __init__(self, A, prof, dist, n, group, world, rank, dev, toy=False):
+        self.n, self.L = n, prof.n_ops
+        per_batch = A.tiled_bytes(n, self.L) + 8 * n
+        self.nbuf = max(2, int(np.ceil(1.3 * L2_BYTES / per_batch)))
+        self.host, self.dev = [], []
+        if toy:  # the whole space, replicated into distinct buffers
+            import aceso_inputs as ai
+            codes, hdr = toy_space(prof)
+            tiled = ai.tile(codes)
+            for b in range(self.nbuf):
+                self.host.append((tiled, hdr, 0))
+                self.dev.append(A.upload_candidates(tiled, hdr, dev.index))
+            self.rowmajor = (codes, hdr)
+            return
+        for b in range(self.nbuf):
+            first = (b * world + rank) * n  # global indices of this rank's shard of batch b
+            codes, hdr = gen_batch(prof, dist, first, n, group, tiled=True)
+            self.host.append((codes, hdr, first))
+            self.dev.append(A.upload_candidates(codes, hdr, dev.index))
+        self.rowmajor = None
+        self.bytes = self.nbuf * per_batch
+
+
+def time_steps(A, ctx, bt, steps, warmup, nstr, overlap, world, rank, hint, kpa, dist=None):
+    """K steps (one aceso_eval per step; N > 1: the packed keys of every `kpa` steps in one NCCL
+    all-reduce MIN on a communication stream) captured in one CUDA graph, replayed once between
+    CUDA events. Steps are issued round-robin on `nstr` streams (independent batches overlap).
+    Returns timing, per-launch concurrent kernel time, clocks and the last step's selection."""
+    import torch
+    from paper_conf_eurosys_liumlsmybw24_b200.api import Selection
+    n, dev = bt.n, torch.device("cuda", torch.cuda.current_device())
+    n_total = n * world
+    nsel = nstr * ((bt.nbuf + nstr - 1) // nstr)  # multiple of nstr: a buffer stays on one stream
+    sels = [ctx.alloc_select(n) for _ in range(nsel)]
+    outs = [ctx.alloc_outputs(n) for _ in range(nstr)]
+    side = [torch.cuda.Stream() for _ in range(nstr)]
+    comm = torch.cuda.Stream()
+    keyvec = torch.empty(max(1, steps), dtype=torch.int64, device=dev)
+    red = dist is not None  # packed keys all-reduced (N > 1, or the one-rank NCCL test mode)
+
+    def launch(s, st, ev0=None, ev1=None):
+        c, h = bt.dev[s % bt.nbuf]
+        if ev0 is not None:
+            ev0.record(st)
+        ctx.eval(c, h, n=n, global_offset=rank * n, n_total=n_total, summary=True, select=True,
+                 out=outs[s % nstr], sel=sels[s % nsel], stream=st, dense_hint=hint, overlap_hint=overlap)
+        if ev1 is not None:
+            ev1.record(st)
+
+    for s in range(max(warmup, nstr)):  # warm-up: every stream and select buffer used once
+        launch(s, side[s % nstr])
+    torch.cuda.synchronize()
+    ev_s = [torch.cuda.Event(enable_timing=True, external=True) for _ in range(steps)]
+    ev_k = [torch.cuda.Event(enable_timing=True, external=True) for _ in range(steps)]
+
+    def issue():
+        cs = torch.cuda.current_stream()
+        fork = torch.cuda.Event()
+        fork.record(cs)
+        for st in side + [comm]:
+            st.wait_event(fork)
+        comm_done = {}
+        for s in range(steps):
+            st = side[s % nstr]
+            if s - nsel in comm_done:  # the select buffer's previous all-reduce has read it
+                st.wait_event(comm_done.pop(s - nsel))
+            launch(s, st, ev_s[s], ev_k[s])
+            if red:
+                done = torch.cuda.Event()
+                done.record(st)
+                comm.wait_event(done)
+                with torch.cuda.stream(comm):
+                    keyvec[s:s + 1].copy_(sels[s % nsel][0:8].view(torch.int64))
+                    if (s + 1) % kpa == 0 or s == steps - 1:
+                        s0 = (s // kpa) * kpa
+                        dist.all_reduce(keyvec[s0:s + 1], op=dist.ReduceOp.MIN)
+                cd = torch.cuda.Event()
+                cd.record(comm)
+                comm_done[s] = cd
+        for st in side + [comm]:
+            j = torch.cuda.Event()
+            j.record(st)
+            cs.wait_event(j)
+
+    mode = "graph"
+    graph = torch.cuda.CUDAGraph()
+    try:
+        with torch.cuda.graph(graph):
+            issue()
+        torch.cuda.synchronize()
+        graph.replay()  # untimed replay (upload)
+        torch.cuda.synchronize()
+    except Exception as e:  # a collective that cannot be captured: time eager issue
+        mode = f"eager ({type(e).__name__} during graph capture)"
+        print(f"[bench] graph capture failed ({e}); timing eagerly issued steps", file=sys.stderr)
+        torch.cuda.synchronize()
+        ev_s = [torch.cuda.Event(enable_timing=True) for _ in range(steps)]
+        ev_k = [torch.cuda.Event(enable_timing=True) for _ in range(steps)]
+        issue()
+        torch.cuda.synchronize()
+    clocks = ClockSampler(torch.cuda.current_device())
+    t0, t1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    if red:
+        dist.barrier()
+    torch.cuda.synchronize()
+    clocks.start()
+    cs = torch.cuda.current_stream()
+    t0.record(cs)
+    if mode == "graph":
+        graph.replay()
+    else:
+        issue()
+    t1.record(cs)
+    torch.cuda.synchronize()
+    if red:
+        dist.barrier()
+    clk = clocks.stop()
+    t = torch.tensor([t0.elapsed_time(t1), float(np.mean([ev_s[s].elapsed_time(ev_k[s]) for s in range(steps)]))],
+                     dtype=torch.float64, device=dev)
+    if red:
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)  # max over ranks
+    elapsed_ms, kern_ms = float(t[0]), float(t[1])
+    last = sels[(steps - 1) % nsel]
+    best = Selection.from_buffer(last)
+    if red:
+        from paper_conf_eurosys_liumlsmybw24_b200 import dist as adist
+        kl = int(keyvec[steps - 1].item())
+        gc, gcost, gidx, sat = A.decode_key(kl, n_total)
+        best = adist.global_select(last, n_total) if sat else Selection(gc, gcost, gidx, kl)
+    return {"elapsed_ms": elapsed_ms, "ms_per_step": elapsed_ms / steps, "kern_ms": kern_ms,
+            "mode": mode, "clocks": clk, "best": best, "last_batch": (steps - 1) % bt.nbuf}
+
+
+def time_serial(ctx, bt, k, rank, world, hint):
+    """The same kernel launched back to back on one stream (CUDA events around each launch)."""
+    import torch
+    n = bt.n
+    out = ctx.alloc_outputs(n)
+    sel = ctx.alloc_select(n)
+    evs = [torch.cuda.Event(enable_timing=True, external=True) for _ in range(k)]
+    eve = [torch.cuda.Event(enable_timing=True, external=True) for _ in range(k)]
+    g = torch.cuda.CUDAGraph()
+    torch.cuda.synchronize()
+    with torch.cuda.graph(g):
+        cs = torch.cuda.current_stream()
+        for s in range(k):
+            c, h = bt.dev[s % bt.nbuf]
+            evs[s].record(cs)
+            ctx.eval(c, h, n=n, global_offset=rank * n, n_total=n * world, summary=True, select=True,
+                     out=out, sel=sel, stream=cs, dense_hint=hint)
+            eve[s].record(cs)
+    g.replay()
+    torch.cuda.synchronize()
+    g.replay()
+    torch.cuda.synchronize()
+    return float(np.mean([evs[s].elapsed_time(eve[s]) for s in range(k)]))
+
+
+def e2e_pipelined(A, ctx, bt, steps, rank, world, hint, dist=None):
+    """The metric end to end through the public API: each step copies its inputs (tiled codes +
+    headers) from pinned host memory to the device, evaluates them (aceso_eval, fused select;
+    N > 1: all-reduce MIN of the key) and reads the 32-byte result back to pinned host memory.
+    Two device buffers: the copy engine loads step k+1 while the SMs evaluate step k."""
+    import torch
+    n, L = bt.n, bt.L
+    dev = torch.device("cuda", torch.cuda.current_device())
+    pinned = [(torch.from_numpy(c).pin_memory(), torch.from_numpy(h.view(np.int64)).pin_memory())
+              for c, h, _ in bt.host[:2]]
+    dbuf = [(torch.empty(A.tiled_bytes(n, L), dtype=torch.uint8, device=dev),
+             torch.empty(n, dtype=torch.int64, device=dev)) for _ in range(2)]
+    sel = [ctx.alloc_select(n) for _ in range(2)]
+    out = ctx.alloc_outputs(n)
+    res = torch.empty((steps, 32), dtype=torch.uint8).pin_memory()
+    cp, cs = torch.cuda.Stream(), torch.cuda.Stream()
+    loaded = [torch.cuda.Event() for _ in range(steps)]
+    freed = [torch.cuda.Event() for _ in range(steps)]
+
+    def run(k_steps):
+        for k in range(k_steps):
+            b = k % 2
+            with torch.cuda.stream(cp):
+                if k >= 2:
+                    cp.wait_event(freed[k - 2])  # evaluation of step k-2 has read this buffer
+                dbuf[b][0].copy_(pinned[k % 2][0], non_blocking=True)
+                dbuf[b][1].copy_(pinned[k % 2][1], non_blocking=True)
+                loaded[k].record(cp)
+            cs.wait_event(loaded[k])
+            ctx.eval(dbuf[b][0], dbuf[b][1], n=n, global_offset=rank * n, n_total=n * world, summary=True,
+                     select=True, out=out, sel=sel[b], stream=cs, dense_hint=hint)
+            with torch.cuda.stream(cs):
+                if dist is not None:
+                    dist.all_reduce(sel[b][0:8].view(torch.int64), op=dist.ReduceOp.MIN)
+                res[k].copy_(sel[b][:32], non_blocking=True)
+            freed[k].record(cs)
+
+    run(min(steps, 3))
+    torch.cuda.synchronize()
+    if dist is not None:
+        dist.barrier()
+    t0, t1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    t0.record(cp)
+    cs.wait_event(t0)
+    run(steps)
+    t1.record(cs)
+    torch.cuda.synchronize()
+    te = torch.tensor([t0.elapsed_time(t1)], dtype=torch.float64, device=dev)
+    if dist is not None:
+        dist.all_reduce(te, op=dist.ReduceOp.MAX)
+    return {"value": n * world * steps / (float(te[0]) * 1e-3), "unit": "configs/s",
+            "h2d_bytes_per_step": int(A.tiled_bytes(n, L) + 8 * n), "d2h_bytes_per_step": 32,
+            "steps": steps,
+            "pipeline": "pinned host codes+headers -> H2D (copy stream, double-buffered) -> "
+                        "aceso_eval (fused select) -> D2H 32-byte result; copies overlap evaluation"}
+
+
+def e2e_descriptors(A, ctx, prof, n, steps):
+    """The search driver's real host input (NEXT(2)): every candidate as a 56-byte descriptor
+    (base index + Table-1 primitive patches, search.Primitives.describe_all on evaluated bases).
+    Per step: H2D of the descriptors (pinned, copy stream, double-buffered), aceso_expand,
+    aceso_eval (fused select), D2H of the 32-byte result. The bases are uploaded once."""
+    import torch
+    from paper_conf_eurosys_liumlsmybw24_b200 import candidates as C
+    from paper_conf_eurosys_liumlsmybw24_b200 import search as S
+    from paper_conf_eurosys_liumlsmybw24_b200.api import as_u32, as_u64
+    dev = torch.device("cuda", torch.cuda.current_device())
+    L, stride = prof.n_ops, C.stride_of(prof.n_ops)
+    codes, hdr = gen_batch(prof, "search", 0, 2048, 64, tiled=False)
+    out, _ = ctx.eval(ctx.pack_rowmajor(torch.from_numpy(codes).to(dev)),
+                      torch.from_numpy(hdr.view(np.int64)).to(dev), full=True, select=False)
+    torch.cuda.synchronize()
+    info = as_u32(out.info)
+    pm = out.p_max
+    st_T, st_c, st_m = (as_u64(getattr(out, k)).reshape(pm, -1).T for k in ("stage_T", "stage_comp", "stage_comm"))
+    ok = np.nonzero((info & (1 << 17)) == 0)[0][:32]
+    prim = S.Primitives(prof)
+    bases = np.zeros((len(ok), stride), np.uint8)
+    ranks = np.zeros((len(ok), 2, stride), np.uint16)
+    chunks = []
+    for bi, i in enumerate(ok):
+        bases[bi, :L] = codes[i]
+        cd, rk = prim.describe_all(codes[i], int(hdr[i] & 0xFF), int(info[i]), st_c[i], st_m[i], st_T[i])
+        cd["base"] = bi
+        ranks[bi] = rk
+        chunks.append(cd)
+    allc = np.concatenate(chunks)
+    tb = torch.from_numpy(bases).to(dev)
+    tr = torch.from_numpy(ranks.view(np.int16)).to(dev)
+    hc = [torch.from_numpy(allc[(np.arange(n) + k * 7919) % len(allc)].view(np.uint8).copy()).pin_memory()
+          for k in range(2)]
+    dcd = [torch.empty(n * 56, dtype=torch.uint8, device=dev) for _ in range(2)]
+    tiled = ctx.alloc_tiled(n)
+    thd = torch.empty(n, dtype=torch.int64, device=dev)
+    sel = ctx.alloc_select(n)
+    o2 = ctx.alloc_outputs(n)
+    res = torch.empty((steps, 32), dtype=torch.uint8).pin_memory()
+    cp, cs = torch.cuda.Stream(), torch.cuda.Stream()
+    loaded = [torch.cuda.Event() for _ in range(steps)]
+    freed = [torch.cuda.Event() for _ in range(steps)]
+
+    def run(k_steps):
+        for k in range(k_steps):
+            b = k % 2
+            with torch.cuda.stream(cp):
+                if k >= 2:
+                    cp.wait_event(freed[k - 2])
+                dcd[b].copy_(hc[k % 2], non_blocking=True)
+                loaded[k].record(cp)
+            cs.wait_event(loaded[k])
+            ctx.expand(tb, dcd[b], tr, n=n, tiled=tiled, hdr=thd, stream=cs)
+            freed[k].record(cs)
+            ctx.eval(tiled, thd, n=n, summary=True, select=True, out=o2, sel=sel, stream=cs)
+            with torch.cuda.stream(cs):
+                res[k].copy_(sel[:32], non_blocking=True)
+
+    run(min(steps, 3))
+    torch.cuda.synchronize()
+    t0, t1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    t0.record(cp)
+    cs.wait_event(t0)
+    run(steps)
+    t1.record(cs)
+    torch.cuda.synchronize()
+    ms = t0.elapsed_time(t1) / steps
+    return {"value": n / (ms * 1e-3), "unit": "configs/s", "h2d_bytes_per_step": n * 56,
+            "d2h_bytes_per_step": 32, "steps": steps, "bases": int(len(ok)),
+            "distinct_descriptors": int(len(allc)),
+            "pipeline": "pinned 56-byte descriptors -> H2D (copy stream, double-buffered) -> "
+                        "aceso_expand -> aceso_eval (fused select) -> D2H 32-byte result"}
+
+
+def measure_dedup(A, bt, hbm, reps=100):
     """NEXT(3) kernels on the bench batches: aceso_hash (streaming: reads the tiled codes and
     headers, writes 8 B per candidate) and aceso_dedup (visited-set insert + flag)."""
     import torch
-    hs = [torch.empty(n, dtype=torch.int64, device=dev_batches[0][0].device) for _ in dev_batches]
-    for (c, h), o in zip(dev_batches, hs):
+    n, L = bt.n, bt.L
+    hs = [torch.empty(n, dtype=torch.int64, device=bt.dev[0][0].device) for _ in bt.dev]
+    for (c, h), o in zip(bt.dev, hs):
         A.hash_candidates(c, h, L, out=o)
     torch.cuda.synchronize()
     ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    g = torch.cuda.CUDAGraph()  # launches captured: host call overhead must not pace the GPU
+    g = torch.cuda.CUDAGraph()
     with torch.cuda.graph(g):
         for r in range(reps):
-            c, h = dev_batches[r % len(dev_batches)]
+            c, h = bt.dev[r % len(bt.dev)]
             A.hash_candidates(c, h, L, out=hs[r % len(hs)])
     g.replay()
     torch.cuda.synchronize()
@@ -185,16 +496,15 @@ def measure_dedup(A, dev_batches, n, L, hbm, reps=200):
     ev1.record()
     torch.cuda.synchronize()
     ms = ev0.elapsed_time(ev1) / reps
-    hbytes = n * (L + 8 + 8)  # codes + header read, hash written
-    # visited set sized for every batch's hashes at <= 50% load
+    hbytes = n * (L + 8 + 8)
     slots = 1 << int(np.ceil(np.log2(2 * n * len(hs))))
     vs = A.VisitedSet(slots, device=hs[0].device.index)
     dup = torch.empty(n, dtype=torch.uint8, device=hs[0].device)
-    vs.insert(hs[0][:1], dup=dup)  # warm-up (epoch 1)
+    vs.insert(hs[0][:1], dup=dup)
     torch.cuda.synchronize()
     gv = torch.cuda.CUDAGraph()
     with torch.cuda.graph(gv):
-        for o in hs:  # distinct batches (later epochs): duplicates are the generator's own
+        for o in hs:
             vs.insert(o, dup=dup)
     ev0.record()
     gv.replay()
@@ -212,107 +522,70 @@ def measure_dedup(A, dev_batches, n, L, hbm, reps=200):
                     "visited set (aceso_dedup) on the bench batches; not part of the timed step"}
 
 
-def measure_incr(A, ctx, prof, n, hbm, seed=SEED, reps=100):
-    """NEXT(2): the same metric for candidates given as base + patches (the search driver's
-    Table-1 primitives, 56-byte descriptors) evaluated by aceso_eval_incr against per-base
-    stage caches. Bases: valid search-shaped configurations; every base gets the driver's
-    primitives for a bottleneck taken from its own evaluation (FULL outputs from aceso_eval,
-    so no oracle on this path); descriptors are tiled to n candidates."""
-    import torch
-    from paper_conf_eurosys_liumlsmybw24_b200 import candidates as C
+def measure_search(A, ctx, prof, budget):
     from paper_conf_eurosys_liumlsmybw24_b200 import search as S
-    from paper_conf_eurosys_liumlsmybw24_b200.api import as_u32, as_u64
-    dev = torch.device("cuda", torch.cuda.current_device())
-    L, stride = prof.n_ops, C.stride_of(prof.n_ops)
-    codes, hdr = gen_batch(prof, "search", 0, 4096, 64, tiled=False)
-    out, _ = ctx.eval(ctx.pack_rowmajor(torch.from_numpy(codes).to(dev)), torch.from_numpy(hdr.view(np.int64)).to(dev),
-                      full=True, select=False)
-    torch.cuda.synchronize()
-    info = as_u32(out.info)
-    pm = out.p_max
-    st_T, st_c, st_m = (as_u64(getattr(out, k)).reshape(pm, -1).T for k in ("stage_T", "stage_comp", "stage_comm"))
-    ok = np.nonzero((info & (1 << 17)) == 0)[0][:64]
-    prim = S.Primitives(prof)
-    bases = np.zeros((len(ok), stride), np.uint8)
-    bhdr = np.zeros(len(ok), np.uint64)
-    ranks = np.zeros((len(ok), 2, stride), np.uint16)
-    chunks = []
-    for bi, i in enumerate(ok):
-        bases[bi, :L] = codes[i]
-        bhdr[bi] = hdr[i]
-        cd, rk = prim.describe_all(codes[i], int(hdr[i] & 0xFF), int(info[i]), st_c[i], st_m[i], st_T[i])
-        cd["base"] = bi
-        ranks[bi] = rk
-        chunks.append(cd)
-    allc = np.concatenate(chunks)
-    cands = allc[np.arange(n) % len(allc)]
-    tb = torch.from_numpy(bases).to(dev)
-    th = torch.from_numpy(bhdr.view(np.int64)).to(dev)
-    tr = torch.from_numpy(ranks.view(np.int16)).to(dev)
-    tc = torch.from_numpy(cands.view(np.uint8)).to(dev)
-    o2 = ctx.alloc_outputs(n)
-    sel = ctx.alloc_select(n)
-    from paper_conf_eurosys_liumlsmybw24_b200 import _lib
-    work = torch.empty(int(_lib.load().aceso_incr_work_bytes(ctx._h, len(ok))), dtype=torch.uint8, device=dev)
-    for _ in range(3):
-        ctx.eval_incr(tb, th, tc, tr, n=n, out=o2, sel=sel, work=work)
-    torch.cuda.synchronize()
-    g = torch.cuda.CUDAGraph()
-    with torch.cuda.graph(g):
-        for _ in range(reps):
-            ctx.eval_incr(tb, th, tc, tr, n=n, out=o2, sel=sel, work=work)
-    g.replay()
-    torch.cuda.synchronize()
-    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    e0.record()
-    g.replay()
-    e1.record()
-    torch.cuda.synchronize()
-    ms = e0.elapsed_time(e1) / reps
-    b = n * (56 + 20)
-    # end to end through the public API with descriptors as the host-side input: per step
-    # H2D of the 56-byte descriptors (pinned), aceso_expand, aceso_eval (fused select), D2H of
-    # the 32-byte result; the bases are uploaded once (like the profile)
-    hc = [torch.from_numpy(allc[(np.arange(n) + k * 7919) % len(allc)].view(np.uint8).copy()).pin_memory()
-          for k in range(2)]
-    dcd = torch.empty(n * 56, dtype=torch.uint8, device=dev)
-    tiled = ctx.alloc_tiled(n)
-    thd = torch.empty(n, dtype=torch.int64, device=dev)
-    sel2 = ctx.alloc_select(n)
-    res_host = torch.empty(32, dtype=torch.uint8).pin_memory()
-    stream = torch.cuda.current_stream()
+    ev = S.GPUEvaluator(ctx)
+    res, st = S.search(prof, ev, budget_s=budget, patience=8)
+    init_best = None
+    for p in [1, 2, 4, 8, 16, 32, 64]:
+        r0 = S.initial_config(prof, p) if p <= prof.n_devices else None
+        if r0 is None:
+            continue
+        o = ev.evaluate(r0[0][None, :], np.array([S.header(r0[1], p)], np.uint64))
+        pf = S.perf_of(int(o["info"][0]), o["iter"][0], o["max_mem"][0])
+        init_best = pf if init_best is None or pf < init_best else init_best
+    return {"time_s": st["time_s"], "time_to_best_s": st["time_to_best_s"], "evaluated": st["evaluated"],
+            "batches": st["batches"], "improvements": st["improvements"],
+            "best": {"class": res.perf[0], "cost": res.perf[1], "iter_ns": res.iter_ns,
+                     "p": int((res.codes & 1).sum()), "mbs_log2": res.mbs},
+            "initial_best": {"class": init_best[0], "cost": init_best[1]} if init_best else None,
+            "note": "batched Alg. 1/2 (MaxHops 7) over all stage counts on one GPU, stops after 8 hops "
+                    "without a new best or at the budget; context: the paper's searches use a 200 s "
+                    "budget on its own hosts (P:L313, P:L339)"}
 
-    def e2e_step(k):
-        dcd.copy_(hc[k % 2], non_blocking=True)
-        ctx.expand(tb, dcd, tr, n=n, tiled=tiled, hdr=thd, stream=stream)
-        ctx.eval(tiled, thd, n=n, summary=True, select=True, out=o2, sel=sel2, stream=stream)
-        res_host.copy_(sel2[:32], non_blocking=True)
 
-    for k in range(3):
-        e2e_step(k)
-    torch.cuda.synchronize()
-    ke = 50
-    e0.record(stream)
-    for k in range(ke):
-        e2e_step(k)
-    e1.record(stream)
-    torch.cuda.synchronize()
-    ems = e0.elapsed_time(e1) / ke
-    e2e_d = {"value": n / (ems * 1e-3), "unit": "configs/s", "h2d_bytes_per_step": n * 56,
-             "d2h_bytes_per_step": 32, "steps": ke,
-             "pipeline": "pinned descriptors -> H2D -> aceso_expand -> aceso_eval (fused select) -> D2H result"}
-    return {"configs_per_s": n / (ms * 1e-3), "ms_per_batch": ms, "batch": n, "bases": int(len(ok)),
-            "e2e_descriptors": e2e_d,
-            "distinct_descriptors": int(len(allc)),
-            "roofline": {"bound": "hbm", "achieved": b / (ms * 1e-3) / 1e9, "peak": hbm, "unit": "GB/s",
-                         "frac": b / (ms * 1e-3) / 1e9 / hbm, "bytes_per_candidate": 76},
-            "note": "SURVEY 8(f) NEXT(2): candidates as base + patches (56 B descriptor + 20 B "
-                    "summary), aceso_eval_incr with fused select, one stream, CUDA graph; not part "
-                    "of the timed step"}
+def measure_dp(A, ctx, prof, budget, search=None):
+    from paper_conf_eurosys_liumlsmybw24_b200 import exhaustive as X
+    from paper_conf_eurosys_liumlsmybw24_b200 import search as S
+    dp = X.exhaustive_best(prof, ctx)
+    dcodes, dhdr = dp.pop("codes", None), dp.pop("hdr", None)
+    if search is not None and dp["best"]:
+        sb = search["best"]
+        dp["search_vs_exhaustive"] = {"search_best": [sb["class"], sb["cost"]],
+                                      "exhaustive_best": [dp["best"]["class"], dp["best"]["cost"]],
+                                      "search_explored": search["evaluated"]}
+        if dcodes is not None and budget > 0:
+            hres, hst = S.search(prof, S.GPUEvaluator(ctx), budget_s=budget, patience=8,
+                                 starts=[(dcodes, int(dhdr & np.uint64(0xFF)))])
+            dp["search_vs_exhaustive"]["hybrid_best"] = [hres.perf[0], hres.perf[1]]
+            dp["search_vs_exhaustive"]["hybrid_time_s"] = hst["time_s"] + dp["time_s"]
+    dp["note"] = ("SURVEY 8(f) NEXT(4), Exp#4 (P:L343-357): the pruned stage-uniform space (p = 1, 2, "
+                  "4, ... stages with every op-level cut set, one (tp, dp) for all stages, recompute "
+                  "all or none, every valid microbatch) enumerated and evaluated exhaustively")
+    return dp
+
+
+def roofline(n, L, ms_per_step, kern_ms_serial, hbm, src, traffic_key):
+    bpc = bytes_per_cand(L)
+    achieved = n * bpc / (ms_per_step * 1e-3) / 1e9
+    achieved_serial = n * bpc / (kern_ms_serial * 1e-3) / 1e9
+    traffic = None
+    try:
+        with open(os.path.join(ROOT, "profiles", "ncu_traffic.json")) as f:
+            traffic = json.load(f).get(traffic_key)
+    except Exception:
+        pass
+    return {"bound": "hbm", "achieved": achieved, "peak": hbm, "unit": "GB/s", "frac": achieved / hbm,
+            "traffic": traffic, "bytes_per_candidate": bpc, "bytes_per_launch": n * bpc,
+            "launch_interval_ms": ms_per_step, "kernel_ms_serial": kern_ms_serial,
+            "achieved_serial": achieved_serial, "frac_serial": achieved_serial / hbm, "peak_source": src,
+            "note": "achieved = algorithmic bytes per launch (L codes + 8 header + 20 summary per "
+                    "candidate) / effective launch interval of the timed region (independent batches "
+                    "overlap on streams); *_serial = the same kernel launched back to back on one stream"}
 
 
 def run_reference(args):
-    """Reference arm of this tier: the CPU oracle, timed as it stands."""
+    """Reference arm of this tier: the CPU oracle, timed as it stands (rank 0 only)."""
     import aceso_inputs as ai  # noqa: F401
     import oracle
     from aceso_inputs import profiles as P
@@ -321,12 +594,17 @@ def run_reference(args):
         return 0
     prof = P.WORKLOADS[args.config]()
     threads = len(os.sched_getaffinity(0))
-    per_step = 4096  # bounded sample per step (CPU)
-    n = per_step * max(1, min(args.steps + args.warmup, 64))
-    codes, hdr = gen_batch(prof, args.dist, 0, n, args.group, tiled=False)
+    L = prof.n_ops
+    per_step = int(max(256, min(4096, (1 << 22) // L)))  # bounded sample per step
+    if BATCH[args.config] == 0:
+        codes, hdr = toy_space(prof)
+        n = len(hdr)
+    else:
+        n = per_step * max(1, min(args.steps + args.warmup, 64))
+        codes, hdr = gen_batch(prof, args.dist, 0, n, args.group, tiled=False)
     times = []
     for s in range(args.warmup + args.steps):
-        k = s % (n // per_step)
+        k = s % max(1, n // per_step)
         c = codes[k * per_step:(k + 1) * per_step]
         h = hdr[k * per_step:(k + 1) * per_step]
         t0 = time.perf_counter()
@@ -343,7 +621,7 @@ def run_reference(args):
         "ms_per_step": 1e3 * total / len(times), "higher_is_better": True, "scaling": "weak",
         "vs_baseline": None, "dtype": "u64", "data": "synthetic",
         "config": {"workload": prof.name, "batch": per_step, "distribution": args.dist,
-                   "note": "CPU oracle: each step a bounded 4096-candidate sample of the workload"},
+                   "note": f"CPU oracle: each step a bounded {per_step}-candidate sample of the workload"},
         "cpu_baseline": {"value": value, "unit": "configs/s", "cores": threads, "kind": "oracle",
                          "sample": f"{per_step} candidates per step x {len(times)} steps"},
         "e2e": {"value": value, "unit": "configs/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
@@ -352,363 +630,155 @@ def run_reference(args):
     return 0
 
 
-HINT = False  # ACESO_HINT_DENSE for every aceso_eval of the run (set in main)
+def measure_workload(A, name, args, dev, hbm, src, world=1, rank=0, dist=None, steps=None, with_extras=True):
+    """One BASELINE workload: timed steps (overlapped streams), serial launches, and on request
+    the oracle baseline, search time and Exp#4 baseline."""
+    import torch
+    from aceso_inputs import profiles as P
+    prof = P.WORKLOADS[name]()
+    ctx = A.Context(prof, dev.index)
+    toy = BATCH[name] == 0
+    hint = args.dist == "dense" and not args.no_hint
+    if toy:
+        n = int(len(toy_space(prof)[1]))
+    else:
+        n = args.batch if (args.batch and name == args.config) else BATCH[name]
+    bt = Batches(A, prof, "search" if toy else args.dist, n, args.group, world, rank, dev, toy=toy)
+    per_batch = A.tiled_bytes(n, prof.n_ops) + 8 * n
+    nstr = args.streams or (8 if per_batch < 64 * 2 ** 20 else 2)
+    nstr = max(1, min(nstr, bt.nbuf))
+    overlap = nstr > 1 and not args.no_overlap_hint
+    k = steps or args.steps
+    r = time_steps(A, ctx, bt, k, args.warmup, nstr, overlap, world, rank, hint, args.keys_per_allreduce, dist)
+    ks = min(k, 64)
+    kern_serial = time_serial(ctx, bt, ks, rank, world, hint)
+    if dist is not None:
+        t = torch.tensor([kern_serial], dtype=torch.float64, device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        kern_serial = float(t[0])
+    rec = {
+        "workload": prof.name, "n_ops": prof.n_ops, "batch_per_gpu": n,
+        "distribution": "exhaustive" if toy else args.dist, "value": n * world * k / (r["elapsed_ms"] * 1e-3),
+        "unit": "configs/s", "steps": k, "ms_per_step": r["ms_per_step"], "streams": nstr, "overlap_hint": overlap,
+        "schedule": ctx.schedule(hint), "timing_mode": r["mode"],
+        "roofline": roofline(n, prof.n_ops, r["ms_per_step"], kern_serial, hbm, src,
+                             f"{name}/{'exhaustive' if toy else args.dist}/{n}"),
+        "kernel_ms_concurrent": r["kern_ms"], "clocks": r["clocks"],
+        "result": {"cls": r["best"].cls, "cost": r["best"].cost, "index": r["best"].index},
+        "l2": f"{bt.nbuf} distinct device-resident batches rotated ({bt.nbuf * per_batch / 2**20:.0f} MiB > 126 MiB L2)",
+    }
+    if with_extras and rank == 0 and world == 1:
+        if not args.no_cpu:
+            if toy:
+                rc, rh = bt.rowmajor
+            else:
+                m = int(min(n, max(2048, (1 << 27) // prof.n_ops)))
+                rc, rh = gen_batch(prof, args.dist, rank * n, m, args.group, tiled=False)
+            rec["cpu_baseline"] = cpu_baseline(prof, rc, rh, target_core_s=8.0)
+        if args.search_budget > 0:
+            rec["search"] = measure_search(A, ctx, prof, args.search_budget)
+        if not args.no_dp:
+            rec["dp_baseline"] = measure_dp(A, ctx, prof, args.search_budget, rec.get("search"))
+    return prof, ctx, bt, rec
 
 
 def main():
     args = parse()
+    world_env = os.environ.get("WORLD_SIZE")
+    if args.gpus > 1 and world_env is None:
+        return relaunch(args)
+    if world_env is not None and int(world_env) != args.gpus and not os.environ.get("ACESO_BENCH_BACKEND"):
+        print(f"bench.py: --gpus {args.gpus} but WORLD_SIZE={world_env}", file=sys.stderr)
+        return 2
     if args.impl == "reference":
         return run_reference(args)
 
     import torch
     import torch.distributed as dist
 
-    import aceso_inputs as ai  # noqa: F401
-    from aceso_inputs import profiles as P
     import paper_conf_eurosys_liumlsmybw24_b200 as A
-    from paper_conf_eurosys_liumlsmybw24_b200 import dist as adist
-    from paper_conf_eurosys_liumlsmybw24_b200.api import Selection
 
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
-    # ACESO_BENCH_BACKEND=gloo (test only): several ranks sharing one GPU exercise the N > 1
-    # host path (shards, key vectors, max-over-ranks timing) where NCCL refuses duplicate GPUs
+    # ACESO_BENCH_BACKEND=gloo (test only): ranks sharing one GPU exercise the N > 1 host path;
+    # ACESO_BENCH_FORCE_DIST=1 (test only): a one-rank NCCL group, so the graph-captured
+    # key-vector all-reduce path runs on a single GPU
     backend = os.environ.get("ACESO_BENCH_BACKEND", "nccl")
+    force = os.environ.get("ACESO_BENCH_FORCE_DIST") == "1"
     local = local % torch.cuda.device_count() if backend != "nccl" else local
-    if world > 1:
-        torch.cuda.set_device(local)
+    use_dist = world > 1 or force
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    if use_dist:
         if backend == "nccl":
-            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+            dist.init_process_group("nccl", device_id=dev)
         else:
             dist.init_process_group(backend)
-    dev = torch.device("cuda", local)
-    torch.cuda.set_device(dev)
-
-    prof = P.WORKLOADS[args.config]()
-    L = prof.n_ops
-    n = args.batch
-    ctx = A.Context(prof, local)
-    global HINT
-    HINT = args.dist == "dense" and not args.no_hint
-    env_k = os.environ.get("ACESO_KERNEL")
-    dense_k = "per-op kernel" if os.environ.get("ACESO_DENSE_KERNEL") == "quad" else "dense kernel"
-    schedule = (f"{dense_k} (ACESO_HINT_DENSE)" if HINT else
-                "per-op kernel" if env_k == "quad" else
-                "dense kernel" if env_k == "dense" or (env_k != "events" and L <= 64) else "event kernel")
-
-    # distinct device-resident batches, rotating, together larger than L2
-    per_batch = A.tiled_bytes(n, L) + 8 * n
-    nbuf = max(2, int(np.ceil(1.3 * L2_BYTES / per_batch)))
-    host = []
-    dev_batches = []
-    for b in range(nbuf):
-        first = (b * world + rank) * n  # global indices of this rank's shard of batch b
-        codes, hdr = gen_batch(prof, args.dist, first, n, args.group, tiled=True)
-        host.append((codes, hdr, first))
-        dev_batches.append(A.upload_candidates(codes, hdr, local))
-    out = ctx.alloc_outputs(n)
-    sels = [ctx.alloc_select(n) for _ in range(nbuf)]
-    n_total = n * world
-    stream = torch.cuda.current_stream()
-
-    def step(s):
-        b = s % nbuf
-        codes_d, hdr_d = dev_batches[b]
-        gofs = rank * n
-        ctx.eval(codes_d, hdr_d, n=n, global_offset=gofs, n_total=n_total, summary=True, full=False,
-                 select=True, out=out, sel=sels[b], stream=stream, dense_hint=HINT)
-        if world > 1:
-            key = sels[b][0:8].view(torch.int64)
-            dist.all_reduce(key, op=dist.ReduceOp.MIN)
-
-    # warm-up
-    for s in range(args.warmup):
-        step(s)
-    torch.cuda.synchronize()
-
-    # The K timed steps are captured once into a CUDA graph (64K-candidate batches
-    # take microseconds; host launch overhead must not pace the GPU), then the
-    # graph is replayed once inside the timed region: exactly K steps.
-    # per-launch kernel times: external timing events captured as graph nodes
-    ev_s = [torch.cuda.Event(enable_timing=True, external=True) for _ in range(args.steps)]
-    ev_k = [torch.cuda.Event(enable_timing=True, external=True) for _ in range(args.steps)]
-    graph = torch.cuda.CUDAGraph()
-    if world > 1:
-        dist.barrier()
-    torch.cuda.synchronize()
-    nstr = max(1, min(args.streams, nbuf))
-    OVERLAP = nstr > 1 and not args.no_overlap_hint  # ACESO_HINT_OVERLAP: batches overlap on streams
-    outs = [out] + [ctx.alloc_outputs(n) for _ in range(nstr - 1)]
-    side = [torch.cuda.Stream() for _ in range(nstr)]
-    comm = torch.cuda.Stream()  # all-reduces in step order on one stream (same on every rank)
-    for si, st in enumerate(side):  # untimed warm-up of every side stream (per-stream state)
-        ctx.eval(dev_batches[si % nbuf][0], dev_batches[si % nbuf][1], n=n, global_offset=rank * n,
-                 n_total=n_total, summary=True, select=True, out=outs[si], sel=sels[si % nbuf], stream=st,
-                 dense_hint=HINT, overlap_hint=OVERLAP)
-    torch.cuda.synchronize()
-    keyvec = torch.empty(args.steps, dtype=torch.int64, device=dev)  # per-step global keys
-    kpa = max(1, args.keys_per_allreduce)
-    def issue_steps():
-        """The K steps on the side streams (+ all-reduces in step order on `comm`)."""
-        cs = torch.cuda.current_stream()
-        fork = torch.cuda.Event()
-        fork.record(cs)
-        for st in side + [comm]:
-            st.wait_event(fork)
-        comm_done = {}
-        for s in range(args.steps):
-            b = s % nbuf
-            st = side[s % nstr] if nstr > 1 else cs
-            codes_d, hdr_d = dev_batches[b]
-            if s - nbuf in comm_done:  # the select buffer's previous all-reduce has read it
-                st.wait_event(comm_done.pop(s - nbuf))
-            ev_s[s].record(st)
-            ctx.eval(codes_d, hdr_d, n=n, global_offset=rank * n, n_total=n_total, summary=True,
-                     select=True, out=outs[s % nstr], sel=sels[b], stream=st, dense_hint=HINT,
-                     overlap_hint=OVERLAP)
-            ev_k[s].record(st)
-            if world > 1:
-                # the step's packed key joins a vector of keys; one all-reduce MIN per
-                # `keys_per_allreduce` steps (SURVEY 8(e): 8*K bytes for K batches)
-                done = torch.cuda.Event()
-                done.record(st)
-                comm.wait_event(done)
-                with torch.cuda.stream(comm):
-                    keyvec[s:s + 1].copy_(sels[b][0:8].view(torch.int64))
-                    if (s + 1) % kpa == 0 or s == args.steps - 1:
-                        s0 = (s // kpa) * kpa
-                        dist.all_reduce(keyvec[s0:s + 1], op=dist.ReduceOp.MIN)
-                cd = torch.cuda.Event()
-                cd.record(comm)
-                comm_done[s] = cd
-        for st in side + [comm]:
-            j = torch.cuda.Event()
-            j.record(st)
-            cs.wait_event(j)
-
-    timing_mode = "graph"
-    try:
-        with torch.cuda.graph(graph):
-            issue_steps()
-        torch.cuda.synchronize()
-        graph.replay()  # one untimed replay (graph upload)
-        torch.cuda.synchronize()
-    except Exception as e:  # e.g. a collective that cannot be captured: time eager issue
-        timing_mode = f"eager ({type(e).__name__} during graph capture)"
-        print(f"[bench] graph capture failed ({e}); timing eagerly issued steps", file=sys.stderr)
-        torch.cuda.synchronize()
-        ev_s = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps)]
-        ev_k = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps)]
-        issue_steps()  # untimed pass
-        torch.cuda.synchronize()
-
-    clocks = ClockSampler(local)
-    t_start = torch.cuda.Event(enable_timing=True)
-    t_end = torch.cuda.Event(enable_timing=True)
-    if world > 1:
-        dist.barrier()
-    torch.cuda.synchronize()
-    clocks.start()
-    t_start.record(stream)
-    if timing_mode == "graph":
-        graph.replay()
-    else:
-        issue_steps()
-    t_end.record(stream)
-    torch.cuda.synchronize()
-    if world > 1:
-        dist.barrier()
-    clk = clocks.stop()
-    elapsed_ms = t_start.elapsed_time(t_end)
-    kern_ms = float(np.mean([ev_s[s].elapsed_time(ev_k[s]) for s in range(args.steps)]))
-    t = torch.tensor([elapsed_ms, kern_ms], dtype=torch.float64, device=dev)
-    if world > 1:
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-    elapsed_ms, kern_ms = float(t[0]), float(t[1])
-    ms_per_step = elapsed_ms / args.steps
-    value = n * world * args.steps / (elapsed_ms * 1e-3)
-
-    # per-launch kernel duration with launches serialized on one stream (roofline of
-    # the kernel alone; the timed region above overlaps independent batches)
-    ks = min(args.steps, 64)
-    evs = [torch.cuda.Event(enable_timing=True, external=True) for _ in range(ks)]
-    eve = [torch.cuda.Event(enable_timing=True, external=True) for _ in range(ks)]
-    g_ser = torch.cuda.CUDAGraph()
-    torch.cuda.synchronize()
-    with torch.cuda.graph(g_ser):
-        cs = torch.cuda.current_stream()
-        for s in range(ks):
-            b = s % nbuf
-            codes_d, hdr_d = dev_batches[b]
-            evs[s].record(cs)
-            ctx.eval(codes_d, hdr_d, n=n, global_offset=rank * n, n_total=n_total, summary=True,
-                     select=True, out=out, sel=sels[b], stream=cs, dense_hint=HINT)
-            eve[s].record(cs)
-    g_ser.replay()
-    torch.cuda.synchronize()
-    g_ser.replay()
-    torch.cuda.synchronize()
-    kern_ms_serial = float(np.mean([evs[s].elapsed_time(eve[s]) for s in range(ks)]))
-
-    # correctness of the timed result of the last step (global select over ranks)
-    last = (args.steps - 1) % nbuf
-    best = Selection.from_buffer(sels[last])
-    if world > 1:  # the global key of the last step (vector all-reduce); exact fallback if saturated
-        kl = int(keyvec[args.steps - 1].item())
-        gc, gcost, gidx, sat = A.decode_key(kl, n_total)
-        best = adist.global_select(sels[last], n_total) if sat else Selection(gc, gcost, gidx, kl)
-
-    # ---- end to end through the public API: host (pinned) -> device -> result -> host
+    dwd = world if use_dist else 1
+    hbm, src = peaks()
+    dd = dist if use_dist else None
+    prof, ctx, bt, rec = measure_workload(A, args.config, args, dev, hbm, src, dwd, rank, dd, with_extras=False)
+    # in the one-rank forced-dist test mode the key vector is still all-reduced (world = 1 math)
     e2e = None
     if not args.no_e2e:
-        pinned = [(torch.from_numpy(c).pin_memory(), torch.from_numpy(h.view(np.int64)).pin_memory())
-                  for c, h, _ in host[:2]]
-        dc = torch.empty(A.tiled_bytes(n, L), dtype=torch.uint8, device=dev)
-        dh = torch.empty(n, dtype=torch.int64, device=dev)
-        res_host = torch.empty(32, dtype=torch.uint8).pin_memory()
-        sel_e = ctx.alloc_select(n)
-        k_e2e = max(3, min(args.steps, 50))
-
-        def e2e_step(s):
-            c, h = pinned[s % 2]
-            dc.copy_(c, non_blocking=True)
-            dh.copy_(h, non_blocking=True)
-            ctx.eval(dc, dh, n=n, global_offset=rank * n, n_total=n_total, summary=True, select=True,
-                     out=out, sel=sel_e, stream=stream, dense_hint=HINT)
-            if world > 1:
-                dist.all_reduce(sel_e[0:8].view(torch.int64), op=dist.ReduceOp.MIN)
-            res_host.copy_(sel_e[:32], non_blocking=True)
-
-        for s in range(3):
-            e2e_step(s)
-        torch.cuda.synchronize()
-        if world > 1:
-            dist.barrier()
-        a = torch.cuda.Event(enable_timing=True)
-        z = torch.cuda.Event(enable_timing=True)
-        a.record(stream)
-        for s in range(k_e2e):
-            e2e_step(s)
-        z.record(stream)
-        torch.cuda.synchronize()
-        te = torch.tensor([a.elapsed_time(z)], dtype=torch.float64, device=dev)
-        if world > 1:
-            dist.all_reduce(te, op=dist.ReduceOp.MAX)
-        e2e = {"value": n * world * k_e2e / (float(te[0]) * 1e-3), "unit": "configs/s",
-               "h2d_bytes_per_step": int(A.tiled_bytes(n, L) + 8 * n), "d2h_bytes_per_step": 32,
-               "steps": k_e2e}
-
+        e2e = e2e_pipelined(A, ctx, bt, max(3, min(args.steps, 20)), rank, dwd,
+                            args.dist == "dense" and not args.no_hint, dd)
     if rank == 0:
-        hbm, src = peaks()
-        bpc = bytes_per_cand(L)
-        # effective per-launch interval in the timed region (one launch per step)
-        achieved = n * bpc / (ms_per_step * 1e-3) / 1e9
-        achieved_serial = n * bpc / (kern_ms_serial * 1e-3) / 1e9
-        traffic = None
-        try:
-            with open(os.path.join(ROOT, "profiles", "ncu_traffic.json")) as f:
-                tr = json.load(f)
-            key = f"{args.config}/{args.dist}/{n}"
-            if key in tr:
-                traffic = tr[key]
-        except Exception:
-            pass
         line = {
             "metric": "candidate configs evaluated/sec",
-            "value": value, "unit": "configs/s", "n_gpus": world, "steps": args.steps,
-            "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True,
+            "value": rec["value"], "unit": "configs/s", "n_gpus": dwd, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": rec["ms_per_step"], "higher_is_better": True,
             "scaling": "weak", "vs_baseline": None, "dtype": "u64", "data": "synthetic",
-            "config": {"workload": prof.name, "batch_per_gpu": n, "n_ops": L,
-                       "distribution": args.dist, "group_size": args.group, "schedule": schedule,
-                       "streams": nstr, "overlap_hint": OVERLAP,
-                       "l2": f"{nbuf} distinct device-resident batches rotated "
-                             f"({nbuf * per_batch / 2**20:.0f} MiB > 126 MiB L2)",
-                       "parallelism": f"dp{world} (candidate shards) + " + ("NCCL" if backend == "nccl" else backend + " (test backend)") + " all-reduce MIN"},
-            "roofline": {"bound": "hbm", "achieved": achieved, "peak": hbm, "unit": "GB/s",
-                         "frac": achieved / hbm, "traffic": traffic,
-                         "bytes_per_candidate": bpc, "bytes_per_launch": n * bpc,
-                         "launch_interval_ms": ms_per_step,
-                         "kernel_ms_concurrent": kern_ms,
-                         "kernel_ms_serial": kern_ms_serial,
-                         "achieved_serial": achieved_serial,
-                         "frac_serial": achieved_serial / hbm,
-                         "peak_source": src,
-                         "note": "achieved = algorithmic bytes per launch / effective launch "
-                                 "interval of the timed region (independent batches overlap "
-                                 "on streams); *_serial = same kernel launched back to back "
-                                 "on one stream"},
+            "config": {"workload": prof.name, "batch_per_gpu": rec["batch_per_gpu"], "n_ops": prof.n_ops,
+                       "global_batch_per_step": rec["batch_per_gpu"] * dwd,
+                       "distribution": rec["distribution"], "group_size": args.group,
+                       "schedule": rec["schedule"], "streams": rec["streams"], "overlap_hint": rec["overlap_hint"],
+                       "l2": rec["l2"],
+                       "parallelism": f"dp{dwd} (candidate shards) + " +
+                                      ("NCCL" if backend == "nccl" else backend + " (test backend)") +
+                                      " all-reduce MIN of packed keys"},
+            "roofline": rec["roofline"],
+            "kernel_ms_concurrent": rec["kernel_ms_concurrent"],
             "gpu_launches": args.steps,
-            "timing": (f"K steps captured in one CUDA graph ({nstr} streams, independent batches "
-                       f"round-robin), replayed once between CUDA events") if timing_mode == "graph" else
-                      (f"K steps issued eagerly ({nstr} streams) between CUDA events: {timing_mode}"),
-            "clocks": clk,
-            "result": {"cls": best.cls, "cost": best.cost, "index": best.index},
+            "timing": (f"K steps captured in one CUDA graph ({rec['streams']} streams, independent batches "
+                       f"round-robin), replayed once between CUDA events; max over ranks")
+            if rec["timing_mode"] == "graph" else f"K steps issued eagerly: {rec['timing_mode']}",
+            "clocks": rec["clocks"],
+            "result": rec["result"],
         }
         if e2e is not None:
             line["e2e"] = e2e
-        if not args.no_dedup:
-            line["dedup"] = measure_dedup(A, dev_batches, n, L, hbm)
-        if not args.no_incr:
-            line["incremental"] = measure_incr(A, ctx, prof, n, hbm)
-        if args.search_budget > 0 and world == 1:
-            from paper_conf_eurosys_liumlsmybw24_b200 import search as S
-            ev = S.GPUEvaluator(ctx)
-            res, st = S.search(prof, ev, budget_s=args.search_budget, patience=8)
-            init_best = None
-            for p in [1, 2, 4, 8, 16, 32, 64]:
-                r0 = S.initial_config(prof, p) if p <= prof.n_devices else None
-                if r0 is None:
+        if world == 1 and not force:
+            if not args.no_e2e:
+                line["e2e_descriptors"] = e2e_descriptors(A, ctx, prof, min(rec["batch_per_gpu"], 65536),
+                                                          max(3, min(args.steps, 20)))
+            if not args.no_cpu:
+                m = int(min(rec["batch_per_gpu"], max(2048, (1 << 28) // prof.n_ops)))
+                rc, rh = gen_batch(prof, args.dist, 0, m, args.group, tiled=False)
+                line["cpu_baseline"] = cpu_baseline(prof, rc, rh, target_core_s=20.0)
+            if not args.no_dedup:
+                line["dedup"] = measure_dedup(A, bt, hbm)
+            if args.search_budget > 0:
+                line["search"] = measure_search(A, ctx, prof, args.search_budget)
+            if not args.no_dp:
+                line["dp_baseline"] = measure_dp(A, ctx, prof, args.search_budget, line.get("search"))
+        del bt
+        ctx.close()
+        torch.cuda.empty_cache()
+        if world == 1 and not force and not args.no_all:
+            allw = {}
+            for name in ALL_WORKLOADS:
+                if name == args.config:
                     continue
-                o = ev.evaluate(r0[0][None, :], np.array([S.header(r0[1], p)], np.uint64))
-                pf = S.perf_of(int(o["info"][0]), o["iter"][0], o["max_mem"][0])
-                init_best = pf if init_best is None or pf < init_best else init_best
-            line["search"] = {
-                "time_s": st["time_s"], "time_to_best_s": st["time_to_best_s"],
-                "evaluated": st["evaluated"], "batches": st["batches"],
-                "improvements": st["improvements"],
-                "best": {"class": res.perf[0], "cost": res.perf[1], "iter_ns": res.iter_ns,
-                         "p": int((res.codes & 1).sum()), "mbs_log2": res.mbs},
-                "initial_best": {"class": init_best[0], "cost": init_best[1]},
-                "note": "batched Alg. 1/2 (MaxHops 7, beam 4) over all stage counts, stops "
-                        "after 8 hops without a new best or at the budget; context: the "
-                        "paper's searches use a 200 s budget (P:L313)"}
-        if not args.no_dp and world == 1:
-            from paper_conf_eurosys_liumlsmybw24_b200 import exhaustive as X
-            dp = X.exhaustive_best(prof, ctx)
-            dcodes, dhdr = dp.pop("codes", None), dp.pop("hdr", None)
-            dp["space"] = ("stage-uniform: p = 1, 2, 4, ... stages (all C(L-1, p-1) op-level cut sets "
-                           "up to 2^27 per p), G/p devices per stage with one (tp, dp), recompute all "
-                           "or none, every valid microbatch")
-            if "search" in line:
-                sb = line["search"]["best"]
-                dp["search_vs_exhaustive"] = {
-                    "search_best": [sb["class"], sb["cost"]], "exhaustive_best":
-                    [dp["best"]["class"], dp["best"]["cost"]] if dp["best"] else None,
-                    "search_explored": line["search"]["evaluated"]}
-                if dcodes is not None:  # hybrid: the search also starts from the exhaustive optimum
-                    hres, hst = S.search(prof, S.GPUEvaluator(ctx), budget_s=args.search_budget, patience=8,
-                                         starts=[(dcodes, int(dhdr & np.uint64(0xFF)))])
-                    dp["search_vs_exhaustive"]["hybrid_best"] = [hres.perf[0], hres.perf[1]]
-                    dp["search_vs_exhaustive"]["hybrid_time_s"] = hst["time_s"] + dp["time_s"]
-            dp["note"] = ("SURVEY 8(f) NEXT(4), Exp#4 (P:L343-357): the paper's DP baseline explores "
-                          "1e7-4.3e7 configurations of a pruned space; here the pruned stage-uniform "
-                          "space is enumerated and evaluated exhaustively on the device (its exact optimum); "
-                          "the search's space is larger (non-uniform stages, per-op tp/dp and recompute)")
-            line["dp_baseline"] = dp
-        if not args.no_cpu and world == 1:
-            import aceso_inputs as ai  # noqa: F811
-            rowm = []
-            need = 0
-            for c, h, first in host:
-                if need >= 2 * 65536:
-                    break
-                cr, hr = gen_batch(prof, args.dist, first, n, args.group, tiled=False)
-                rowm.append((cr, hr))
-                need += n
-            line["cpu_baseline"] = cpu_baseline(prof, rowm, 2 * 65536)
+                _, c2, b2, r2 = measure_workload(A, name, args, dev, hbm, src, steps=args.all_steps)
+                allw[name] = r2
+                del b2
+                c2.close()
+                torch.cuda.empty_cache()
+            line["all_workloads"] = allw
         print(json.dumps(line), flush=True)
-    if world > 1:
+    if use_dist:
         dist.destroy_process_group()
     return 0
 

@@ -86,12 +86,13 @@ typedef struct aceso_ctx aceso_ctx; /* opaque; owned by the library */
  * context. Synchronous. Range rules (ACESO_ERANGE on violation):
  *  - time fields (ns) and dps in [0, 2^32); memory fields (act, keep, peak) and
  *    each wmem entry in [0, 2^40];  keep <= act;
- *  - fwd_comp+fwd_comm+bwd_comp+bwd_comm + (fwd_comp+fwd_comm) < 2^32;
- *  - memory is packed exactly in units of 2^m bytes, m = the largest power of two
- *    (<= 16) dividing every memory value; act, peak + act - keep and
- *    param+optimizer bytes must each be < 2^(32+m);
  *  - model-wide: a conservative bound on every iteration time and stage memory
  *    (L * max per-op cost * (Bg + 1)) is < 2^62, so packed keys are exact.
+ * Every profile within these rules is evaluated exactly. Schedules: the event,
+ * dense and per-op kernels hold per-op values in 32-bit fields (memory in units
+ * of 2^m bytes, m = the largest power of two <= 16 dividing every memory value;
+ * a recomputed op's time 2(fwd) + bwd < 2^32 ns); a profile outside those
+ * fields is served by the scan kernel (exact 64-bit tables) for every call.
  * Returns ACESO_OK and sets *out, or a negative status (see aceso_last_error). */
 int aceso_load_profile(const aceso_profile_desc *desc, int cuda_device, aceso_ctx **out);
 
@@ -225,15 +226,20 @@ size_t aceso_select_buf_bytes(const aceso_ctx *ctx, int64_t n);
  *             stage heads and tp/dp changes and takes run sums from position-prefix
  *             tables; the dense kernel (default for n_ops <= 64, and with
  *             ACESO_HINT_DENSE) accumulates every op branch-free under its own record;
- *             the per-op kernel accumulates every op with quad-signature sums. The
- *             dense and per-op kernels stage their tables in shared memory, so for
- *             profiles whose tables exceed ~200 KB only the event kernel is used (the
- *             hint is then ignored). Environment variables read by aceso_load_profile
- *             (measurement and test knobs; results never change):
- *             ACESO_KERNEL=quad|events|dense (default schedule), ACESO_DENSE_KERNEL=quad
- *             (schedule of the dense hint), ACESO_SPLIT=2 (per-op kernel: warp pair per
- *             tile), ACESO_MINB=2|3 (register target: resident CTAs per SM),
- *             ACESO_TILES_PER_WARP=k (event kernel: tiles per warp per launch).
+ *             the per-op kernel accumulates every op with quad-signature sums; the
+ *             scan kernel streams each warp's tiles as one contiguous range and walks
+ *             the dirty chunks (heads, tp/dp changes, recompute flags) with exact
+ *             64-bit prefix tables (the schedule for profiles outside the packed
+ *             fields, see aceso_load_profile). The dense and per-op kernels stage
+ *             their tables in shared memory, so for profiles whose tables exceed
+ *             ~200 KB the event (or scan) kernel serves the hint too. Environment
+ *             variables read by aceso_load_profile (measurement and test knobs;
+ *             results never change): ACESO_KERNEL=quad|events|dense|scan (default
+ *             schedule), ACESO_DENSE_KERNEL=quad (schedule of the dense hint),
+ *             ACESO_SPLIT=2 (per-op kernel: warp pair per tile), ACESO_MINB=2|3
+ *             (register target: resident CTAs per SM), ACESO_TILES_PER_WARP=k
+ *             (event / scan kernel: tiles per warp per launch), ACESO_SCAN_NORESOLVE=1
+ *             (scan kernel: recompute-only chunks resolved in the per-lane walk).
  *   out     : host struct of device pointers (may be null if no OUT_* flag)
  *   d_sel   : select buffer (device), required with ACESO_FUSED_SELECT
  *   stream  : cudaStream_t
@@ -243,6 +249,11 @@ size_t aceso_select_buf_bytes(const aceso_ctx *ctx, int64_t n);
 int aceso_eval(aceso_ctx *ctx, const uint8_t *d_codes, const uint64_t *d_hdr, int64_t n,
                int64_t global_offset, int64_t n_total, uint32_t flags,
                const aceso_eval_out *out, void *d_sel, void *stream);
+
+/* Name of the kernel aceso_eval runs for `flags` on this context ("event kernel",
+ * "dense kernel", "per-op kernel" or "scan kernel"; "" for a null context). Static
+ * string, owned by the library. Host only. */
+const char *aceso_schedule_name(const aceso_ctx *ctx, uint32_t flags);
 
 /* Argmin over an already written summary (iter_ns, max_mem, info) of n
  * candidates; same order and result layout as the fused select. Async. */
@@ -296,21 +307,6 @@ typedef struct {
 int aceso_expand(const uint8_t *d_bases, const uint16_t *d_ranks, int32_t n_bases, int32_t n_ops,
                  const aceso_cand *d_cands, int64_t n, uint8_t *d_tiled, uint64_t *d_hdr,
                  void *stream);
-
-/* Incremental evaluation ("re-reduce only the touched
- * stages"): same outputs, flags and select semantics as aceso_eval for the
- * candidates of aceso_expand, without expanding them. d_base_hdr: [n_bases]
- * headers of the bases. The bases are evaluated once into d_work (per-stage
- * sums, an op -> stage map); each candidate then re-walks only the ops of the
- * stages its patch ranges [a-1, b) touch and takes every other stage from the
- * cache. Candidates whose microbatch or stage count differ from their base's,
- * or whose base is invalid or has more than 64 stages, are walked over all ops.
- * ACESO_HINT_DENSE is ignored. Two launches on `stream`. */
-size_t aceso_incr_work_bytes(const aceso_ctx *ctx, int32_t n_bases);
-int aceso_eval_incr(aceso_ctx *ctx, const uint8_t *d_bases, const uint64_t *d_base_hdr,
-                    const uint16_t *d_ranks, int32_t n_bases, const aceso_cand *d_cands, int64_t n,
-                    int64_t global_offset, int64_t n_total, uint32_t flags,
-                    const aceso_eval_out *out, void *d_sel, void *d_work, void *stream);
 
 /* ------------------------------------------------------------------------- */
 /* Exhaustive stage-partition enumeration (the Exp#4     */

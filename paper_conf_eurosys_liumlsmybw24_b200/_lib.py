@@ -14,8 +14,8 @@ INFO_INVALID = 1 << 17
 
 SYMBOLS = ["aceso_load_profile", "aceso_free", "aceso_tiled_bytes", "aceso_pack_rowmajor",
            "aceso_select_buf_bytes", "aceso_eval", "aceso_select", "aceso_decode_key",
-           "aceso_last_error", "aceso_version", "aceso_hash", "aceso_visited_bytes", "aceso_dedup", "aceso_expand", "aceso_incr_work_bytes", "aceso_eval_incr",
-           "aceso_enum_cuts_count", "aceso_enum_cuts"]
+           "aceso_last_error", "aceso_version", "aceso_hash", "aceso_visited_bytes", "aceso_dedup", "aceso_expand",
+           "aceso_enum_cuts_count", "aceso_enum_cuts", "aceso_schedule_name"]
 
 
 class ProfileDesc(ctypes.Structure):
@@ -66,6 +66,8 @@ def load():
     lib.aceso_last_error.restype = ctypes.c_char_p
     lib.aceso_version.argtypes = []
     lib.aceso_version.restype = ctypes.c_char_p
+    lib.aceso_schedule_name.argtypes = [P, c_u32]
+    lib.aceso_schedule_name.restype = ctypes.c_char_p
     lib.aceso_hash.argtypes = [P, P, c_i64, c_i32, P, P]
     lib.aceso_hash.restype = ctypes.c_int
     lib.aceso_visited_bytes.argtypes = [c_i64]
@@ -78,10 +80,5 @@ def load():
     lib.aceso_enum_cuts_count.restype = c_i64
     lib.aceso_enum_cuts.argtypes = [c_i32, c_i32, ctypes.c_uint8, ctypes.c_uint64, c_i64, c_i64, P, P, P]
     lib.aceso_enum_cuts.restype = ctypes.c_int
-    lib.aceso_incr_work_bytes.argtypes = [P, c_i32]
-    lib.aceso_incr_work_bytes.restype = c_sz
-    lib.aceso_eval_incr.argtypes = [P, P, P, P, c_i32, P, c_i64, c_i64, c_i64, c_u32, ctypes.POINTER(EvalOut),
-                                    P, P, P]
-    lib.aceso_eval_incr.restype = ctypes.c_int
     _lib = lib
     return lib

@@ -125,6 +125,10 @@ class Context:
         except Exception:
             pass
 
+    def schedule(self, dense_hint: bool = False) -> str:
+        """aceso_schedule_name: the kernel aceso_eval runs on this context."""
+        return L.load().aceso_schedule_name(self._h, L.HINT_DENSE if dense_hint else 0).decode()
+
     # -- buffers --------------------------------------------------------------
     def alloc_outputs(self, n: int, full: bool = False) -> Outputs:
         d = self._dev
@@ -200,30 +204,6 @@ class Context:
                                      self.n_ops, _ptr(cands), n, _ptr(tiled), _ptr(hdr), _stream(stream)),
                "aceso_expand")
         return tiled, hdr[:n]
-
-    def eval_incr(self, bases: torch.Tensor, base_hdr: torch.Tensor, cands: torch.Tensor,
-                  ranks: torch.Tensor | None = None, n: int | None = None, global_offset: int = 0,
-                  n_total: int | None = None, summary: bool = True, full: bool = False, select: bool = True,
-                  out: Outputs | None = None, sel: torch.Tensor | None = None, work: torch.Tensor | None = None,
-                  stream=None):
-        """aceso_eval_incr: candidates as base + patches (uint8 view of aceso_cand rows), evaluated
-        incrementally against per-base stage caches. Returns (out, sel) like eval()."""
-        n = int(cands.numel() // 56) if n is None else int(n)
-        nb = int(bases.shape[0])
-        n_total = global_offset + n if n_total is None else int(n_total)
-        flags = (L.OUT_SUMMARY if summary else 0) | (L.OUT_FULL if full else 0) | (L.FUSED_SELECT if select else 0)
-        if (summary or full) and out is None:
-            out = self.alloc_outputs(n, full=full)
-        if select and sel is None:
-            sel = self.alloc_select(n)
-        if work is None:
-            work = torch.empty(int(L.load().aceso_incr_work_bytes(self._h, nb)), dtype=torch.uint8, device=self._dev)
-        cs = out.c_struct() if out is not None else None
-        _check(L.load().aceso_eval_incr(self._h, _ptr(bases), _ptr(base_hdr), _ptr(ranks) if ranks is not None else None,
-                                        nb, _ptr(cands), n, int(global_offset), n_total, flags,
-                                        ctypes.byref(cs) if cs is not None else None, _ptr(sel), _ptr(work),
-                                        _stream(stream)), "aceso_eval_incr")
-        return out, sel
 
     def select(self, out: Outputs, n: int | None = None, global_offset: int = 0,
                n_total: int | None = None, sel: torch.Tensor | None = None, stream=None):

@@ -18,11 +18,11 @@
 #include "common.cuh"
 #include "dedup_kernels.cuh"
 #include "expand_kernel.cuh"
-#include "incr_kernel.cuh"
 #include "eval_kernel.cuh"
 #include "event_kernel.cuh"
 #include "dense_kernel.cuh"
 #include "enum_kernel.cuh"
+#include "scan_kernel.cuh"
 
 using namespace aceso;
 
@@ -94,9 +94,30 @@ void *dense_kernel_for(uint32_t mode) {
   }
 }
 
+template <bool E64, int B>
+void *scan_kernel_for(uint32_t mode) {
+  switch (mode) {
+    case 1: return reinterpret_cast<void *>(&scan_kernel<1, E64, B>);
+    case 2: return reinterpret_cast<void *>(&scan_kernel<2, E64, B>);
+    case 3: return reinterpret_cast<void *>(&scan_kernel<3, E64, B>);
+    case 4: return reinterpret_cast<void *>(&scan_kernel<4, E64, B>);
+    case 5: return reinterpret_cast<void *>(&scan_kernel<5, E64, B>);
+    case 6: return reinterpret_cast<void *>(&scan_kernel<6, E64, B>);
+    case 7: return reinterpret_cast<void *>(&scan_kernel<7, E64, B>);
+    default: return nullptr;
+  }
+}
+
 // kernel 0: per-op/quad kernel (eval_kernel.cuh); kernel 1: event kernel (event_kernel.cuh);
-// kernel 2: dense kernel (dense_kernel.cuh, ACESO_HINT_DENSE)
-void *eval_kernel_for(uint32_t mode, int split, int minb, int kernel) {
+// kernel 2: dense kernel (dense_kernel.cuh, ACESO_HINT_DENSE); kernel 3: scan kernel
+// (scan_kernel.cuh, exact u64 tables; e64: wide transient-memory table)
+void *eval_kernel_for(uint32_t mode, int split, int minb, int kernel, int e64 = 0) {
+  if (kernel == 3) {
+    // the scan kernel's default register target is 2 CTAs per SM (its ring and lists take
+    // ~100 KB of shared memory per CTA); ACESO_MINB=3 selects the 80-register build
+    if (minb == 3 && getenv("ACESO_MINB")) return e64 ? scan_kernel_for<true, 3>(mode) : scan_kernel_for<false, 3>(mode);
+    return e64 ? scan_kernel_for<true, 2>(mode) : scan_kernel_for<false, 2>(mode);
+  }
   if (kernel == 1) return minb == 2 ? event_kernel_for<2>(mode) : event_kernel_for<3>(mode);
   if (kernel == 2) return minb == 2 ? dense_kernel_for<2>(mode) : dense_kernel_for<3>(mode);
   if (minb == 2) return split == 2 ? eval_kernel_split<2, 2>(mode) : eval_kernel_split<1, 2>(mode);
@@ -129,15 +150,21 @@ struct aceso_ctx {
   int split;        // warps per tile (1 or 2)
   int minb;         // register target: 2 or 3 resident CTAs per SM
   int tiles_per_warp;  // ACESO_TILES_PER_WARP (measurement knob): tiles each warp walks per launch (default 1)
-  int max_ctas[3][8];  // per kernel and mode: resident CTAs (occupancy x SMs)
+  int max_ctas[4][8];  // per kernel and mode: resident CTAs (occupancy x SMs)
   int dense_kernel;    // schedule of ACESO_HINT_DENSE: 2 dense kernel (default), 0 per-op kernel (ACESO_DENSE_KERNEL=quad)
-  size_t smem[3][8];
+  size_t smem[4][8];
+  int packed_ok;       // memory values fit the 32-bit packed tables of kernels 0-2 (else: scan kernel only)
+  void *d_sc;          // scan-kernel tables
+  const uint4 *sx, *sk, *sq;
+  const uint64_t *sd;
+  const void *ss;
+  const uint32_t *sqo;
+  uint32_t qo_words, es;
+  int e64;             // scan kernel: transient-memory table in u64 (values >= 2^32 units)
+  uint32_t sc_resolve; // scan kernel: resolve recompute-only chunks in the compacted pass (ACESO_SCAN_NORESOLVE=1: in the walk)
 };
 
 namespace {
-template <uint32_t M>
-void *incr_kernel_ptr() { return reinterpret_cast<void *>(&incr_kernel<M>); }
-
 // kernel parameter block of a call (tables, outputs, selection); codes/hdr set by the caller
 EvalParams make_params(const aceso_ctx *ctx, int64_t n, int64_t global_offset, int64_t n_total,
                        const aceso_eval_out *out, void *d_sel) {
@@ -180,6 +207,15 @@ EvalParams make_params(const aceso_ctx *ctx, int64_t n, int64_t global_offset, i
   P.qo_bytes = ctx->qo_bytes;
   P.qo_off = ctx->qo_off;
   P.evblob = reinterpret_cast<const unsigned char *>(ctx->d_ev);
+  P.sx = ctx->sx;
+  P.sk = ctx->sk;
+  P.sd = ctx->sd;
+  P.ss = ctx->ss;
+  P.sq = ctx->sq;
+  P.sqo = ctx->sqo;
+  P.qo_words = ctx->qo_words;
+  P.es = ctx->es;
+  P.sc_resolve = ctx->sc_resolve;
   return P;
 }
 }  // namespace
@@ -227,7 +263,6 @@ int aceso_load_profile(const aceso_profile_desc *d, int cuda_device, aceso_ctx *
         if (keep > act) return fail(ACESO_ERANGE, "keep > act at rec[%d][%d][%d]", t, tp, b);
         uint64_t s1 = 2 * (fc + fm) + bc + bm;
         uint64_t e1 = peak + act - keep;
-        if (s1 > U32) return fail(ACESO_ERANGE, "recomputed op time > 2^32-1 at rec[%d][%d][%d]", t, tp, b);
         maxSop = std::max(maxSop, s1);
         maxRes = std::max(maxRes, (uint64_t)R(t, tp, b, 7));
         maxP2P = std::max(maxP2P, (uint64_t)std::max(R(t, tp, b, 8), R(t, tp, b, 9)));
@@ -253,10 +288,10 @@ int aceso_load_profile(const aceso_profile_desc *d, int cuda_device, aceso_ctx *
         tz(d->wmem[((int64_t)t * NT + tp) * 2]);
         tz(d->wmem[((int64_t)t * NT + tp) * 2 + 1]);
       }
-    if ((maxA >> ms) > U32) return fail(ACESO_ERANGE, "act exceeds 2^32 units of 2^%u bytes", ms);
-    if ((maxE >> ms) > U32) return fail(ACESO_ERANGE, "peak + act - keep exceeds 2^32 units of 2^%u bytes", ms);
-    if ((maxW >> ms) > U32) return fail(ACESO_ERANGE, "param+optimizer bytes exceed 2^32 units of 2^%u bytes", ms);
   }
+  // the packed kernels (per-op, event v2, dense) hold per-op values in 32-bit fields: memory in
+  // units of 2^ms bytes, recomputed op times in ns; the scan kernel is exact for every profile
+  const bool packed_ok = (maxA >> ms) <= U32 && (maxE >> ms) <= U32 && (maxW >> ms) <= U32 && maxSop <= U32;
   {
     // model-wide bounds: every iteration time / stage memory < 2^62 (exact keys)
     typedef unsigned __int128 u128;
@@ -519,6 +554,120 @@ int aceso_load_profile(const aceso_profile_desc *d, int cuda_device, aceso_ctx *
     for (int q = 0; q < nq; ++q) put32(ev_qo + (size_t)q * 4, eqo[q]);
   }
 
+  // ---- scan-kernel tables (scan_kernel.cuh): exact u64 prefixes, no packing ----
+  // transient-memory values (peak, peak + act - keep) in units of 2^es bytes: u32 when every
+  // value fits, else u64 (es = 0)
+  uint32_t es = 16;
+  uint64_t emax = 0;
+  for (int t = 0; t < T; ++t)
+    for (int tp = 0; tp < NT; ++tp)
+      for (int b = 0; b < NB; ++b) {
+        for (int f : {ACESO_F_ACT, ACESO_F_KEEP, ACESO_F_PEAK})
+          if (R(t, tp, b, f) != 0) es = std::min<uint32_t>(es, (uint32_t)__builtin_ctzll((uint64_t)R(t, tp, b, f)));
+        emax = std::max(emax, (uint64_t)R(t, tp, b, ACESO_F_PEAK) + R(t, tp, b, ACESO_F_ACT) - R(t, tp, b, ACESO_F_KEEP));
+      }
+  const bool e64 = (emax >> es) > U32;
+  if (e64) es = 0;
+  const size_t ew = e64 ? 8 : 4;
+  const int nqs = 4 * nch;  // quads incl. the zero-padded tail (4 per chunk)
+  std::vector<uint32_t> sqo(nqs, 0u);
+  std::vector<std::array<int, 4>> ssig;
+  {
+    std::map<std::array<int, 4>, int> seen;
+    for (int q = 0; q < nqs; ++q) {
+      if (4 * q >= L) continue;  // pad quads carry no recompute flags
+      std::array<int, 4> key;
+      for (int k = 0; k < 4; ++k) key[k] = 4 * q + k < L ? (int)d->op_type[4 * q + k] : -1;
+      auto it = seen.find(key);
+      if (it == seen.end()) {
+        it = seen.emplace(key, (int)ssig.size()).first;
+        ssig.push_back(key);
+      }
+      sqo[q] = (uint32_t)it->second * RUNS * 16u;
+    }
+  }
+  const size_t sc_sx = 0;
+  const size_t sc_sk = al(sc_sx + (size_t)RUNS * Lp1 * 32);
+  const size_t sc_sd = al(sc_sk + (size_t)RUNS * Lp1 * 16);
+  const size_t sc_ss = al(sc_sd + (size_t)NT * ND * Lp1 * 8);
+  const size_t sc_sq = al(sc_ss + (size_t)levels * RUNS * L * ew);
+  const size_t sc_qo = al(sc_sq + ssig.size() * RUNS * 16 * 32);
+  const size_t sc_bytes = al(sc_qo + (size_t)nqs * 4);
+  std::vector<unsigned char> sc(sc_bytes, 0);
+  {
+    auto put64 = [&](size_t off, uint64_t v) { memcpy(&sc[off], &v, 8); };
+    auto put32 = [&](size_t off, uint32_t v) { memcpy(&sc[off], &v, 4); };
+    auto pute = [&](size_t idx, uint64_t v) {
+      if (e64) put64(sc_ss + idx * 8, v);
+      else put32(sc_ss + idx * 4, (uint32_t)v);
+    };
+    auto gete = [&](size_t idx) -> uint64_t {
+      if (e64) { uint64_t v; memcpy(&v, &sc[sc_ss + idx * 8], 8); return v; }
+      uint32_t v; memcpy(&v, &sc[sc_ss + idx * 4], 4); return v;
+    };
+    auto Wof = [&](int t, int tp) -> uint64_t {
+      return (uint64_t)d->wmem[((int64_t)t * NT + tp) * 2] + (uint64_t)d->wmem[((int64_t)t * NT + tp) * 2 + 1];
+    };
+    for (int b = 0; b < NB; ++b)
+      for (int tp = 0; tp < NT; ++tp) {
+        const uint32_t rr = (uint32_t)(b * NT + tp);
+        uint64_t PS = 0, PA = 0, PW = 0, PC = 0;
+        for (uint32_t j = 0; j <= (uint32_t)L; ++j) {
+          const size_t o = (size_t)rr * Lp1 + j;
+          put64(sc_sx + o * 32, PS);
+          put64(sc_sx + o * 32 + 8, PA);
+          put64(sc_sx + o * 32 + 16, PW);
+          put64(sc_sx + o * 32 + 24, PC);
+          if (j < (uint32_t)L) {
+            const int t = d->op_type[j];
+            PS += (uint64_t)R(t, tp, b, ACESO_F_FWD_COMP) + R(t, tp, b, ACESO_F_FWD_COMM) +
+                  R(t, tp, b, ACESO_F_BWD_COMP) + R(t, tp, b, ACESO_F_BWD_COMM);
+            PA += (uint64_t)R(t, tp, b, ACESO_F_ACT);
+            PW += Wof(t, tp);
+            PC += (uint64_t)R(t, tp, b, ACESO_F_FWD_COMP) + R(t, tp, b, ACESO_F_BWD_COMP);
+            put32(sc_sk + o * 16, (uint32_t)R(t, tp, b, ACESO_F_RESHARD));
+            put32(sc_sk + o * 16 + 4, (uint32_t)R(t, tp, b, ACESO_F_P2P_BWD));
+            pute((size_t)rr * L + j, (uint64_t)R(t, tp, b, ACESO_F_PEAK) >> es);
+          }
+          if (j > 0) put32(sc_sk + o * 16 + 8, (uint32_t)R(d->op_type[j - 1], tp, b, ACESO_F_P2P_FWD));
+        }
+        for (int k = 1; k < levels; ++k)
+          for (int j = 0; j < L; ++j) {
+            const int j2 = std::min(j + (1 << (k - 1)), L - 1);
+            const uint64_t v1 = gete(((size_t)(k - 1) * RUNS + rr) * L + j);
+            const uint64_t v2 = gete(((size_t)(k - 1) * RUNS + rr) * L + j2);
+            pute(((size_t)k * RUNS + rr) * L + j, std::max(v1, v2));
+          }
+        for (size_t sg = 0; sg < ssig.size(); ++sg)
+          for (uint32_t m = 1; m < 16; ++m) {
+            uint64_t dS = 0, dA = 0, dC = 0, E1 = 0;
+            for (int k = 0; k < 4; ++k) {
+              const int t = ssig[sg][k];
+              if (t < 0 || !((m >> k) & 1u)) continue;
+              dS += (uint64_t)R(t, tp, b, ACESO_F_FWD_COMP) + R(t, tp, b, ACESO_F_FWD_COMM);
+              dA += (uint64_t)(R(t, tp, b, ACESO_F_ACT) - R(t, tp, b, ACESO_F_KEEP));
+              dC += (uint64_t)R(t, tp, b, ACESO_F_FWD_COMP);
+              E1 = std::max(E1, ((uint64_t)R(t, tp, b, ACESO_F_PEAK) + R(t, tp, b, ACESO_F_ACT) -
+                                 R(t, tp, b, ACESO_F_KEEP)) >> es);
+            }
+            const size_t o = sc_sq + (((size_t)sg * RUNS + rr) * 16 + m) * 32;
+            put64(o, dS);
+            put64(o + 8, dA);
+            put64(o + 16, E1);
+            put64(o + 24, dC);
+          }
+      }
+    for (int tp = 0; tp < NT; ++tp)
+      for (int dp = 0; dp < ND; ++dp) {
+        uint64_t acc = 0;
+        for (uint32_t j = 0; j <= (uint32_t)L; ++j) {
+          put64(sc_sd + (((size_t)tp * ND + dp) * Lp1 + j) * 8, acc);
+          if (j < (uint32_t)L) acc += dps_of(d->op_type[j], tp, dp);
+        }
+      }
+    for (int q = 0; q < nqs; ++q) put32(sc_qo + (size_t)q * 4, sqo[q]);
+  }
+
   // ---- device ----
   int ndev = 0;
   if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev == 0) return fail(ACESO_ENODEV, "no CUDA device");
@@ -542,15 +691,22 @@ int aceso_load_profile(const aceso_profile_desc *d, int cuda_device, aceso_ctx *
   ctx->mem_shift = ms;
   ctx->d_blob = nullptr;
   ctx->d_ev = nullptr;
-  ctx->quad_ok = quad_ok ? 1 : 0;
-  // short models: per-tile event overheads outweigh the per-op work; the dense kernel's
-  // branch-free per-op accumulation beats the per-op kernel there (toy-A 25.1 vs 21.4, toy-B
-  // 20.1 vs 16.4 G configs/s, search-shaped)
-  ctx->kernel = L > 64 ? 1 : dense_ok ? 2 : quad_ok ? 0 : 1;
+  ctx->packed_ok = packed_ok ? 1 : 0;
+  ctx->quad_ok = (quad_ok && packed_ok) ? 1 : 0;
+  ctx->d_sc = nullptr;
+  ctx->es = es;
+  ctx->e64 = e64 ? 1 : 0;
+  ctx->qo_words = (uint32_t)nqs;
+  ctx->sc_resolve = getenv("ACESO_SCAN_NORESOLVE") ? 0u : 1u;
+  // default schedule: the event kernel (its packed tables hold the profile), for short models
+  // (<= 64 ops) the dense kernel's branch-free per-op accumulation; the scan kernel (exact
+  // 64-bit tables) for profiles whose per-op values exceed the packed 32-bit fields
+  ctx->kernel = !packed_ok ? 3 : (L <= 64 && dense_ok) ? 2 : 1;
   if (const char *env = getenv("ACESO_KERNEL")) {
-    if (!strcmp(env, "quad") && quad_ok) ctx->kernel = 0;
-    else if (!strcmp(env, "events")) ctx->kernel = 1;
-    else if (!strcmp(env, "dense")) ctx->kernel = 2;  // validated against dense_ok below
+    if (!strcmp(env, "quad") && quad_ok && packed_ok) ctx->kernel = 0;
+    else if (!strcmp(env, "events") && packed_ok) ctx->kernel = 1;
+    else if (!strcmp(env, "dense") && packed_ok) ctx->kernel = 2;  // validated against dense_ok below
+    else if (!strcmp(env, "scan")) ctx->kernel = 3;
   }
   ctx->qo_off = (uint32_t)ev_qo;
   ctx->qo_bytes = qo_bytes;
@@ -562,6 +718,8 @@ int aceso_load_profile(const aceso_profile_desc *d, int cuda_device, aceso_ctx *
     if (e == cudaSuccess) e = cudaMemcpyAsync(ctx->d_blob, blob.data(), blob_bytes, cudaMemcpyHostToDevice, st);
     if (e == cudaSuccess) e = cudaMalloc(&ctx->d_ev, ev_bytes);
     if (e == cudaSuccess) e = cudaMemcpyAsync(ctx->d_ev, ev.data(), ev_bytes, cudaMemcpyHostToDevice, st);
+    if (e == cudaSuccess) e = cudaMalloc(&ctx->d_sc, sc_bytes);
+    if (e == cudaSuccess) e = cudaMemcpyAsync(ctx->d_sc, sc.data(), sc_bytes, cudaMemcpyHostToDevice, st);
     if (e == cudaSuccess) e = cudaStreamSynchronize(st);
     cudaStreamDestroy(st);
     if (e != cudaSuccess) { rc = fail(e == cudaErrorMemoryAllocation ? ACESO_ENOMEM : ACESO_ECUDA, "upload: %s", cudaGetErrorString(e)); break; }
@@ -588,25 +746,35 @@ int aceso_load_profile(const aceso_profile_desc *d, int cuda_device, aceso_ctx *
       ctx->pd = reinterpret_cast<const uint64_t *>(eb + ev_pd);
       ctx->st = reinterpret_cast<const uint32_t *>(eb + ev_st);
       ctx->qr = reinterpret_cast<const uint4 *>(eb + ev_qr);
+      const unsigned char *cb = reinterpret_cast<const unsigned char *>(ctx->d_sc);
+      ctx->sx = reinterpret_cast<const uint4 *>(cb + sc_sx);
+      ctx->sk = reinterpret_cast<const uint4 *>(cb + sc_sk);
+      ctx->sd = reinterpret_cast<const uint64_t *>(cb + sc_sd);
+      ctx->ss = reinterpret_cast<const void *>(cb + sc_ss);
+      ctx->sq = reinterpret_cast<const uint4 *>(cb + sc_sq);
+      ctx->sqo = reinterpret_cast<const uint32_t *>(cb + sc_qo);
     }
-    ctx->dense_kernel = dense_ok ? 2 : 0;  // its tables must fit in shared memory
-    if (ctx->kernel == 2 && !dense_ok) ctx->kernel = (L > 64 || !quad_ok) ? 1 : 0;  // ACESO_KERNEL=dense
+    // ACESO_HINT_DENSE: the dense kernel when its tables fit shared memory and the profile fits
+    // its packed fields, else the scan kernel
+    ctx->dense_kernel = (dense_ok && packed_ok) ? 2 : ctx->quad_ok ? 0 : 3;
+    if (ctx->kernel == 2 && !dense_ok) ctx->kernel = packed_ok ? 1 : 3;  // ACESO_KERNEL=dense
     if (const char *env = getenv("ACESO_DENSE_KERNEL"))
-      if (!strcmp(env, "quad")) ctx->dense_kernel = 0;
-    for (int kern = 0; kern < 3 && rc == ACESO_OK; ++kern)
+      if (!strcmp(env, "quad") && ctx->quad_ok) ctx->dense_kernel = 0;
+    for (int kern = 0; kern < 4 && rc == ACESO_OK; ++kern)
       for (uint32_t mode = 1; mode < 8; ++mode) {
-        if ((kern == 0 && !quad_ok) || (kern == 2 && !dense_ok)) {
+        if ((kern == 0 && !ctx->quad_ok) || (kern == 2 && !(dense_ok && packed_ok)) || (kern == 1 && !packed_ok)) {
           ctx->smem[kern][mode] = 0;
           ctx->max_ctas[kern][mode] = 0;
           continue;
         }
         const size_t tabs = ((mode & ACESO_OUT_FULL) ? tab.bytes_full : tab.bytes) + (tab.k_smem ? bytesK : 0u);
         const size_t smem =
-            kern == 1   ? (size_t)qo_bytes + ev_ring_bytes() + ev_list_bytes((mode & ACESO_OUT_FULL) != 0)
+            kern == 3   ? (size_t)sc_smem_bytes((uint32_t)(nqs * 4 + 15) & ~15u)
+            : kern == 1 ? (size_t)qo_bytes + ev_ring_bytes() + ev_list_bytes((mode & ACESO_OUT_FULL) != 0)
             : kern == 2 ? ((mode & ACESO_OUT_FULL) ? tab.dbytes_full : tab.dbytes) + kRingBytesPerCta
                         : tabs + kRingBytesPerCta + (ctx->split == 2 ? (size_t)(kWarps / 2) * 32 * sizeof(Xchg) : 0);
         ctx->smem[kern][mode] = smem;
-        void *k = eval_kernel_for(mode, ctx->split, ctx->minb, kern);
+        void *k = eval_kernel_for(mode, ctx->split, ctx->minb, kern, ctx->e64);
         e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
         int occ = 0;
         if (e == cudaSuccess) e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k, kThreads, smem);
@@ -621,6 +789,7 @@ int aceso_load_profile(const aceso_profile_desc *d, int cuda_device, aceso_ctx *
   if (rc != ACESO_OK) {
     if (ctx->d_blob) cudaFree(ctx->d_blob);
     if (ctx->d_ev) cudaFree(ctx->d_ev);
+    if (ctx->d_sc) cudaFree(ctx->d_sc);
     delete ctx;
     return rc;
   }
@@ -635,6 +804,7 @@ void aceso_free(aceso_ctx *ctx) {
   cudaSetDevice(ctx->device);
   cudaFree(ctx->d_blob);
   cudaFree(ctx->d_ev);
+  cudaFree(ctx->d_sc);
   cudaSetDevice(prev);
   delete ctx;
 }
@@ -643,7 +813,7 @@ size_t aceso_select_buf_bytes(const aceso_ctx *ctx, int64_t n) {
   (void)n;
   if (!ctx) return 0;
   int m = 0;
-  for (int kern = 0; kern < 3; ++kern)
+  for (int kern = 0; kern < 4; ++kern)
     for (int k = 1; k < 8; ++k) m = std::max(m, ctx->max_ctas[kern][k]);
   m = std::max(m, 4 * ctx->sms);  // per-CTA partials of the eval kernels; select kernel grid
   return (size_t)kSelPartialOff + 16 * (size_t)m;
@@ -658,7 +828,7 @@ int aceso_eval(aceso_ctx *ctx, const uint8_t *d_codes, const uint64_t *d_hdr, in
   if (n >= (1ll << 37)) return fail(ACESO_EINVAL, "n >= 2^37");
   const uint32_t mode = flags & 7u;
   if (mode == 0 || (flags & ~(7u | ACESO_HINT_DENSE | ACESO_HINT_OVERLAP))) return fail(ACESO_EINVAL, "bad flags 0x%x", flags);
-  const int kern = ((flags & ACESO_HINT_DENSE) && ctx->quad_ok) ? ctx->dense_kernel : ctx->kernel;
+  const int kern = (flags & ACESO_HINT_DENSE) ? ctx->dense_kernel : ctx->kernel;
   if (n > 0 && (!d_codes || !d_hdr)) return fail(ACESO_EINVAL, "null codes/headers");
   if ((mode & (ACESO_OUT_SUMMARY | ACESO_OUT_FULL)) && !out) return fail(ACESO_EINVAL, "null outputs");
   if ((mode & ACESO_OUT_SUMMARY) && n > 0 && (!out->iter_ns || !out->max_mem || !out->info)) return fail(ACESO_EINVAL, "null summary array");
@@ -678,20 +848,33 @@ int aceso_eval(aceso_ctx *ctx, const uint8_t *d_codes, const uint64_t *d_hdr, in
   // the per-launch prologue and epilogue (measured, 8 streams: GPT-3 1.3B 5.39 / 5.83 / 5.97 G/s
   // with 1 / 2 / 3 tiles; Wide-ResNet 4.66 / 5.04 / 4.99; GPT-3 13B 3.21 / 2.96 / 2.35)
   const int tpw_hint = P.nch <= 20 ? 3 : P.nch <= 24 ? 2 : 1;
-  const int tpw = (kern == 1 && (flags & ACESO_HINT_OVERLAP) && tpw_hint > 1) ? std::max(tpw_hint, ctx->tiles_per_warp)
+  const int tpw = ((kern == 1 || kern == 3) && (flags & ACESO_HINT_OVERLAP) && tpw_hint > 1) ? std::max(tpw_hint, ctx->tiles_per_warp)
                                                                           : ctx->tiles_per_warp;
   const int tiles_per_cta = (kern != 0 ? kWarps : kWarps / ctx->split) * tpw;
   const int64_t need = (P.n_tiles + tiles_per_cta - 1) / tiles_per_cta;
   int grid = (int)std::max<int64_t>(1, std::min<int64_t>(need, ctx->max_ctas[kern][mode]));
+  if (kern == 3) {
+    const int64_t nw = (int64_t)grid * kWarps;
+    P.tw_q = (uint32_t)(P.n_tiles / nw);
+    P.tw_r = (uint32_t)(P.n_tiles % nw);
+    if ((uint64_t)(P.tw_q + 1) * (uint64_t)P.nch >= (1ull << 32) || P.n_tiles >= (1ll << 32))
+      return fail(ACESO_EINVAL, "batch too large for one launch (per-warp chunk count >= 2^32)");
+  }
   int prev = 0;
   CUDA_TRY(cudaGetDevice(&prev));
   if (prev != ctx->device) CUDA_TRY(cudaSetDevice(ctx->device));
   void *args[] = {&P};
-  cudaError_t e = cudaLaunchKernel(eval_kernel_for(mode, ctx->split, ctx->minb, kern), dim3(grid), dim3(kThreads), args, ctx->smem[kern][mode],
+  cudaError_t e = cudaLaunchKernel(eval_kernel_for(mode, ctx->split, ctx->minb, kern, ctx->e64), dim3(grid), dim3(kThreads), args, ctx->smem[kern][mode],
                                    reinterpret_cast<cudaStream_t>(stream));
   if (prev != ctx->device) cudaSetDevice(prev);
   if (e != cudaSuccess) return fail(ACESO_ECUDA, "eval launch: %s", cudaGetErrorString(e));
   return ACESO_OK;
+}
+
+const char *aceso_schedule_name(const aceso_ctx *ctx, uint32_t flags) {
+  if (!ctx) return "";
+  static const char *const names[4] = {"per-op kernel", "event kernel", "dense kernel", "scan kernel"};
+  return names[(flags & ACESO_HINT_DENSE) ? ctx->dense_kernel : ctx->kernel];
 }
 
 int aceso_select(aceso_ctx *ctx, const aceso_eval_out *out, int64_t n, int64_t global_offset,
@@ -740,65 +923,6 @@ int aceso_pack_rowmajor(const uint8_t *d_rowmajor, int64_t n, int32_t n_ops, uin
   pack_kernel<<<grid, 256, 0, reinterpret_cast<cudaStream_t>(stream)>>>(d_rowmajor, n, n_ops, reinterpret_cast<uint4 *>(d_tiled), total_vec);
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return fail(ACESO_ECUDA, "pack launch: %s", cudaGetErrorString(e));
-  return ACESO_OK;
-}
-
-size_t aceso_incr_work_bytes(const aceso_ctx *ctx, int32_t n_bases) {
-  if (!ctx || n_bases < 1) return 0;
-  auto al = [](size_t v) { return (v + 255) & ~(size_t)255; };
-  return al((size_t)n_bases * sizeof(IncrBaseHdr)) + al((size_t)n_bases * ctx->G * sizeof(IncrBaseStage)) +
-         al((size_t)n_bases * ctx->L);
-}
-
-int aceso_eval_incr(aceso_ctx *ctx, const uint8_t *d_bases, const uint64_t *d_base_hdr,
-                    const uint16_t *d_ranks, int32_t n_bases, const aceso_cand *d_cands, int64_t n,
-                    int64_t global_offset, int64_t n_total, uint32_t flags,
-                    const aceso_eval_out *out, void *d_sel, void *d_work, void *stream) {
-  if (!ctx) return fail(ACESO_EINVAL, "null context");
-  if (n < 0 || global_offset < 0 || n_total < global_offset + n) return fail(ACESO_EINVAL, "bad n / global_offset / n_total");
-  if (n_total >= (1ll << 40)) return fail(ACESO_EINVAL, "n_total >= 2^40");
-  const uint32_t mode = flags & 7u;
-  if (mode == 0 || (flags & ~(7u | ACESO_HINT_DENSE))) return fail(ACESO_EINVAL, "bad flags 0x%x", flags);
-  if (n_bases < 1 || !d_bases || !d_base_hdr || !d_work || (n > 0 && !d_cands)) return fail(ACESO_EINVAL, "null argument");
-  if ((mode & (ACESO_OUT_SUMMARY | ACESO_OUT_FULL)) && !out) return fail(ACESO_EINVAL, "null outputs");
-  if ((mode & ACESO_OUT_SUMMARY) && n > 0 && (!out->iter_ns || !out->max_mem || !out->info)) return fail(ACESO_EINVAL, "null summary array");
-  if (mode & ACESO_OUT_FULL) {
-    if (out->p_max < ctx->G) return fail(ACESO_EINVAL, "p_max %d < n_devices %d", out->p_max, ctx->G);
-    if (n > 0 && (!out->stage_T || !out->stage_mem || !out->stage_comp || !out->stage_comm)) return fail(ACESO_EINVAL, "null stage array");
-  }
-  if ((mode & ACESO_FUSED_SELECT) && !d_sel) return fail(ACESO_EINVAL, "null select buffer");
-  EvalParams P = make_params(ctx, n, global_offset, n_total, out, d_sel);
-  auto al = [](size_t v) { return (v + 255) & ~(size_t)255; };
-  unsigned char *w = reinterpret_cast<unsigned char *>(d_work);
-  IncrBaseHdr *hdrs = reinterpret_cast<IncrBaseHdr *>(w);
-  IncrBaseStage *stages = reinterpret_cast<IncrBaseStage *>(w + al((size_t)n_bases * sizeof(IncrBaseHdr)));
-  uint8_t *smap = w + al((size_t)n_bases * sizeof(IncrBaseHdr)) + al((size_t)n_bases * ctx->G * sizeof(IncrBaseStage));
-  int prev = 0;
-  CUDA_TRY(cudaGetDevice(&prev));
-  if (prev != ctx->device) CUDA_TRY(cudaSetDevice(ctx->device));
-  cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
-  base_cache_kernel<<<(n_bases + 127) / 128, 128, 0, st>>>(P, d_bases, d_base_hdr, n_bases, hdrs, stages, smap);
-  void *k = nullptr;
-  switch (mode) {
-    case 1: k = incr_kernel_ptr<1>(); break;
-    case 2: k = incr_kernel_ptr<2>(); break;
-    case 3: k = incr_kernel_ptr<3>(); break;
-    case 4: k = incr_kernel_ptr<4>(); break;
-    case 5: k = incr_kernel_ptr<5>(); break;
-    case 6: k = incr_kernel_ptr<6>(); break;
-    default: k = incr_kernel_ptr<7>(); break;
-  }
-  const int grid = (int)std::max<int64_t>(1, std::min<int64_t>((n + 255) / 256, (int64_t)ctx->sms * 8));
-  const uint8_t *b = d_bases;
-  const uint16_t *r = d_ranks;
-  const IncrBaseHdr *ch = hdrs;
-  const IncrBaseStage *cs = stages;
-  const uint8_t *cm = smap;
-  void *args[] = {&P, &b, &r, &n_bases, &d_cands, &ch, &cs, &cm};
-  cudaError_t e = cudaLaunchKernel(k, dim3(grid), dim3(256), args, 0, st);
-  if (e == cudaSuccess) e = cudaGetLastError();
-  if (prev != ctx->device) cudaSetDevice(prev);
-  if (e != cudaSuccess) return fail(ACESO_ECUDA, "incremental eval launch: %s", cudaGetErrorString(e));
   return ACESO_OK;
 }
 

@@ -78,6 +78,17 @@ struct EvalParams {
   uint32_t qo_bytes;      // bytes of the per-quad signature table staged to shared memory
   uint32_t qo_off;        // its byte offset in the event blob
   const unsigned char *evblob;
+  // scan kernel (scan_kernel.cuh), exact u64 tables in global memory:
+  const uint4 *sx;        // [RUNS][L+1] x 2: {PS, PA} {PW, PC}  u64 prefix sums at rc = 0
+  const uint4 *sk;        // [RUNS][L+1]    : {reshard_j, p2p_bwd_j, p2p_fwd_{j-1}, 0} (u32 ns)
+  const uint64_t *sd;     // [n_tp * n_dp][L+1] DP all-reduce prefix sums
+  const void *ss;         // [levels][RUNS][L] range-max table of peak >> es (u32, or u64 when wide)
+  const uint4 *sq;        // [nsig][RUNS][16] x 2: {dS, dA} {e1 >> es, dC} u64 recompute deltas
+  const uint32_t *sqo;    // [4 * nch] per-quad signature record offset (staged to shared memory)
+  uint32_t qo_words;
+  uint32_t es;            // transient-memory values are stored in units of 2^es bytes
+  uint32_t tw_q, tw_r;    // scan kernel: tiles per warp (quotient / remainder over all warps)
+  uint32_t sc_resolve;    // scan kernel: resolve recompute-only chunks in the compacted pass
 };
 
 // select buffer layout: [0,32) result, [32,40) completion counter, [64, ...) partials (16 B each)

@@ -34,7 +34,22 @@ def test_reference_arm_json_line():
 
 
 def test_reference_arm_other_ranks_exit_quietly():
-    r = _run(["--impl", "reference", "--steps", "1", "--warmup", "3", "--config", "toy-a"],
+    r = _run(["--impl", "reference", "--gpus", "2", "--steps", "1", "--warmup", "3", "--config", "toy-a"],
              env={"RANK": "1", "WORLD_SIZE": "2"})
     assert r.returncode == 0, r.stderr
     assert r.stdout.strip() == ""
+
+
+def test_gpus_mismatch_with_world_size_is_refused():
+    r = _run(["--impl", "reference", "--gpus", "4", "--steps", "1", "--config", "toy-a"],
+             env={"RANK": "0", "WORLD_SIZE": "2"})
+    assert r.returncode == 2 and "WORLD_SIZE" in r.stderr
+
+
+def test_gpus_n_self_launches_n_ranks():
+    """--gpus 2 without torchrun relaunches under torch.distributed.run: two ranks, rank 0
+    alone prints (the reference arm needs no GPU)."""
+    r = _run(["--impl", "reference", "--gpus", "2", "--steps", "1", "--warmup", "1", "--config", "toy-a"])
+    assert r.returncode == 0, r.stderr[-2000:]
+    lines = [l for l in r.stdout.splitlines() if l.startswith("{")]
+    assert len(lines) == 1 and json.loads(lines[0])["n_gpus"] == 2

@@ -84,7 +84,12 @@ def _load(prof):
     (lambda p: p.rec.__setitem__((0, 0, 0, 5), p.rec[0, 0, 0, 4] + 1), L.ACESO_ERANGE),   # keep > act
     (lambda p: p.rec.__setitem__((0, 0, 0, 0), 1 << 32), L.ACESO_ERANGE),               # > u32
     (lambda p: p.rec.__setitem__((0, 0, 0, 2), -1), L.ACESO_ERANGE),                    # negative
-    (lambda p: p.wmem.__setitem__((0, 0, 0), (1 << 32) - 1), L.ACESO_ERANGE),           # W overflow
+    (lambda p: p.wmem.__setitem__((0, 0, 0), (1 << 40) + 1), L.ACESO_ERANGE),           # W > 2^40
+    (lambda p: p.rec.__setitem__((0, 0, 0, 6), (1 << 40) + 1), L.ACESO_ERANGE),         # peak > 2^40
+    # wide but valid memory values are accepted (served by the exact 64-bit scan kernel); on a
+    # box without a GPU the load then stops at the device probe
+    (lambda p: p.wmem.__setitem__((0, 0, 0), (1 << 40) - 1), L.ACESO_ENODEV),
+    (lambda p: p.rec.__setitem__((0, 0, 0, 4), (1 << 39) + 1), L.ACESO_ENODEV),
     (lambda p: p.op_type.__setitem__(0, 999), L.ACESO_EINVAL),                          # bad type
     (lambda p: setattr(p, "global_batch", 0), L.ACESO_EINVAL),
     (lambda p: setattr(p, "n_devices", 256), L.ACESO_EINVAL),

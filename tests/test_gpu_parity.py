@@ -395,7 +395,7 @@ def test_random_bytes_never_crash_and_match():
 # forward+reverse warp pair; 2 or 3 resident CTAs per SM
 # ---------------------------------------------------------------------------
 @pytest.mark.parametrize("minb", ["2", "3"])
-@pytest.mark.parametrize("kernel,split", [("events", "1"), ("quad", "1"), ("quad", "2")])
+@pytest.mark.parametrize("kernel,split", [("scan", "1"), ("events", "1"), ("quad", "1"), ("quad", "2")])
 @pytest.mark.parametrize("name", ["gpt3-1.3b", "t5", "wrn", "gpt3-13b", "toy-a"])
 def test_kernel_variants_parity(kernel, split, minb, name, monkeypatch):
     monkeypatch.setenv("ACESO_KERNEL", kernel)
@@ -529,3 +529,123 @@ def test_event_kernel_recompute_attribution_parity(name):
     g, o, sel, _, _ = compare(prof, codes, hdr, full=True)
     assert ((o["info"] & oracle.INFO_INVALID) == 0).mean() > 0.5  # the sums are really compared
     compare(prof, codes, hdr)
+
+
+# ---------------------------------------------------------------------------
+# memory values of any width: no common power-of-two factor above 2^shift (shift 0 = odd
+# byte counts), and values beyond 32-bit units (scale 64: up to ~2^38 bytes per op)
+# ---------------------------------------------------------------------------
+def _jit_batches(prof, seed):
+    codes, hdr = ai.search_shaped(prof, seed, 0, 1500, group_size=16)
+    rng = np.random.default_rng(seed)
+    rcodes = rng.integers(0, 256, size=(200, prof.n_ops), dtype=np.uint8)
+    rhdr = rng.integers(0, 1 << 16, size=200, dtype=np.uint64)
+    dcodes, dhdr = ai.dense_random(prof, seed + 1, 0, 300)
+    return [(codes, hdr), (rcodes, rhdr), (dcodes, dhdr)]
+
+
+@pytest.mark.parametrize("shift", list(range(10)))
+@pytest.mark.parametrize("name", ["gpt3-1.3b", "toy-b", "t5"])
+def test_memory_units_parity(name, shift):
+    prof = P.jittered(P.WORKLOADS[name](), 300 + shift, shift)
+    try:
+        for codes, hdr in _jit_batches(prof, SEED + 60 + shift):
+            compare(prof, codes, hdr, full=True)
+            compare(prof, codes, hdr, dense_hint=True)
+    finally:
+        _, ctx = _ctx_cache.pop(id(prof))
+        ctx.close()
+
+
+@pytest.mark.parametrize("kernel", ["events", "quad", "dense"])
+@pytest.mark.parametrize("shift", [0, 5, 9])
+def test_memory_units_packed_kernels_parity(kernel, shift, monkeypatch):
+    """The 32-bit packed kernels at every memory unit they accept."""
+    monkeypatch.setenv("ACESO_KERNEL", kernel)
+    prof = P.jittered(P.WORKLOADS["gpt3-1.3b"](), 400 + shift, shift)
+    try:
+        for codes, hdr in _jit_batches(prof, SEED + 70 + shift):
+            compare(prof, codes, hdr, full=True)
+    finally:
+        _, ctx = _ctx_cache.pop(id(prof))
+        ctx.close()
+
+
+@pytest.mark.parametrize("name", ["gpt3-1.3b", "gpt3-13b", "toy-a", "wrn"])
+def test_wide_memory_values_parity(name):
+    """Per-op memory beyond 2^32 units (scaled by 64, odd byte counts): the packed kernels
+    decline the profile and the scan kernel's 64-bit transient table serves every call."""
+    prof = P.jittered(P.WORKLOADS[name](), 500, 0, scale=64)
+    assert prof.rec[..., 6].max() + prof.rec[..., 4].max() > (1 << 32)
+    try:
+        for codes, hdr in _jit_batches(prof, SEED + 80):
+            compare(prof, codes, hdr, full=True)
+            compare(prof, codes, hdr, dense_hint=True)
+    finally:
+        _, ctx = _ctx_cache.pop(id(prof))
+        ctx.close()
+
+
+@pytest.mark.parametrize("case", ["memory", "fig3", "fingerprint", "recompute", "p2p"])
+def test_pin_profiles_parity(case):
+    """The hand-built profiles of tests/test_oracle_pins.py on the GPU (every candidate of
+    each pin through the C-ABI, bit-exact)."""
+    from tests import test_oracle_pins as T
+    profs = []
+    if case == "memory":
+        vals = [(10, 3, 7, 5), (20, 20, 40, 1), (30, 0, 11, 9)]
+        recs = {t: (lambda v: (lambda tpl, b: [1, 0, 1, 0, v[0], v[1], v[2], 0, 0, 0]))(v)
+                for t, v in enumerate(vals)}
+        wm = np.array([[[v[3], 0]] for v in vals], np.int64)
+        prof = T.mkprof(recs, [0, 1, 2], G=1, Bg=1, wmem=wm)
+        rows = [T.cand([3]), T.cand([3], rc=[1, 0, 0]), T.cand([3], rc=[1, 1, 1])]
+        profs.append((prof, rows, [ai.header(0, 1)] * 3))
+    elif case == "fig3":
+        prof = T.fig3_profile()
+        rows = [T.cand([2, 2], tpdp=[(0, 0), (0, 1)]), T.cand([2, 2], tpdp=[(1, 0), (0, 0)]),
+                T.cand([3, 1], tpdp=[(1, 0), (0, 0)])]
+        profs.append((prof, rows, [ai.header(1, 2)] * 3))
+    elif case == "fingerprint":
+        n_tp = n_dp = n_b = 4
+        recs = {t: (lambda t: (lambda tpl, b: [1 + b + 10 * tpl + 100 * t, 0, 0, 0, 0, 0, 0, 0, 0, 0]))(t)
+                for t in range(2)}
+        dps = np.zeros((2, n_tp, n_dp), np.int64)
+        for t in range(2):
+            for tpl in range(n_tp):
+                for dpl in range(n_dp):
+                    dps[t, tpl, dpl] = 1000 * (1 + dpl + 10 * tpl + 100 * t)
+        for t in range(2):
+            for G in [1, 2, 4, 8]:
+                kG = G.bit_length() - 1
+                prof = T.mkprof(recs, [t], n_tp=n_tp, n_b=n_b, n_dp=n_dp, G=G, Bg=64, dps=dps)
+                rows, hdrs = [], []
+                for tpl in range(kG + 1):
+                    dpl = kG - tpl
+                    for mbs_log2 in range(dpl, dpl + n_b):
+                        rows.append([ai.code(1, tpl, dpl, 0)])
+                        hdrs.append(ai.header(mbs_log2, 1))
+                profs.append((prof, rows, hdrs))
+    elif case == "recompute":
+        prof = T.mkprof({0: lambda tpl, b: [1, 10, 100, 1000, 0, 0, 0, 10 ** 4, 10 ** 5, 10 ** 6]},
+                        [0] * 5, n_tp=2, n_b=2, n_dp=2, G=4, Bg=8, dps=[[[0, 10 ** 7], [0, 10 ** 7]]])
+        row = [ai.code(1, 1, 0, 0), ai.code(0, 0, 1, 0), ai.code(0, 0, 1, 1),
+               ai.code(1, 0, 1, 0), ai.code(0, 0, 1, 1)]
+        profs.append((prof, [row], [ai.header(1, 2)]))
+    else:
+        k, f, b, c = 3, 7, 13, 5
+        recs = {0: lambda tpl, bb: [f, 0, b, 0, 0, 0, 0, 0, 1000, 1000],
+                1: lambda tpl, bb: [f, 0, b, 0, 0, 0, 0, 0, c, c],
+                2: lambda tpl, bb: [f + c, 0, b + c, 0, 0, 0, 0, 0, 3000, 3000]}
+        for p in [2, 3, 4, 5]:
+            types = [2] + [0] * (k - 2) + [1] + ([1] + [0] * (k - 2) + [1]) * (p - 2) + [1] + [0] * (k - 2) + [2]
+            prof = T.mkprof(recs, types, G=p, Bg=8)
+            profs.append((prof, [T.cand([k] * p)] * 4, [ai.header(m, p) for m in [0, 1, 2, 3]]))
+    for prof, rows, hdrs in profs:
+        codes = np.array(rows, np.uint8)
+        hdr = np.array(hdrs, np.uint64)
+        try:
+            for flags in [dict(), dict(dense_hint=True)]:
+                compare(prof, codes, hdr, full=True, **flags)
+        finally:
+            _, ctx = _ctx_cache.pop(id(prof))
+            ctx.close()
