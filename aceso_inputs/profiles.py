@@ -38,6 +38,9 @@ class Profile:
     n_devices: int
     mem_capacity: int
     global_batch: int
+    # records of each type's alternative tensor-parallel partition dimension (§4.2, P:L263-265:
+    # row- vs column-wise MatMul, input- vs output-channel convolution); None: no alternative
+    rec_alt: np.ndarray | None = None
 
     @property
     def n_ops(self):

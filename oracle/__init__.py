@@ -38,7 +38,7 @@ def _load():
         lib = ctypes.CDLL(path)
         P = ctypes.c_void_p
         i32, i64 = ctypes.c_int32, ctypes.c_int64
-        lib.oracle_eval.argtypes = [i32, i32, i32, i32, i32, i32, P, P, P, P, i64, i64, P, P, i64,
+        lib.oracle_eval.argtypes = [i32, i32, i32, i32, i32, i32, P, P, P, P, P, i64, i64, P, P, P, i64,
                                     i32, P, P, P, P, P, P, P, ctypes.c_int]
         lib.oracle_eval.restype = ctypes.c_int
         lib.oracle_select.argtypes = [P, P, P, i64, i64, P, P, P]
@@ -50,13 +50,19 @@ def _ptr(a):
     return None if a is None else a.ctypes.data
 
 
-def evaluate(prof, codes, hdr, full=False, threads=1):
-    """Evaluates row-major codes [n][L] with headers [n].
+def evaluate(prof, codes, hdr, full=False, threads=1, dims=None):
+    """Evaluates row-major codes [n][L] with headers [n]; dims (optional, row-major [n][L],
+    nonzero = the op's alternative tensor-parallel partition dimension) needs prof.rec_alt.
 
     Returns dict(iter, max_mem, info[, stage_T, stage_mem, stage_comp, stage_comm]);
     stage arrays are [n][G] (rows i >= p and rows of invalid candidates are 0)."""
     lib = _load()
     codes = np.ascontiguousarray(codes, dtype=np.uint8)
+    if dims is not None:
+        dims = np.ascontiguousarray(dims, dtype=np.uint8)
+        assert dims.shape == codes.shape
+    rec_alt = getattr(prof, "rec_alt", None)
+    rec_alt = None if rec_alt is None else np.ascontiguousarray(rec_alt, dtype=np.int64)
     hdr = np.ascontiguousarray(hdr, dtype=np.uint64)
     n = int(hdr.shape[0])
     L = int(prof.op_type.shape[0])
@@ -75,8 +81,9 @@ def evaluate(prof, codes, hdr, full=False, threads=1):
         for k, name in enumerate(["stage_T", "stage_mem", "stage_comp", "stage_comm"]):
             out[name] = np.zeros((n, G), np.uint64)
             st[k] = out[name]
-    rc = lib.oracle_eval(L, T, n_tp, n_dp, n_b, G, _ptr(op_type), _ptr(rec), _ptr(wmem), _ptr(dps),
-                         int(prof.mem_capacity), int(prof.global_batch), _ptr(codes), _ptr(hdr), n,
+    rc = lib.oracle_eval(L, T, n_tp, n_dp, n_b, G, _ptr(op_type), _ptr(rec), _ptr(rec_alt), _ptr(wmem),
+                         _ptr(dps), int(prof.mem_capacity), int(prof.global_batch), _ptr(codes), _ptr(dims),
+                         _ptr(hdr), n,
                          G, _ptr(out["iter"]), _ptr(out["max_mem"]), _ptr(out["info"]),
                          _ptr(st[0]), _ptr(st[1]), _ptr(st[2]), _ptr(st[3]), int(threads))
     assert rc == 0

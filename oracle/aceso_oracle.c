@@ -61,18 +61,23 @@ typedef struct {
   int32_t L, T, n_tp, n_dp, n_b, G;
   const uint16_t *op_type;
   const int64_t *rec;  /* [T][n_tp][n_b][NF] */
+  const int64_t *rec_alt; /* [T][n_tp][n_b][NF] records of the alternative partition dimension, or 0 */
   const int64_t *wmem; /* [T][n_tp][2] */
   const int64_t *dps;  /* [T][n_tp][n_dp] */
   int64_t C, Bg;
 } oracle_profile;
 
-static u64 rec_field(const oracle_profile *P, int type, int tpl, int b, int f) {
-  return (u64)P->rec[(((int64_t)type * P->n_tp + tpl) * P->n_b + b) * NF + f];
+/* record field of an op of `type` at (tpl, b); dim = 1 reads the records profiled for the
+ * op's alternative tensor-parallel partition dimension (§4.2: row- vs
+ * column-wise MatMul, input- vs output-channel convolution) */
+static u64 rec_field(const oracle_profile *P, int dim, int type, int tpl, int b, int f) {
+  const int64_t *r = dim ? P->rec_alt : P->rec;
+  return (u64)r[(((int64_t)type * P->n_tp + tpl) * P->n_b + b) * NF + f];
 }
 
 /* Evaluates one candidate. codes: [L] bytes, hdr: header. Stage outputs (if
  * non-null) are rows of p_max entries for this candidate. */
-static void eval_one(const oracle_profile *P, const uint8_t *codes, u64 hdr, int32_t p_max,
+static void eval_one(const oracle_profile *P, const uint8_t *codes, const uint8_t *dims, u64 hdr, int32_t p_max,
                      u64 *iter_out, u64 *mem_out, uint32_t *info_out, u64 *sT, u64 *sM, u64 *sC,
                      u64 *sK) {
   const int L = P->L;
@@ -94,12 +99,14 @@ static void eval_one(const oracle_profile *P, const uint8_t *codes, u64 hdr, int
   int *tpl = (int *)malloc(sizeof(int) * L);
   int *dpl = (int *)malloc(sizeof(int) * L);
   int *rc = (int *)malloc(sizeof(int) * L);
+  int *dim = (int *)malloc(sizeof(int) * L);
   for (int j = 0; j < L; ++j) {
     uint8_t c = codes[j];
     head[j] = c & 1;
     tpl[j] = (c >> 1) & 7;
     rc[j] = (c >> 4) & 1;
     dpl[j] = (c >> 5) & 7;
+    dim[j] = dims ? (dims[j] != 0) : 0; /* tensor-parallel partition dimension of op j */
   }
 
   /* --- structural checks ------------------------------------------------- */
@@ -128,7 +135,7 @@ static void eval_one(const oracle_profile *P, const uint8_t *codes, u64 hdr, int
     *iter_out = 0;
     *mem_out = 0;
     *info_out = (p << 8) | O_INVALID | (reasons << 18);
-    free(head); free(tpl); free(dpl); free(rc);
+    free(head); free(tpl); free(dpl); free(rc); free(dim);
     return;
   }
 
@@ -154,13 +161,13 @@ static void eval_one(const oracle_profile *P, const uint8_t *codes, u64 hdr, int
     int i = sid[j];
     int t = P->op_type[j];
     int b = (int)mbs_log2 - dpl[j]; /* per-GPU batch = mbs / dp (R8) */
-    u64 fc = rec_field(P, t, tpl[j], b, FWD_COMP);
-    u64 fm = rec_field(P, t, tpl[j], b, FWD_COMM);
-    u64 bc = rec_field(P, t, tpl[j], b, BWD_COMP);
-    u64 bm = rec_field(P, t, tpl[j], b, BWD_COMM);
-    u64 act = rec_field(P, t, tpl[j], b, ACT);
-    u64 keep = rec_field(P, t, tpl[j], b, KEEP);
-    u64 peak = rec_field(P, t, tpl[j], b, PEAK);
+    u64 fc = rec_field(P, dim[j], t, tpl[j], b, FWD_COMP);
+    u64 fm = rec_field(P, dim[j], t, tpl[j], b, FWD_COMM);
+    u64 bc = rec_field(P, dim[j], t, tpl[j], b, BWD_COMP);
+    u64 bm = rec_field(P, dim[j], t, tpl[j], b, BWD_COMM);
+    u64 act = rec_field(P, dim[j], t, tpl[j], b, ACT);
+    u64 keep = rec_field(P, dim[j], t, tpl[j], b, KEEP);
+    u64 peak = rec_field(P, dim[j], t, tpl[j], b, PEAK);
     u64 F = fc + fm;                           /* forward of one microbatch */
     u64 Bp = bc + bm + (rc[j] ? F : 0);        /* recompute adds the forward (R7) */
     u64 Aj = rc[j] ? keep : act;               /* R3 */
@@ -170,7 +177,7 @@ static void eval_one(const oracle_profile *P, const uint8_t *codes, u64 hdr, int
     u64 dj = (u64)P->dps[((int64_t)t * P->n_tp + tpl[j]) * P->n_dp + dpl[j]];
     u64 rs = 0; /* P:L261, R13: reshard when the tp/dp mix changes inside a stage */
     if (j > 0 && !head[j] && (tpl[j] != tpl[j - 1] || dpl[j] != dpl[j - 1]))
-      rs = rec_field(P, t, tpl[j], b, RESHARD);
+      rs = rec_field(P, dim[j], t, tpl[j], b, RESHARD);
     S[i] += F + Bp + rs;
     comp[i] += fc + bc + (rc[j] ? fc : 0);
     comm[i] += fm + bm + (rc[j] ? fm : 0) + rs;
@@ -189,13 +196,13 @@ static void eval_one(const oracle_profile *P, const uint8_t *codes, u64 hdr, int
       }
     if (i + 1 < p) {
       int t = P->op_type[last];
-      u64 v = rec_field(P, t, tpl[last], (int)mbs_log2 - dpl[last], P2P_FWD);
+      u64 v = rec_field(P, dim[last], t, tpl[last], (int)mbs_log2 - dpl[last], P2P_FWD);
       S[i] += v;
       comm[i] += v;
     }
     if (i > 0) {
       int t = P->op_type[first];
-      u64 v = rec_field(P, t, tpl[first], (int)mbs_log2 - dpl[first], P2P_BWD);
+      u64 v = rec_field(P, dim[first], t, tpl[first], (int)mbs_log2 - dpl[first], P2P_BWD);
       S[i] += v;
       comm[i] += v;
     }
@@ -226,12 +233,13 @@ static void eval_one(const oracle_profile *P, const uint8_t *codes, u64 hdr, int
   *info_out = bottleneck | (p << 8) | (oom ? O_OOM : 0);
 
   free(sid); free(S); free(Dd); free(Wst); free(A); free(E); free(comp); free(comm);
-  free(head); free(tpl); free(dpl); free(rc);
+  free(head); free(tpl); free(dpl); free(rc); free(dim);
 }
 
 typedef struct {
   const oracle_profile *P;
   const uint8_t *codes;
+  const uint8_t *dims;
   const uint64_t *hdr;
   int64_t lo, hi;
   int32_t p_max;
@@ -243,7 +251,8 @@ static void *run_job(void *arg) {
   job_t *J = (job_t *)arg;
   for (int64_t c = J->lo; c < J->hi; ++c) {
     int64_t o = c * J->p_max;
-    eval_one(J->P, J->codes + c * (int64_t)J->P->L, J->hdr[c], J->p_max, &J->iter[c], &J->mem[c],
+    eval_one(J->P, J->codes + c * (int64_t)J->P->L, J->dims ? J->dims + c * (int64_t)J->P->L : 0,
+             J->hdr[c], J->p_max, &J->iter[c], &J->mem[c],
              &J->info[c], J->sT ? J->sT + o : 0, J->sM ? J->sM + o : 0, J->sC ? J->sC + o : 0,
              J->sK ? J->sK + o : 0);
   }
@@ -251,26 +260,29 @@ static void *run_job(void *arg) {
 }
 
 /* Public entry: evaluates n candidates (row-major codes [n][L]) on n_threads
- * host threads (contiguous blocks). Stage arrays are [n][p_max] (nullable);
+ * host threads (contiguous blocks). rec_alt / dims (nullable): records of each op type's
+ * alternative tensor-parallel partition dimension and the per-op choice (row-major [n][L],
+ * nonzero = alternative; dims require rec_alt). Stage arrays are [n][p_max] (nullable);
  * entries i >= p are left untouched; for invalid candidates nothing is written.
  * Returns 0, or -1 on bad arguments. */
 int oracle_eval(int32_t L, int32_t T, int32_t n_tp, int32_t n_dp, int32_t n_b, int32_t G,
-                const uint16_t *op_type, const int64_t *rec, const int64_t *wmem,
-                const int64_t *dps, int64_t C, int64_t Bg, const uint8_t *codes,
+                const uint16_t *op_type, const int64_t *rec, const int64_t *rec_alt, const int64_t *wmem,
+                const int64_t *dps, int64_t C, int64_t Bg, const uint8_t *codes, const uint8_t *dims,
                 const uint64_t *hdr, int64_t n, int32_t p_max, uint64_t *iter, uint64_t *max_mem,
                 uint32_t *info, uint64_t *stage_T, uint64_t *stage_mem, uint64_t *stage_comp,
                 uint64_t *stage_comm, int n_threads) {
   if (L < 1 || T < 1 || n < 0 || !op_type || !rec || !wmem || !dps || (n && (!codes || !hdr)))
     return -1;
   if ((stage_T || stage_mem || stage_comp || stage_comm) && p_max < G) return -1;
-  oracle_profile P = {L, T, n_tp, n_dp, n_b, G, op_type, rec, wmem, dps, C, Bg};
+  if (dims && !rec_alt) return -1;
+  oracle_profile P = {L, T, n_tp, n_dp, n_b, G, op_type, rec, rec_alt, wmem, dps, C, Bg};
   if (n_threads < 1) n_threads = 1;
   if (n_threads > 256) n_threads = 256;
   if ((int64_t)n_threads > n) n_threads = n > 0 ? (int)n : 1;
   job_t jobs[256];
   pthread_t th[256];
   for (int k = 0; k < n_threads; ++k) {
-    jobs[k] = (job_t){&P, codes, hdr, n * k / n_threads, n * (k + 1) / n_threads, p_max,
+    jobs[k] = (job_t){&P, codes, dims, hdr, n * k / n_threads, n * (k + 1) / n_threads, p_max,
                       iter, max_mem, stage_T, stage_mem, stage_comp, stage_comm, info};
   }
   if (n_threads == 1) {

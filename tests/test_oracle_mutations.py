@@ -66,10 +66,10 @@ MUTATIONS = [
      "u64 dj = (u64)P->dps[((int64_t)t * P->n_tp + dpl[j]) * P->n_dp + tpl[j]];"),
     ("r5-drop-p2p-fwd", "R5, P:L241", "if (i + 1 < p) {", "if (0) {"),
     ("r5-p2p-bwd-of-last-op", "R5, P:L241",
-     "int t = P->op_type[first];\n      u64 v = rec_field(P, t, tpl[first], (int)mbs_log2 - dpl[first], P2P_BWD);",
-     "int t = P->op_type[last];\n      u64 v = rec_field(P, t, tpl[last], (int)mbs_log2 - dpl[last], P2P_BWD);"),
+     "int t = P->op_type[first];\n      u64 v = rec_field(P, dim[first], t, tpl[first], (int)mbs_log2 - dpl[first], P2P_BWD);",
+     "int t = P->op_type[last];\n      u64 v = rec_field(P, dim[last], t, tpl[last], (int)mbs_log2 - dpl[last], P2P_BWD);"),
     ("r13-drop-reshard", "R13, P:L261",
-     "rs = rec_field(P, t, tpl[j], b, RESHARD);", "rs = 0;"),
+     "rs = rec_field(P, dim[j], t, tpl[j], b, RESHARD);", "rs = 0;"),
     ("r9-no-gsum-check", "R9, P:L151", "if (gsum != (u64)P->G) reasons |= O_R_GSUM;", ";"),
     ("select-tie-highest-index", "R11 (selection)", "else better = g < best_idx;",
      "else better = g > best_idx;"),
