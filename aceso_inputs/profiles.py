@@ -129,6 +129,27 @@ class OpCost:
     inp: float = 0.0  # input bytes, full (for reshard / p2p)
     params: float = 0.0  # parameters per GPU
     workspace: float = 0.0
+    # tensor-parallel partition dimension: "col" (MatMul split along its output
+    # features: input replicated, output sharded), "row" (split along its input features:
+    # input sharded, partial outputs all-reduced), "out" / "in" (convolution output / input
+    # channels); "" = no alternative dimension
+    part: str = ""
+
+
+def _alternative(c: OpCost, tp: int) -> OpCost:
+    """The op's cost under its other partition dimension (Megatron's column/row pairing for
+    MatMul, output/input channels for convolution)."""
+    import dataclasses as dc
+    if c.part == "col":  # -> row-wise: input sharded, partial outputs all-reduced forward
+        return dc.replace(c, act=c.act / tp, out=c.out * tp, tp_fwd_bytes=c.tp_fwd_bytes + c.out * tp,
+                          tp_bwd_bytes=0.0, part="row")
+    if c.part == "row":  # -> column-wise: input replicated, output gathered, input grads all-reduced
+        return dc.replace(c, act=c.act * tp, out=c.out / tp, tp_fwd_bytes=0.0, tp_fwd_gather=c.out,
+                          tp_bwd_bytes=c.tp_bwd_bytes + c.act * tp, part="col")
+    if c.part == "out":  # -> input channels: input sharded, partial outputs all-reduced
+        return dc.replace(c, act=c.act / tp, out=c.out * tp, tp_fwd_gather=0.0, tp_fwd_bytes=c.out * tp,
+                          tp_bwd_bytes=0.0, part="in")
+    return c
 
 
 def _mem(x):
@@ -173,15 +194,21 @@ def _build(name, ops, type_of, n_devices, global_batch, n_b_max, hw, bytes_per_p
     n_b = n_b_max
     while True:
         rec = np.zeros((T, n_tp, n_b, NF), dtype=np.int64)
+        rec_alt = np.zeros((T, n_tp, n_b, NF), dtype=np.int64)
         for t, k in enumerate(keys):
             for tpl in range(n_tp):
                 for b in range(n_b):
-                    rec[t, tpl, b] = _record(hw, type_of[k](1 << b, 1 << tpl), 1 << tpl, n_devices)
-        times = rec[..., [0, 1, 2, 3, 7, 8, 9]]
+                    c = type_of[k](1 << b, 1 << tpl)
+                    rec[t, tpl, b] = _record(hw, c, 1 << tpl, n_devices)
+                    # tp = 1: nothing is partitioned, both dimensions cost the same
+                    rec_alt[t, tpl, b] = (_record(hw, _alternative(c, 1 << tpl), 1 << tpl, n_devices)
+                                          if tpl > 0 else rec[t, tpl, b])
+        times = np.concatenate([rec, rec_alt])[..., [0, 1, 2, 3, 7, 8, 9]]
         if times.max() <= U32 or n_b == 1:
             break
         n_b -= 1
-    assert rec[..., [0, 1, 2, 3, 7, 8, 9]].max() <= U32, name
+    assert np.concatenate([rec, rec_alt])[..., [0, 1, 2, 3, 7, 8, 9]].max() <= U32, name
+    assert (rec_alt[..., 5] <= rec_alt[..., 4]).all()
     wmem = np.zeros((T, n_tp, 2), dtype=np.int64)
     dps = np.zeros((T, n_tp, n_dp), dtype=np.int64)
     for t, k in enumerate(keys):
@@ -196,7 +223,7 @@ def _build(name, ops, type_of, n_devices, global_batch, n_b_max, hw, bytes_per_p
     assert dps.max() <= U32, name
     return Profile(name=name, op_type=op_type, type_names=[str(k) for k in keys], rec=rec, wmem=wmem,
                    dps=dps, n_devices=n_devices, mem_capacity=int(mem_capacity),
-                   global_batch=int(global_batch))
+                   global_batch=int(global_batch), rec_alt=rec_alt)
 
 
 # ----------------------------------------------------------------------------
@@ -217,7 +244,7 @@ def _xf_ops(h, a, ff, inner, s, V, dtype_b=2.0, s_kv=None):
         return OpCost(flops=2 * t * h * 3 * inner / tp, mbytes=(t * h + 3 * t * inner / tp) * dtype_b,
                       tp_bwd_bytes=t * h * dtype_b, act=t * h * dtype_b, keep_frac=1.0,
                       out=3 * t * inner * dtype_b / tp, inp=t * h * dtype_b,
-                      params=(3 * h * inner + 3 * inner) / tp, workspace=ws)
+                      params=(3 * h * inner + 3 * inner) / tp, workspace=ws, part="col")
 
     def xq(b, tp):  # cross-attention q (decoder) + kv (encoder output)
         t, tk = b * s, b * s_kv
@@ -225,7 +252,7 @@ def _xf_ops(h, a, ff, inner, s, V, dtype_b=2.0, s_kv=None):
                       mbytes=(t * h + tk * h + 3 * t * inner / tp) * dtype_b,
                       tp_bwd_bytes=(t + tk) * h * dtype_b, act=(t + tk) * h * dtype_b, keep_frac=1.0,
                       out=(t + 2 * tk) * inner * dtype_b / tp, inp=t * h * dtype_b,
-                      params=3 * h * inner / tp, workspace=ws)
+                      params=3 * h * inner / tp, workspace=ws, part="col")
 
     def score(b, tp):
         t = b * s
@@ -256,7 +283,7 @@ def _xf_ops(h, a, ff, inner, s, V, dtype_b=2.0, s_kv=None):
         return OpCost(flops=2 * t * inner * h / tp, mbytes=(t * inner / tp + t * h) * dtype_b,
                       tp_fwd_bytes=t * h * dtype_b, act=t * inner * dtype_b / tp, keep_frac=0.5,
                       out=t * h * dtype_b, inp=t * inner * dtype_b, params=inner * h / tp + h,
-                      workspace=ws)
+                      workspace=ws, part="row")
 
     def resid(b, tp):
         t = b * s
@@ -268,7 +295,7 @@ def _xf_ops(h, a, ff, inner, s, V, dtype_b=2.0, s_kv=None):
         return OpCost(flops=2 * t * h * ff / tp, mbytes=(t * h + t * ff / tp) * dtype_b,
                       tp_bwd_bytes=t * h * dtype_b, act=t * h * dtype_b, keep_frac=1.0,
                       out=t * ff * dtype_b / tp, inp=t * h * dtype_b, params=(h * ff + ff) / tp,
-                      workspace=ws)
+                      workspace=ws, part="col")
 
     def gelu(b, tp):
         t = b * s
@@ -279,7 +306,8 @@ def _xf_ops(h, a, ff, inner, s, V, dtype_b=2.0, s_kv=None):
         t = b * s
         return OpCost(flops=2 * t * ff * h / tp, mbytes=(t * ff / tp + t * h) * dtype_b,
                       tp_fwd_bytes=t * h * dtype_b, act=t * ff * dtype_b / tp, keep_frac=0.5,
-                      out=t * h * dtype_b, inp=t * ff * dtype_b, params=ff * h / tp + h, workspace=ws)
+                      out=t * h * dtype_b, inp=t * ff * dtype_b, params=ff * h / tp + h, workspace=ws,
+                      part="row")
 
     def emb(b, tp):
         t = b * s
@@ -290,7 +318,7 @@ def _xf_ops(h, a, ff, inner, s, V, dtype_b=2.0, s_kv=None):
         t = b * s
         return OpCost(flops=2 * t * h * V / tp, mbytes=(t * h + 2 * t * V / tp * 2) * dtype_b,
                       tp_fwd_bytes=t * 12.0, act=t * h * dtype_b + t * V * 4.0 / tp, keep_frac=0.25,
-                      out=t * V * 4.0 / tp, inp=t * h * dtype_b, params=0.0, workspace=ws)
+                      out=t * V * 4.0 / tp, inp=t * h * dtype_b, params=0.0, workspace=ws, part="col")
 
     return dict(ln=ln, qkv=qkv, xq=xq, score=score, softmax=softmax, dropout=dropout, context=context,
                 outproj=outproj, resid=resid, fc1=fc1, gelu=gelu, fc2=fc2, emb=emb, head=head)
@@ -392,7 +420,7 @@ def wrn(n_devices=16, width=480, blocks=(3, 4, 23, 3), global_batch=1536, mem_ca
             return OpCost(flops=2 * b * Ho * Ho * cout * cin * k * k / tp, mbytes=inp + out,
                           tp_fwd_gather=inp if k > 1 else 0.0, tp_bwd_bytes=inp, act=inp,
                           keep_frac=0.5, out=out, inp=inp, params=cin * cout * k * k / tp,
-                          workspace=ws)
+                          workspace=ws, part="out")
         return f
 
     def elt(C, H, kind):

@@ -71,6 +71,17 @@ MUTATIONS = [
     ("r13-drop-reshard", "R13, P:L261",
      "rs = rec_field(P, dim[j], t, tpl[j], b, RESHARD);", "rs = 0;"),
     ("r9-no-gsum-check", "R9, P:L151", "if (gsum != (u64)P->G) reasons |= O_R_GSUM;", ";"),
+    ("dim-ignored-for-compute", "TP dimension, P:L263-265",
+     "u64 fc = rec_field(P, dim[j], t, tpl[j], b, FWD_COMP);", "u64 fc = rec_field(P, 0, t, tpl[j], b, FWD_COMP);"),
+    ("dim-ignored-for-memory", "TP dimension, P:L263-265",
+     "u64 act = rec_field(P, dim[j], t, tpl[j], b, ACT);", "u64 act = rec_field(P, 0, t, tpl[j], b, ACT);"),
+    ("dim-ignored-for-reshard", "TP dimension + R13",
+     "rs = rec_field(P, dim[j], t, tpl[j], b, RESHARD);", "rs = rec_field(P, 0, t, tpl[j], b, RESHARD);"),
+    ("dim-ignored-for-p2p-fwd", "TP dimension + R5",
+     "u64 v = rec_field(P, dim[last], t, tpl[last], (int)mbs_log2 - dpl[last], P2P_FWD);",
+     "u64 v = rec_field(P, 0, t, tpl[last], (int)mbs_log2 - dpl[last], P2P_FWD);"),
+    ("dim-of-previous-op", "TP dimension, P:L263-265",
+     "dim[j] = dims ? (dims[j] != 0) : 0;", "dim[j] = dims ? (dims[j > 0 ? j - 1 : 0] != 0) : 0;"),
     ("select-tie-highest-index", "R11 (selection)", "else better = g < best_idx;",
      "else better = g > best_idx;"),
     ("select-oom-before-feasible", "P:L138 better", "else if (k != best_cls) better = k < best_cls;",

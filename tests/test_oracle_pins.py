@@ -572,3 +572,103 @@ def test_heuristic1_memory_first_when_oom():
         assert out["stage_T"][0, 1] > out["stage_T"][0, 0]
         assert bool(out["info"][0] & oracle.INFO_OOM) == oom
         assert out["info"][0] & 0xFF == neck
+
+
+# --------------------------------------------------------------------------
+# Tensor-parallel partition dimension (§4.2): an op can run under its
+# alternative partition dimension (row- vs column-wise MatMul, input- vs output-channel
+# convolution); choosing it reads the records profiled for that dimension in every term.
+# --------------------------------------------------------------------------
+DEF_FP = [1, 2, 4, 8, 16, 0, 32, 64, 128, 256]        # fc fm bc bm act keep peak rs p2pf p2pb
+ALT_FP = [1000 * v for v in DEF_FP]
+
+
+def _dim_prof(op_type, n_tp=2, n_dp=2, G=2, Bg=8):
+    T = max(op_type) + 1
+    prof = mkprof({t: (lambda tpl, b: DEF_FP) for t in range(T)}, op_type, n_tp=n_tp, n_dp=n_dp,
+                  n_b=4, G=G, Bg=Bg)
+    prof.rec_alt = np.zeros_like(prof.rec)
+    prof.rec_alt[...] = np.array(ALT_FP, np.int64)
+    return prof
+
+
+@pytest.mark.parametrize("d0,d1", [(0, 0), (0, 1), (1, 0), (1, 1)])
+def test_dimension_fingerprint_two_stages(d0, d1):
+    """Two single-op stages: each stage's time reads its op's own dimension's compute,
+    collectives and send (stage 0 pays op 0's p2p_fwd, stage 1 op 1's p2p_bwd, R5)."""
+    prof = _dim_prof([0, 0])
+    out = oracle.evaluate(prof, np.array([cand([1, 1])], np.uint8), np.array([ai.header(1, 2)], np.uint64),
+                          full=True, dims=np.array([[d0, d1]], np.uint8))
+    assert out["info"][0] & oracle.INFO_INVALID == 0
+    fp = [DEF_FP, ALT_FP]
+    f0, f1 = fp[d0], fp[d1]
+    N = 4
+    S0 = f0[0] + f0[1] + f0[2] + f0[3] + f0[8]
+    S1 = f1[0] + f1[1] + f1[2] + f1[3] + f1[9]
+    assert list(out["stage_T"][0, :2]) == [S0 + S1 + (N - 1) * S0, S0 + S1 + (N - 1) * S1]
+    assert list(out["stage_comp"][0, :2]) == [N * (f0[0] + f0[2]), N * (f1[0] + f1[2])]
+    assert list(out["stage_comm"][0, :2]) == [N * (f0[1] + f0[3] + f0[8]), N * (f1[1] + f1[3] + f1[9])]
+    assert list(out["stage_mem"][0, :2]) == [min(2, N) * f0[4] + f0[6], 1 * f1[4] + f1[6]]
+
+
+@pytest.mark.parametrize("d1", [0, 1])
+def test_dimension_fingerprint_reshard_and_recompute(d1):
+    """One stage of two ops with a tp/dp change at op 1 (R13 reshard into op 1) and op 1
+    recomputed (R3, R4): the reshard, the recomputed forward and the kept /
+    transient bytes all come from op 1's dimension."""
+    prof = _dim_prof([0, 0])
+    row = [ai.code(1, 1, 0, 0), ai.code(0, 0, 1, 1)]  # (tp2, dp1) then (tp1, dp2), op 1 recomputed
+    out = oracle.evaluate(prof, np.array([row], np.uint8), np.array([ai.header(1, 1)], np.uint64),
+                          full=True, dims=np.array([[0, d1]], np.uint8))
+    assert out["info"][0] & oracle.INFO_INVALID == 0
+    f0, f1 = DEF_FP, [DEF_FP, ALT_FP][d1]
+    N = 4
+    S = (f0[0] + f0[1] + f0[2] + f0[3]) + (f1[0] + f1[1] + f1[2] + f1[3]) + (f1[0] + f1[1]) + f1[7]
+    assert int(out["stage_T"][0, 0]) == N * S
+    assert int(out["stage_mem"][0, 0]) == f0[4] + f1[5] + max(f0[6], f1[6] + f1[4] - f1[5])
+
+
+def test_dimension_choice_with_identical_records_changes_nothing():
+    prof = P.WORKLOADS["gpt3-1.3b"]()
+    prof.rec_alt = prof.rec.copy()
+    codes, hdr = ai.search_shaped(prof, 31, 0, 300, group_size=16)
+    rng = np.random.default_rng(2)
+    dims = rng.integers(0, 2, size=codes.shape, dtype=np.uint8)
+    a = oracle.evaluate(prof, codes, hdr, full=True)
+    b = oracle.evaluate(prof, codes, hdr, full=True, dims=dims)
+    for k in a:
+        assert np.array_equal(a[k], b[k]), k
+
+
+def test_dimension_flip_is_local_to_its_op():
+    """Flipping the dimension of op j (not a stage edge) changes stage i's per-microbatch time by
+    the op's own difference d = S_alt(j) - S_def(j): T_i by N d, every other T_k by d (Eq. 2)."""
+    prof = P.WORKLOADS["gpt3-1.3b"]()
+    codes, hdr = ai.search_shaped(prof, 33, 0, 200, group_size=16, invalid_permille=0)
+    base = oracle.evaluate(prof, codes, hdr, full=True)
+    rng = np.random.default_rng(4)
+    checked = 0
+    for c in range(len(hdr)):
+        if base["info"][c] & oracle.INFO_INVALID:
+            continue
+        heads = np.nonzero(codes[c] & 1)[0]
+        j = int(rng.integers(1, prof.n_ops - 1))
+        if j in heads or (j + 1) in heads or codes[c, j] & 0x10:
+            continue
+        if (codes[c, j] ^ codes[c, j - 1]) & 0xEE:
+            continue
+        dims = np.zeros((1, prof.n_ops), np.uint8)
+        dims[0, j] = 1
+        new = oracle.evaluate(prof, codes[c:c + 1], hdr[c:c + 1], full=True, dims=dims)
+        tpl, dpl = (int(codes[c, j]) >> 1) & 7, (int(codes[c, j]) >> 5) & 7
+        b = (int(hdr[c]) & 0xFF) - dpl
+        t = prof.op_type[j]
+        d = int(prof.rec_alt[t, tpl, b, :4].sum()) - int(prof.rec[t, tpl, b, :4].sum())
+        i = int(np.sum(codes[c, :j + 1] & 1)) - 1
+        N = prof.global_batch >> (int(hdr[c]) & 0xFF)
+        p = (int(hdr[c]) >> 8) & 0xFF
+        for k in range(p):
+            delta = int(new["stage_T"][0, k]) - int(base["stage_T"][c, k])
+            assert delta == (N * d if k == i else d)
+        checked += 1
+    assert checked > 50
