@@ -140,6 +140,23 @@ def tile(codes: np.ndarray):
     return out
 
 
+def dims_bytes(n, L):
+    return ((n + 31) // 32) * ((L + 15) // 16) * 64
+
+
+def tile_dims(dims: np.ndarray):
+    """Row-major dimension bytes [n][L] (nonzero = alternative) -> the tiled plane
+    (include/aceso.h: one little-endian u16 per candidate and 16-op chunk)."""
+    dims = np.ascontiguousarray(dims != 0, dtype=np.uint8)
+    n, L = dims.shape
+    nch = (L + 15) // 16
+    pad = np.zeros(((n + 31) // 32 * 32, nch * 16), np.uint8)
+    pad[:n, :L] = dims
+    bits = pad.reshape(-1, 32, nch, 16).astype(np.uint16) << np.arange(16, dtype=np.uint16)
+    plane = bits.sum(axis=3, dtype=np.uint16).transpose(0, 2, 1)  # [tile][chunk][lane]
+    return np.ascontiguousarray(plane).view(np.uint8).reshape(-1)
+
+
 def code(head, tpl, dpl, rc):
     return (head & 1) | ((tpl & 7) << 1) | ((rc & 1) << 4) | ((dpl & 7) << 5)
 

@@ -78,6 +78,13 @@ typedef struct {
   const int64_t *dps;       /* [n_types][n_tp][n_dp]: DP gradient all-reduce ns */
   int64_t mem_capacity;     /* C: device memory in bytes (OOM iff Mem_i > C, R10) */
   int64_t global_batch;     /* Bg: samples per iteration, 1..2^31             */
+  const int64_t *rec_alt;   /* nullable; [n_types][n_tp][n_b][ACESO_REC_FIELDS]: the records
+                               of each op type under its alternative tensor-parallel
+                               partition dimension (§4.2: row- vs column-wise
+                               MatMul, input- vs output-channel convolution), same range
+                               rules as rec; read for ops a candidate's dimension plane
+                               flips (aceso_eval_dims). Parameter bytes and DP sync are
+                               those of the default dimension. */
 } aceso_profile_desc;
 
 typedef struct aceso_ctx aceso_ctx; /* opaque; owned by the library */
@@ -254,6 +261,33 @@ int aceso_eval(aceso_ctx *ctx, const uint8_t *d_codes, const uint64_t *d_hdr, in
  * "dense kernel", "per-op kernel" or "scan kernel"; "" for a null context). Static
  * string, owned by the library. Host only. */
 const char *aceso_schedule_name(const aceso_ctx *ctx, uint32_t flags);
+
+/* ------------------------------------------------------------------------- */
+/* Tensor-parallel partition dimension per operator (§4.2 fine-tuning,        */
+/* P:L263-265).                                                               */
+/* ------------------------------------------------------------------------- */
+/* Dimension plane: one bit per op (1 = the op runs under its alternative
+ * partition dimension and reads rec_alt), tiled like the codes: the 16 bits of
+ * chunk k of candidate c are the little-endian u16 at
+ *   ((c / 32) * nch + k) * 64 + (c % 32) * 2,   bit (j % 16) = op j = 16 k + j % 16.
+ * Bits of pad ops (j >= n_ops) are ignored. */
+size_t aceso_dims_bytes(int64_t n, int32_t n_ops);
+
+/* Row-major dimension bytes [n][n_ops] (device, nonzero = alternative) -> the tiled
+ * plane (device, 2-byte aligned; pad bits zero). Async on `stream`. */
+int aceso_pack_dims(const uint8_t *d_rowmajor, int64_t n, int32_t n_ops, uint8_t *d_plane, void *stream);
+
+/* aceso_eval with a dimension plane (nullable: identical to aceso_eval). Every op
+ * whose bit is set uses the alternative-dimension records in every term of the
+ * model (its compute, collectives, memory, reshard and p2p). Same flags, outputs,
+ * selection and errors as aceso_eval, plus: ACESO_EINVAL if the context has no
+ * rec_alt or d_dims is not 2-byte aligned; ACESO_ERANGE if the profile's values
+ * exceed the 32-bit packed fields (see aceso_load_profile). Schedule: the dense
+ * kernel (per-op accumulation, records read per op under type or type + T), its
+ * tables in shared memory when they fit, else in global memory. */
+int aceso_eval_dims(aceso_ctx *ctx, const uint8_t *d_codes, const uint8_t *d_dims, const uint64_t *d_hdr,
+                    int64_t n, int64_t global_offset, int64_t n_total, uint32_t flags,
+                    const aceso_eval_out *out, void *d_sel, void *stream);
 
 /* Argmin over an already written summary (iter_ns, max_mem, info) of n
  * candidates; same order and result layout as the fused select. Async. */

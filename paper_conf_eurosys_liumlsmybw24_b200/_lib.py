@@ -15,13 +15,14 @@ INFO_INVALID = 1 << 17
 SYMBOLS = ["aceso_load_profile", "aceso_free", "aceso_tiled_bytes", "aceso_pack_rowmajor",
            "aceso_select_buf_bytes", "aceso_eval", "aceso_select", "aceso_decode_key",
            "aceso_last_error", "aceso_version", "aceso_hash", "aceso_visited_bytes", "aceso_dedup", "aceso_expand",
-           "aceso_enum_cuts_count", "aceso_enum_cuts", "aceso_schedule_name"]
+           "aceso_enum_cuts_count", "aceso_enum_cuts", "aceso_schedule_name", "aceso_dims_bytes",
+           "aceso_pack_dims", "aceso_eval_dims"]
 
 
 class ProfileDesc(ctypes.Structure):
     _fields_ = [("n_ops", c_i32), ("n_types", c_i32), ("n_tp", c_i32), ("n_dp", c_i32),
                 ("n_b", c_i32), ("n_devices", c_i32), ("op_type", P), ("rec", P), ("wmem", P),
-                ("dps", P), ("mem_capacity", c_i64), ("global_batch", c_i64)]
+                ("dps", P), ("mem_capacity", c_i64), ("global_batch", c_i64), ("rec_alt", P)]
 
 
 class EvalOut(ctypes.Structure):
@@ -68,6 +69,12 @@ def load():
     lib.aceso_version.restype = ctypes.c_char_p
     lib.aceso_schedule_name.argtypes = [P, c_u32]
     lib.aceso_schedule_name.restype = ctypes.c_char_p
+    lib.aceso_dims_bytes.argtypes = [c_i64, c_i32]
+    lib.aceso_dims_bytes.restype = c_sz
+    lib.aceso_pack_dims.argtypes = [P, c_i64, c_i32, P, P]
+    lib.aceso_pack_dims.restype = ctypes.c_int
+    lib.aceso_eval_dims.argtypes = [P, P, P, P, c_i64, c_i64, c_i64, c_u32, ctypes.POINTER(EvalOut), P, P]
+    lib.aceso_eval_dims.restype = ctypes.c_int
     lib.aceso_hash.argtypes = [P, P, c_i64, c_i32, P, P]
     lib.aceso_hash.restype = ctypes.c_int
     lib.aceso_visited_bytes.argtypes = [c_i64]

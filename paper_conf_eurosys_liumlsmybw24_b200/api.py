@@ -97,15 +97,17 @@ class Context:
         lib = L.load()
         self.device = int(device)
         self.profile = profile
+        alt = getattr(profile, "rec_alt", None)
         self._keep = [np.ascontiguousarray(profile.op_type, dtype=np.uint16),
                       np.ascontiguousarray(profile.rec, dtype=np.int64),
                       np.ascontiguousarray(profile.wmem, dtype=np.int64),
-                      np.ascontiguousarray(profile.dps, dtype=np.int64)]
-        ot, rec, wm, dps = self._keep
+                      np.ascontiguousarray(profile.dps, dtype=np.int64),
+                      None if alt is None else np.ascontiguousarray(alt, dtype=np.int64)]
+        ot, rec, wm, dps, ra = self._keep
         desc = L.ProfileDesc(int(ot.shape[0]), int(rec.shape[0]), int(rec.shape[1]), int(dps.shape[2]),
                              int(rec.shape[2]), int(profile.n_devices), ot.ctypes.data, rec.ctypes.data,
                              wm.ctypes.data, dps.ctypes.data, int(profile.mem_capacity),
-                             int(profile.global_batch))
+                             int(profile.global_batch), None if ra is None else ra.ctypes.data)
         h = ctypes.c_void_p()
         _check(lib.aceso_load_profile(ctypes.byref(desc), self.device, ctypes.byref(h)),
                "aceso_load_profile")
@@ -165,12 +167,14 @@ class Context:
     def eval(self, codes: torch.Tensor, hdr: torch.Tensor, n: int | None = None, global_offset: int = 0,
              n_total: int | None = None, summary: bool = True, full: bool = False, select: bool = True,
              out: Outputs | None = None, sel: torch.Tensor | None = None, stream=None,
-             dense_hint: bool = False, overlap_hint: bool = False):
+             dense_hint: bool = False, overlap_hint: bool = False, dims: torch.Tensor | None = None):
         """aceso_eval on tiled device codes and int64 device headers.
 
         dense_hint sets ACESO_HINT_DENSE (per-op kernel; identical results).
         overlap_hint sets ACESO_HINT_OVERLAP (the caller overlaps independent batches on
         several streams: throughput launch geometry; identical results).
+        dims: tiled dimension plane (aceso_eval_dims; pack_dims builds it): ops whose bit is set
+        run under their alternative tensor-parallel partition dimension.
         Returns (out, sel): the output arrays (or None) and the select buffer (or None)."""
         n = int(hdr.shape[0]) if n is None else int(n)
         n_total = global_offset + n if n_total is None else int(n_total)
@@ -184,10 +188,29 @@ class Context:
         if select and sel is None:
             sel = self.alloc_select(n)
         cs = out.c_struct() if out is not None else None
+        if dims is not None:
+            rc = L.load().aceso_eval_dims(self._h, _ptr(codes), _ptr(dims), _ptr(hdr), n, int(global_offset), n_total,
+                                          flags, ctypes.byref(cs) if cs is not None else None, _ptr(sel),
+                                          _stream(stream))
+            _check(rc, "aceso_eval_dims")
+            return out, sel
         rc = L.load().aceso_eval(self._h, _ptr(codes), _ptr(hdr), n, int(global_offset), n_total, flags,
                                  ctypes.byref(cs) if cs is not None else None, _ptr(sel), _stream(stream))
         _check(rc, "aceso_eval")
         return out, sel
+
+    def pack_dims(self, dims: torch.Tensor, plane: torch.Tensor | None = None, stream=None):
+        """aceso_pack_dims: device row-major [n, L] uint8 (nonzero = alternative dimension) ->
+        tiled dimension plane."""
+        assert dims.is_cuda and dims.dtype == torch.uint8 and dims.dim() == 2
+        n = int(dims.shape[0])
+        if plane is None:
+            plane = torch.zeros(max(2, int(L.load().aceso_dims_bytes(n, self.n_ops))), dtype=torch.uint8,
+                                device=self._dev)
+        dims = dims.contiguous()
+        _check(L.load().aceso_pack_dims(_ptr(dims), n, int(dims.shape[1]), _ptr(plane), _stream(stream)),
+               "aceso_pack_dims")
+        return plane
 
     def expand(self, bases: torch.Tensor, cands: torch.Tensor, ranks: torch.Tensor | None = None,
                n: int | None = None, tiled: torch.Tensor | None = None, hdr: torch.Tensor | None = None,

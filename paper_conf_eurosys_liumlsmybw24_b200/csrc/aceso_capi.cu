@@ -94,6 +94,20 @@ void *dense_kernel_for(uint32_t mode) {
   }
 }
 
+template <bool GT>
+void *dense_dims_kernel_for(uint32_t mode) {
+  switch (mode) {
+    case 1: return reinterpret_cast<void *>(&dense_kernel<1, 2, true, GT>);
+    case 2: return reinterpret_cast<void *>(&dense_kernel<2, 2, true, GT>);
+    case 3: return reinterpret_cast<void *>(&dense_kernel<3, 2, true, GT>);
+    case 4: return reinterpret_cast<void *>(&dense_kernel<4, 2, true, GT>);
+    case 5: return reinterpret_cast<void *>(&dense_kernel<5, 2, true, GT>);
+    case 6: return reinterpret_cast<void *>(&dense_kernel<6, 2, true, GT>);
+    case 7: return reinterpret_cast<void *>(&dense_kernel<7, 2, true, GT>);
+    default: return nullptr;
+  }
+}
+
 template <bool E64, int B>
 void *scan_kernel_for(uint32_t mode) {
   switch (mode) {
@@ -162,6 +176,10 @@ struct aceso_ctx {
   uint32_t qo_words, es;
   int e64;             // scan kernel: transient-memory table in u64 (values >= 2^32 units)
   uint32_t sc_resolve; // scan kernel: resolve recompute-only chunks in the compacted pass (ACESO_SCAN_NORESOLVE=1: in the walk)
+  int has_alt;         // alternative-dimension records loaded (aceso_eval_dims)
+  int dims_gt;         // aceso_eval_dims: dense tables in global memory (too large for shared memory)
+  size_t dims_smem[8];
+  int dims_max_ctas[8];
 };
 
 namespace {
@@ -247,25 +265,31 @@ int aceso_load_profile(const aceso_profile_desc *d, int cuda_device, aceso_ctx *
     if (d->op_type[j] >= T) return fail(ACESO_EINVAL, "op_type[%d] = %d >= n_types", j, d->op_type[j]);
 
   const uint64_t U32 = 0xffffffffull;
-  auto R = [&](int t, int tp, int b, int f) { return d->rec[(((int64_t)t * NT + tp) * NB + b) * ACESO_REC_FIELDS + f]; };
+  const int n_alt = d->rec_alt ? 2 : 1;  // record sets: default dimension (+ the alternative)
+  auto RA = [&](int alt, int t, int tp, int b, int f) {
+    return (alt ? d->rec_alt : d->rec)[(((int64_t)t * NT + tp) * NB + b) * ACESO_REC_FIELDS + f];
+  };
+  auto R = [&](int t, int tp, int b, int f) { return RA(0, t, tp, b, f); };
   uint64_t maxSop = 0, maxRes = 0, maxP2P = 0, maxA = 0, maxE = 0, maxW = 0, maxD = 0;
   for (int t = 0; t < T; ++t)
     for (int tp = 0; tp < NT; ++tp) {
+      for (int alt = 0; alt < n_alt; ++alt)
       for (int b = 0; b < NB; ++b) {
         for (int f = 0; f < ACESO_REC_FIELDS; ++f) {
-          int64_t v = R(t, tp, b, f);
+          int64_t v = RA(alt, t, tp, b, f);
           const bool memf = (f == ACESO_F_ACT || f == ACESO_F_KEEP || f == ACESO_F_PEAK);
           if (v < 0 || (uint64_t)v > (memf ? (1ull << 40) : U32))
-            return fail(ACESO_ERANGE, "rec[%d][%d][%d][%d] = %lld out of range", t, tp, b, f, (long long)v);
+            return fail(ACESO_ERANGE, "%s[%d][%d][%d][%d] = %lld out of range", alt ? "rec_alt" : "rec", t, tp, b,
+                        f, (long long)v);
         }
-        uint64_t fc = R(t, tp, b, 0), fm = R(t, tp, b, 1), bc = R(t, tp, b, 2), bm = R(t, tp, b, 3);
-        uint64_t act = R(t, tp, b, 4), keep = R(t, tp, b, 5), peak = R(t, tp, b, 6);
-        if (keep > act) return fail(ACESO_ERANGE, "keep > act at rec[%d][%d][%d]", t, tp, b);
+        uint64_t fc = RA(alt, t, tp, b, 0), fm = RA(alt, t, tp, b, 1), bc = RA(alt, t, tp, b, 2), bm = RA(alt, t, tp, b, 3);
+        uint64_t act = RA(alt, t, tp, b, 4), keep = RA(alt, t, tp, b, 5), peak = RA(alt, t, tp, b, 6);
+        if (keep > act) return fail(ACESO_ERANGE, "keep > act at %s[%d][%d][%d]", alt ? "rec_alt" : "rec", t, tp, b);
         uint64_t s1 = 2 * (fc + fm) + bc + bm;
         uint64_t e1 = peak + act - keep;
         maxSop = std::max(maxSop, s1);
-        maxRes = std::max(maxRes, (uint64_t)R(t, tp, b, 7));
-        maxP2P = std::max(maxP2P, (uint64_t)std::max(R(t, tp, b, 8), R(t, tp, b, 9)));
+        maxRes = std::max(maxRes, (uint64_t)RA(alt, t, tp, b, 7));
+        maxP2P = std::max(maxP2P, (uint64_t)std::max(RA(alt, t, tp, b, 8), RA(alt, t, tp, b, 9)));
         maxA = std::max(maxA, act);
         maxE = std::max(maxE, e1);
       }
@@ -284,7 +308,8 @@ int aceso_load_profile(const aceso_profile_desc *d, int cuda_device, aceso_ctx *
     auto tz = [&](int64_t v) { if (v != 0) ms = std::min<uint32_t>(ms, (uint32_t)__builtin_ctzll((uint64_t)v)); };
     for (int t = 0; t < T; ++t)
       for (int tp = 0; tp < NT; ++tp) {
-        for (int b = 0; b < NB; ++b) { tz(R(t, tp, b, 4)); tz(R(t, tp, b, 5)); tz(R(t, tp, b, 6)); }
+        for (int alt = 0; alt < n_alt; ++alt)
+          for (int b = 0; b < NB; ++b) { tz(RA(alt, t, tp, b, 4)); tz(RA(alt, t, tp, b, 5)); tz(RA(alt, t, tp, b, 6)); }
         tz(d->wmem[((int64_t)t * NT + tp) * 2]);
         tz(d->wmem[((int64_t)t * NT + tp) * 2 + 1]);
       }
@@ -353,14 +378,16 @@ int aceso_load_profile(const aceso_profile_desc *d, int cuda_device, aceso_ctx *
   // the per-op kernel stages its tables in shared memory; larger profiles use the event
   // kernel only (its tables are in global memory)
   const bool quad_ok = tab.bytes_full + kRingBytesPerCta + 16384u <= 220u * 1024u;
+  // dense-kernel tables: 2T types when alternative-dimension records are given (type + T)
+  const uint32_t T2 = (uint32_t)(n_alt * T);
   tab.dOff = a16(tab.offK + bytesK);
   tab.dR = 0;
-  tab.dD = tab.dR + bytesR;
-  tab.dK = tab.dD + bytesD;
-  tab.dT = tab.dK + bytesK;
+  tab.dD = tab.dR + RUNS * T2 * S;
+  tab.dK = tab.dD + (uint32_t)NT * T2 * S;
+  tab.dT = tab.dK + RUNS * T2 * 16;
   tab.dbytes = tab.dT + bytesT;
   tab.dF = tab.dbytes;
-  tab.dbytes_full = tab.dF + bytesF;
+  tab.dbytes_full = tab.dF + a16(RUNS * T2 * 8);
   const bool dense_ok = tab.dbytes_full + kRingBytesPerCta + 16384u <= 220u * 1024u;
   const uint32_t blob_bytes = tab.dOff + tab.dbytes_full;
   std::vector<uint32_t> blob(blob_bytes / 4, 0u);
@@ -395,27 +422,35 @@ int aceso_load_profile(const aceso_profile_desc *d, int cuda_device, aceso_ctx *
         k[0] = (uint32_t)R(t, tp, b, 7);
         k[1] = (uint32_t)R(t, tp, b, 8);
         k[2] = (uint32_t)R(t, tp, b, 9);
-        // dense-kernel copies, type-major
-        const uint32_t tr = (uint32_t)t * RUNS + (uint32_t)(b * NT + tp);  // (type, run) index
+      }
+  // dense-kernel copies, type-major; types T..2T-1: the alternative dimension's records (same
+  // parameter bytes and DP sync: the partition dimension does not change the weights per GPU)
+  for (uint32_t t2 = 0; t2 < T2; ++t2)
+    for (int b = 0; b < NB; ++b)
+      for (int tp = 0; tp < NT; ++tp) {
+        const int t = (int)(t2 % (uint32_t)T), alt = t2 >= (uint32_t)T;
+        auto F = [&](int f) { return (uint64_t)RA(alt, t, tp, b, f); };
+        const uint32_t tr = t2 * RUNS + (uint32_t)(b * NT + tp);  // (type, run) index
         for (int rc = 0; rc < 2; ++rc) {
+          const uint64_t Fw = F(0) + F(1);
           uint32_t *r = &blob[(tab.dOff + tab.dR) / 4 + tr * 8 + rc * 4];
-          r[0] = (uint32_t)rec_S(t, tp, b, rc);
-          r[1] = (uint32_t)rec_A(t, tp, b, rc);
-          r[2] = (uint32_t)rec_e(t, tp, b, rc);
+          r[0] = (uint32_t)(Fw + F(2) + F(3) + (rc ? Fw : 0));
+          r[1] = (uint32_t)((rc ? F(5) : F(4)) >> ms);
+          r[2] = (uint32_t)((F(6) + (rc ? F(4) - F(5) : 0)) >> ms);
           r[3] = (uint32_t)rec_W(t, tp);
-          blob[(tab.dOff + tab.dF) / 4 + tr * 2 + rc] = (uint32_t)rec_C(t, tp, b, rc);
+          blob[(tab.dOff + tab.dF) / 4 + tr * 2 + rc] = (uint32_t)(F(0) + F(2) + (rc ? F(0) : 0));
         }
         uint32_t *dk = &blob[(tab.dOff + tab.dK) / 4 + tr * 4];
-        dk[0] = k[0];
-        dk[1] = k[1];
-        dk[2] = k[2];
+        dk[0] = (uint32_t)F(7);
+        dk[1] = (uint32_t)F(8);
+        dk[2] = (uint32_t)F(9);
       }
   for (int tp = 0; tp < NT; ++tp)
     for (int t = 0; t < T; ++t)
-      for (int dp = 0; dp < ND; ++dp)
-      {
+      for (int dp = 0; dp < ND; ++dp) {
         blob[(tab.offD + ((uint32_t)tp * T + t) * S) / 4 + dp] = (uint32_t)dps_of(t, tp, dp);
-        blob[(tab.dOff + tab.dD) / 4 + ((uint32_t)t * NT + tp) * 8 + dp] = (uint32_t)dps_of(t, tp, dp);
+        for (int alt = 0; alt < n_alt; ++alt)
+          blob[(tab.dOff + tab.dD) / 4 + (((uint32_t)(t + alt * T)) * NT + tp) * 8 + dp] = (uint32_t)dps_of(t, tp, dp);
       }
   {
     uint16_t *tt = reinterpret_cast<uint16_t *>(&blob[tab.offT / 4]);
@@ -698,6 +733,8 @@ int aceso_load_profile(const aceso_profile_desc *d, int cuda_device, aceso_ctx *
   ctx->e64 = e64 ? 1 : 0;
   ctx->qo_words = (uint32_t)nqs;
   ctx->sc_resolve = getenv("ACESO_SCAN_NORESOLVE") ? 0u : 1u;
+  ctx->has_alt = d->rec_alt ? 1 : 0;
+  ctx->dims_gt = dense_ok ? 0 : 1;
   // default schedule: the event kernel (its packed tables hold the profile), for short models
   // (<= 64 ops) the dense kernel's branch-free per-op accumulation; the scan kernel (exact
   // 64-bit tables) for profiles whose per-op values exceed the packed 32-bit fields
@@ -784,6 +821,19 @@ int aceso_load_profile(const aceso_profile_desc *d, int cuda_device, aceso_ctx *
         }
         ctx->max_ctas[kern][mode] = occ * ctx->sms;
       }
+    for (uint32_t mode = 1; mode < 8 && rc == ACESO_OK && ctx->has_alt && packed_ok; ++mode) {
+      const size_t smem = (ctx->dims_gt ? 0 : ((mode & ACESO_OUT_FULL) ? tab.dbytes_full : tab.dbytes)) + kRingBytesPerCta;
+      void *k = ctx->dims_gt ? dense_dims_kernel_for<true>(mode) : dense_dims_kernel_for<false>(mode);
+      e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+      int occ = 0;
+      if (e == cudaSuccess) e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k, kThreads, smem);
+      if (e != cudaSuccess || occ < 1) {
+        rc = fail(ACESO_ECUDA, "kernel setup (dimension plane, mode %u, %zu B smem): %s", mode, smem, cudaGetErrorString(e));
+        break;
+      }
+      ctx->dims_smem[mode] = smem;
+      ctx->dims_max_ctas[mode] = occ * ctx->sms;
+    }
   } while (0);
   cudaSetDevice(prev_dev);
   if (rc != ACESO_OK) {
@@ -814,7 +864,7 @@ size_t aceso_select_buf_bytes(const aceso_ctx *ctx, int64_t n) {
   if (!ctx) return 0;
   int m = 0;
   for (int kern = 0; kern < 4; ++kern)
-    for (int k = 1; k < 8; ++k) m = std::max(m, ctx->max_ctas[kern][k]);
+    for (int k = 1; k < 8; ++k) m = std::max(m, std::max(ctx->max_ctas[kern][k], ctx->dims_max_ctas[k]));
   m = std::max(m, 4 * ctx->sms);  // per-CTA partials of the eval kernels; select kernel grid
   return (size_t)kSelPartialOff + 16 * (size_t)m;
 }
@@ -868,6 +918,63 @@ int aceso_eval(aceso_ctx *ctx, const uint8_t *d_codes, const uint64_t *d_hdr, in
                                    reinterpret_cast<cudaStream_t>(stream));
   if (prev != ctx->device) cudaSetDevice(prev);
   if (e != cudaSuccess) return fail(ACESO_ECUDA, "eval launch: %s", cudaGetErrorString(e));
+  return ACESO_OK;
+}
+
+size_t aceso_dims_bytes(int64_t n, int32_t n_ops) {
+  if (n < 0 || n_ops < 1) return 0;
+  return (size_t)((n + 31) / 32) * (size_t)((n_ops + 15) / 16) * 64;
+}
+
+int aceso_pack_dims(const uint8_t *d_rowmajor, int64_t n, int32_t n_ops, uint8_t *d_plane, void *stream) {
+  if (n < 0 || n_ops < 1 || n_ops > kMaxOps || (n > 0 && (!d_rowmajor || !d_plane))) return fail(ACESO_EINVAL, "bad argument");
+  if (((uintptr_t)d_plane & 1) != 0) return fail(ACESO_EINVAL, "dimension plane not 2-byte aligned");
+  if (n == 0) return ACESO_OK;
+  const int64_t total = (int64_t)aceso_dims_bytes(n, n_ops) / 2;
+  const int grid = (int)std::min<int64_t>((total + 255) / 256, 148 * 16);
+  pack_dims_kernel<<<grid, 256, 0, reinterpret_cast<cudaStream_t>(stream)>>>(d_rowmajor, n, n_ops,
+                                                                            reinterpret_cast<uint16_t *>(d_plane), total);
+  cudaError_t e = cudaGetLastError();
+  if (e != cudaSuccess) return fail(ACESO_ECUDA, "pack_dims launch: %s", cudaGetErrorString(e));
+  return ACESO_OK;
+}
+
+int aceso_eval_dims(aceso_ctx *ctx, const uint8_t *d_codes, const uint8_t *d_dims, const uint64_t *d_hdr,
+                    int64_t n, int64_t global_offset, int64_t n_total, uint32_t flags,
+                    const aceso_eval_out *out, void *d_sel, void *stream) {
+  if (!d_dims) return aceso_eval(ctx, d_codes, d_hdr, n, global_offset, n_total, flags, out, d_sel, stream);
+  if (!ctx) return fail(ACESO_EINVAL, "null context");
+  if (!ctx->has_alt) return fail(ACESO_EINVAL, "dimension plane given but the profile has no rec_alt");
+  if (!ctx->packed_ok) return fail(ACESO_ERANGE, "dimension plane: the profile's values exceed the dense kernel's 32-bit fields");
+  if (((uintptr_t)d_dims & 1) != 0) return fail(ACESO_EINVAL, "dimension plane not 2-byte aligned");
+  if (n < 0 || global_offset < 0 || n_total < global_offset + n) return fail(ACESO_EINVAL, "bad n / global_offset / n_total");
+  if (n_total >= (1ll << 40)) return fail(ACESO_EINVAL, "n_total >= 2^40");
+  if (n >= (1ll << 37)) return fail(ACESO_EINVAL, "n >= 2^37");
+  const uint32_t mode = flags & 7u;
+  if (mode == 0 || (flags & ~(7u | ACESO_HINT_DENSE | ACESO_HINT_OVERLAP))) return fail(ACESO_EINVAL, "bad flags 0x%x", flags);
+  if (n > 0 && (!d_codes || !d_hdr)) return fail(ACESO_EINVAL, "null codes/headers");
+  if ((mode & (ACESO_OUT_SUMMARY | ACESO_OUT_FULL)) && !out) return fail(ACESO_EINVAL, "null outputs");
+  if ((mode & ACESO_OUT_SUMMARY) && n > 0 && (!out->iter_ns || !out->max_mem || !out->info)) return fail(ACESO_EINVAL, "null summary array");
+  if (mode & ACESO_OUT_FULL) {
+    if (out->p_max < ctx->G) return fail(ACESO_EINVAL, "p_max %d < n_devices %d", out->p_max, ctx->G);
+    if (n > 0 && (!out->stage_T || !out->stage_mem || !out->stage_comp || !out->stage_comm)) return fail(ACESO_EINVAL, "null stage array");
+  }
+  if ((mode & ACESO_FUSED_SELECT) && !d_sel) return fail(ACESO_EINVAL, "null select buffer");
+  if (((uintptr_t)d_codes & 15) != 0) return fail(ACESO_EINVAL, "codes not 16-byte aligned");
+  EvalParams P = make_params(ctx, n, global_offset, n_total, out, d_sel);
+  P.codes = reinterpret_cast<const uint4 *>(d_codes);
+  P.hdr = d_hdr;
+  P.dims = d_dims;
+  const int64_t need = (P.n_tiles + kWarps - 1) / kWarps;
+  const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(need, ctx->dims_max_ctas[mode]));
+  int prev = 0;
+  CUDA_TRY(cudaGetDevice(&prev));
+  if (prev != ctx->device) CUDA_TRY(cudaSetDevice(ctx->device));
+  void *args[] = {&P};
+  void *k = ctx->dims_gt ? dense_dims_kernel_for<true>(mode) : dense_dims_kernel_for<false>(mode);
+  cudaError_t e = cudaLaunchKernel(k, dim3(grid), dim3(kThreads), args, ctx->dims_smem[mode], reinterpret_cast<cudaStream_t>(stream));
+  if (prev != ctx->device) cudaSetDevice(prev);
+  if (e != cudaSuccess) return fail(ACESO_ECUDA, "eval_dims launch: %s", cudaGetErrorString(e));
   return ACESO_OK;
 }
 

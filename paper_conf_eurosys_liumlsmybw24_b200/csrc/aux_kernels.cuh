@@ -55,4 +55,23 @@ __global__ void __launch_bounds__(256) pack_kernel(const uint8_t *__restrict__ s
   }
 }
 
+// row-major dimension bytes [n][L] -> tiled plane: one u16 per (candidate, 16-op chunk)
+__global__ void __launch_bounds__(256) pack_dims_kernel(const uint8_t *__restrict__ src, int64_t n, int L,
+                                                        uint16_t *__restrict__ dst, int64_t total) {
+  const int nch = (L + 15) / 16;
+  for (int64_t u = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; u < total; u += (int64_t)gridDim.x * blockDim.x) {
+    // u enumerates the plane: ((tile * nch + k) * 32 + lane)
+    const int64_t lane = u & 31, tk = u >> 5;
+    const int64_t tile = tk / nch, k = tk % nch;
+    const int64_t c = tile * 32 + lane;
+    uint32_t v = 0;
+    if (c < n)
+      for (int i = 0; i < 16; ++i) {
+        const int64_t j = k * 16 + i;
+        if (j < L && src[c * L + j]) v |= 1u << i;
+      }
+    dst[u] = (uint16_t)v;
+  }
+}
+
 }  // namespace aceso

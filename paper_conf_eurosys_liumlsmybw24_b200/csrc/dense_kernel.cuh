@@ -18,12 +18,34 @@
 //   every op      : S += fwd+bwd (+fwd if rc, R7), A += act or keep (R3),
 //                   E = max(E, peak (+act-keep if rc)) (R4), W += param+opt, D += DP sync (R6)
 // Readings R1-R13, R18-R20 in DESIGN.md §3.
+//
+// Tensor-parallel partition dimension (§4.2): with DIMS the candidates carry a
+// dimension bit per op (aceso_eval_dims); an op on its alternative dimension reads the records
+// of type + T (the tables then hold 2T types: the alternative dimension's records, same
+// parameter and DP-sync entries). GT: the tables stay in global memory (L2) when they do not
+// fit shared memory (e.g. Wide-ResNet with alternative records).
 #pragma once
+#include <type_traits>
+
 #include "eval_kernel.cuh"
 
 namespace aceso {
 
-template <uint32_t MODE, int MINB>
+// table accessors: shared memory (staged once per CTA) or global memory (L2-resident)
+struct DTabS {
+  uint32_t b;
+  __device__ __forceinline__ uint32_t u32(uint32_t o) const { return lds32(b + o); }
+  __device__ __forceinline__ uint2 u64(uint32_t o) const { return lds64(b + o); }
+  __device__ __forceinline__ uint4 u128(uint32_t o) const { return lds128(b + o); }
+};
+struct DTabG {
+  const unsigned char *b;
+  __device__ __forceinline__ uint32_t u32(uint32_t o) const { return __ldg(reinterpret_cast<const uint32_t *>(b + o)); }
+  __device__ __forceinline__ uint2 u64(uint32_t o) const { return __ldg(reinterpret_cast<const uint2 *>(b + o)); }
+  __device__ __forceinline__ uint4 u128(uint32_t o) const { return __ldg(reinterpret_cast<const uint4 *>(b + o)); }
+};
+
+template <uint32_t MODE, int MINB, bool DIMS = false, bool GT = false>
 __global__ void __launch_bounds__(kThreads, MINB) dense_kernel(const __grid_constant__ EvalParams P) {
   extern __shared__ __align__(128) unsigned char sm_raw[];
   __shared__ __align__(8) uint64_t s_tbar;
@@ -32,10 +54,13 @@ __global__ void __launch_bounds__(kThreads, MINB) dense_kernel(const __grid_cons
   __shared__ int64_t s_idx[kWarps];
 
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-  const uint32_t stage_bytes = (MODE & kFull) ? P.tab.dbytes_full : P.tab.dbytes;
+  const uint32_t stage_bytes = GT ? 0u : (MODE & kFull) ? P.tab.dbytes_full : P.tab.dbytes;
   const uint32_t sb = smem_addr(sm_raw);
-  const uint32_t DR = sb + P.tab.dR, DD = sb + P.tab.dD, DK = sb + P.tab.dK, DT = sb + P.tab.dT,
-                 DF = sb + P.tab.dF;
+  typename std::conditional<GT, DTabG, DTabS>::type tb;
+  if constexpr (GT) tb.b = reinterpret_cast<const unsigned char *>(P.blob) + P.tab.dOff;
+  else tb.b = sb;
+  const uint32_t DR = P.tab.dR, DD = P.tab.dD, DK = P.tab.dK, DT = P.tab.dT, DF = P.tab.dF;
+  const uint32_t T = (uint32_t)P.T;  // alternative-dimension records: type + T
   const uint32_t runs = (uint32_t)(P.n_b * P.n_tp);
   const uint32_t ring = sb + stage_bytes + (uint32_t)warp * kRingSlots * kSlotBytes;
   Smem sm;  // init_cand's table bases (unused here)
@@ -52,8 +77,12 @@ __global__ void __launch_bounds__(kThreads, MINB) dense_kernel(const __grid_cons
   __syncthreads();
   if (threadIdx.x == 0) {
     const uint32_t bar = smem_addr(&s_tbar);
-    mbar_expect_tx(bar, stage_bytes);
-    bulk_g2s(sb, reinterpret_cast<const unsigned char *>(P.blob) + P.tab.dOff, stage_bytes, bar);
+    if (GT) {
+      asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(bar) : "memory");
+    } else {
+      mbar_expect_tx(bar, stage_bytes);
+      bulk_g2s(sb, reinterpret_cast<const unsigned char *>(P.blob) + P.tab.dOff, stage_bytes, bar);
+    }
   }
 
   const uint32_t nch = (uint32_t)P.nch;
@@ -112,25 +141,25 @@ __global__ void __launch_bounds__(kThreads, MINB) dense_kernel(const __grid_cons
     const uint32_t kofs = DK + tr * 16u;
     if ((c & 1u) || j == 0) {
       if ((c & 1u) && j > 0) {
-        s.S += lds32(pk + 4u);  // R5: p2p_fwd of the stage's last op (j-1)
+        s.S += tb.u32(pk + 4u);  // R5: p2p_fwd of the stage's last op (j-1)
         stage_commit<MODE>(s, P, cand, active, false);
         s.i += 1;
-        s.S += lds32(kofs + 8u);  // R5: p2p_bwd of the stage's first op
+        s.S += tb.u32(kofs + 8u);  // R5: p2p_bwd of the stage's first op
       }
       s.gst = gg;
       s.gsum += 1u << gg;  // R9
       s.nheads += c & 1u;
     } else {
       if (gg != s.gst) s.reasons |= ACESO_R_GSTAGE;  // P:L151 in-stage symmetry
-      if ((c ^ prev) & 0xeeu) s.S += lds32(kofs);     // R13: reshard into op j
+      if ((c ^ prev) & 0xeeu) s.S += tb.u32(kofs);     // R13: reshard into op j
     }
-    const uint4 r = lds128(DR + tr * 32u + rc * 16u);
+    const uint4 r = tb.u128(DR + tr * 32u + rc * 16u);
     s.S += r.x;
     s.A += r.y;
     s.E = max(s.E, r.z);
     s.W += r.w;
-    s.D += lds32(DD + (ty * n_tp + tplc) * 32u + dpl * 4u);
-    if (MODE & kFull) s.comp += lds32(DF + tr * 8u + rc * 4u);
+    s.D += tb.u32(DD + (ty * n_tp + tplc) * 32u + dpl * 4u);
+    if (MODE & kFull) s.comp += tb.u32(DF + tr * 8u + rc * 4u);
     prev = c;
     pk = kofs;
   };
@@ -149,21 +178,27 @@ __global__ void __launch_bounds__(kThreads, MINB) dense_kernel(const __grid_cons
 #pragma unroll 1
     for (uint32_t ch = a; ch < b; ++ch) {
       const uint4 w4 = lds128(slot_a + (ch - a) * 512u);
+      // dimension bits of the chunk's 16 ops (bit k = op 16 ch + k): alternative type = type + T
+      uint32_t dm = 0;
+      if (DIMS)
+        dm = __ldg(reinterpret_cast<const unsigned short *>(P.dims + ((size_t)tile * nch + ch) * 64u) + lane);
       const uint32_t nq = min(4u, (L - ch * 16u + 3u) >> 2);  // quads inside L
 #pragma unroll 1
       for (uint32_t q = 0; q < nq; ++q) {
         const uint32_t w = q == 0 ? w4.x : q == 1 ? w4.y : q == 2 ? w4.z : w4.w;
         const uint32_t j0 = ch * 16u + q * 4u;
-        const uint2 tt = lds64(DT + 2u * j0);  // the quad's 4 u16 types
+        const uint2 tt = tb.u64(DT + 2u * j0);  // the quad's 4 u16 types
+        const uint32_t dq = DIMS ? (dm >> (4u * q)) & 0xfu : 0u;
         if (j0 + 4u <= L) {  // full quad
-          op(j0, w & 0xffu, tt.x & 0xffffu);
-          op(j0 + 1u, (w >> 8) & 0xffu, tt.x >> 16);
-          op(j0 + 2u, (w >> 16) & 0xffu, tt.y & 0xffffu);
-          op(j0 + 3u, w >> 24, tt.y >> 16);
+          op(j0, w & 0xffu, (tt.x & 0xffffu) + (dq & 1u) * T);
+          op(j0 + 1u, (w >> 8) & 0xffu, (tt.x >> 16) + ((dq >> 1) & 1u) * T);
+          op(j0 + 2u, (w >> 16) & 0xffu, (tt.y & 0xffffu) + ((dq >> 2) & 1u) * T);
+          op(j0 + 3u, w >> 24, (tt.y >> 16) + (dq >> 3) * T);
         } else {
 #pragma unroll 1
           for (uint32_t k = 0; j0 + k < L; ++k)
-            op(j0 + k, (w >> (8u * k)) & 0xffu, (k < 2 ? tt.x >> (16u * k) : tt.y >> (16u * (k - 2))) & 0xffffu);
+            op(j0 + k, (w >> (8u * k)) & 0xffu,
+               ((k < 2 ? tt.x >> (16u * k) : tt.y >> (16u * (k - 2))) & 0xffffu) + ((dq >> k) & 1u) * T);
         }
       }
     }
