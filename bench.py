@@ -540,14 +540,23 @@ def measure_search(A, ctx, prof, budget):
         o = ev.evaluate(r0[0][None, :], np.array([S.header(r0[1], p)], np.uint64))
         pf = S.perf_of(int(o["info"][0]), o["iter"][0], o["max_mem"][0])
         init_best = pf if init_best is None or pf < init_best else init_best
+    t1 = time.perf_counter()
+    dims, dperf, dst = S.finetune_dims(prof, ev, res.codes, res.mbs, max_rounds=16)
+    t_dims = time.perf_counter() - t1
     return {"time_s": st["time_s"], "time_to_best_s": st["time_to_best_s"], "evaluated": st["evaluated"],
             "batches": st["batches"], "improvements": st["improvements"],
             "best": {"class": res.perf[0], "cost": res.perf[1], "iter_ns": res.iter_ns,
                      "p": int((res.codes & 1).sum()), "mbs_log2": res.mbs},
             "initial_best": {"class": init_best[0], "cost": init_best[1]} if init_best else None,
-            "note": "batched Alg. 1/2 (MaxHops 7) over all stage counts on one GPU, stops after 8 hops "
-                    "without a new best or at the budget; context: the paper's searches use a 200 s "
-                    "budget on its own hosts (P:L313, P:L339)"}
+            "dims_finetune": {"time_s": t_dims, "rounds": dst["rounds"], "evaluated": dst["evaluated"],
+                              "switched_ops": len(dst["switched"]), "best": {"class": dperf[0], "cost": dperf[1]},
+                              "note": "op-level tensor-parallel dimension fine-tune of the best "
+                                      "configuration (§4.2, P:L263-265), aceso_eval_dims"},
+            "note": "batched Alg. 1/2 (MaxHops 7) over all stage counts on one GPU: Heuristic-2 over "
+                    "computation, communication and memory, inc/dec-rc attached to the primitives "
+                    "(P:L273), root retries on the next resource and the secondary bottleneck "
+                    "(P:L219); stops after 8 hops without a new best or at the budget; context: the "
+                    "paper's searches use a 200 s budget on its own hosts (P:L313, P:L339)"}
 
 
 def measure_dp(A, ctx, prof, budget, search=None):

@@ -165,6 +165,35 @@ def _rc_order(prof, codes, s, mbs, st=None):
     return j[np.argsort(-act, kind="stable")]
 
 
+RESOURCES = ("comp", "comm", "mem")
+
+
+def resource_order(info, comp, comm, mem, p, bn):
+    """Heuristic-2: the bottleneck stage's resources by consumption proportion
+    (its consumption divided by the consumption of all stages), highest first; an OOM
+    configuration puts memory first (Heuristic-1's safety-first priority). Without
+    per-stage memory (mem None) only computation and communication are ranked."""
+    shares = {"comp": int(comp[bn]) / max(int(comp[:p].sum()), 1),
+              "comm": int(comm[bn]) / max(int(comm[:p].sum()), 1)}
+    if mem is not None:
+        shares["mem"] = int(mem[bn]) / max(int(mem[:p].sum()), 1)
+    order = sorted(shares, key=lambda r: -shares[r])  # stable: comp, comm, mem on ties
+    if info & INFO_OOM:
+        order = ["mem"] + [r for r in order if r != "mem"]
+    return order
+
+
+def bottleneck_rank(info, mem, stage_time, p, rank):
+    """The stage of Heuristic-1's order at `rank` (0: the bottleneck of the info word; 1: the
+    secondary bottleneck): stages by memory if OOM, else by time, highest first,
+    lowest index on ties."""
+    if rank == 0 or p <= 1:
+        return int(info & 0xFF)
+    key = mem if info & INFO_OOM else stage_time
+    order = sorted(range(p), key=lambda i: (-int(key[i]), i))
+    return order[min(rank, p - 1)]
+
+
 class Primitives:
     def __init__(self, prof, heuristic2=True, max_k=None):
         self.prof = prof
@@ -290,7 +319,7 @@ class Primitives:
         return out
 
 
-    def describe_all(self, codes, mbs, info, comp, comm, stage_time):
+    def describe_all(self, codes, mbs, info, comp, comm, stage_time, mem=None, bn=None, resource=None):
         """The candidates of apply_all, in the same order, as base + patches
         (candidates.CAND_DTYPE rows with base = 0) plus the two rank rows of this base
         used by the recompute patches. Nothing is materialised on the host; the families
@@ -301,11 +330,16 @@ class Primitives:
         L = len(codes)
         heads, ends = stages_of(codes)
         p = len(heads)
-        bn = int(info & 0xFF)
+        if bn is None:
+            bn = int(info & 0xFF)
         if bn >= p:
             bn = 0
         oom = bool(info & INFO_OOM)
-        if oom:
+        if resource is not None:
+            want = {resource}
+        elif mem is not None:
+            want = {resource_order(info, comp, comm, mem, p, bn)[0]}
+        elif oom:
             want = {"mem"}
         else:
             cs, ms = max(int(comp[:p].sum()), 1), max(int(comm[:p].sum()), 1)
@@ -462,8 +496,10 @@ class GPUEvaluator:
         self.calls = 0
         self.evaluated = 0
 
-    def evaluate(self, codes, hdr):
-        from .api import as_u32, as_u64
+    def evaluate(self, codes, hdr, dims=None, hashes=False):
+        """Row-major codes [n][L] (+ optional dimension bytes [n][L]) -> FULL outputs
+        (+ configuration hashes, aceso_hash)."""
+        from .api import as_u32, as_u64, hash_candidates
         n = int(hdr.shape[0])
         self.calls += 1
         self.evaluated += n
@@ -471,10 +507,15 @@ class GPUEvaluator:
         c = torch.from_numpy(np.ascontiguousarray(codes)).to(dev)
         h = torch.from_numpy(np.ascontiguousarray(hdr, np.uint64).view(np.int64)).to(dev)
         tiled = self.ctx.pack_rowmajor(c)
-        out, _ = self.ctx.eval(tiled, h, n=n, full=True, select=False)
+        plane = None
+        if dims is not None:
+            plane = self.ctx.pack_dims(torch.from_numpy(np.ascontiguousarray(dims, np.uint8)).to(dev))
+        out, _ = self.ctx.eval(tiled, h, n=n, full=True, select=False, dims=plane)
         res = dict(iter=as_u64(out.iter_ns), max_mem=as_u64(out.max_mem), info=as_u32(out.info))
         for k in ["stage_T", "stage_mem", "stage_comp", "stage_comm"]:
             res[k] = as_u64(getattr(out, k)).reshape(out.p_max, n).T
+        if hashes:
+            res["hash"] = hash_candidates(tiled, h, self.ctx.n_ops, n=n).cpu().numpy().view(np.uint64)
         return res
 
     def evaluate_cands(self, bases, ranks, cands):
@@ -514,8 +555,9 @@ class _Node:
     time: np.ndarray
     iter_ns: int
     max_mem: int
-    src: tuple          # (base row, rank rows, descriptor, n_ops): materialised on demand
+    src: tuple | None   # (base row, rank rows, descriptor, n_ops): materialised on demand
     _codes: np.ndarray | None = None
+    mem: np.ndarray | None = None  # per-stage memory (Heuristic-2's third resource)
 
     @property
     def codes(self):
@@ -560,33 +602,52 @@ def _key(perf):
     return (int(perf[0]) << 62) | int(perf[1])
 
 
+def _keys_of(r):
+    info = np.asarray(r["info"], np.uint64)
+    cls = np.where(info & INFO_INVALID, 2, np.where(info & INFO_OOM, 1, 0)).astype(np.uint64)
+    cost = np.where(cls == 2, 0, np.where(cls == 1, r["max_mem"], r["iter"])).astype(np.uint64)
+    return (cls << np.uint64(62)) | cost  # perf_of as one ordered integer
+
+
 class _Chunk:
     """The configurations one hop added to a search's unexplored set, kept as arrays in
     best-performance-first order (stable: generation order among equals). Nodes are only
     materialised when the search takes them; they leave the set from the front (the
-    improving node, GetBestOf)."""
+    improving node, the next frontier, GetBestOf)."""
 
-    def __init__(self, keys, idx, r, bases, ranks, cands, L):
+    def __init__(self, keys, idx, r, bases, ranks, cands, L, codes=None, mbs=None):
         self.keys = keys[idx]
         self.idx = idx
         self.hash = r["hash"][idx]
         self.info = r["info"][idx]
         self.iter = r["iter"][idx]
         self.mem = r["max_mem"][idx]
-        self.stage = (r["stage_comp"], r["stage_comm"], r["stage_T"])  # [n][p_max], host or device
-        self.cands = cands[idx]
+        self.stage = (r["stage_comp"], r["stage_comm"], r["stage_T"], r["stage_mem"])  # [n][p_max]
+        self.cands = None if cands is None else cands[idx]
+        self.codes = None if codes is None else codes[idx]  # materialised rows (recompute attachment)
+        self.mbs = None if mbs is None else mbs[idx]
         self.bases, self.ranks, self.L = bases, ranks, L
         self.head = 0
 
     def node(self, t):
         info = int(self.info[t])
-        c = self.cands[t]
-        b = int(c["base"])
         i = int(self.idx[t])
         rows = [_row(x, i) for x in self.stage]
+        if self.codes is not None:
+            return _Node(int(self.hash[t]), int(self.mbs[t]), perf_of(info, self.iter[t], self.mem[t]), info,
+                         rows[0], rows[1], rows[2], int(self.iter[t]), int(self.mem[t]), None,
+                         self.codes[t], rows[3])
+        c = self.cands[t]
+        b = int(c["base"])
         return _Node(int(self.hash[t]), int(c["mbs"]), perf_of(info, self.iter[t], self.mem[t]), info,
                      rows[0], rows[1], rows[2], int(self.iter[t]), int(self.mem[t]),
-                     (self.bases[b], self.ranks[b], c, self.L))
+                     (self.bases[b], self.ranks[b], c, self.L), None, rows[3])
+
+
+# the root of a failed multi-hop search is retried on Heuristic-2's next resource (backtracking
+# over the primitive groups, P:L207-211), then on the secondary bottleneck (P:L219), before
+# GetBestOf(unexplored) (Alg. 1 line 13)
+ROOT_MODES = ((0, 0), (0, 1), (0, 2), (1, 0))
 
 
 class _Search:
@@ -598,7 +659,8 @@ class _Search:
         self.init_perf = start.perf
         self.frontier = [start]
         self.hop = 0
-        self.chunks = []  # unexplored configurations, in insertion order (_Chunk)
+        self.mode = 0      # index into ROOT_MODES for the current root
+        self.chunks = []   # unexplored configurations, in insertion order (_Chunk)
         self.done = False
         self.improvements = 0
 
@@ -615,9 +677,51 @@ class _Search:
         best.head += 1
         return nd
 
+    def take_best(self, chunks, k):
+        """The k best configurations of this hop's chunks (removed from the unexplored set)."""
+        out = []
+        for _ in range(k):
+            best = None
+            for ch in chunks:
+                if ch.head < len(ch.keys) and (best is None or ch.keys[ch.head] < best.keys[best.head]):
+                    best = ch
+            if best is None:
+                break
+            out.append(best.node(best.head))
+            best.head += 1
+        return out
+
+
+def _rc_variants(prof, codes, mbs, info, mem, stage_time, max_n=4096):
+    """Recomputation attached to a primitive's result (greedy as in P:L255): on its
+    memory bottleneck (if OOM) the largest-activation ops not yet recomputed, k = 1.. in
+    order (inc-rc); otherwise on its time bottleneck the recomputed ops released smallest
+    activation first (dec-rc). Returns a list of code rows (same header)."""
+    heads, ends = stages_of(codes)
+    p = len(heads)
+    bn = int(info & 0xFF)
+    if bn >= p:
+        return []
+    order = _rc_order(prof, codes, bn, mbs, (heads, ends))
+    rc = (codes[order] >> 4) & 1
+    out = []
+    if info & INFO_OOM:
+        todo = order[rc == 0]
+        for k in range(1, min(len(todo), max_n) + 1):
+            c = codes.copy()
+            c[todo[:k]] |= 0x10
+            out.append(c)
+    else:
+        have = order[rc == 1][::-1]
+        for k in range(1, min(len(have), max_n) + 1):
+            c = codes.copy()
+            c[have[:k]] &= 0xEF
+            out.append(c)
+    return out
+
 
 def search(prof, evaluator, p_values=None, budget_s=10.0, max_hops=7, beam=4, heuristic2=True,
-           max_batch=200000, max_k=None, patience=None, starts=None):
+           max_batch=200000, max_k=None, patience=None, starts=None, attach_rc=8, root_modes=ROOT_MODES):
     """Runs the batched Aceso search. Returns (best Result, stats dict).
 
     starts: optional extra initial configurations [(codes, mbs_log2)], each searched like the
@@ -627,7 +731,11 @@ def search(prof, evaluator, p_values=None, budget_s=10.0, max_hops=7, beam=4, he
     Every hop's candidates are generated as base + patches (Primitives.describe_all) and
     evaluated by `evaluator.evaluate_cands(bases, ranks, cands)`, which also returns each
     candidate's configuration hash; configurations are deduplicated by hash in
-    generation order, and only the ones the search keeps are materialised on the host."""
+    generation order, and only the ones the search keeps are materialised on the host.
+    attach_rc: per search and hop, the best `attach_rc` new configurations also get greedy
+    inc/dec-rc attached (evaluated as rows in a second batch of the hop).
+    root_modes: (bottleneck rank, resource rank) tried at the root of a failed multi-hop
+    search before GetBestOf: Heuristic-2's next resources, then the secondary bottleneck."""
     from . import candidates as C
     t0 = time.perf_counter()
     L = prof.n_ops
@@ -655,7 +763,7 @@ def search(prof, evaluator, p_values=None, budget_s=10.0, max_hops=7, beam=4, he
         info = int(r["info"][i])
         nd = _Node(int(r["hash"][i]), int(cand["mbs"]), perf_of(info, r["iter"][i], r["max_mem"][i]), info,
                    _row(r["stage_comp"], i), _row(r["stage_comm"], i), _row(r["stage_T"], i), int(r["iter"][i]),
-                   int(r["max_mem"][i]), (base_row, rank_rows, cand, L))
+                   int(r["max_mem"][i]), (base_row, rank_rows, cand, L), None, _row(r["stage_mem"], i))
         return nd
 
     searches = []
@@ -677,10 +785,17 @@ def search(prof, evaluator, p_values=None, budget_s=10.0, max_hops=7, beam=4, he
         for si, s in enumerate(searches):
             if s.done:
                 continue
+            bn_rank, res_rank = root_modes[s.mode] if s.hop == 0 else (0, 0)
             for nd in s.frontier:
                 if nd.perf[0] == 2 or total >= max_batch:
                     continue
-                cd, rk = prims.describe_all(nd.codes, nd.mbs, nd.info, nd.comp, nd.comm, nd.time)
+                p = int((nd.codes & 1).sum())
+                kw = {}
+                if nd.mem is not None and heuristic2:
+                    bn = bottleneck_rank(nd.info, nd.mem, nd.time, p, bn_rank)
+                    order = resource_order(nd.info, nd.comp, nd.comm, nd.mem, p, bn)
+                    kw = dict(mem=nd.mem, bn=bn, resource=order[min(res_rank, len(order) - 1)])
+                cd, rk = prims.describe_all(nd.codes, nd.mbs, nd.info, nd.comp, nd.comm, nd.time, **kw)
                 if len(cd) == 0:
                     continue
                 cd = cd[: max_batch - total]
@@ -705,38 +820,77 @@ def search(prof, evaluator, p_values=None, budget_s=10.0, max_hops=7, beam=4, he
         owner = np.concatenate(owners)
         # configurations seen before (or earlier in this batch) are dropped
         keep, visited = _first_new(np.asarray(r["hash"], np.uint64), visited)
-        info = np.asarray(r["info"], np.uint64)
-        cls = np.where(info & INFO_INVALID, 2, np.where(info & INFO_OOM, 1, 0)).astype(np.uint64)
-        cost = np.where(cls == 2, 0, np.where(cls == 1, r["max_mem"], r["iter"])).astype(np.uint64)
-        keys = (cls << np.uint64(62)) | cost  # perf_of as one ordered integer
-        improved_any = False
+        keys = _keys_of(r)
+        hop_chunks = {}
         for si, s in enumerate(searches):
             if s.done:
                 continue
             idx = np.nonzero(keep & (owner == si))[0]
             # Heuristic-2: best estimated performance first (stable: generation order)
             idx = idx[np.argsort(keys[idx], kind="stable")]
-            ch = _Chunk(keys, idx, r, bases, ranks, cands, L) if len(idx) else None
-            if ch is not None:
-                s.chunks.append(ch)
-            if ch is not None and int(ch.keys[0]) < _key(s.init_perf):
+            hop_chunks[si] = [_Chunk(keys, idx, r, bases, ranks, cands, L)] if len(idx) else []
+        # recomputation attached to the primitives' results: a second batch of the hop
+        if attach_rc:
+            rows, hdrs, mbss, rowner = [], [], [], []
+            for si, chs in hop_chunks.items():
+                if not chs:
+                    continue
+                ch = chs[0]
+                for t in range(min(attach_rc, len(ch.keys))):
+                    if int(ch.info[t]) & INFO_INVALID:
+                        continue
+                    nd = ch.node(t)
+                    p = int((nd.codes & 1).sum())
+                    for c in _rc_variants(prof, nd.codes, nd.mbs, nd.info, nd.mem, nd.time):
+                        rows.append(c)
+                        hdrs.append(header(nd.mbs, p))
+                        mbss.append(nd.mbs)
+                        rowner.append(si)
+            if rows:
+                rc_codes = np.stack(rows)
+                rr = evaluator.evaluate(rc_codes, np.array(hdrs, np.uint64), hashes=True)
+                batches += 1
+                evaluated += len(rows)
+                keep2, visited = _first_new(np.asarray(rr["hash"], np.uint64), visited)
+                keys2 = _keys_of(rr)
+                rowner = np.array(rowner)
+                mbss = np.array(mbss)
+                for si in hop_chunks:
+                    idx = np.nonzero(keep2 & (rowner == si))[0]
+                    if len(idx):
+                        idx = idx[np.argsort(keys2[idx], kind="stable")]
+                        hop_chunks[si].append(_Chunk(keys2, idx, rr, None, None, None, L, codes=rc_codes, mbs=mbss))
+        for si, s in enumerate(searches):
+            if s.done:
+                continue
+            chs = hop_chunks.get(si, [])
+            s.chunks.extend(chs)
+            first = min((int(ch.keys[0]) for ch in chs), default=None)
+            if first is not None and first < _key(s.init_perf):
                 # Alg. 2 returns the improved configuration; Alg. 1 restarts from it
-                nd0 = ch.node(0)
-                ch.head = 1  # leaves the unexplored set
+                nd0 = s.take_best(chs, 1)[0]  # leaves the unexplored set
                 s.cur = nd0
                 if nd0.perf < s.best.perf:
                     s.best = nd0
                 s.init_perf = nd0.perf
                 s.frontier = [nd0]
                 s.hop = 0
+                s.mode = 0
                 s.improvements += 1
-                improved_any = True
                 continue
             s.hop += 1
-            if s.hop < max_hops and ch is not None:
-                s.frontier = [ch.node(t) for t in range(min(beam, len(ch.keys)))]
+            if s.hop < max_hops and chs:
+                # the next hop explores the best configurations of this one (they leave the
+                # unexplored set, Alg. 2 line 1)
+                s.frontier = s.take_best(chs, beam)
                 continue
-            # MultiHop failed within MaxHops: Alg. 1 continues from GetBestOf(unexplored)
+            # MultiHop failed within MaxHops: retry the root on the next resource / the
+            # secondary bottleneck, then Alg. 1 continues from GetBestOf(unexplored)
+            if s.mode + 1 < len(root_modes):
+                s.mode += 1
+                s.frontier = [s.cur]
+                s.hop = 0
+                continue
             nd = s.get_best_of_unexplored()
             if nd is None:
                 s.done = True
@@ -745,6 +899,7 @@ def search(prof, evaluator, p_values=None, budget_s=10.0, max_hops=7, beam=4, he
             s.init_perf = nd.perf
             s.frontier = [nd]
             s.hop = 0
+            s.mode = 0
         cur_best = min((s.best for s in searches), key=lambda n: n.perf)
         if cur_best.perf < best.perf:
             best = cur_best
@@ -760,3 +915,41 @@ def search(prof, evaluator, p_values=None, budget_s=10.0, max_hops=7, beam=4, he
                  searches=len(searches), history=history,
                  improvements=sum(s.improvements for s in searches))
     return Result(best.codes, best.mbs, best.perf, best.iter_ns, best.max_mem, best.info), stats
+
+
+def finetune_dims(prof, evaluator, codes, mbs, dims=None, max_rounds=64):
+    """Op-level fine-tuning of the tensor-parallel partition dimension (§4.2):
+    "we check the partition options for each operator to determine if there is a better
+    dimension". Each round evaluates, as one batch, the configuration with every single op
+    whose alternative records differ switched to its other dimension, and keeps the best
+    improving switch; stops when none improves. Returns (dims [L] u8, perf, stats)."""
+    rec_alt = getattr(prof, "rec_alt", None)
+    L = prof.n_ops
+    dims = np.zeros(L, np.uint8) if dims is None else np.asarray(dims, np.uint8).copy()
+    p = int((codes & 1).sum())
+    hdr1 = np.array([header(mbs, p)], np.uint64)
+    cur = evaluator.evaluate(codes[None, :], hdr1, dims=dims[None, :])
+    perf = perf_of(int(cur["info"][0]), cur["iter"][0], cur["max_mem"][0])
+    stats = dict(rounds=0, evaluated=1, switched=[])
+    if rec_alt is None:
+        return dims, perf, stats
+    tpl = np.minimum((codes >> 1) & 7, prof.n_tp - 1)
+    b = np.clip(mbs - ((codes >> 5) & 7).astype(np.int64), 0, prof.n_b - 1)
+    differs = np.nonzero((rec_alt[prof.op_type, tpl, b] != prof.rec[prof.op_type, tpl, b]).any(axis=1))[0]
+    for _ in range(max_rounds):
+        if len(differs) == 0:
+            break
+        cand = np.repeat(dims[None, :], len(differs), axis=0)
+        cand[np.arange(len(differs)), differs] ^= 1
+        r = evaluator.evaluate(np.repeat(codes[None, :], len(differs), axis=0),
+                               np.repeat(hdr1, len(differs)), dims=cand)
+        stats["rounds"] += 1
+        stats["evaluated"] += len(differs)
+        keys = _keys_of(r)
+        t = int(np.argmin(keys))  # the lowest index among equals
+        if int(keys[t]) >= _key(perf):
+            break
+        dims = cand[t]
+        perf = perf_of(int(r["info"][t]), r["iter"][t], r["max_mem"][t])
+        stats["switched"].append(int(differs[t]))
+    return dims, perf, stats

@@ -15,9 +15,12 @@ class OracleEvaluator:
         self.prof = prof
         self.evaluated = 0
 
-    def evaluate(self, codes, hdr):
+    def evaluate(self, codes, hdr, dims=None, hashes=False):
         self.evaluated += len(hdr)
-        return oracle.evaluate(self.prof, codes, hdr, full=True, threads=8)
+        r = oracle.evaluate(self.prof, codes, hdr, full=True, threads=8, dims=dims)
+        if hashes:
+            r["hash"] = config_hash(codes, hdr)
+        return r
 
     def evaluate_cands(self, bases, ranks, cands):
         from paper_conf_eurosys_liumlsmybw24_b200 import candidates as C

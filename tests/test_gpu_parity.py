@@ -469,21 +469,51 @@ def test_nccl_allreduce_min_single_rank():
         dist.destroy_process_group()
 
 
-def test_search_driver_gpu_matches_oracle_trajectory():
-    """The batched search (Alg. 1/2) driven by aceso_eval follows exactly the trajectory
-    of the same search driven by the oracle (bit-exact evaluations)."""
+@pytest.mark.parametrize("name,kw", [
+    ("gpt3-1.3b", dict(p_values=[2, 4, 8], max_hops=3, beam=2, max_k=8, patience=3)),
+    ("toy-a", dict(max_hops=7, beam=4, patience=6)),
+    ("toy-b", dict(max_hops=7, beam=4, patience=6)),
+    ("gpt3-13b", dict(p_values=[4, 8], max_hops=2, beam=2, max_k=4, patience=2)),
+    ("t5", dict(p_values=[4], max_hops=2, beam=2, max_k=4, patience=2)),
+    ("wrn", dict(p_values=[2, 4], max_hops=2, beam=2, max_k=6, patience=2)),
+    ("gpt-1k", dict(p_values=[8], max_hops=2, beam=1, max_k=2, patience=1, attach_rc=1)),
+])
+def test_search_driver_gpu_matches_oracle_trajectory(name, kw):
+    """The batched search (Alg. 1/2 with Heuristic-2 over three resources, recomputation
+    attached to the primitives, root retries on the next resource and the secondary
+    bottleneck) driven by aceso_eval follows exactly the trajectory of the same search driven
+    by the oracle (bit-exact evaluations), on every BASELINE workload."""
     import os
     import sys
     from paper_conf_eurosys_liumlsmybw24_b200 import search as S
     sys.path.insert(0, os.path.dirname(__file__))
     from oracle_evaluator import OracleEvaluator
 
-    prof = P.WORKLOADS["gpt3-1.3b"]()
-    kw = dict(p_values=[2, 4, 8], budget_s=120, max_hops=3, beam=2, max_k=8, patience=3)
+    prof = P.WORKLOADS[name]()
+    kw = dict(kw, budget_s=300)
     rg, sg = S.search(prof, S.GPUEvaluator(ctx_for(prof)), **kw)
     ro, so = S.search(prof, OracleEvaluator(prof), **kw)
     assert rg.perf == ro.perf and rg.mbs == ro.mbs and np.array_equal(rg.codes, ro.codes)
     assert sg["evaluated"] == so["evaluated"] and sg["batches"] == so["batches"]
+    assert [h[1] for h in sg["history"]] == [h[1] for h in so["history"]]
+
+
+def test_dimension_finetune_gpu_matches_oracle():
+    """§4.2 op-level dimension fine-tune driven by aceso_eval_dims equals the oracle-driven one."""
+    import os
+    import sys
+    from paper_conf_eurosys_liumlsmybw24_b200 import search as S
+    sys.path.insert(0, os.path.dirname(__file__))
+    from oracle_evaluator import OracleEvaluator
+    prof = P.WORKLOADS["wrn"]()
+    for p in (2, 4):
+        codes, mbs = S.initial_config(prof, p)
+        for s in range(p):
+            c2 = S._recode_stage(codes, s, 1, -1)
+            codes = c2 if c2 is not None else codes
+        dg, pg, sg = S.finetune_dims(prof, S.GPUEvaluator(ctx_for(prof)), codes, mbs, max_rounds=8)
+        do, po, so = S.finetune_dims(prof, OracleEvaluator(prof), codes, mbs, max_rounds=8)
+        assert pg == po and np.array_equal(dg, do) and sg == so
 
 
 def _attribution_candidates(prof, n, seed):

@@ -169,3 +169,68 @@ def test_first_new_dedup_is_first_occurrence_against_visited():
         keep, visited = S._first_new(hs, visited)
         assert np.array_equal(keep, want)
         assert np.array_equal(visited, np.array(sorted(visited_set), np.uint64))
+
+
+def test_heuristic2_resource_order_and_secondary_bottleneck():
+    """Heuristic-2 (P:L206-211): resources by the bottleneck stage's consumption proportion;
+    an OOM configuration puts memory first. The secondary bottleneck is the next
+    stage of Heuristic-1's order."""
+    comp = np.array([10, 30, 60], np.uint64)   # stage 1: 30% of compute
+    comm = np.array([50, 40, 10], np.uint64)   # stage 1: 40% of communication
+    mem = np.array([20, 50, 30], np.uint64)    # stage 1: 50% of memory
+    assert S.resource_order(1, comp, comm, mem, 3, 1) == ["mem", "comm", "comp"]
+    assert S.resource_order(1, comp, comm, None, 3, 1) == ["comm", "comp"]
+    assert S.resource_order(S.INFO_OOM | 2, comp, comm, mem, 3, 2)[0] == "mem"
+    assert S.resource_order(2, comp, comm, mem, 3, 2) == ["comp", "mem", "comm"]
+    t = np.array([5, 9, 7], np.uint64)
+    assert S.bottleneck_rank(1, mem, t, 3, 0) == 1
+    assert S.bottleneck_rank(1, mem, t, 3, 1) == 2           # by time
+    assert S.bottleneck_rank(S.INFO_OOM | 1, mem, t, 3, 1) == 2  # by memory: 50 > 30 > 20
+
+
+def test_rc_attachment_is_greedy_by_activation():
+    """Attached inc-rc: the k-th variant recomputes the k largest-activation
+    ops of the memory bottleneck that were not recomputed; dec-rc releases smallest first."""
+    prof = P.WORKLOADS["gpt3-1.3b"]()
+    codes, mbs = S.initial_config(prof, 4)
+    heads, ends = S.stages_of(codes)
+    a, e = int(heads[2]), int(ends[2])
+    vs = S._rc_variants(prof, codes, mbs, S.INFO_OOM | 2, None, None)
+    assert len(vs) == e - a
+    tpl, dpl = (codes[a] >> 1) & 7, (codes[a] >> 5) & 7
+    act = prof.rec[prof.op_type[a:e], tpl, mbs - dpl, 4]
+    prev = set()
+    for k, v in enumerate(vs, 1):
+        on = set(np.nonzero(v & 0x10)[0].tolist())
+        assert len(on) == k and prev < on and all(a <= j < e for j in on)
+        new = (on - prev).pop()
+        assert act[new - a] == max(act[j - a] for j in range(a, e) if j not in prev)
+        prev = on
+    full = vs[-1]
+    back = S._rc_variants(prof, full, mbs, 2, None, None)
+    assert len(back) == e - a and not (back[-1] & 0x10).any()
+
+
+def test_search_with_attachment_and_root_modes_returns_a_reproducible_configuration():
+    prof = P.WORKLOADS["gpt3-13b"]()
+    r, st = S.search(prof, OracleEvaluator(prof), p_values=[4, 8], budget_s=120, max_hops=2, beam=2,
+                     max_k=4, patience=3, attach_rc=4)
+    o = oracle.evaluate(prof, r.codes[None, :], np.array([S.header(r.mbs, int((r.codes & 1).sum()))], np.uint64))
+    assert perf_tuple(o, 0) == r.perf and st["evaluated"] > 0
+
+
+def test_dimension_finetune_improves_or_keeps():
+    """§4.2: the greedy per-op dimension fine-tune never returns a worse
+    configuration, and its result re-evaluates to the reported performance."""
+    prof = P.WORKLOADS["gpt3-1.3b"]()
+    codes, mbs = S.initial_config(prof, 2)
+    for s in range(2):  # 4 devices per stage as tp 2 x dp 2: MatMuls have two dimensions
+        codes = S._recode_stage(codes, s, 1, -1)
+    ev = OracleEvaluator(prof)
+    base = ev.evaluate(codes[None, :], np.array([S.header(mbs, 2)], np.uint64))
+    assert not base["info"][0] & oracle.INFO_INVALID
+    dims, perf, st = S.finetune_dims(prof, ev, codes, mbs, max_rounds=6)
+    assert perf <= perf_tuple(base, 0) and st["rounds"] >= 1
+    o = oracle.evaluate(prof, codes[None, :], np.array([S.header(mbs, 2)], np.uint64), dims=dims[None, :])
+    assert perf_tuple(o, 0) == perf
+    assert len(st["switched"]) == int(dims.sum())
