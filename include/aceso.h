@@ -202,6 +202,11 @@ typedef struct {
                                  unaffected.
                                  Results are identical.                         */
 
+#define ACESO_PIPE_LITERAL 32u /* Eq. 2 as printed: the steady phase runs N
+                                 microbatches of stage i, T_i = sum_k S_k + N S_i + D_i;
+                                 default (reading R1): N - 1, the 1F1B
+                                 makespan on uniform stages. Applies to every output. */
+
 /* ------------------------------------------------------------------------- */
 /* Selection (Alg. 1 GetBestOf P:L543, Alg. 2 `perf < init_perf` P:L576).     */
 /* ------------------------------------------------------------------------- */

@@ -39,7 +39,7 @@ def _load():
         P = ctypes.c_void_p
         i32, i64 = ctypes.c_int32, ctypes.c_int64
         lib.oracle_eval.argtypes = [i32, i32, i32, i32, i32, i32, P, P, P, P, P, i64, i64, P, P, P, i64,
-                                    i32, P, P, P, P, P, P, P, ctypes.c_int]
+                                    i32, P, P, P, P, P, P, P, ctypes.c_int, ctypes.c_int]
         lib.oracle_eval.restype = ctypes.c_int
         lib.oracle_select.argtypes = [P, P, P, i64, i64, P, P, P]
         _lib = lib
@@ -50,12 +50,13 @@ def _ptr(a):
     return None if a is None else a.ctypes.data
 
 
-def evaluate(prof, codes, hdr, full=False, threads=1, dims=None):
+def evaluate(prof, codes, hdr, full=False, threads=1, dims=None, literal=False):
     """Evaluates row-major codes [n][L] with headers [n]; dims (optional, row-major [n][L],
     nonzero = the op's alternative tensor-parallel partition dimension) needs prof.rec_alt.
 
     Returns dict(iter, max_mem, info[, stage_T, stage_mem, stage_comp, stage_comm]);
-    stage arrays are [n][G] (rows i >= p and rows of invalid candidates are 0)."""
+    stage arrays are [n][G] (rows i >= p and rows of invalid candidates are 0).
+    literal: Eq. 2 as printed (steady phase of N microbatches; reading R1 uses N - 1)."""
     lib = _load()
     codes = np.ascontiguousarray(codes, dtype=np.uint8)
     if dims is not None:
@@ -85,7 +86,8 @@ def evaluate(prof, codes, hdr, full=False, threads=1, dims=None):
                          _ptr(dps), int(prof.mem_capacity), int(prof.global_batch), _ptr(codes), _ptr(dims),
                          _ptr(hdr), n,
                          G, _ptr(out["iter"]), _ptr(out["max_mem"]), _ptr(out["info"]),
-                         _ptr(st[0]), _ptr(st[1]), _ptr(st[2]), _ptr(st[3]), int(threads))
+                         _ptr(st[0]), _ptr(st[1]), _ptr(st[2]), _ptr(st[3]), int(threads),
+                         int(bool(literal)))
     assert rc == 0
     return out
 

@@ -65,6 +65,7 @@ typedef struct {
   const int64_t *wmem; /* [T][n_tp][2] */
   const int64_t *dps;  /* [T][n_tp][n_dp] */
   int64_t C, Bg;
+  int literal; /* R1 variant: the literal reading of Eq. 2 */
 } oracle_profile;
 
 /* record field of an op of `type` at (tpl, b); dim = 1 reads the records profiled for the
@@ -216,6 +217,7 @@ static void eval_one(const oracle_profile *P, const uint8_t *codes, const uint8_
   int oom = 0;
   for (unsigned i = 0; i < p; ++i) {
     u64 Ti = sumS + (N - 1) * S[i] + Dd[i];
+    if (P->literal) Ti += S[i]; /* R1 variant: Eq. 2 as printed (steady phase N, not N-1, microbatches) */
     u64 inflight = (u64)(p - i) < N ? (u64)(p - i) : N;
     u64 Mi = Wst[i] + inflight * A[i] + E[i];
     if (Mi > (u64)P->C) oom = 1; /* R10 */
@@ -270,12 +272,12 @@ int oracle_eval(int32_t L, int32_t T, int32_t n_tp, int32_t n_dp, int32_t n_b, i
                 const int64_t *dps, int64_t C, int64_t Bg, const uint8_t *codes, const uint8_t *dims,
                 const uint64_t *hdr, int64_t n, int32_t p_max, uint64_t *iter, uint64_t *max_mem,
                 uint32_t *info, uint64_t *stage_T, uint64_t *stage_mem, uint64_t *stage_comp,
-                uint64_t *stage_comm, int n_threads) {
+                uint64_t *stage_comm, int n_threads, int literal) {
   if (L < 1 || T < 1 || n < 0 || !op_type || !rec || !wmem || !dps || (n && (!codes || !hdr)))
     return -1;
   if ((stage_T || stage_mem || stage_comp || stage_comm) && p_max < G) return -1;
   if (dims && !rec_alt) return -1;
-  oracle_profile P = {L, T, n_tp, n_dp, n_b, G, op_type, rec, rec_alt, wmem, dps, C, Bg};
+  oracle_profile P = {L, T, n_tp, n_dp, n_b, G, op_type, rec, rec_alt, wmem, dps, C, Bg, literal};
   if (n_threads < 1) n_threads = 1;
   if (n_threads > 256) n_threads = 256;
   if ((int64_t)n_threads > n) n_threads = n > 0 ? (int)n : 1;

@@ -8,7 +8,7 @@ c_i32, c_i64, c_u32, c_u64, c_sz, P = (ctypes.c_int32, ctypes.c_int64, ctypes.c_
                                         ctypes.c_uint64, ctypes.c_size_t, ctypes.c_void_p)
 
 ACESO_OK, ACESO_EINVAL, ACESO_ERANGE, ACESO_ECUDA, ACESO_ENOMEM, ACESO_ENODEV = 0, -1, -2, -3, -4, -5
-OUT_SUMMARY, OUT_FULL, FUSED_SELECT, HINT_DENSE, HINT_OVERLAP = 1, 2, 4, 8, 16
+OUT_SUMMARY, OUT_FULL, FUSED_SELECT, HINT_DENSE, HINT_OVERLAP, PIPE_LITERAL = 1, 2, 4, 8, 16, 32
 INFO_OOM = 1 << 16
 INFO_INVALID = 1 << 17
 

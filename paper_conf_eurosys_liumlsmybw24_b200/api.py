@@ -167,7 +167,8 @@ class Context:
     def eval(self, codes: torch.Tensor, hdr: torch.Tensor, n: int | None = None, global_offset: int = 0,
              n_total: int | None = None, summary: bool = True, full: bool = False, select: bool = True,
              out: Outputs | None = None, sel: torch.Tensor | None = None, stream=None,
-             dense_hint: bool = False, overlap_hint: bool = False, dims: torch.Tensor | None = None):
+             dense_hint: bool = False, overlap_hint: bool = False, dims: torch.Tensor | None = None,
+             literal: bool = False):
         """aceso_eval on tiled device codes and int64 device headers.
 
         dense_hint sets ACESO_HINT_DENSE (per-op kernel; identical results).
@@ -183,6 +184,8 @@ class Context:
             flags |= L.HINT_DENSE
         if overlap_hint:
             flags |= L.HINT_OVERLAP
+        if literal:
+            flags |= L.PIPE_LITERAL  # Eq. 2 as printed (R1 variant)
         if (summary or full) and out is None:
             out = self.alloc_outputs(n, full=full)
         if select and sel is None:

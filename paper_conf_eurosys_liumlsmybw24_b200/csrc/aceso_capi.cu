@@ -234,6 +234,7 @@ EvalParams make_params(const aceso_ctx *ctx, int64_t n, int64_t global_offset, i
   P.qo_words = ctx->qo_words;
   P.es = ctx->es;
   P.sc_resolve = ctx->sc_resolve;
+  P.n_minus = 1;
   return P;
 }
 }  // namespace
@@ -877,7 +878,7 @@ int aceso_eval(aceso_ctx *ctx, const uint8_t *d_codes, const uint64_t *d_hdr, in
   if (n_total >= (1ll << 40)) return fail(ACESO_EINVAL, "n_total >= 2^40");
   if (n >= (1ll << 37)) return fail(ACESO_EINVAL, "n >= 2^37");
   const uint32_t mode = flags & 7u;
-  if (mode == 0 || (flags & ~(7u | ACESO_HINT_DENSE | ACESO_HINT_OVERLAP))) return fail(ACESO_EINVAL, "bad flags 0x%x", flags);
+  if (mode == 0 || (flags & ~(7u | ACESO_HINT_DENSE | ACESO_HINT_OVERLAP | ACESO_PIPE_LITERAL))) return fail(ACESO_EINVAL, "bad flags 0x%x", flags);
   const int kern = (flags & ACESO_HINT_DENSE) ? ctx->dense_kernel : ctx->kernel;
   if (n > 0 && (!d_codes || !d_hdr)) return fail(ACESO_EINVAL, "null codes/headers");
   if ((mode & (ACESO_OUT_SUMMARY | ACESO_OUT_FULL)) && !out) return fail(ACESO_EINVAL, "null outputs");
@@ -892,6 +893,7 @@ int aceso_eval(aceso_ctx *ctx, const uint8_t *d_codes, const uint64_t *d_hdr, in
   EvalParams P = make_params(ctx, n, global_offset, n_total, out, d_sel);
   P.codes = reinterpret_cast<const uint4 *>(d_codes);
   P.hdr = d_hdr;
+  if (flags & ACESO_PIPE_LITERAL) P.n_minus = 0;
 
   // tiles per warp: 1 (latency); with ACESO_HINT_OVERLAP on the event kernel, 3 for models of at
   // most 20 chunks (320 ops) and 2 for at most 24 (384 ops), whose per-tile work does not amortise
@@ -951,7 +953,7 @@ int aceso_eval_dims(aceso_ctx *ctx, const uint8_t *d_codes, const uint8_t *d_dim
   if (n_total >= (1ll << 40)) return fail(ACESO_EINVAL, "n_total >= 2^40");
   if (n >= (1ll << 37)) return fail(ACESO_EINVAL, "n >= 2^37");
   const uint32_t mode = flags & 7u;
-  if (mode == 0 || (flags & ~(7u | ACESO_HINT_DENSE | ACESO_HINT_OVERLAP))) return fail(ACESO_EINVAL, "bad flags 0x%x", flags);
+  if (mode == 0 || (flags & ~(7u | ACESO_HINT_DENSE | ACESO_HINT_OVERLAP | ACESO_PIPE_LITERAL))) return fail(ACESO_EINVAL, "bad flags 0x%x", flags);
   if (n > 0 && (!d_codes || !d_hdr)) return fail(ACESO_EINVAL, "null codes/headers");
   if ((mode & (ACESO_OUT_SUMMARY | ACESO_OUT_FULL)) && !out) return fail(ACESO_EINVAL, "null outputs");
   if ((mode & ACESO_OUT_SUMMARY) && n > 0 && (!out->iter_ns || !out->max_mem || !out->info)) return fail(ACESO_EINVAL, "null summary array");
@@ -964,6 +966,7 @@ int aceso_eval_dims(aceso_ctx *ctx, const uint8_t *d_codes, const uint8_t *d_dim
   EvalParams P = make_params(ctx, n, global_offset, n_total, out, d_sel);
   P.codes = reinterpret_cast<const uint4 *>(d_codes);
   P.hdr = d_hdr;
+  if (flags & ACESO_PIPE_LITERAL) P.n_minus = 0;
   P.dims = d_dims;
   const int64_t need = (P.n_tiles + kWarps - 1) / kWarps;
   const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(need, ctx->dims_max_ctas[mode]));

@@ -90,6 +90,7 @@ struct EvalParams {
   uint32_t tw_q, tw_r;    // scan kernel: tiles per warp (quotient / remainder over all warps)
   uint32_t sc_resolve;    // scan kernel: resolve recompute-only chunks in the compacted pass
   const unsigned char *dims;  // dense kernel with DIMS: tiled dimension plane (aceso_eval_dims)
+  uint32_t n_minus;       // Eq. 2 steady-phase microbatches N - n_minus: 1 (reading R1), 0 (ACESO_PIPE_LITERAL)
 };
 
 // select buffer layout: [0,32) result, [32,40) completion counter, [64, ...) partials (16 B each)

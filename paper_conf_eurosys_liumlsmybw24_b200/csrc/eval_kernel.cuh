@@ -149,7 +149,7 @@ template <uint32_t MODE, class St>
 __device__ __forceinline__ void stage_commit(St &s, const EvalParams &P, int64_t c, bool active,
                                              bool reverse) {
   s.sumS += s.S;
-  const uint64_t tk = (uint64_t)(s.N - 1) * s.S + s.D;  // T_i - sum_k S_k (Eq. 2, R1, R6)
+  const uint64_t tk = (uint64_t)(s.N - P.n_minus) * s.S + s.D;  // T_i - sum_k S_k (Eq. 2, R1, R6)
   const uint64_t infl = s.p > s.i ? (uint64_t)min(s.p - s.i, s.N) : 0ull;  // R2
   const uint64_t M = (s.W + infl * s.A + s.E) << P.mem_shift;              // Eq. 1 (R3, R4)
   // argmax with the lowest stage index on ties (R11): forward visits ascending

@@ -131,7 +131,7 @@ __device__ __forceinline__ void ev_init(EvCand &s, const EvalParams &P, uint64_t
 template <uint32_t MODE>
 __device__ __forceinline__ void ev_commit(EvCand &s, const EvalParams &P, int64_t c, bool active) {
   s.sumS += s.S;
-  const uint64_t tk = (uint64_t)(s.N - 1) * s.S + s.D;  // T_i - sum_k S_k (Eq. 2, R1, R6)
+  const uint64_t tk = (uint64_t)(s.N - P.n_minus) * s.S + s.D;  // T_i - sum_k S_k (Eq. 2, R1, R6)
   const uint32_t p = s.p();
   const uint64_t infl = p > s.i ? (uint64_t)min(p - s.i, s.N) : 0ull;  // R2
   const uint64_t M = (s.W + infl * s.A + s.E) << P.mem_shift;         // Eq. 1 (R3, R4)

@@ -99,7 +99,7 @@ __device__ __forceinline__ void sc_init(ScCand<E64> &s, const EvalParams &P, uin
 template <uint32_t MODE, bool E64>
 __device__ __forceinline__ void sc_commit(ScCand<E64> &s, const EvalParams &P, int64_t c, bool active) {
   s.sumS += s.S;
-  const uint64_t tk = (uint64_t)(s.N - 1) * s.S + s.D;
+  const uint64_t tk = (uint64_t)(s.N - P.n_minus) * s.S + s.D;
   const uint32_t p = s.p();
   const uint64_t infl = p > s.i ? (uint64_t)min(p - s.i, s.N) : 0ull;
   const uint64_t M = s.W + infl * s.A + ((uint64_t)s.E << P.es);

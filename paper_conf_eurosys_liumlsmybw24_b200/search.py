@@ -692,11 +692,23 @@ class _Search:
         return out
 
 
+def _greedy_counts(n):
+    """How many ops the greedy recompute steps try: every k up to 16, then k growing by 25%
+    (the smallest fitting k of the batch is within 25% of the exact greedy stopping point),
+    and all n."""
+    ks, k = list(range(1, min(n, 16) + 1)), 16
+    while k < n:
+        k = min(n, max(k + 1, int(k * 1.25)))
+        ks.append(k)
+    return ks
+
+
 def _rc_variants(prof, codes, mbs, info, mem, stage_time, max_n=4096):
     """Recomputation attached to a primitive's result (greedy as in P:L255): on its
-    memory bottleneck (if OOM) the largest-activation ops not yet recomputed, k = 1.. in
+    memory bottleneck (if OOM) the largest-activation ops not yet recomputed, the first k in
     order (inc-rc); otherwise on its time bottleneck the recomputed ops released smallest
-    activation first (dec-rc). Returns a list of code rows (same header)."""
+    activation first (dec-rc); k from _greedy_counts. Returns a list of code rows (same
+    header)."""
     heads, ends = stages_of(codes)
     p = len(heads)
     bn = int(info & 0xFF)
@@ -707,13 +719,13 @@ def _rc_variants(prof, codes, mbs, info, mem, stage_time, max_n=4096):
     out = []
     if info & INFO_OOM:
         todo = order[rc == 0]
-        for k in range(1, min(len(todo), max_n) + 1):
+        for k in _greedy_counts(min(len(todo), max_n)):
             c = codes.copy()
             c[todo[:k]] |= 0x10
             out.append(c)
     else:
         have = order[rc == 1][::-1]
-        for k in range(1, min(len(have), max_n) + 1):
+        for k in _greedy_counts(min(len(have), max_n)):
             c = codes.copy()
             c[have[:k]] &= 0xEF
             out.append(c)
@@ -721,7 +733,8 @@ def _rc_variants(prof, codes, mbs, info, mem, stage_time, max_n=4096):
 
 
 def search(prof, evaluator, p_values=None, budget_s=10.0, max_hops=7, beam=4, heuristic2=True,
-           max_batch=200000, max_k=None, patience=None, starts=None, attach_rc=8, root_modes=ROOT_MODES):
+           max_batch=200000, max_k=None, patience=None, starts=None, attach_rc=8, root_modes=ROOT_MODES,
+           max_batches=None):
     """Runs the batched Aceso search. Returns (best Result, stats dict).
 
     starts: optional extra initial configurations [(codes, mbs_log2)], each searched like the
@@ -735,7 +748,8 @@ def search(prof, evaluator, p_values=None, budget_s=10.0, max_hops=7, beam=4, he
     attach_rc: per search and hop, the best `attach_rc` new configurations also get greedy
     inc/dec-rc attached (evaluated as rows in a second batch of the hop).
     root_modes: (bottleneck rank, resource rank) tried at the root of a failed multi-hop
-    search before GetBestOf: Heuristic-2's next resources, then the secondary bottleneck."""
+    search before GetBestOf: Heuristic-2's next resources, then the secondary bottleneck.
+    max_batches: stop after this many evaluation batches (a budget independent of speed)."""
     from . import candidates as C
     t0 = time.perf_counter()
     L = prof.n_ops
@@ -778,7 +792,8 @@ def search(prof, evaluator, p_values=None, budget_s=10.0, max_hops=7, beam=4, he
     evaluated = len(init)
     history = [(t_best, best.perf)]
     stale = 0
-    while time.perf_counter() - t0 < budget_s and any(not s.done for s in searches):
+    while time.perf_counter() - t0 < budget_s and any(not s.done for s in searches) and \
+            (max_batches is None or batches < max_batches):
         # one hop of every active search, generated into one batch of descriptors
         owners, chunks, base_rows, rank_rows = [], [], [], []
         total = 0

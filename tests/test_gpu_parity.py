@@ -36,7 +36,7 @@ def ctx_for(prof):
 
 
 def run_gpu(prof, codes, hdr, full=False, gofs=0, n_total=None, pack_on_device=False, select=True,
-            dense_hint=False, overlap_hint=False):
+            dense_hint=False, overlap_hint=False, literal=False):
     ctx = ctx_for(prof)
     n = len(hdr)
     if pack_on_device:
@@ -45,7 +45,7 @@ def run_gpu(prof, codes, hdr, full=False, gofs=0, n_total=None, pack_on_device=F
         tiled = torch.from_numpy(ai.tile(codes)).cuda()
     hd = torch.from_numpy(np.ascontiguousarray(hdr, np.uint64).view(np.int64)).cuda()
     out, sel = ctx.eval(tiled, hd, n=n, global_offset=gofs, n_total=n_total, full=full, select=select,
-                        dense_hint=dense_hint, overlap_hint=overlap_hint)
+                        dense_hint=dense_hint, overlap_hint=overlap_hint, literal=literal)
     torch.cuda.synchronize()
     g = dict(iter=as_u64(out.iter_ns), max_mem=as_u64(out.max_mem), info=as_u32(out.info))
     if full:
@@ -55,10 +55,10 @@ def run_gpu(prof, codes, hdr, full=False, gofs=0, n_total=None, pack_on_device=F
 
 
 def compare(prof, codes, hdr, full=False, gofs=0, n_total=None, pack_on_device=False, dense_hint=False,
-            overlap_hint=False):
+            overlap_hint=False, literal=False):
     g, sel, out, ctx = run_gpu(prof, codes, hdr, full, gofs, n_total, pack_on_device, dense_hint=dense_hint,
-                               overlap_hint=overlap_hint)
-    o = oracle.evaluate(prof, codes, hdr, full=full, threads=8)
+                               overlap_hint=overlap_hint, literal=literal)
+    o = oracle.evaluate(prof, codes, hdr, full=full, threads=8, literal=literal)
     for k in ["iter", "max_mem", "info"]:
         bad = np.nonzero(g[k] != o[k])[0]
         assert bad.size == 0, (k, bad[:5], g[k][bad[:5]], o[k][bad[:5]])
@@ -476,7 +476,7 @@ def test_nccl_allreduce_min_single_rank():
     ("gpt3-13b", dict(p_values=[4, 8], max_hops=2, beam=2, max_k=4, patience=2)),
     ("t5", dict(p_values=[4], max_hops=2, beam=2, max_k=4, patience=2)),
     ("wrn", dict(p_values=[2, 4], max_hops=2, beam=2, max_k=6, patience=2)),
-    ("gpt-1k", dict(p_values=[8], max_hops=2, beam=1, max_k=2, patience=1, attach_rc=1)),
+    ("gpt-1k", dict(p_values=[8], max_hops=2, beam=1, max_k=2, patience=2, attach_rc=1, max_batches=8)),
 ])
 def test_search_driver_gpu_matches_oracle_trajectory(name, kw):
     """The batched search (Alg. 1/2 with Heuristic-2 over three resources, recomputation
@@ -490,7 +490,7 @@ def test_search_driver_gpu_matches_oracle_trajectory(name, kw):
     from oracle_evaluator import OracleEvaluator
 
     prof = P.WORKLOADS[name]()
-    kw = dict(kw, budget_s=300)
+    kw = dict(kw, budget_s=1e9)  # bounded by patience / max_batches, not by the clock
     rg, sg = S.search(prof, S.GPUEvaluator(ctx_for(prof)), **kw)
     ro, so = S.search(prof, OracleEvaluator(prof), **kw)
     assert rg.perf == ro.perf and rg.mbs == ro.mbs and np.array_equal(rg.codes, ro.codes)
@@ -679,3 +679,20 @@ def test_pin_profiles_parity(case):
         finally:
             _, ctx = _ctx_cache.pop(id(prof))
             ctx.close()
+
+
+@pytest.mark.parametrize("kernel", ["events", "scan", "quad", "dense"])
+@pytest.mark.parametrize("name", ["gpt3-1.3b", "toy-b", "wrn"])
+def test_literal_eq2_flag_parity(kernel, name, monkeypatch):
+    """ACESO_PIPE_LITERAL (Eq. 2 as printed, R1's variant) on every schedule."""
+    monkeypatch.setenv("ACESO_KERNEL", kernel)
+    prof = P.WORKLOADS[name]()
+    ctx = A.Context(prof, 0)
+    _ctx_cache[id(prof)] = (prof, ctx)
+    try:
+        codes, hdr = ai.search_shaped(prof, SEED + 95, 0, 1200, group_size=16)
+        compare(prof, codes, hdr, full=True, literal=True)
+        compare(prof, codes, hdr, dense_hint=True, literal=True)
+    finally:
+        _ctx_cache.pop(id(prof), None)
+        ctx.close()

@@ -82,6 +82,7 @@ MUTATIONS = [
      "u64 v = rec_field(P, 0, t, tpl[last], (int)mbs_log2 - dpl[last], P2P_FWD);"),
     ("dim-of-previous-op", "TP dimension, P:L263-265",
      "dim[j] = dims ? (dims[j] != 0) : 0;", "dim[j] = dims ? (dims[j > 0 ? j - 1 : 0] != 0) : 0;"),
+    ("literal-eq2-ignored", "R1 variant, P:L238-241", "if (P->literal) Ti += S[i];", ";"),
     ("select-tie-highest-index", "R11 (selection)", "else better = g < best_idx;",
      "else better = g > best_idx;"),
     ("select-oom-before-feasible", "P:L138 better", "else if (k != best_cls) better = k < best_cls;",

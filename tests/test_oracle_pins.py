@@ -672,3 +672,18 @@ def test_dimension_flip_is_local_to_its_op():
             assert delta == (N * d if k == i else d)
         checked += 1
     assert checked > 50
+
+
+@pytest.mark.parametrize("p", [1, 2, 3, 5])
+@pytest.mark.parametrize("mbs_log2", [0, 2])
+def test_literal_eq2_counts_one_more_microbatch(p, mbs_log2):
+    """ACESO_PIPE_LITERAL (reading R1's variant): Eq. 2 as printed -- warm-up of a
+    microbatch through all stages, N steady microbatches of stage i, cool-down -- is the 1F1B
+    makespan of uniform stages plus one more stage time: (N+p)(f+b)."""
+    k, f_op, b_op = 2, 5, 11
+    prof = mkprof({0: lambda tpl, b: [f_op, 0, b_op, 0, 1, 0, 0, 0, 0, 0]}, [0] * (p * k), G=p, Bg=8)
+    N = 8 >> mbs_log2
+    out = oracle.evaluate(prof, np.array([cand([k] * p)], np.uint8), np.array([ai.header(mbs_log2, p)], np.uint64),
+                          literal=True)
+    mk, _ = simulate([f_op * k] * p, [b_op * k] * p, N)
+    assert int(out["iter"][0]) == mk + (f_op + b_op) * k == (N + p) * (f_op + b_op) * k

@@ -196,19 +196,21 @@ def test_rc_attachment_is_greedy_by_activation():
     heads, ends = S.stages_of(codes)
     a, e = int(heads[2]), int(ends[2])
     vs = S._rc_variants(prof, codes, mbs, S.INFO_OOM | 2, None, None)
-    assert len(vs) == e - a
+    ks = S._greedy_counts(e - a)
+    assert len(vs) == len(ks) and ks[:16] == list(range(1, 17)) and ks[-1] == e - a
     tpl, dpl = (codes[a] >> 1) & 7, (codes[a] >> 5) & 7
     act = prof.rec[prof.op_type[a:e], tpl, mbs - dpl, 4]
     prev = set()
-    for k, v in enumerate(vs, 1):
+    for k, v in zip(ks, vs):
         on = set(np.nonzero(v & 0x10)[0].tolist())
         assert len(on) == k and prev < on and all(a <= j < e for j in on)
-        new = (on - prev).pop()
-        assert act[new - a] == max(act[j - a] for j in range(a, e) if j not in prev)
+        # the added ops are the largest activations among those not yet recomputed
+        rest = sorted((act[j - a] for j in range(a, e) if j not in prev), reverse=True)
+        assert sorted((act[j - a] for j in on - prev), reverse=True) == rest[:len(on - prev)]
         prev = on
     full = vs[-1]
     back = S._rc_variants(prof, full, mbs, 2, None, None)
-    assert len(back) == e - a and not (back[-1] & 0x10).any()
+    assert len(back) == len(ks) and not (back[-1] & 0x10).any()
 
 
 def test_search_with_attachment_and_root_modes_returns_a_reproducible_configuration():
