@@ -767,7 +767,11 @@ int aceso_load_profile(const aceso_profile_desc *d, int cuda_device, aceso_ctx *
       int v = atoi(env);
       if (v == 1 || (v == 2 && nch >= 2)) ctx->split = v;
     }
-    ctx->minb = 3;  // ACESO_MINB=2 selects the ~96-register variant (lower single-launch latency)
+    // register target: 3 resident CTAs per SM (80 registers) for models of up to 128 chunks;
+    // the long models' event kernel runs faster at 2 (measured, 1K-layer GPT: 0.608 vs 0.571 of
+    // the HBM roofline at 131,072 candidates, 0.641 vs 0.589 at 1M; GPT-3 1.3B / 13B, T5 and
+    // Wide-ResNet lose 11-17% at 2). ACESO_MINB=2|3 overrides.
+    ctx->minb = nch > 128 ? 2 : 3;
     ctx->tiles_per_warp = 1;
     if (const char *env = getenv("ACESO_TILES_PER_WARP")) {
       int v = atoi(env);
