@@ -1,0 +1,13 @@
+#!/bin/bash
+# Round-2 evidence: default bench line, ncu launch list of the headline bench command, full ncu
+# capture of one headline launch and of one GPT-3 1.3B 64K launch (event kernel).
+mkdir -p gpurun_out
+python -c "import oracle, aceso_inputs; oracle.build(); aceso_inputs.build()"
+nvidia-smi --query-gpu=index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active --format=csv -lms 500 > gpurun_out/r2_clocks.csv &
+SMI=$!
+timeout 900 python bench.py > gpurun_out/r2_bench.json 2> gpurun_out/r2_bench.err; echo "bench rc=$?"
+kill $SMI
+timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none -c 400 --csv --log-file gpurun_out/r2_launches.csv \
+  python bench.py --steps 20 --warmup 5 --no-all --no-e2e --no-cpu --no-dedup --no-dp --search-budget 0 > gpurun_out/r2_launches.log 2>&1; echo "launches rc=$?"
+timeout 900 ncu --set full --clock-control none --import-source on -k regex:event_kernel -s 1 -c 1 -o gpurun_out/r2_ev1k python tools/prof_one.py gpt-1k 131072 2 > gpurun_out/r2_ev1k.log 2>&1; echo "ncu 1k rc=$?"
+timeout 900 ncu --set full --clock-control none --import-source on -k regex:event_kernel -s 1 -c 1 -o gpurun_out/r2_ev13 python tools/prof_one.py gpt3-1.3b 65536 2 > gpurun_out/r2_ev13.log 2>&1; echo "ncu 1.3b rc=$?"
