@@ -42,9 +42,10 @@ def load():
     global _lib
     if _lib is not None:
         return _lib
-    if not os.path.exists(LIB):
-        raise ImportError(f"libaceso.so not built ({LIB}); run __graft_entry__.build()")
-    lib = ctypes.CDLL(LIB)
+    path = os.environ.get("ACESO_LIB_PATH") or LIB  # measurement knob: an alternative build
+    if not os.path.exists(path):
+        raise ImportError(f"libaceso.so not built ({path}); run __graft_entry__.build()")
+    lib = ctypes.CDLL(path)
     lib.aceso_load_profile.argtypes = [ctypes.POINTER(ProfileDesc), ctypes.c_int, ctypes.POINTER(P)]
     lib.aceso_load_profile.restype = ctypes.c_int
     lib.aceso_free.argtypes = [P]
