@@ -282,6 +282,7 @@ __device__ __forceinline__ void sc_drain(ScCand<E64> &s, const EvalParams &P, ui
   constexpr bool RESOLVE = !E64 && !(MODE & kFull);
   const uint32_t wm0 = wl + kScListW, wm1 = wm0 + kScMetaW;  // warp bases of the meta / e1 arrays
   if (RESOLVE && P.sc_resolve) {
+    __syncwarp();  // the lanes' list writes are visible to the compacted pass
     uint32_t incl = cnt;
 #pragma unroll
     for (uint32_t o = 1; o < 32; o <<= 1) {
