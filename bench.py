@@ -59,6 +59,9 @@ def parse():
                     help="do not pass ACESO_HINT_OVERLAP when several streams are in flight")
     ap.add_argument("--keys-per-allreduce", type=int, default=16,
                     help="N > 1: packed keys of this many steps per all-reduce MIN")
+    ap.add_argument("--global-select", default="nccl", choices=["nccl", "symm"],
+                    help="N > 1: global key by NCCL all-reduce MIN of key vectors, or fused into each "
+                         "launch as an atomic MIN on rank 0's symmetric memory (NVLink peer mapping)")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--no-dedup", action="store_true", help="skip the hash / visited-set measurement")
@@ -213,7 +216,7 @@ class Batches:
         self.bytes = self.nbuf * per_batch
 
 
-def time_steps(A, ctx, bt, steps, warmup, nstr, overlap, world, rank, hint, kpa, dist=None):
+def time_steps(A, ctx, bt, steps, warmup, nstr, overlap, world, rank, hint, kpa, dist=None, symm=False):
     """K steps (one aceso_eval per step; N > 1: the packed keys of every `kpa` steps in one NCCL
     all-reduce MIN on a communication stream) captured in one CUDA graph, replayed once between
     CUDA events. Steps are issued round-robin on `nstr` streams (independent batches overlap).
@@ -229,13 +232,18 @@ def time_steps(A, ctx, bt, steps, warmup, nstr, overlap, world, rank, hint, kpa,
     comm = torch.cuda.Stream()
     keyvec = torch.empty(max(1, steps), dtype=torch.int64, device=dev)
     red = dist is not None  # packed keys all-reduced (N > 1, or the one-rank NCCL test mode)
+    gk = None
+    if red and symm:  # the global key fused into every launch (atomic MIN on rank 0's slot)
+        from paper_conf_eurosys_liumlsmybw24_b200.dist import SymmetricKeys
+        gk = SymmetricKeys(max(1, steps))
 
-    def launch(s, st, ev0=None, ev1=None):
+    def launch(s, st, ev0=None, ev1=None, timed=False):
         c, h = bt.dev[s % bt.nbuf]
         if ev0 is not None:
             ev0.record(st)
         ctx.eval(c, h, n=n, global_offset=rank * n, n_total=n_total, summary=True, select=True,
-                 out=outs[s % nstr], sel=sels[s % nsel], stream=st, dense_hint=hint, overlap_hint=overlap)
+                 out=outs[s % nstr], sel=sels[s % nsel], stream=st, dense_hint=hint, overlap_hint=overlap,
+                 global_key=gk.slot(s) if (gk is not None and timed) else None)
         if ev1 is not None:
             ev1.record(st)
 
@@ -256,8 +264,8 @@ def time_steps(A, ctx, bt, steps, warmup, nstr, overlap, world, rank, hint, kpa,
             st = side[s % nstr]
             if s - nsel in comm_done:  # the select buffer's previous all-reduce has read it
                 st.wait_event(comm_done.pop(s - nsel))
-            launch(s, st, ev_s[s], ev_k[s])
-            if red:
+            launch(s, st, ev_s[s], ev_k[s], timed=True)
+            if red and gk is None:
                 done = torch.cuda.Event()
                 done.record(st)
                 comm.wait_event(done)
@@ -280,6 +288,8 @@ def time_steps(A, ctx, bt, steps, warmup, nstr, overlap, world, rank, hint, kpa,
         with torch.cuda.graph(graph):
             issue()
         torch.cuda.synchronize()
+        if gk is not None:
+            gk.reset()
         graph.replay()  # untimed replay (upload)
         torch.cuda.synchronize()
     except Exception as e:  # a collective that cannot be captured: time eager issue
@@ -292,6 +302,8 @@ def time_steps(A, ctx, bt, steps, warmup, nstr, overlap, world, rank, hint, kpa,
         torch.cuda.synchronize()
     clocks = ClockSampler(torch.cuda.current_device())
     t0, t1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    if gk is not None:
+        gk.reset()
     if red:
         dist.barrier()
     torch.cuda.synchronize()
@@ -316,6 +328,10 @@ def time_steps(A, ctx, bt, steps, warmup, nstr, overlap, world, rank, hint, kpa,
     best = Selection.from_buffer(last)
     if red:
         from paper_conf_eurosys_liumlsmybw24_b200 import dist as adist
+        if gk is not None:  # rank 0 holds the fused keys; every rank needs the last one
+            kt = torch.tensor([gk.read(steps - 1) if rank == 0 else 0], dtype=torch.int64, device=dev)
+            dist.broadcast(kt, 0)
+            keyvec[steps - 1] = kt[0]
         kl = int(keyvec[steps - 1].item())
         gc, gcost, gidx, sat = A.decode_key(kl, n_total)
         best = adist.global_select(last, n_total) if sat else Selection(gc, gcost, gidx, kl)
@@ -664,7 +680,8 @@ def measure_workload(A, name, args, dev, hbm, src, world=1, rank=0, dist=None, s
     nstr = max(1, min(nstr, bt.nbuf))
     overlap = nstr > 1 and not args.no_overlap_hint
     k = steps or args.steps
-    r = time_steps(A, ctx, bt, k, args.warmup, nstr, overlap, world, rank, hint, args.keys_per_allreduce, dist)
+    r = time_steps(A, ctx, bt, k, args.warmup, nstr, overlap, world, rank, hint, args.keys_per_allreduce, dist,
+                   symm=args.global_select == "symm")
     ks = min(k, 64)
     kern_serial = time_serial(ctx, bt, ks, rank, world, hint)
     if dist is not None:
@@ -751,8 +768,10 @@ def main():
                        "schedule": rec["schedule"], "streams": rec["streams"], "overlap_hint": rec["overlap_hint"],
                        "l2": rec["l2"],
                        "parallelism": f"dp{dwd} (candidate shards) + " +
-                                      ("NCCL" if backend == "nccl" else backend + " (test backend)") +
-                                      " all-reduce MIN of packed keys"},
+                                      (("global key fused into every launch: atomic MIN on rank 0's symmetric "
+                                        "memory (NVLink peer mapping)") if args.global_select == "symm" else
+                                       ("NCCL" if backend == "nccl" else backend + " (test backend)") +
+                                       " all-reduce MIN of packed keys")},
             "roofline": rec["roofline"],
             "kernel_ms_concurrent": rec["kernel_ms_concurrent"],
             "gpu_launches": args.steps,

@@ -294,6 +294,19 @@ int aceso_eval_dims(aceso_ctx *ctx, const uint8_t *d_codes, const uint8_t *d_dim
                     int64_t n, int64_t global_offset, int64_t n_total, uint32_t flags,
                     const aceso_eval_out *out, void *d_sel, void *stream);
 
+/* aceso_eval with the global selection fused into the launch (§8e, NVSwitch-native
+ * variant): flags must include ACESO_FUSED_SELECT; after writing the batch's select
+ * result, the grid's last CTA also applies atomicMin_system of the packed key to
+ * *d_global_key — a device address on this GPU or an NVLink peer-mapped address of
+ * another GPU's memory (e.g. the rank-0 buffer of a symmetric-memory allocation), so
+ * every rank's launch joins one job-wide key without a separate collective. The
+ * caller initialises the key to INT64_MAX and reads it after all ranks' launches
+ * complete; decode it with aceso_decode_key (a saturated key needs the exact
+ * pairs of the select buffers, as with the NCCL path). 8-byte aligned. */
+int aceso_eval_global(aceso_ctx *ctx, const uint8_t *d_codes, const uint64_t *d_hdr, int64_t n,
+                      int64_t global_offset, int64_t n_total, uint32_t flags, const aceso_eval_out *out,
+                      void *d_sel, int64_t *d_global_key, void *stream);
+
 /* Argmin over an already written summary (iter_ns, max_mem, info) of n
  * candidates; same order and result layout as the fused select. Async. */
 int aceso_select(aceso_ctx *ctx, const aceso_eval_out *out, int64_t n, int64_t global_offset,

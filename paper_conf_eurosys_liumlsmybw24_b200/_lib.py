@@ -16,7 +16,7 @@ SYMBOLS = ["aceso_load_profile", "aceso_free", "aceso_tiled_bytes", "aceso_pack_
            "aceso_select_buf_bytes", "aceso_eval", "aceso_select", "aceso_decode_key",
            "aceso_last_error", "aceso_version", "aceso_hash", "aceso_visited_bytes", "aceso_dedup", "aceso_expand",
            "aceso_enum_cuts_count", "aceso_enum_cuts", "aceso_schedule_name", "aceso_dims_bytes",
-           "aceso_pack_dims", "aceso_eval_dims"]
+           "aceso_pack_dims", "aceso_eval_dims", "aceso_eval_global"]
 
 
 class ProfileDesc(ctypes.Structure):
@@ -76,6 +76,8 @@ def load():
     lib.aceso_pack_dims.restype = ctypes.c_int
     lib.aceso_eval_dims.argtypes = [P, P, P, P, c_i64, c_i64, c_i64, c_u32, ctypes.POINTER(EvalOut), P, P]
     lib.aceso_eval_dims.restype = ctypes.c_int
+    lib.aceso_eval_global.argtypes = [P, P, P, c_i64, c_i64, c_i64, c_u32, ctypes.POINTER(EvalOut), P, P, P]
+    lib.aceso_eval_global.restype = ctypes.c_int
     lib.aceso_hash.argtypes = [P, P, c_i64, c_i32, P, P]
     lib.aceso_hash.restype = ctypes.c_int
     lib.aceso_visited_bytes.argtypes = [c_i64]

@@ -168,7 +168,7 @@ class Context:
              n_total: int | None = None, summary: bool = True, full: bool = False, select: bool = True,
              out: Outputs | None = None, sel: torch.Tensor | None = None, stream=None,
              dense_hint: bool = False, overlap_hint: bool = False, dims: torch.Tensor | None = None,
-             literal: bool = False):
+             literal: bool = False, global_key: int | torch.Tensor | None = None):
         """aceso_eval on tiled device codes and int64 device headers.
 
         dense_hint sets ACESO_HINT_DENSE (per-op kernel; identical results).
@@ -176,6 +176,8 @@ class Context:
         several streams: throughput launch geometry; identical results).
         dims: tiled dimension plane (aceso_eval_dims; pack_dims builds it): ops whose bit is set
         run under their alternative tensor-parallel partition dimension.
+        global_key: int64 tensor element or raw device address (e.g. a peer-mapped symmetric-
+        memory pointer): aceso_eval_global joins the batch's packed key into it (atomic MIN).
         Returns (out, sel): the output arrays (or None) and the select buffer (or None)."""
         n = int(hdr.shape[0]) if n is None else int(n)
         n_total = global_offset + n if n_total is None else int(n_total)
@@ -191,6 +193,14 @@ class Context:
         if select and sel is None:
             sel = self.alloc_select(n)
         cs = out.c_struct() if out is not None else None
+        if global_key is not None:
+            assert dims is None and select
+            gk = global_key.data_ptr() if isinstance(global_key, torch.Tensor) else int(global_key)
+            rc = L.load().aceso_eval_global(self._h, _ptr(codes), _ptr(hdr), n, int(global_offset), n_total, flags,
+                                            ctypes.byref(cs) if cs is not None else None, _ptr(sel),
+                                            ctypes.c_void_p(gk), _stream(stream))
+            _check(rc, "aceso_eval_global")
+            return out, sel
         if dims is not None:
             rc = L.load().aceso_eval_dims(self._h, _ptr(codes), _ptr(dims), _ptr(hdr), n, int(global_offset), n_total,
                                           flags, ctypes.byref(cs) if cs is not None else None, _ptr(sel),

@@ -874,9 +874,28 @@ size_t aceso_select_buf_bytes(const aceso_ctx *ctx, int64_t n) {
   return (size_t)kSelPartialOff + 16 * (size_t)m;
 }
 
+static int eval_impl(aceso_ctx *ctx, const uint8_t *d_codes, const uint64_t *d_hdr, int64_t n,
+                     int64_t global_offset, int64_t n_total, uint32_t flags, const aceso_eval_out *out,
+                     void *d_sel, unsigned long long *d_global_key, void *stream);
+
 int aceso_eval(aceso_ctx *ctx, const uint8_t *d_codes, const uint64_t *d_hdr, int64_t n,
                int64_t global_offset, int64_t n_total, uint32_t flags, const aceso_eval_out *out,
                void *d_sel, void *stream) {
+  return eval_impl(ctx, d_codes, d_hdr, n, global_offset, n_total, flags, out, d_sel, nullptr, stream);
+}
+
+int aceso_eval_global(aceso_ctx *ctx, const uint8_t *d_codes, const uint64_t *d_hdr, int64_t n,
+                      int64_t global_offset, int64_t n_total, uint32_t flags, const aceso_eval_out *out,
+                      void *d_sel, int64_t *d_global_key, void *stream) {
+  if (!(flags & ACESO_FUSED_SELECT) || !d_global_key) return fail(ACESO_EINVAL, "aceso_eval_global needs ACESO_FUSED_SELECT and a key address");
+  if (((uintptr_t)d_global_key & 7) != 0) return fail(ACESO_EINVAL, "global key not 8-byte aligned");
+  return eval_impl(ctx, d_codes, d_hdr, n, global_offset, n_total, flags, out, d_sel,
+                   reinterpret_cast<unsigned long long *>(d_global_key), stream);
+}
+
+static int eval_impl(aceso_ctx *ctx, const uint8_t *d_codes, const uint64_t *d_hdr, int64_t n,
+                     int64_t global_offset, int64_t n_total, uint32_t flags, const aceso_eval_out *out,
+                     void *d_sel, unsigned long long *d_global_key, void *stream) {
   if (!ctx) return fail(ACESO_EINVAL, "null context");
   if (n < 0 || global_offset < 0 || n_total < global_offset + n) return fail(ACESO_EINVAL, "bad n / global_offset / n_total");
   if (n_total >= (1ll << 40)) return fail(ACESO_EINVAL, "n_total >= 2^40");
@@ -897,6 +916,7 @@ int aceso_eval(aceso_ctx *ctx, const uint8_t *d_codes, const uint64_t *d_hdr, in
   EvalParams P = make_params(ctx, n, global_offset, n_total, out, d_sel);
   P.codes = reinterpret_cast<const uint4 *>(d_codes);
   P.hdr = d_hdr;
+  P.gkey = d_global_key;
   if (flags & ACESO_PIPE_LITERAL) P.n_minus = 0;
 
   // tiles per warp: 1 (latency); with ACESO_HINT_OVERLAP on the event kernel, 3 for models of at

@@ -91,6 +91,7 @@ struct EvalParams {
   uint32_t sc_resolve;    // scan kernel: resolve recompute-only chunks in the compacted pass
   const unsigned char *dims;  // dense kernel with DIMS: tiled dimension plane (aceso_eval_dims)
   uint32_t n_minus;       // Eq. 2 steady-phase microbatches N - n_minus: 1 (reading R1), 0 (ACESO_PIPE_LITERAL)
+  unsigned long long *gkey;  // aceso_eval_global: the job's global key (local or peer-mapped), or null
 };
 
 // select buffer layout: [0,32) result, [32,40) completion counter, [64, ...) partials (16 B each)
@@ -118,7 +119,8 @@ __device__ __forceinline__ void warp_argmin(uint64_t &ck, int64_t &idx) {
 // writes the final result). Called by every thread of the CTA.
 __device__ __forceinline__ void block_select_finish(uint64_t ck, int64_t idx, unsigned char *sel,
                                                     int64_t n_total, uint32_t ib,
-                                                    uint64_t *s_ck, int64_t *s_idx) {
+                                                    uint64_t *s_ck, int64_t *s_idx,
+                                                    unsigned long long *gkey = nullptr) {
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nw = blockDim.x >> 5;
   warp_argmin(ck, idx);
   if (lane == 0) {
@@ -185,6 +187,10 @@ __device__ __forceinline__ void block_select_finish(uint64_t ck, int64_t idx, un
     }
     res->reserved = 0;
     *reinterpret_cast<unsigned int *>(sel + kSelCounterOff) = 0;  // reusable
+    // global selection fused into the launch (aceso_eval_global): the packed key joins the
+    // job's key by a system-scope atomic MIN on a local or NVLink peer-mapped address (the
+    // key's top bit is 0, so unsigned order = signed order; "nothing valid" = INT64_MAX)
+    if (gkey) atomicMin_system(gkey, (unsigned long long)res->key);
   }
 }
 
@@ -194,7 +200,7 @@ __device__ __forceinline__ void block_select_finish(uint64_t ck, int64_t idx, un
 // Called by all 32 lanes of every warp of the grid.
 __device__ __forceinline__ void warp_select_finish(uint64_t ck, int64_t idx, unsigned char *sel,
                                                    int64_t n_total, uint32_t ib, uint64_t *s_ck,
-                                                   int64_t *s_idx) {
+                                                   int64_t *s_idx, unsigned long long *gkey = nullptr) {
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   const uint32_t wpb = blockDim.x >> 5;
   warp_argmin(ck, idx);
@@ -254,6 +260,10 @@ __device__ __forceinline__ void warp_select_finish(uint64_t ck, int64_t idx, uns
     }
     res->reserved = 0;
     *reinterpret_cast<unsigned int *>(sel + kSelCounterOff) = 0;  // reusable
+    // global selection fused into the launch (aceso_eval_global): the packed key joins the
+    // job's key by a system-scope atomic MIN on a local or NVLink peer-mapped address (the
+    // key's top bit is 0, so unsigned order = signed order; "nothing valid" = INT64_MAX)
+    if (gkey) atomicMin_system(gkey, (unsigned long long)res->key);
   }
 }
 

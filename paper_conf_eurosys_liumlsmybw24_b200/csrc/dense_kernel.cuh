@@ -220,7 +220,7 @@ __global__ void __launch_bounds__(kThreads, MINB) dense_kernel(const __grid_cons
     }
   }
 
-  if (MODE & kSelect) block_select_finish(best_ck, best_idx, P.sel, P.n_total, P.ib, s_ck, s_idx);
+  if (MODE & kSelect) block_select_finish(best_ck, best_idx, P.sel, P.n_total, P.ib, s_ck, s_idx, P.gkey);
 }
 
 }  // namespace aceso

@@ -644,7 +644,7 @@ __global__ void __launch_bounds__(kThreads, MINB) eval_kernel(const __grid_const
   }
 
   if (MODE & kSelect)
-    block_select_finish(best_ck, best_idx, P.sel, P.n_total, P.ib, s_ck, s_idx);
+    block_select_finish(best_ck, best_idx, P.sel, P.n_total, P.ib, s_ck, s_idx, P.gkey);
 }
 
 }  // namespace aceso

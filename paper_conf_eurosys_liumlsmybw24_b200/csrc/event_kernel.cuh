@@ -581,7 +581,7 @@ __global__ void __launch_bounds__(kThreads, MINB) event_kernel(const __grid_cons
     ev_finish<MODE>(s, P, cand, active, best_ck, best_idx);
   }
 
-  if (MODE & kSelect) warp_select_finish(best_ck, best_idx, P.sel, P.n_total, P.ib, s_ck, s_idx);
+  if (MODE & kSelect) warp_select_finish(best_ck, best_idx, P.sel, P.n_total, P.ib, s_ck, s_idx, P.gkey);
 }
 
 }  // namespace aceso

@@ -496,7 +496,7 @@ __global__ void __launch_bounds__(kThreads, MINB) scan_kernel(const __grid_const
     }
   }
 
-  if (MODE & kSelect) warp_select_finish(best_ck, best_idx, P.sel, P.n_total, P.ib, s_ck, s_idx);
+  if (MODE & kSelect) warp_select_finish(best_ck, best_idx, P.sel, P.n_total, P.ib, s_ck, s_idx, P.gkey);
 }
 
 }  // namespace aceso

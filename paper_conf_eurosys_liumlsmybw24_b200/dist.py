@@ -46,3 +46,34 @@ def global_select(sel: torch.Tensor, n_total: int, group=None) -> Selection:
         if best is None or (cc, ix) < best:
             best = (cc, ix)
     return Selection(best[0] >> 62, best[0] & ((1 << 62) - 1), best[1], k)
+
+
+class SymmetricKeys:
+    """Global selection fused into the evaluation launches (§8e, NVSwitch-native variant): a
+    symmetric-memory vector of packed keys (torch.distributed._symmetric_memory); every rank's
+    aceso_eval_global applies an atomic MIN of its batch key to rank 0's slot through the
+    NVLink peer mapping, so a step needs no collective call. Slots are reset to INT64_MAX
+    (`reset`, then a barrier) before the steps that use them; `read` after every rank's
+    launches have completed (stream synchronised + barrier)."""
+
+    def __init__(self, n_slots: int, group=None):
+        import torch.distributed._symmetric_memory as symm
+        self.group = group or dist.group.WORLD
+        self.buf = symm.empty(int(n_slots), dtype=torch.int64, device=torch.device("cuda", torch.cuda.current_device()))
+        self.handle = symm.rendezvous(self.buf, self.group)
+        self.root = int(self.handle.buffer_ptrs[0])  # rank 0's buffer, mapped into this rank
+        self.rank = dist.get_rank(self.group)
+
+    def slot(self, s: int) -> int:
+        """Device address of slot s on rank 0 (valid in this rank's kernels)."""
+        return self.root + 8 * int(s)
+
+    def reset(self):
+        if self.rank == 0:
+            self.buf.fill_((1 << 63) - 1)
+        torch.cuda.synchronize()
+        dist.barrier(group=self.group)
+
+    def read(self, s: int) -> int:
+        """Rank 0: the job-wide packed key of slot s."""
+        return int(self.buf[s].item())

@@ -73,3 +73,28 @@ def test_bench_captured_nccl_key_vector_one_rank():
     codes, hdr = ai.search_shaped(prof, 20240422, b * n, n, group_size=1024)
     o = oracle.evaluate(prof, codes, hdr, threads=16)
     assert (d["result"]["cls"], d["result"]["cost"], d["result"]["index"]) == oracle.select(o)
+
+
+@pytest.mark.gpu
+def test_bench_fused_global_key_symmetric_memory_one_rank():
+    """--global-select symm: every timed launch joins rank 0's symmetric-memory key slot by an
+    atomic MIN (aceso_eval_global through the peer mapping; here one rank maps its own buffer);
+    no collective per step. The last step's global selection equals the oracle's."""
+    steps = 24
+    env = dict(os.environ, ACESO_BENCH_FORCE_DIST="1", WORLD_SIZE="1", RANK="0", LOCAL_RANK="0",
+               MASTER_ADDR="127.0.0.1", MASTER_PORT=str(_free_port()))
+    cmd = [sys.executable, "bench.py", "--gpus", "1", "--steps", str(steps), "--warmup", "3",
+           "--config", "gpt3-1.3b", "--no-cpu", "--no-e2e", "--no-dedup", "--no-dp", "--no-all",
+           "--search-budget", "0", "--global-select", "symm"]
+    r = subprocess.run(cmd, cwd=ROOT, env=env, capture_output=True, text=True, timeout=900)
+    assert r.returncode == 0, r.stderr[-3000:]
+    d = json.loads([l for l in r.stdout.strip().splitlines() if l.startswith("{")][-1])
+    assert d["timing"].startswith("K steps captured in one CUDA graph"), d["timing"]
+    assert "symmetric" in d["config"]["parallelism"]
+    n = d["config"]["batch_per_gpu"]
+    nbuf = int(d["config"]["l2"].split()[0])
+    b = (steps - 1) % nbuf
+    prof = P.WORKLOADS["gpt3-1.3b"]()
+    codes, hdr = ai.search_shaped(prof, 20240422, b * n, n, group_size=1024)
+    o = oracle.evaluate(prof, codes, hdr, threads=16)
+    assert (d["result"]["cls"], d["result"]["cost"], d["result"]["index"]) == oracle.select(o)

@@ -696,3 +696,28 @@ def test_literal_eq2_flag_parity(kernel, name, monkeypatch):
     finally:
         _ctx_cache.pop(id(prof), None)
         ctx.close()
+
+
+@pytest.mark.parametrize("name", ["gpt3-1.3b", "toy-b", "gpt-1k"])
+def test_eval_global_fuses_the_cross_shard_selection(name):
+    """aceso_eval_global: each shard's launch applies an atomic MIN of its packed key to one
+    job-wide key (here a local int64; on NVLink a peer-mapped address): after all shards the
+    key decodes to the oracle's selection over their union, and equals the NCCL path's key."""
+    prof = P.WORKLOADS[name]()
+    ctx = ctx_for(prof)
+    shards = 3
+    n = 1000 if name != "gpt-1k" else 200
+    codes, hdr = ai.search_shaped(prof, SEED + 97, 0, shards * n, group_size=16)
+    key = torch.full((1,), (1 << 63) - 1, dtype=torch.int64, device="cuda")
+    keys = []
+    for r in range(shards):
+        c = torch.from_numpy(ai.tile(codes[r * n:(r + 1) * n])).cuda()
+        h = torch.from_numpy(np.ascontiguousarray(hdr[r * n:(r + 1) * n]).view(np.int64)).cuda()
+        _, sel = ctx.eval(c, h, n=n, global_offset=r * n, n_total=shards * n, select=True, global_key=key)
+        keys.append(int(sel[0:8].view(torch.int64).item()))
+    torch.cuda.synchronize()
+    k = int(key.item())
+    assert k == min(keys)  # = the all-reduce MIN of the shards' packed keys
+    cls, cost, idx, sat = A.decode_key(k, shards * n)
+    o = oracle.evaluate(prof, codes, hdr, threads=8)
+    assert not sat and (cls, cost, idx) == oracle.select(o)
