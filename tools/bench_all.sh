@@ -8,7 +8,7 @@ for cfg in toy-a toy-b gpt3-1.3b gpt3-13b t5 wrn gpt-1k; do
     if [ "$cfg" = "gpt-1k" ]; then b=65536; st=20; fi
     if [ "$cfg" = "toy-a" ] || [ "$cfg" = "toy-b" ]; then b=262144; fi
     timeout 900 python bench.py --config $cfg --dist $dist --batch $b --steps $st --warmup 3 \
-      --no-e2e --no-cpu --no-dedup --no-incr --no-dp --search-budget 0 2>/dev/null | tail -1 >> $out
+      --no-e2e --no-cpu --no-dedup --no-dp --no-all --search-budget 0 2>/dev/null | tail -1 >> $out
   done
 done
 python - "$out" <<'PY'
