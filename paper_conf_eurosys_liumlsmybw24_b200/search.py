@@ -515,8 +515,13 @@ class GPUEvaluator:
         for k in ["stage_T", "stage_mem", "stage_comp", "stage_comm"]:
             res[k] = as_u64(getattr(out, k)).reshape(out.p_max, n).T
         if hashes:
-            res["hash"] = hash_candidates(tiled, h, self.ctx.n_ops, n=n).cpu().numpy().view(np.uint64)
+            hs = hash_candidates(tiled, h, self.ctx.n_ops, n=n)
+            res["hash"], res["hash_dev"] = hs.cpu().numpy().view(np.uint64), hs
         return res
+
+    def visited(self):
+        """The search's visited set on this device (aceso_dedup)."""
+        return DeviceVisited(self.ctx.device)
 
     def evaluate_cands(self, bases, ranks, cands):
         """Candidates as base + patches: aceso_expand -> aceso_eval (FULL) -> aceso_hash on the
@@ -533,7 +538,7 @@ class GPUEvaluator:
         out, _ = self.ctx.eval(tiled, hdr, n=n, full=True, select=False)
         hs = hash_candidates(tiled, hdr, self.ctx.n_ops, n=n)
         res = dict(iter=as_u64(out.iter_ns), max_mem=as_u64(out.max_mem), info=as_u32(out.info),
-                   hash=hs.cpu().numpy().view(np.uint64))
+                   hash=hs.cpu().numpy().view(np.uint64), hash_dev=hs)
         # per-stage rows stay on the device ([n][p_max] views): the search reads the few rows
         # of the configurations it takes (Heuristic-2 needs them), not the whole batch
         for k in ["stage_T", "stage_mem", "stage_comp", "stage_comm"]:
@@ -590,6 +595,56 @@ def _first_new(hs, visited):
         idx, h = idx[~seen], h[~seen]
     keep[idx] = True
     return keep, np.insert(visited, np.searchsorted(visited, h), h)
+
+
+class _HostVisited:
+    """Visited set of an evaluator without a device one: sorted host hashes (_first_new)."""
+
+    def __init__(self):
+        self.h = np.zeros(0, np.uint64)
+
+    def first_new(self, r):
+        keep, self.h = _first_new(np.asarray(r["hash"], np.uint64), self.h)
+        return keep
+
+
+class DeviceVisited:
+    """Configuration dedup on the device: every batch's hashes (r["hash_dev"], left
+    on the device by aceso_hash) go through aceso_dedup's open-addressing table, first
+    occurrence in generation order across batches, the same rule as _first_new. Before the
+    load factor would pass 1/2 the table is rebuilt 4x larger from the device list of every
+    configuration seen, so the insert never fills it; only the keep mask (1 byte per
+    candidate) comes back to the host."""
+
+    def __init__(self, device, slots=1 << 16):
+        from .api import VisitedSet
+        self._cls = VisitedSet
+        self.device = device
+        self.vs = VisitedSet(slots, device)
+        self.seen = []   # device tensors of first-occurrence hashes (re-inserted on growth)
+        self.count = 0
+
+    def _grow(self, need):
+        slots = self.vs.slots
+        while slots < 4 * need:
+            slots *= 2
+        self.vs = self._cls(slots, self.device)
+        if self.seen:
+            self.seen = [torch.cat(self.seen)]
+            self.vs.insert(self.seen[0])
+
+    def first_new(self, r):
+        hs = r["hash_dev"]
+        n = int(hs.shape[0])
+        if 2 * (self.count + n) > self.vs.slots:
+            self._grow(self.count + n)
+        new = self.vs.insert(hs) == 0
+        if self.vs.overflowed():
+            raise RuntimeError("aceso_dedup: visited table full")  # unreachable at load <= 1/2
+        self.seen.append(hs[new])
+        keep = new.cpu().numpy()
+        self.count += int(keep.sum())
+        return keep
 
 
 def _row(x, i):
@@ -744,7 +799,8 @@ def search(prof, evaluator, p_values=None, budget_s=10.0, max_hops=7, beam=4, he
     Every hop's candidates are generated as base + patches (Primitives.describe_all) and
     evaluated by `evaluator.evaluate_cands(bases, ranks, cands)`, which also returns each
     candidate's configuration hash; configurations are deduplicated by hash in
-    generation order, and only the ones the search keeps are materialised on the host.
+    generation order (the evaluator's device visited set, `evaluator.visited()`, else the
+    host statement), and only the ones the search keeps are materialised on the host.
     attach_rc: per search and hop, the best `attach_rc` new configurations also get greedy
     inc/dec-rc attached (evaluated as rows in a second batch of the hop).
     root_modes: (bottleneck rank, resource rank) tried at the root of a failed multi-hop
@@ -757,7 +813,8 @@ def search(prof, evaluator, p_values=None, budget_s=10.0, max_hops=7, beam=4, he
     prims = Primitives(prof, heuristic2=heuristic2, max_k=max_k)
     if p_values is None:
         p_values = [p for p in (1, 2, 3, 4, 6, 8, 12, 16, 24, 32, 48, 64) if p <= min(prof.n_devices, prof.n_ops)]
-    visited = np.zeros(0, np.uint64)  # sorted hashes of every configuration seen
+    # every configuration seen: the evaluator's device set, else sorted host hashes
+    seen = evaluator.visited() if hasattr(evaluator, "visited") else _HostVisited()
     init = []
     for p in p_values:
         r = initial_config(prof, p)
@@ -772,6 +829,7 @@ def search(prof, evaluator, p_values=None, budget_s=10.0, max_hops=7, beam=4, he
         bases[i, :L] = c
         cands[i]["base"], cands[i]["mbs"], cands[i]["p"] = i, m, int((c & 1).sum())
     res = evaluator.evaluate_cands(bases, ranks, cands)
+    seen.first_new(res)
 
     def node(i, r, base_row, rank_rows, cand):
         info = int(r["info"][i])
@@ -784,7 +842,6 @@ def search(prof, evaluator, p_values=None, budget_s=10.0, max_hops=7, beam=4, he
     for i in range(len(init)):
         n0 = node(i, res, bases[i], ranks[i], cands[i])
         n0._codes = init[i][0]
-        _, visited = _first_new(np.array([n0.key], np.uint64), visited)
         searches.append(_Search(n0))
     best = min((s.best for s in searches), key=lambda n: n.perf)
     t_best = time.perf_counter() - t0
@@ -834,7 +891,7 @@ def search(prof, evaluator, p_values=None, budget_s=10.0, max_hops=7, beam=4, he
         evaluated += len(cands)
         owner = np.concatenate(owners)
         # configurations seen before (or earlier in this batch) are dropped
-        keep, visited = _first_new(np.asarray(r["hash"], np.uint64), visited)
+        keep = seen.first_new(r)
         keys = _keys_of(r)
         hop_chunks = {}
         for si, s in enumerate(searches):
@@ -866,7 +923,7 @@ def search(prof, evaluator, p_values=None, budget_s=10.0, max_hops=7, beam=4, he
                 rr = evaluator.evaluate(rc_codes, np.array(hdrs, np.uint64), hashes=True)
                 batches += 1
                 evaluated += len(rows)
-                keep2, visited = _first_new(np.asarray(rr["hash"], np.uint64), visited)
+                keep2 = seen.first_new(rr)
                 keys2 = _keys_of(rr)
                 rowner = np.array(rowner)
                 mbss = np.array(mbss)

@@ -83,3 +83,19 @@ def test_visited_set_overflow_is_reported():
     vs.insert(hs)
     torch.cuda.synchronize()
     assert vs.overflowed()
+
+
+def test_search_device_visited_set_equals_host_statement_through_growth():
+    """search.DeviceVisited (aceso_dedup inside the search driver, rebuilt 4x larger before
+    its load factor passes 1/2) keeps exactly what the host statement _first_new keeps, batch
+    after batch, with repeats inside a batch and across batches and several table rebuilds."""
+    from paper_conf_eurosys_liumlsmybw24_b200 import search as S
+    rng = np.random.default_rng(11)
+    pool = rng.integers(1, 2**63, 5000, dtype=np.int64).view(np.uint64)
+    dv = S.DeviceVisited(0, slots=64)
+    hv = S._HostVisited()
+    for b in range(12):
+        hs = pool[rng.integers(0, 300 + 400 * b, int(rng.integers(1, 900)))]
+        r = dict(hash=hs, hash_dev=torch.from_numpy(hs.view(np.int64)).cuda())
+        assert np.array_equal(dv.first_new(r), hv.first_new(r)), b
+    assert dv.vs.slots > 64 and dv.count == len(hv.h)
