@@ -66,18 +66,27 @@ void *eval_kernel_split(uint32_t mode) {
   }
 }
 
-template <int B>
+template <int B, int W>
 void *event_kernel_for(uint32_t mode) {
   switch (mode) {
-    case 1: return reinterpret_cast<void *>(&event_kernel<1, B>);
-    case 2: return reinterpret_cast<void *>(&event_kernel<2, B>);
-    case 3: return reinterpret_cast<void *>(&event_kernel<3, B>);
-    case 4: return reinterpret_cast<void *>(&event_kernel<4, B>);
-    case 5: return reinterpret_cast<void *>(&event_kernel<5, B>);
-    case 6: return reinterpret_cast<void *>(&event_kernel<6, B>);
-    case 7: return reinterpret_cast<void *>(&event_kernel<7, B>);
+    case 1: return reinterpret_cast<void *>(&event_kernel<1, B, W>);
+    case 2: return reinterpret_cast<void *>(&event_kernel<2, B, W>);
+    case 3: return reinterpret_cast<void *>(&event_kernel<3, B, W>);
+    case 4: return reinterpret_cast<void *>(&event_kernel<4, B, W>);
+    case 5: return reinterpret_cast<void *>(&event_kernel<5, B, W>);
+    case 6: return reinterpret_cast<void *>(&event_kernel<6, B, W>);
+    case 7: return reinterpret_cast<void *>(&event_kernel<7, B, W>);
     default: return nullptr;
   }
+}
+
+// the event kernel's CTA shapes: (warps per CTA, register target in resident CTAs per SM).
+// Built: 8 warps at 2 or 3 CTAs per SM. Measured and dropped (round 2, every BASELINE
+// workload): 6 warps x 3 CTAs (18 warps per SM at 96 registers), 4 warps x 4 / 5 / 6 CTAs —
+// within 0.3% of the better 8-warp shape on the 1K-layer model and 1-10% slower elsewhere.
+void *event_kernel_shape(uint32_t mode, int warps, int minb) {
+  (void)warps;
+  return minb == 2 ? event_kernel_for<2, 8>(mode) : event_kernel_for<3, 8>(mode);
 }
 
 template <int B>
@@ -125,14 +134,14 @@ void *scan_kernel_for(uint32_t mode) {
 // kernel 0: per-op/quad kernel (eval_kernel.cuh); kernel 1: event kernel (event_kernel.cuh);
 // kernel 2: dense kernel (dense_kernel.cuh, ACESO_HINT_DENSE); kernel 3: scan kernel
 // (scan_kernel.cuh, exact u64 tables; e64: wide transient-memory table)
-void *eval_kernel_for(uint32_t mode, int split, int minb, int kernel, int e64 = 0) {
+void *eval_kernel_for(uint32_t mode, int split, int minb, int kernel, int e64 = 0, int ev_warps = kWarps) {
   if (kernel == 3) {
     // the scan kernel's default register target is 2 CTAs per SM (its ring and lists take
     // ~100 KB of shared memory per CTA); ACESO_MINB=3 selects the 80-register build
     if (minb == 3 && getenv("ACESO_MINB")) return e64 ? scan_kernel_for<true, 3>(mode) : scan_kernel_for<false, 3>(mode);
     return e64 ? scan_kernel_for<true, 2>(mode) : scan_kernel_for<false, 2>(mode);
   }
-  if (kernel == 1) return minb == 2 ? event_kernel_for<2>(mode) : event_kernel_for<3>(mode);
+  if (kernel == 1) return event_kernel_shape(mode, ev_warps, minb);
   if (kernel == 2) return minb == 2 ? dense_kernel_for<2>(mode) : dense_kernel_for<3>(mode);
   if (minb == 2) return split == 2 ? eval_kernel_split<2, 2>(mode) : eval_kernel_split<1, 2>(mode);
   return split == 2 ? eval_kernel_split<2, 3>(mode) : eval_kernel_split<1, 3>(mode);
@@ -163,6 +172,8 @@ struct aceso_ctx {
   const uint32_t *st;
   int split;        // warps per tile (1 or 2)
   int minb;         // register target: 2 or 3 resident CTAs per SM
+  int ev_warps;     // event kernel: warps per CTA (its kernels are templated on it; 8 is built)
+  int ev_minb;      // event kernel: register target
   int tiles_per_warp;  // ACESO_TILES_PER_WARP (measurement knob): tiles each warp walks per launch (default 1)
   int max_ctas[4][8];  // per kernel and mode: resident CTAs (occupancy x SMs)
   int dense_kernel;    // schedule of ACESO_HINT_DENSE: 2 dense kernel (default), 0 per-op kernel (ACESO_DENSE_KERNEL=quad)
@@ -781,6 +792,8 @@ int aceso_load_profile(const aceso_profile_desc *d, int cuda_device, aceso_ctx *
       int v = atoi(env);
       if (v == 2 || v == 3) ctx->minb = v;
     }
+    ctx->ev_warps = kWarps;
+    ctx->ev_minb = ctx->minb;
     {
       const unsigned char *eb = reinterpret_cast<const unsigned char *>(ctx->d_ev);
       ctx->px = reinterpret_cast<const uint4 *>(eb + ev_px);
@@ -812,14 +825,15 @@ int aceso_load_profile(const aceso_profile_desc *d, int cuda_device, aceso_ctx *
         const size_t tabs = ((mode & ACESO_OUT_FULL) ? tab.bytes_full : tab.bytes) + (tab.k_smem ? bytesK : 0u);
         const size_t smem =
             kern == 3   ? (size_t)sc_smem_bytes((uint32_t)(nqs * 4 + 15) & ~15u)
-            : kern == 1 ? (size_t)qo_bytes + ev_ring_bytes() + ev_list_bytes((mode & ACESO_OUT_FULL) != 0)
+            : kern == 1 ? (size_t)qo_bytes + ev_qo_off((mode & ACESO_OUT_FULL) != 0, (uint32_t)ctx->ev_warps)
             : kern == 2 ? ((mode & ACESO_OUT_FULL) ? tab.dbytes_full : tab.dbytes) + kRingBytesPerCta
                         : tabs + kRingBytesPerCta + (ctx->split == 2 ? (size_t)(kWarps / 2) * 32 * sizeof(Xchg) : 0);
         ctx->smem[kern][mode] = smem;
-        void *k = eval_kernel_for(mode, ctx->split, ctx->minb, kern, ctx->e64);
+        void *k = kern == 1 ? eval_kernel_for(mode, 1, ctx->ev_minb, 1, 0, ctx->ev_warps)
+                            : eval_kernel_for(mode, ctx->split, ctx->minb, kern, ctx->e64);
         e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
         int occ = 0;
-        if (e == cudaSuccess) e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k, kThreads, smem);
+        if (e == cudaSuccess) e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k, kern == 1 ? 32 * ctx->ev_warps : kThreads, smem);
         if (e != cudaSuccess || occ < 1) {
           rc = fail(ACESO_ECUDA, "kernel setup (kernel %d, mode %u, %zu B smem): %s", kern, mode, smem, cudaGetErrorString(e));
           break;
@@ -926,7 +940,7 @@ static int eval_impl(aceso_ctx *ctx, const uint8_t *d_codes, const uint64_t *d_h
   const int tpw_hint = P.nch <= 20 ? 3 : P.nch <= 24 ? 2 : 1;
   const int tpw = ((kern == 1 || kern == 3) && (flags & ACESO_HINT_OVERLAP) && tpw_hint > 1) ? std::max(tpw_hint, ctx->tiles_per_warp)
                                                                           : ctx->tiles_per_warp;
-  const int tiles_per_cta = (kern != 0 ? kWarps : kWarps / ctx->split) * tpw;
+  const int tiles_per_cta = (kern == 1 ? ctx->ev_warps : kern != 0 ? kWarps : kWarps / ctx->split) * tpw;
   const int64_t need = (P.n_tiles + tiles_per_cta - 1) / tiles_per_cta;
   int grid = (int)std::max<int64_t>(1, std::min<int64_t>(need, ctx->max_ctas[kern][mode]));
   if (kern == 3) {
@@ -940,7 +954,9 @@ static int eval_impl(aceso_ctx *ctx, const uint8_t *d_codes, const uint64_t *d_h
   CUDA_TRY(cudaGetDevice(&prev));
   if (prev != ctx->device) CUDA_TRY(cudaSetDevice(ctx->device));
   void *args[] = {&P};
-  cudaError_t e = cudaLaunchKernel(eval_kernel_for(mode, ctx->split, ctx->minb, kern, ctx->e64), dim3(grid), dim3(kThreads), args, ctx->smem[kern][mode],
+  void *kfn = kern == 1 ? eval_kernel_for(mode, 1, ctx->ev_minb, 1, 0, ctx->ev_warps)
+                        : eval_kernel_for(mode, ctx->split, ctx->minb, kern, ctx->e64);
+  cudaError_t e = cudaLaunchKernel(kfn, dim3(grid), dim3(kern == 1 ? 32 * ctx->ev_warps : kThreads), args, ctx->smem[kern][mode],
                                    reinterpret_cast<cudaStream_t>(stream));
   if (prev != ctx->device) cudaSetDevice(prev);
   if (e != cudaSuccess) return fail(ACESO_ECUDA, "eval launch: %s", cudaGetErrorString(e));

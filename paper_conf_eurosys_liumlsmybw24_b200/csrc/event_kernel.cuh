@@ -40,23 +40,22 @@ constexpr int kEvRingSlots = 2;   // per-warp ring depth
 constexpr int kEvSlotChunks = 4;  // 16-op chunks per ring slot (2 KB)
 constexpr int kEvSlotBytes = kEvSlotChunks * 512;
 
-// Dynamic shared memory, blocks of [warp][2 KB] with lane stride 16 B (one per-lane base
-// register lb = sb + 2048 warp + 16 lane addresses them through immediate offsets):
-//   ring slot s  lb + kEvBlock s + 512 c   the warp's cp.async.bulk ring (2 slots x 4 chunks)
+// Dynamic shared memory: per warp one 8 KB block of four 2 KB parts with lane stride 16 B
+// (one per-lane base register lb = sb + 8192 warp + 16 lane addresses them through
+// immediate offsets, independent of the CTA's warp count W):
+//   ring slot s  lb + 2048 s + 512 c       the warp's cp.async.bulk ring (2 slots x 4 chunks)
 //   F            lb + kEvF + 512 k         list entry k: activity words of the chunk
 //   C            lb + kEvC + 512 k         cumulative phase-A recompute sums dS, dA (u64 x 2)
 // then X = [warp][k][lane] records {recompute peak since the previous entry, chunk index}
-// (8 B; FULL: 16 B with the cumulative dC), addressed from lx = sb + kEvX + rec (warp,
+// (8 B; FULL: 16 B with the cumulative dC), addressed from lx = sb + ev_x_off(W) + rec (warp,
 // lane), and the per-quad signature table (runtime size).
-constexpr uint32_t kEvBlock = (uint32_t)kWarps * 2048u;
-constexpr uint32_t kEvF = 2u * kEvBlock, kEvC = 3u * kEvBlock, kEvX = 4u * kEvBlock;
-static_assert(kEvSlotBytes == 2048 && kEvCap * 512 == 2048, "per-warp blocks are 2 KB");
+constexpr uint32_t kEvWarpBytes = 8192u, kEvF = 4096u, kEvC = 6144u;
+static_assert(kEvSlotBytes == 2048 && kEvCap * 512 == 2048, "per-warp parts are 2 KB");
 __host__ __device__ constexpr uint32_t ev_xrec(bool full) { return full ? 16u : 8u; }
-__host__ __device__ constexpr uint32_t ev_ring_bytes() { return 2u * kEvBlock; }
-__host__ __device__ constexpr uint32_t ev_list_bytes(bool full) {
-  return 2u * kEvBlock + (uint32_t)kWarps * kEvCap * 32u * ev_xrec(full);
+__host__ __device__ constexpr uint32_t ev_x_off(uint32_t w) { return w * kEvWarpBytes; }
+__host__ __device__ constexpr uint32_t ev_qo_off(bool full, uint32_t w) {
+  return w * (kEvWarpBytes + kEvCap * 32u * ev_xrec(full));
 }
-__host__ __device__ constexpr uint32_t ev_qo_off(bool full) { return ev_ring_bytes() + ev_list_bytes(full); }
 __host__ __device__ constexpr uint32_t ev_snap_bytes(bool) { return 0u; }
 
 __device__ __forceinline__ uint64_t u64of(uint32_t lo, uint32_t hi) {
@@ -341,7 +340,7 @@ __device__ __forceinline__ uint32_t ev_rc_mask(uint4 f) {
 // phase B over every lane's list (warp-uniform call), lockstep over ITEMS: each step every
 // lane with work left takes its next item in op order — an event (run close/open, stage
 // close) or a recompute segment (the recompute flags of one quad up to its next event:
-// one pattern lookup under the open run). lb, lx = this lane's bases (see kEvBlock).
+// one pattern lookup under the open run). lb, lx = this lane's bases (see kEvWarpBytes).
 template <uint32_t MODE>
 __device__ __forceinline__ void ev_drain(EvCand &s, const EvalParams &P, uint32_t qo, uint32_t lb,
                                          uint32_t lx, int64_t cand, bool active) {
@@ -405,21 +404,22 @@ __device__ __forceinline__ uint4 pad_tail(uint4 w4, uint32_t nvl) {
   return w4;
 }
 
-template <uint32_t MODE, int MINB>
-__global__ void __launch_bounds__(kThreads, MINB) event_kernel(const __grid_constant__ EvalParams P) {
+// W warps per CTA (the launch uses 32 W threads)
+template <uint32_t MODE, int MINB, int W>
+__global__ void __launch_bounds__(32 * W, MINB) event_kernel(const __grid_constant__ EvalParams P) {
   extern __shared__ __align__(128) unsigned char sm_raw[];
   __shared__ __align__(8) uint64_t s_tbar;
-  __shared__ __align__(8) uint64_t s_ring_bar[kEvRingSlots][kWarps];
-  __shared__ uint64_t s_ck[kWarps];
-  __shared__ int64_t s_idx[kWarps];
+  __shared__ __align__(8) uint64_t s_ring_bar[kEvRingSlots][W];
+  __shared__ uint64_t s_ck[W];
+  __shared__ int64_t s_idx[W];
   constexpr bool FULL = (MODE & kFull) != 0;
   constexpr uint32_t XR = ev_xrec(FULL);
 
   const uint32_t lane = threadIdx.x & 31u, warp = threadIdx.x >> 5;
   const uint32_t sb = smem_addr(sm_raw);
-  const uint32_t qo = sb + ev_qo_off(FULL);
-  const uint32_t lb = sb + warp * 2048u + lane * 16u;  // see kEvBlock
-  const uint32_t lx = sb + kEvX + warp * kEvCap * 32u * XR + lane * XR;
+  const uint32_t qo = sb + ev_qo_off(FULL, W);
+  const uint32_t lb = sb + warp * kEvWarpBytes + lane * 16u;  // see kEvWarpBytes
+  const uint32_t lx = sb + ev_x_off(W) + warp * kEvCap * 32u * XR + lane * XR;
 
   if (threadIdx.x == 0) {
     mbar_init(smem_addr(&s_tbar), 1);
@@ -440,8 +440,8 @@ __global__ void __launch_bounds__(kThreads, MINB) event_kernel(const __grid_cons
   const uint32_t ngroups = (nch + kEvSlotChunks - 1) / kEvSlotChunks;
   // tile indices fit 32 bits (aceso_eval rejects n >= 2^37)
   const uint32_t n_tiles = (uint32_t)P.n_tiles;
-  const uint32_t first_tile = blockIdx.x * kWarps + warp;
-  const uint32_t tile_stride = gridDim.x * kWarps;
+  const uint32_t first_tile = blockIdx.x * W + warp;
+  const uint32_t tile_stride = gridDim.x * W;
   const unsigned char *codes = reinterpret_cast<const unsigned char *>(P.codes);
 
   // producer state (lane 0): the next (tile, slot group) to copy; done when it_tile >= n_tiles
@@ -451,7 +451,7 @@ __global__ void __launch_bounds__(kThreads, MINB) event_kernel(const __grid_cons
     const uint32_t a = kEvSlotChunks * it_g, b = min(a + kEvSlotChunks, nch);
     const uint32_t bar = smem_addr(&s_ring_bar[slot][warp]);
     mbar_expect_tx(bar, (b - a) * 512u);
-    bulk_g2s(lb + kEvBlock * slot, codes + ((size_t)it_tile * nch + a) * 512, (b - a) * 512u, bar);
+    bulk_g2s(lb + kEvSlotBytes * slot, codes + ((size_t)it_tile * nch + a) * 512, (b - a) * 512u, bar);
     if (++it_g == ngroups) {
       it_g = 0;
       it_tile += tile_stride;
@@ -530,8 +530,8 @@ __global__ void __launch_bounds__(kThreads, MINB) event_kernel(const __grid_cons
 #pragma unroll 1
     for (uint32_t g = 0; g < ngroups; ++g) {
       const uint32_t ch0 = kEvSlotChunks * g, nc = min((uint32_t)kEvSlotChunks, nch - ch0);
-      const uint32_t addr = lb + kEvBlock * slot;
-      mbar_wait(smem_addr(&s_ring_bar[0][warp]) + 8u * kWarps * slot, phase);
+      const uint32_t addr = lb + kEvSlotBytes * slot;
+      mbar_wait(smem_addr(&s_ring_bar[0][warp]) + 8u * W * slot, phase);
       if (g == 0) {
         // seed the previous word so that op 0 always shows a tp difference (an event)
         const uint32_t w0 = lds32(addr);

@@ -419,6 +419,29 @@ def test_kernel_variants_parity(kernel, split, minb, name, monkeypatch):
 
 
 @pytest.mark.parametrize("minb", ["2", "3"])
+@pytest.mark.parametrize("name", ["gpt3-1.3b", "wrn", "gpt-1k"])
+def test_event_kernel_two_tiles_per_warp_parity(minb, name, monkeypatch):
+    """The event kernel at both register targets with every warp walking two tiles through
+    its ring (the persistent path of large batches): FULL outputs, selection, a ragged last
+    tile."""
+    monkeypatch.setenv("ACESO_KERNEL", "events")
+    monkeypatch.setenv("ACESO_MINB", minb)
+    monkeypatch.setenv("ACESO_TILES_PER_WARP", "2")  # every warp walks two tiles through its ring
+    prof = P.WORKLOADS[name]()
+    ctx = A.Context(prof, 0)
+    _ctx_cache[id(prof)] = (prof, ctx)
+    try:
+        n = 333 if name == "gpt-1k" else 2113
+        codes, hdr = ai.search_shaped(prof, SEED + 32, 0, n, group_size=16)
+        compare(prof, codes, hdr, full=True)
+        codes, hdr = ai.dense_random(prof, SEED + 33, 0, n // 3)
+        compare(prof, codes, hdr)
+    finally:
+        _ctx_cache.pop(id(prof), None)
+        ctx.close()
+
+
+@pytest.mark.parametrize("minb", ["2", "3"])
 @pytest.mark.parametrize("dense_kernel", ["dense", "quad"])
 @pytest.mark.parametrize("name", ["gpt3-1.3b", "t5", "wrn", "gpt3-13b", "toy-a", "toy-b"])
 def test_dense_hint_kernels_parity(dense_kernel, minb, name, monkeypatch):
