@@ -580,10 +580,18 @@ def measure_dp(A, ctx, prof, budget, search=None):
     from paper_conf_eurosys_liumlsmybw24_b200 import search as S
     dp = X.exhaustive_best(prof, ctx)
     dcodes, dhdr = dp.pop("codes", None), dp.pop("hdr", None)
+    t0 = time.perf_counter()
+    meg = X.megatron_best(prof, S.GPUEvaluator(ctx))
+    meg["time_s"] = time.perf_counter() - t0
+    meg["note"] = ("the paper's Megatron-LM baseline space (P:L304-305): global (pp, tp, dp, "
+                   "microbatch, recompute) over an even op partition, evaluated with the same model")
+    dp["megatron_grid"] = meg
     if search is not None and dp["best"]:
         sb = search["best"]
         dp["search_vs_exhaustive"] = {"search_best": [sb["class"], sb["cost"]],
                                       "exhaustive_best": [dp["best"]["class"], dp["best"]["cost"]],
+                                      "megatron_grid_best": ([meg["best"]["class"], meg["best"]["cost"]]
+                                                             if meg.get("best") else None),
                                       "search_explored": search["evaluated"]}
         if dcodes is not None and budget > 0:
             hres, hst = S.search(prof, S.GPUEvaluator(ctx), budget_s=budget, patience=8,

@@ -22,7 +22,7 @@ import numpy as np
 import torch
 
 from .api import Context, enum_cuts, enum_cuts_count
-from .search import encode, header
+from .search import encode, header, perf_of
 
 
 def families(prof, max_per_family: int = 1 << 27):
@@ -117,3 +117,54 @@ def exhaustive_best(prof, ctx: Context, batch: int = 1 << 22, max_per_family: in
             break
         acc += fam[3]
     return res
+
+
+def megatron_grid(prof):
+    """The paper's Megatron-LM baseline configuration space ("a grid search over
+    all these options using ACESO's performance model"): global settings only -- p pipeline
+    stages (p a power of two dividing the device count), every stage on G/p devices with the
+    same (tp, dp), the ops partitioned evenly (stage i = ops [L i / p, L (i + 1) / p), the
+    search's initial partition), recomputation of every op or none, every microbatch size whose
+    per-GPU batch is in the profile. Returns row-major codes [n][L] and headers [n]."""
+    L, G = prof.n_ops, prof.n_devices
+    rows, hdrs = [], []
+    p = 1
+    while p <= min(G, L):
+        if G % p == 0:
+            g = int(math.log2(G // p))
+            starts = [L * i // p for i in range(p)]
+            for tpl in range(0, min(g, prof.n_tp - 1) + 1):
+                dpl = g - tpl
+                if dpl >= prof.n_dp:
+                    continue
+                for rc in (0, 1):
+                    row = np.full(L, encode(0, tpl, dpl, rc), np.uint8)
+                    row[starts] |= 1
+                    for mbs in range(dpl, dpl + prof.n_b):
+                        if (1 << mbs) > prof.global_batch or prof.global_batch % (1 << mbs):
+                            continue
+                        rows.append(row)
+                        hdrs.append(header(mbs, p))
+        p *= 2
+    if not rows:
+        return np.zeros((0, L), np.uint8), np.zeros(0, np.uint64)
+    return np.stack(rows), np.array(hdrs, np.uint64)
+
+
+def megatron_best(prof, evaluator):
+    """Evaluates the Megatron grid (one batch through `evaluator.evaluate`); the best
+    configuration by (class, cost) with the lowest index on ties (R12)."""
+    codes, hdr = megatron_grid(prof)
+    if len(hdr) == 0:
+        return {"explored": 0, "best": None}
+    r = evaluator.evaluate(codes, hdr)
+    best, bi = None, -1
+    for i in range(len(hdr)):
+        key = perf_of(int(r["info"][i]), r["iter"][i], r["max_mem"][i])
+        if key[0] < 2 and (best is None or key < best):
+            best, bi = key, i
+    out = {"explored": int(len(hdr)), "best": None}
+    if best is not None:
+        out["best"] = {"class": best[0], "cost": best[1], "index": bi, "p": int(hdr[bi] >> np.uint64(8)),
+                       "mbs_log2": int(hdr[bi] & np.uint64(0xFF)), "code": int(codes[bi][0] & 0xFE)}
+    return out

@@ -664,6 +664,29 @@ def _keys_of(r):
     return (cls << np.uint64(62)) | cost  # perf_of as one ordered integer
 
 
+def _oom_excess(r, capacity):
+    """Per candidate: sum over its stages of the memory above the capacity, sum_i max(0,
+    Mem_i - C), for OOM candidates (0 for the others). The search's tie-break among OOM
+    candidates of equal max_i Mem_i (R26): the one closer to feasibility first, so a
+    recompute move that fixes the whole bottleneck stage wins over one that only brings it
+    down to the next stage's memory."""
+    info = np.asarray(r["info"], np.uint64)
+    oom = ((info & np.uint64(INFO_OOM)) != 0) & ((info & np.uint64(INFO_INVALID)) == 0)
+    ex = np.zeros(len(info), np.int64)
+    rows = np.flatnonzero(oom)
+    if len(rows) == 0:
+        return ex
+    sm = r["stage_mem"]
+    if isinstance(sm, torch.Tensor):
+        sm = sm[torch.from_numpy(rows).to(sm.device)].cpu().numpy()
+    else:
+        sm = np.asarray(sm)[rows].view(np.int64)
+    p = ((info[rows] >> np.uint64(8)) & np.uint64(0xFF)).astype(np.int64)
+    live = np.arange(sm.shape[1])[None, :] < p[:, None]
+    ex[rows] = np.where(live, np.maximum(sm.astype(np.int64) - int(capacity), 0), 0).sum(axis=1)
+    return ex
+
+
 class _Chunk:
     """The configurations one hop added to a search's unexplored set, kept as arrays in
     best-performance-first order (stable: generation order among equals). Nodes are only
@@ -718,6 +741,8 @@ class _Search:
         self.chunks = []   # unexplored configurations, in insertion order (_Chunk)
         self.done = False
         self.improvements = 0
+        self.last_best = start.perf  # patience bookkeeping (search())
+        self.stale = 0
 
     def get_best_of_unexplored(self):
         """GetBestOf(unexplored) (Alg. 1): the best remaining configuration, the
@@ -805,7 +830,9 @@ def search(prof, evaluator, p_values=None, budget_s=10.0, max_hops=7, beam=4, he
     inc/dec-rc attached (evaluated as rows in a second batch of the hop).
     root_modes: (bottleneck rank, resource rank) tried at the root of a failed multi-hop
     search before GetBestOf: Heuristic-2's next resources, then the secondary bottleneck.
-    max_batches: stop after this many evaluation batches (a budget independent of speed)."""
+    max_batches: stop after this many evaluation batches (a budget independent of speed).
+    patience: a stage count's search stops after this many batches without improving its own
+    best (None: only the clock budget, max_batches and exhausted searches stop)."""
     from . import candidates as C
     t0 = time.perf_counter()
     L = prof.n_ops
@@ -848,18 +875,21 @@ def search(prof, evaluator, p_values=None, budget_s=10.0, max_hops=7, beam=4, he
     batches = 0
     evaluated = len(init)
     history = [(t_best, best.perf)]
-    stale = 0
     while time.perf_counter() - t0 < budget_s and any(not s.done for s in searches) and \
             (max_batches is None or batches < max_batches):
         # one hop of every active search, generated into one batch of descriptors
         owners, chunks, base_rows, rank_rows = [], [], [], []
         total = 0
+        share = max_batch // max(1, sum(1 for s in searches if not s.done))
         for si, s in enumerate(searches):
             if s.done:
                 continue
             bn_rank, res_rank = root_modes[s.mode] if s.hop == 0 else (0, 0)
+            # every active search (stage count) gets an equal share of the batch, so long
+            # models' many-candidate hops cannot starve the later searches
+            cap = total + share
             for nd in s.frontier:
-                if nd.perf[0] == 2 or total >= max_batch:
+                if nd.perf[0] == 2 or total >= cap:
                     continue
                 p = int((nd.codes & 1).sum())
                 kw = {}
@@ -870,7 +900,7 @@ def search(prof, evaluator, p_values=None, budget_s=10.0, max_hops=7, beam=4, he
                 cd, rk = prims.describe_all(nd.codes, nd.mbs, nd.info, nd.comp, nd.comm, nd.time, **kw)
                 if len(cd) == 0:
                     continue
-                cd = cd[: max_batch - total]
+                cd = cd[: cap - total]
                 cd["base"] = len(base_rows)
                 row = np.zeros(stride, np.uint8)
                 row[:L] = nd.codes
@@ -893,13 +923,14 @@ def search(prof, evaluator, p_values=None, budget_s=10.0, max_hops=7, beam=4, he
         # configurations seen before (or earlier in this batch) are dropped
         keep = seen.first_new(r)
         keys = _keys_of(r)
+        ex = _oom_excess(r, prof.mem_capacity)
         hop_chunks = {}
         for si, s in enumerate(searches):
             if s.done:
                 continue
             idx = np.nonzero(keep & (owner == si))[0]
             # Heuristic-2: best estimated performance first (stable: generation order)
-            idx = idx[np.argsort(keys[idx], kind="stable")]
+            idx = idx[np.lexsort((ex[idx], keys[idx]))]  # stable: generation order among equals
             hop_chunks[si] = [_Chunk(keys, idx, r, bases, ranks, cands, L)] if len(idx) else []
         # recomputation attached to the primitives' results: a second batch of the hop
         if attach_rc:
@@ -925,12 +956,13 @@ def search(prof, evaluator, p_values=None, budget_s=10.0, max_hops=7, beam=4, he
                 evaluated += len(rows)
                 keep2 = seen.first_new(rr)
                 keys2 = _keys_of(rr)
+                ex2 = _oom_excess(rr, prof.mem_capacity)
                 rowner = np.array(rowner)
                 mbss = np.array(mbss)
                 for si in hop_chunks:
                     idx = np.nonzero(keep2 & (rowner == si))[0]
                     if len(idx):
-                        idx = idx[np.argsort(keys2[idx], kind="stable")]
+                        idx = idx[np.lexsort((ex2[idx], keys2[idx]))]
                         hop_chunks[si].append(_Chunk(keys2, idx, rr, None, None, None, L, codes=rc_codes, mbs=mbss))
         for si, s in enumerate(searches):
             if s.done:
@@ -977,11 +1009,19 @@ def search(prof, evaluator, p_values=None, budget_s=10.0, max_hops=7, beam=4, he
             best = cur_best
             t_best = time.perf_counter() - t0
             history.append((t_best, best.perf))
-            stale = 0
-        else:
-            stale += 1
-        if patience is not None and stale >= patience:
-            break
+        # patience per search (stage count): a search stops after `patience` batches without
+        # improving its own best (each stage count is its own Alg. 1 run); the clock
+        # budget stops them all
+        for s in searches:
+            if s.done:
+                continue
+            if s.best.perf < s.last_best:
+                s.last_best = s.best.perf
+                s.stale = 0
+            else:
+                s.stale += 1
+                if patience is not None and s.stale >= patience:
+                    s.done = True
     total_t = time.perf_counter() - t0
     stats = dict(time_s=total_t, time_to_best_s=t_best, batches=batches, evaluated=evaluated,
                  searches=len(searches), history=history,
@@ -1018,6 +1058,7 @@ def finetune_dims(prof, evaluator, codes, mbs, dims=None, max_rounds=64):
         stats["rounds"] += 1
         stats["evaluated"] += len(differs)
         keys = _keys_of(r)
+        ex = _oom_excess(r, prof.mem_capacity)
         t = int(np.argmin(keys))  # the lowest index among equals
         if int(keys[t]) >= _key(perf):
             break

@@ -236,3 +236,54 @@ def test_dimension_finetune_improves_or_keeps():
     o = oracle.evaluate(prof, codes[None, :], np.array([S.header(mbs, 2)], np.uint64), dims=dims[None, :])
     assert perf_tuple(o, 0) == perf
     assert len(st["switched"]) == int(dims.sum())
+
+
+@pytest.mark.parametrize("name", ["toy-a", "gpt3-1.3b", "t5", "wrn"])
+def test_megatron_grid_space(name):
+    """The Megatron-LM baseline space: every configuration is valid under the
+    oracle, uses global settings (one (tp, dp, recompute) for all ops, even op partition),
+    covers each (p, tp, recompute, microbatch) combination once, and megatron_best returns its
+    (class, cost, lowest index) optimum."""
+    from paper_conf_eurosys_liumlsmybw24_b200 import exhaustive as X
+    prof = P.WORKLOADS[name]()
+    codes, hdr = X.megatron_grid(prof)
+    L, G = prof.n_ops, prof.n_devices
+    o = oracle.evaluate(prof, codes, hdr, threads=4)
+    assert not np.any(o["info"] & oracle.INFO_INVALID)
+    seen = set()
+    for c, h in zip(codes, hdr):
+        p, mbs = int(h) >> 8, int(h) & 0xFF
+        heads = np.flatnonzero(c & 1)
+        assert list(heads) == [L * i // p for i in range(p)]
+        body = c & 0xFE
+        assert np.all(body == body[0])
+        tpl, dpl = (int(body[0]) >> 1) & 7, int(body[0]) >> 5
+        assert p << (tpl + dpl) == G
+        key = (p, tpl, (int(body[0]) >> 4) & 1, mbs)
+        assert key not in seen
+        seen.add(key)
+    n_rc = 2
+    assert len(seen) % n_rc == 0
+    r = X.megatron_best(prof, OracleEvaluator(prof))
+    keys = [S.perf_of(int(i), t, m) for i, t, m in zip(o["info"], o["iter"], o["max_mem"])]
+    best = min((k, i) for i, k in enumerate(keys) if k[0] < 2)
+    assert (r["best"]["class"], r["best"]["cost"], r["best"]["index"]) == (best[0][0], best[0][1], best[1])
+
+
+def test_oom_excess_tie_break():
+    """R26: the excess sum_i max(0, Mem_i - C) over a candidate's p stages, OOM candidates only."""
+    C = 100
+    info = np.array([(2 << 8) | S.INFO_OOM, (3 << 8) | S.INFO_OOM, (2 << 8), (2 << 8) | S.INFO_OOM | S.INFO_INVALID],
+                    np.uint32)
+    sm = np.array([[150, 120, 999], [101, 90, 130], [150, 150, 150], [500, 500, 500]], np.uint64)
+    ex = S._oom_excess(dict(info=info, stage_mem=sm), C)
+    assert list(ex) == [70, 31, 0, 0]
+
+
+def test_oom_phase_fixes_a_whole_stage_per_batch():
+    """With R26 the 1K-layer model's 8-stage search (initial configuration OOM: every stage
+    holds its in-flight activations) becomes feasible within ten batches (five hops with their recompute attachment): each recompute move
+    fixes the whole bottleneck stage instead of stopping at the next stage's memory."""
+    prof = P.WORKLOADS["gpt-1k"]()
+    res, st = S.search(prof, OracleEvaluator(prof), p_values=[8], budget_s=1e9, max_batches=10)
+    assert res.perf[0] == 0, res.perf
