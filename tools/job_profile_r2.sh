@@ -1,5 +1,5 @@
 #!/bin/bash
-# Round-2 evidence: default bench line, ncu launch list of the headline bench command, full ncu
+# Round-2 evidence (final): default bench line, ncu launch list of the headline bench command, full ncu
 # capture of one headline launch and of one GPT-3 1.3B 64K launch (event kernel).
 mkdir -p gpurun_out
 python -c "import oracle, aceso_inputs; oracle.build(); aceso_inputs.build()"
