@@ -66,16 +66,16 @@ void *eval_kernel_split(uint32_t mode) {
   }
 }
 
-template <int B, int W>
+template <int B, int W, int SC>
 void *event_kernel_for(uint32_t mode) {
   switch (mode) {
-    case 1: return reinterpret_cast<void *>(&event_kernel<1, B, W>);
-    case 2: return reinterpret_cast<void *>(&event_kernel<2, B, W>);
-    case 3: return reinterpret_cast<void *>(&event_kernel<3, B, W>);
-    case 4: return reinterpret_cast<void *>(&event_kernel<4, B, W>);
-    case 5: return reinterpret_cast<void *>(&event_kernel<5, B, W>);
-    case 6: return reinterpret_cast<void *>(&event_kernel<6, B, W>);
-    case 7: return reinterpret_cast<void *>(&event_kernel<7, B, W>);
+    case 1: return reinterpret_cast<void *>(&event_kernel<1, B, W, SC>);
+    case 2: return reinterpret_cast<void *>(&event_kernel<2, B, W, SC>);
+    case 3: return reinterpret_cast<void *>(&event_kernel<3, B, W, SC>);
+    case 4: return reinterpret_cast<void *>(&event_kernel<4, B, W, SC>);
+    case 5: return reinterpret_cast<void *>(&event_kernel<5, B, W, SC>);
+    case 6: return reinterpret_cast<void *>(&event_kernel<6, B, W, SC>);
+    case 7: return reinterpret_cast<void *>(&event_kernel<7, B, W, SC>);
     default: return nullptr;
   }
 }
@@ -84,9 +84,11 @@ void *event_kernel_for(uint32_t mode) {
 // Built: 8 warps at 2 or 3 CTAs per SM. Measured and dropped (round 2, every BASELINE
 // workload): 6 warps x 3 CTAs (18 warps per SM at 96 registers), 4 warps x 4 / 5 / 6 CTAs —
 // within 0.3% of the better 8-warp shape on the 1K-layer model and 1-10% slower elsewhere.
-void *event_kernel_shape(uint32_t mode, int warps, int minb) {
+// Ring slots: 8 chunks (4 KB) at 2 CTAs per SM, 4 chunks (2 KB) at 3.
+void *event_kernel_shape(uint32_t mode, int warps, int minb, int sc) {
   (void)warps;
-  return minb == 2 ? event_kernel_for<2, 8>(mode) : event_kernel_for<3, 8>(mode);
+  if (minb == 2) return sc == 8 ? event_kernel_for<2, 8, 8>(mode) : event_kernel_for<2, 8, 4>(mode);
+  return event_kernel_for<3, 8, 4>(mode);
 }
 
 template <int B>
@@ -134,14 +136,14 @@ void *scan_kernel_for(uint32_t mode) {
 // kernel 0: per-op/quad kernel (eval_kernel.cuh); kernel 1: event kernel (event_kernel.cuh);
 // kernel 2: dense kernel (dense_kernel.cuh, ACESO_HINT_DENSE); kernel 3: scan kernel
 // (scan_kernel.cuh, exact u64 tables; e64: wide transient-memory table)
-void *eval_kernel_for(uint32_t mode, int split, int minb, int kernel, int e64 = 0, int ev_warps = kWarps) {
+void *eval_kernel_for(uint32_t mode, int split, int minb, int kernel, int e64 = 0, int ev_warps = kWarps, int ev_sc = 4) {
   if (kernel == 3) {
     // the scan kernel's default register target is 2 CTAs per SM (its ring and lists take
     // ~100 KB of shared memory per CTA); ACESO_MINB=3 selects the 80-register build
     if (minb == 3 && getenv("ACESO_MINB")) return e64 ? scan_kernel_for<true, 3>(mode) : scan_kernel_for<false, 3>(mode);
     return e64 ? scan_kernel_for<true, 2>(mode) : scan_kernel_for<false, 2>(mode);
   }
-  if (kernel == 1) return event_kernel_shape(mode, ev_warps, minb);
+  if (kernel == 1) return event_kernel_shape(mode, ev_warps, minb, ev_sc);
   if (kernel == 2) return minb == 2 ? dense_kernel_for<2>(mode) : dense_kernel_for<3>(mode);
   if (minb == 2) return split == 2 ? eval_kernel_split<2, 2>(mode) : eval_kernel_split<1, 2>(mode);
   return split == 2 ? eval_kernel_split<2, 3>(mode) : eval_kernel_split<1, 3>(mode);
@@ -174,6 +176,7 @@ struct aceso_ctx {
   int minb;         // register target: 2 or 3 resident CTAs per SM
   int ev_warps;     // event kernel: warps per CTA (its kernels are templated on it; 8 is built)
   int ev_minb;      // event kernel: register target
+  int ev_sc;        // event kernel: 16-op chunks per ring slot (8 at 2 CTAs per SM, else 4)
   int tiles_per_warp;  // ACESO_TILES_PER_WARP (measurement knob): tiles each warp walks per launch (default 1)
   int max_ctas[4][8];  // per kernel and mode: resident CTAs (occupancy x SMs)
   int dense_kernel;    // schedule of ACESO_HINT_DENSE: 2 dense kernel (default), 0 per-op kernel (ACESO_DENSE_KERNEL=quad)
@@ -192,6 +195,11 @@ struct aceso_ctx {
   size_t dims_smem[8];
   int dims_max_ctas[8];
 };
+
+// chunks per ring slot of the event kernel in this mode: FULL keeps 4 (its 16-byte list records
+// would not leave room for two 8-chunk CTAs per SM)
+static int ev_sc_for(const aceso_ctx *ctx, uint32_t mode) { return (mode & ACESO_OUT_FULL) ? 4 : ctx->ev_sc; }
+
 
 namespace {
 // kernel parameter block of a call (tables, outputs, selection); codes/hdr set by the caller
@@ -794,6 +802,9 @@ int aceso_load_profile(const aceso_profile_desc *d, int cuda_device, aceso_ctx *
     }
     ctx->ev_warps = kWarps;
     ctx->ev_minb = ctx->minb;
+    ctx->ev_sc = ctx->minb == 2 ? 8 : 4;
+    if (const char *env = getenv("ACESO_EV_SLOT"))  // measurement knob: 4 or 8 (8 needs 2 CTAs per SM)
+      if (atoi(env) == 4 || (atoi(env) == 8 && ctx->minb == 2)) ctx->ev_sc = atoi(env);
     {
       const unsigned char *eb = reinterpret_cast<const unsigned char *>(ctx->d_ev);
       ctx->px = reinterpret_cast<const uint4 *>(eb + ev_px);
@@ -825,11 +836,11 @@ int aceso_load_profile(const aceso_profile_desc *d, int cuda_device, aceso_ctx *
         const size_t tabs = ((mode & ACESO_OUT_FULL) ? tab.bytes_full : tab.bytes) + (tab.k_smem ? bytesK : 0u);
         const size_t smem =
             kern == 3   ? (size_t)sc_smem_bytes((uint32_t)(nqs * 4 + 15) & ~15u)
-            : kern == 1 ? (size_t)qo_bytes + ev_qo_off((mode & ACESO_OUT_FULL) != 0, (uint32_t)ctx->ev_warps)
+            : kern == 1 ? (size_t)ev_smem_bytes((mode & ACESO_OUT_FULL) != 0, (uint32_t)ctx->ev_warps, ev_sc_for(ctx, mode), qo_bytes)
             : kern == 2 ? ((mode & ACESO_OUT_FULL) ? tab.dbytes_full : tab.dbytes) + kRingBytesPerCta
                         : tabs + kRingBytesPerCta + (ctx->split == 2 ? (size_t)(kWarps / 2) * 32 * sizeof(Xchg) : 0);
         ctx->smem[kern][mode] = smem;
-        void *k = kern == 1 ? eval_kernel_for(mode, 1, ctx->ev_minb, 1, 0, ctx->ev_warps)
+        void *k = kern == 1 ? eval_kernel_for(mode, 1, ctx->ev_minb, 1, 0, ctx->ev_warps, ev_sc_for(ctx, mode))
                             : eval_kernel_for(mode, ctx->split, ctx->minb, kern, ctx->e64);
         e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
         int occ = 0;
@@ -954,7 +965,7 @@ static int eval_impl(aceso_ctx *ctx, const uint8_t *d_codes, const uint64_t *d_h
   CUDA_TRY(cudaGetDevice(&prev));
   if (prev != ctx->device) CUDA_TRY(cudaSetDevice(ctx->device));
   void *args[] = {&P};
-  void *kfn = kern == 1 ? eval_kernel_for(mode, 1, ctx->ev_minb, 1, 0, ctx->ev_warps)
+  void *kfn = kern == 1 ? eval_kernel_for(mode, 1, ctx->ev_minb, 1, 0, ctx->ev_warps, ev_sc_for(ctx, mode))
                         : eval_kernel_for(mode, ctx->split, ctx->minb, kern, ctx->e64);
   cudaError_t e = cudaLaunchKernel(kfn, dim3(grid), dim3(kern == 1 ? 32 * ctx->ev_warps : kThreads), args, ctx->smem[kern][mode],
                                    reinterpret_cast<cudaStream_t>(stream));

@@ -37,24 +37,30 @@ namespace aceso {
 
 constexpr int kEvCap = 4;         // event chunks per lane between drains (checked every 2 chunks)
 constexpr int kEvRingSlots = 2;   // per-warp ring depth
-constexpr int kEvSlotChunks = 4;  // 16-op chunks per ring slot (2 KB)
-constexpr int kEvSlotBytes = kEvSlotChunks * 512;
 
-// Dynamic shared memory: per warp one 8 KB block of four 2 KB parts with lane stride 16 B
-// (one per-lane base register lb = sb + 8192 warp + 16 lane addresses them through
-// immediate offsets, independent of the CTA's warp count W):
-//   ring slot s  lb + 2048 s + 512 c       the warp's cp.async.bulk ring (2 slots x 4 chunks)
-//   F            lb + kEvF + 512 k         list entry k: activity words of the chunk
-//   C            lb + kEvC + 512 k         cumulative phase-A recompute sums dS, dA (u64 x 2)
+// Dynamic shared memory: per warp one block of parts with lane stride 16 B (one per-lane base
+// register lb = sb + ev_warp_bytes(SC) warp + 16 lane addresses them through immediate
+// offsets, independent of the CTA's warp count W); SC = 16-op chunks per ring slot (4 or 8):
+//   ring slot s  lb + 512 SC s + 512 c     the warp's cp.async.bulk ring (2 slots x SC chunks)
+//   F            lb + ev_f_off(SC) + 512 k list entry k: activity words of the chunk
+//   C            lb + ev_c_off(SC) + 512 k cumulative phase-A recompute sums dS, dA (u64 x 2)
 // then X = [warp][k][lane] records {recompute peak since the previous entry, chunk index}
-// (8 B; FULL: 16 B with the cumulative dC), addressed from lx = sb + ev_x_off(W) + rec (warp,
-// lane), and the per-quad signature table (runtime size).
-constexpr uint32_t kEvWarpBytes = 8192u, kEvF = 4096u, kEvC = 6144u;
-static_assert(kEvSlotBytes == 2048 && kEvCap * 512 == 2048, "per-warp parts are 2 KB");
+// (8 B; FULL: 16 B with the cumulative dC), addressed from lx = sb + ev_x_off(W, SC) + rec
+// (warp, lane), and (SC = 4) the per-quad signature table (runtime size). With SC = 8 the
+// signature table is read through the L1 (__ldg) instead, so two CTAs of 8 warps still fit.
+static_assert(kEvCap * 512 == 2048, "per-warp list parts are 2 KB");
+__host__ __device__ constexpr uint32_t ev_slot_bytes(int sc) { return 512u * (uint32_t)sc; }
+__host__ __device__ constexpr uint32_t ev_f_off(int sc) { return 2u * ev_slot_bytes(sc); }
+__host__ __device__ constexpr uint32_t ev_c_off(int sc) { return ev_f_off(sc) + 2048u; }
+__host__ __device__ constexpr uint32_t ev_warp_bytes(int sc) { return ev_c_off(sc) + 2048u; }
 __host__ __device__ constexpr uint32_t ev_xrec(bool full) { return full ? 16u : 8u; }
-__host__ __device__ constexpr uint32_t ev_x_off(uint32_t w) { return w * kEvWarpBytes; }
-__host__ __device__ constexpr uint32_t ev_qo_off(bool full, uint32_t w) {
-  return w * (kEvWarpBytes + kEvCap * 32u * ev_xrec(full));
+__host__ __device__ constexpr uint32_t ev_x_off(uint32_t w, int sc) { return w * ev_warp_bytes(sc); }
+__host__ __device__ constexpr uint32_t ev_qo_off(bool full, uint32_t w, int sc) {
+  return w * (ev_warp_bytes(sc) + kEvCap * 32u * ev_xrec(full));
+}
+// dynamic shared memory of one CTA (qo_bytes: the signature table's size)
+__host__ __device__ constexpr uint32_t ev_smem_bytes(bool full, uint32_t w, int sc, uint32_t qo_bytes) {
+  return ev_qo_off(full, w, sc) + (sc == 8 ? 0u : qo_bytes);
 }
 __host__ __device__ constexpr uint32_t ev_snap_bytes(bool) { return 0u; }
 
@@ -340,10 +346,11 @@ __device__ __forceinline__ uint32_t ev_rc_mask(uint4 f) {
 // phase B over every lane's list (warp-uniform call), lockstep over ITEMS: each step every
 // lane with work left takes its next item in op order — an event (run close/open, stage
 // close) or a recompute segment (the recompute flags of one quad up to its next event:
-// one pattern lookup under the open run). lb, lx = this lane's bases (see kEvWarpBytes).
-template <uint32_t MODE>
+// one pattern lookup under the open run). lb, lx = this lane's bases (see ev_warp_bytes).
+template <uint32_t MODE, int SC>
 __device__ __forceinline__ void ev_drain(EvCand &s, const EvalParams &P, uint32_t qo, uint32_t lb,
                                          uint32_t lx, int64_t cand, bool active) {
+  constexpr uint32_t kEvF = ev_f_off(SC), kEvC = ev_c_off(SC);
 #ifdef ACESO_EXPERIMENT_NO_PHASEB
   s.ec = 0;
   return;
@@ -379,7 +386,9 @@ __device__ __forceinline__ void ev_drain(EvCand &s, const EvalParams &P, uint32_
         const uint32_t nxt = em & (0xfu << qb);
         const uint32_t lim = nxt ? __ffs(nxt) - 1u : qb + 4u;
         const uint32_t seg = rm & ((1u << lim) - 1u);
-        ev_rc_add<MODE>(s, P, lds32(qo + 4u * (q0 + (j >> 2))), seg >> qb);
+        const uint32_t qsb = SC == 8 ? __ldg(reinterpret_cast<const uint32_t *>(P.evblob + P.qo_off) + (q0 + (j >> 2)))
+                                     : lds32(qo + 4u * (q0 + (j >> 2)));
+        ev_rc_add<MODE>(s, P, qsb, seg >> qb);
         rm &= ~seg;
       }
     }
@@ -404,9 +413,11 @@ __device__ __forceinline__ uint4 pad_tail(uint4 w4, uint32_t nvl) {
   return w4;
 }
 
-// W warps per CTA (the launch uses 32 W threads)
-template <uint32_t MODE, int MINB, int W>
+// W warps per CTA (the launch uses 32 W threads), SC chunks per ring slot
+template <uint32_t MODE, int MINB, int W, int SC>
 __global__ void __launch_bounds__(32 * W, MINB) event_kernel(const __grid_constant__ EvalParams P) {
+  constexpr uint32_t kEvSlotBytes = ev_slot_bytes(SC), kEvF = ev_f_off(SC), kEvC = ev_c_off(SC);
+  constexpr bool QG = SC == 8;  // signature table read through the L1
   extern __shared__ __align__(128) unsigned char sm_raw[];
   __shared__ __align__(8) uint64_t s_tbar;
   __shared__ __align__(8) uint64_t s_ring_bar[kEvRingSlots][W];
@@ -417,9 +428,10 @@ __global__ void __launch_bounds__(32 * W, MINB) event_kernel(const __grid_consta
 
   const uint32_t lane = threadIdx.x & 31u, warp = threadIdx.x >> 5;
   const uint32_t sb = smem_addr(sm_raw);
-  const uint32_t qo = sb + ev_qo_off(FULL, W);
-  const uint32_t lb = sb + warp * kEvWarpBytes + lane * 16u;  // see kEvWarpBytes
-  const uint32_t lx = sb + ev_x_off(W) + warp * kEvCap * 32u * XR + lane * XR;
+  const uint32_t qo = sb + ev_qo_off(FULL, W, SC);
+  const uint32_t lb = sb + warp * ev_warp_bytes(SC) + lane * 16u;  // see ev_warp_bytes
+  const uint32_t lx = sb + ev_x_off(W, SC) + warp * kEvCap * 32u * XR + lane * XR;
+  const uint4 *qg = reinterpret_cast<const uint4 *>(P.evblob + P.qo_off);
 
   if (threadIdx.x == 0) {
     mbar_init(smem_addr(&s_tbar), 1);
@@ -432,12 +444,12 @@ __global__ void __launch_bounds__(32 * W, MINB) event_kernel(const __grid_consta
   __syncthreads();
   if (threadIdx.x == 0) {
     const uint32_t bar = smem_addr(&s_tbar);
-    mbar_expect_tx(bar, P.qo_bytes);
-    bulk_g2s(qo, P.evblob + P.qo_off, P.qo_bytes, bar);
+    mbar_expect_tx(bar, QG ? 0u : P.qo_bytes);  // QG: the arrival alone completes the phase
+    if (!QG) bulk_g2s(qo, P.evblob + P.qo_off, P.qo_bytes, bar);
   }
 
   const uint32_t nch = (uint32_t)P.nch;
-  const uint32_t ngroups = (nch + kEvSlotChunks - 1) / kEvSlotChunks;
+  const uint32_t ngroups = (nch + SC - 1) / SC;
   // tile indices fit 32 bits (aceso_eval rejects n >= 2^37)
   const uint32_t n_tiles = (uint32_t)P.n_tiles;
   const uint32_t first_tile = blockIdx.x * W + warp;
@@ -448,7 +460,7 @@ __global__ void __launch_bounds__(32 * W, MINB) event_kernel(const __grid_consta
   uint32_t it_tile = first_tile;
   uint32_t it_g = 0;
   auto issue_next = [&](uint32_t slot) {
-    const uint32_t a = kEvSlotChunks * it_g, b = min(a + kEvSlotChunks, nch);
+    const uint32_t a = SC * it_g, b = min(a + (uint32_t)SC, nch);
     const uint32_t bar = smem_addr(&s_ring_bar[slot][warp]);
     mbar_expect_tx(bar, (b - a) * 512u);
     bulk_g2s(lb + kEvSlotBytes * slot, codes + ((size_t)it_tile * nch + a) * 512, (b - a) * 512u, bar);
@@ -475,7 +487,7 @@ __global__ void __launch_bounds__(32 * W, MINB) event_kernel(const __grid_consta
   bool active = false;
   // the lists must hold what the next 2 chunks add
   auto drain_check = [&]() {
-    if (__any_sync(0xffffffffu, s.ec + 2u > (uint32_t)kEvCap)) ev_drain<MODE>(s, P, qo, lb, lx, cand, active);
+    if (__any_sync(0xffffffffu, s.ec + 2u > (uint32_t)kEvCap)) ev_drain<MODE, SC>(s, P, qo, lb, lx, cand, active);
   };
   // phase A, one 16-op chunk (ring address a, chunk index ci)
   auto chunk = [&](uint32_t a, uint32_t ci) {
@@ -510,7 +522,7 @@ __global__ void __launch_bounds__(32 * W, MINB) event_kernel(const __grid_consta
         // recompute flags in an event-free chunk: every op is in the open run, whose
         // (tp, dp) is that of op 0 of the chunk
         const uint32_t rr = ev_run(w4.x & 0xffu, s.mbs(), P);
-        const uint4 qs = lds128(qo + 16u * ci);
+        const uint4 qs = QG ? __ldg(qg + ci) : lds128(qo + 16u * ci);
         uint32_t pat;
         if ((pat = quad_rc(f.x))) ev_rc_lookup<MODE>(P, qs.x, rr, pat, cS, cA, rE, cC);
         if ((pat = quad_rc(f.y))) ev_rc_lookup<MODE>(P, qs.y, rr, pat, cS, cA, rE, cC);
@@ -529,7 +541,7 @@ __global__ void __launch_bounds__(32 * W, MINB) event_kernel(const __grid_consta
     pw = 0;
 #pragma unroll 1
     for (uint32_t g = 0; g < ngroups; ++g) {
-      const uint32_t ch0 = kEvSlotChunks * g, nc = min((uint32_t)kEvSlotChunks, nch - ch0);
+      const uint32_t ch0 = SC * g, nc = min((uint32_t)SC, nch - ch0);
       const uint32_t addr = lb + kEvSlotBytes * slot;
       mbar_wait(smem_addr(&s_ring_bar[0][warp]) + 8u * W * slot, phase);
       if (g == 0) {
@@ -548,13 +560,16 @@ __global__ void __launch_bounds__(32 * W, MINB) event_kernel(const __grid_consta
           sts128(la, pad_tail(lds128(la), nvl));
         }
       }
-      if (nc == (uint32_t)kEvSlotChunks) {
-        drain_check();
-        chunk(addr, ch0);
-        chunk(addr + 512u, ch0 + 1u);
-        drain_check();
-        chunk(addr + 1024u, ch0 + 2u);
-        chunk(addr + 1536u, ch0 + 3u);
+      if (nc == (uint32_t)SC) {
+#pragma unroll 1
+        for (uint32_t h = 0; h < (uint32_t)SC; h += 4u) {
+          drain_check();
+          chunk(addr + 512u * h, ch0 + h);
+          chunk(addr + 512u * h + 512u, ch0 + h + 1u);
+          drain_check();
+          chunk(addr + 512u * h + 1024u, ch0 + h + 2u);
+          chunk(addr + 512u * h + 1536u, ch0 + h + 3u);
+        }
       } else {
 #pragma unroll 1
         for (uint32_t c = 0; c < nc; ++c) {
@@ -571,7 +586,7 @@ __global__ void __launch_bounds__(32 * W, MINB) event_kernel(const __grid_consta
       phase ^= slot ^ 1u;  // flips after slot 1
     }
     // ---- tile epilogue: drain, close the last run and stage (no p2p_fwd) ----
-    ev_drain<MODE>(s, P, qo, lb, lx, cand, active);
+    ev_drain<MODE, SC>(s, P, qo, lb, lx, cand, active);
     s.S += cS;  // phase-A recompute deltas after the last event chunk (last stage)
     s.A -= cA;
     s.E = max(s.E, rE);
