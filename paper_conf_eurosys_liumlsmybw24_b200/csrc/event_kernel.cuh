@@ -492,6 +492,11 @@ __global__ void __launch_bounds__(32 * W, MINB) event_kernel(const __grid_consta
   // phase A, one 16-op chunk (ring address a, chunk index ci)
   auto chunk = [&](uint32_t a, uint32_t ci) {
     const uint4 w4 = lds128(a);
+    // QG: the chunk's quad signatures, requested ahead of the activity words (one broadcast
+    // L1 load; its latency is off the recompute lookups' critical path)
+    uint4 qsg = make_uint4(0u, 0u, 0u, 0u);
+    if (QG) asm volatile("ld.global.nc.v4.u32 {%0, %1, %2, %3}, [%4];"
+                         : "=r"(qsg.x), "=r"(qsg.y), "=r"(qsg.z), "=r"(qsg.w) : "l"(qg + ci));
     uint4 f;
     f.x = quad_activity(w4.x, pw);
     f.y = quad_activity(w4.y, w4.x);
@@ -522,7 +527,7 @@ __global__ void __launch_bounds__(32 * W, MINB) event_kernel(const __grid_consta
         // recompute flags in an event-free chunk: every op is in the open run, whose
         // (tp, dp) is that of op 0 of the chunk
         const uint32_t rr = ev_run(w4.x & 0xffu, s.mbs(), P);
-        const uint4 qs = QG ? __ldg(qg + ci) : lds128(qo + 16u * ci);
+        const uint4 qs = QG ? qsg : lds128(qo + 16u * ci);
         uint32_t pat;
         if ((pat = quad_rc(f.x))) ev_rc_lookup<MODE>(P, qs.x, rr, pat, cS, cA, rE, cC);
         if ((pat = quad_rc(f.y))) ev_rc_lookup<MODE>(P, qs.y, rr, pat, cS, cA, rE, cC);
