@@ -11,3 +11,5 @@ timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none -c 400 --c
   python bench.py --steps 20 --warmup 5 --no-all --no-e2e --no-cpu --no-dedup --no-dp --search-budget 0 > gpurun_out/r2_launches.log 2>&1; echo "launches rc=$?"
 timeout 900 ncu --set full --clock-control none --import-source on -k regex:event_kernel -s 1 -c 1 -o gpurun_out/r2_ev1k python tools/prof_one.py gpt-1k 131072 2 > gpurun_out/r2_ev1k.log 2>&1; echo "ncu 1k rc=$?"
 timeout 900 ncu --set full --clock-control none --import-source on -k regex:event_kernel -s 1 -c 1 -o gpurun_out/r2_ev13 python tools/prof_one.py gpt3-1.3b 65536 2 > gpurun_out/r2_ev13.log 2>&1; echo "ncu 1.3b rc=$?"
+timeout 900 python bench.py --batch 1048576 --no-all --no-e2e --no-cpu --no-dedup --no-dp --search-budget 0 --steps 10 --warmup 3 > gpurun_out/r2_bench_1k_1m.json 2> gpurun_out/r2_bench_1k_1m.err; echo "1m rc=$?"
+timeout 2400 python -m pytest tests -m gpu -q -p no:cacheprovider > gpurun_out/gpu_tests_full.log 2>&1; tail -1 gpurun_out/gpu_tests_full.log

@@ -1,7 +1,8 @@
 """Small evaluations for compute-sanitizer (memcheck / racecheck / synccheck) on the round-2
 paths: the scan kernel (wide memory values: u64 transient tables; and the u32 variant via
 ACESO_KERNEL=scan), the dense kernel with a dimension plane (shared-memory and global tables),
-and ACESO_PIPE_LITERAL; every result checked against the oracle."""
+ACESO_PIPE_LITERAL and the event kernel's two ring-slot sizes; every result checked against the
+oracle."""
 import os
 import sys
 
@@ -41,4 +42,10 @@ check(P.WORKLOADS["gpt3-1.3b"](), n, literal=True)                            # 
 del os.environ["ACESO_KERNEL"]
 check(P.WORKLOADS["gpt3-1.3b"](), n, dims=True, full=True)                    # dense + plane, smem tables
 check(P.WORKLOADS["wrn"](), 200, dims=True)                                   # dense + plane, global tables
+# event kernel with 8-chunk ring slots (2 CTAs per SM: SUMMARY + select) and 4-chunk slots
+# (FULL), every warp walking two tiles through its ring
+os.environ["ACESO_TILES_PER_WARP"] = "2"
+check(P.WORKLOADS["gpt-1k"](), 32 * 3 + 5)
+check(P.WORKLOADS["gpt-1k"](), 32 * 3 + 5, full=True)
+del os.environ["ACESO_TILES_PER_WARP"]
 print("round-2 sanitizer run ok")
