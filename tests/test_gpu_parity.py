@@ -746,3 +746,20 @@ def test_eval_global_fuses_the_cross_shard_selection(name):
     cls, cost, idx, sat = A.decode_key(k, shards * n)
     o = oracle.evaluate(prof, codes, hdr, threads=8)
     assert not sat and (cls, cost, idx) == oracle.select(o)
+
+
+@pytest.mark.parametrize("name", ["toy-a", "gpt3-1.3b", "gpt3-13b", "t5", "wrn", "gpt-1k"])
+def test_megatron_grid_gpu_matches_oracle(name):
+    """The Megatron-LM baseline grid evaluated on the GPU (FULL mode through the
+    search's evaluator) selects the same configuration and cost as the oracle."""
+    import os
+    import sys
+    sys.path.insert(0, os.path.dirname(__file__))
+    from oracle_evaluator import OracleEvaluator
+    from paper_conf_eurosys_liumlsmybw24_b200 import exhaustive as X
+    from paper_conf_eurosys_liumlsmybw24_b200 import search as S
+    prof = P.WORKLOADS[name]()
+    ctx = ctx_for(prof)
+    g = X.megatron_best(prof, S.GPUEvaluator(ctx))
+    o = X.megatron_best(prof, OracleEvaluator(prof))
+    assert g == o and g["best"] is not None
