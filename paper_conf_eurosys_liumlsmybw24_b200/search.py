@@ -69,8 +69,9 @@ def _split_devices(p, G):
     return [int(math.log2(x)) for x in g]
 
 
-def initial_config(prof, p):
-    """Even partition, balanced devices, data parallelism first, minimum microbatch."""
+def initial_config(prof, p, first="dp"):
+    """Even partition, balanced devices, minimum microbatch; a stage's devices
+    go to data parallelism first (first="dp") or to tensor parallelism first ("tp"), R28."""
     L, G = prof.n_ops, prof.n_devices
     k = _split_devices(p, G)
     if sum(1 << x for x in k) != G:
@@ -78,8 +79,14 @@ def initial_config(prof, p):
     codes = np.zeros(L, np.uint8)
     starts = [L * i // p for i in range(p)] + [L]
     for i in range(p):
-        d = min(k[i], prof.n_dp - 1)
-        t = k[i] - d
+        if first == "tp":
+            t = min(k[i], prof.n_tp - 1)
+            d = k[i] - t
+            if d >= prof.n_dp:
+                return None
+        else:
+            d = min(k[i], prof.n_dp - 1)
+            t = k[i] - d
         if t >= prof.n_tp:
             return None
         a, b = starts[i], starts[i + 1]
@@ -814,7 +821,7 @@ def _rc_variants(prof, codes, mbs, info, mem, stage_time, max_n=4096):
 
 def search(prof, evaluator, p_values=None, budget_s=10.0, max_hops=7, beam=4, heuristic2=True,
            max_batch=200000, max_k=None, patience=None, starts=None, attach_rc=8, root_modes=ROOT_MODES,
-           max_batches=None):
+           max_batches=None, init_first=("dp", "tp")):
     """Runs the batched Aceso search. Returns (best Result, stats dict).
 
     starts: optional extra initial configurations [(codes, mbs_log2)], each searched like the
@@ -832,7 +839,9 @@ def search(prof, evaluator, p_values=None, budget_s=10.0, max_hops=7, beam=4, he
     search before GetBestOf: Heuristic-2's next resources, then the secondary bottleneck.
     max_batches: stop after this many evaluation batches (a budget independent of speed).
     patience: a stage count's search stops after this many batches without improving its own
-    best (None: only the clock budget, max_batches and exhausted searches stop)."""
+    best (None: only the clock budget, max_batches and exhausted searches stop).
+    init_first: the initial configurations per stage count, devices to data parallelism first
+    and / or to tensor parallelism first (R28)."""
     from . import candidates as C
     t0 = time.perf_counter()
     L = prof.n_ops
@@ -844,9 +853,12 @@ def search(prof, evaluator, p_values=None, budget_s=10.0, max_hops=7, beam=4, he
     seen = evaluator.visited() if hasattr(evaluator, "visited") else _HostVisited()
     init = []
     for p in p_values:
-        r = initial_config(prof, p)
-        if r is not None:
-            init.append(r)
+        seen_p = []
+        for first in init_first:  # R28: both device splits of the paper's initial configuration
+            r = initial_config(prof, p, first)
+            if r is not None and not any(np.array_equal(r[0], c) for c in seen_p):
+                seen_p.append(r[0])
+                init.append(r)
     for c, m in (starts or []):
         init.append((np.asarray(c, np.uint8), int(m)))
     bases = np.zeros((len(init), stride), np.uint8)

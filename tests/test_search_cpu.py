@@ -39,15 +39,27 @@ def test_primitives_keep_encodings_valid_structure():
     assert all(not (np.array_equal(c, codes) and m == mbs) for c, m in cands)
 
 
-def test_initial_configs_are_valid():
+@pytest.mark.parametrize("first", ["dp", "tp"])
+def test_initial_configs_are_valid(first):
+    """Both device splits of the initial configuration (R28) are valid configurations with an
+    even partition and the minimum microbatch; dp-first puts a stage's devices into data
+    parallelism up to the profile's range, tp-first into tensor parallelism."""
     for name in ["toy-a", "gpt3-1.3b", "gpt3-13b", "t5", "wrn"]:
         prof = P.WORKLOADS[name]()
         for p in [1, 2, 4]:
-            r = S.initial_config(prof, p)
+            r = S.initial_config(prof, p, first)
             assert r is not None
             codes, mbs = r
             out = oracle.evaluate(prof, codes[None, :], np.array([S.header(mbs, p)], np.uint64))
             assert not out["info"][0] & oracle.INFO_INVALID, (name, p, out["info"][0] >> 18)
+            assert list(np.flatnonzero(codes & 1)) == [prof.n_ops * i // p for i in range(p)]
+            tpl, dpl = (codes >> 1) & 7, codes >> 5
+            assert mbs == int(dpl.max())
+            k = int(np.log2(prof.n_devices // p))
+            if first == "tp":
+                assert np.all(tpl == min(k, prof.n_tp - 1))
+            else:
+                assert np.all(dpl == min(k, prof.n_dp - 1))
 
 
 def test_search_improves_and_is_deterministic():
