@@ -248,10 +248,11 @@ size_t aceso_select_buf_bytes(const aceso_ctx *ctx, int64_t n);
  *             variables read by aceso_load_profile (measurement and test knobs;
  *             results never change): ACESO_KERNEL=quad|events|dense|scan (default
  *             schedule), ACESO_DENSE_KERNEL=quad (schedule of the dense hint),
- *             ACESO_SPLIT=2 (per-op kernel: warp pair per tile), ACESO_MINB=2|3
- *             (register target: resident CTAs per SM), ACESO_TILES_PER_WARP=k
- *             (event / scan kernel: tiles per warp per launch), ACESO_SCAN_NORESOLVE=1
- *             (scan kernel: recompute-only chunks resolved in the per-lane walk).
+ *             ACESO_MINB=2|3 (register target: resident CTAs per SM),
+ *             ACESO_EV_SLOT=4|8 (event kernel: chunks per ring slot; 8 only at 2
+ *             CTAs per SM), ACESO_TILES_PER_WARP=k (event / scan kernel: tiles per
+ *             warp per launch), ACESO_SCAN_NORESOLVE=1 (scan kernel: recompute-only
+ *             chunks resolved in the per-lane walk).
  *   out     : host struct of device pointers (may be null if no OUT_* flag)
  *   d_sel   : select buffer (device), required with ACESO_FUSED_SELECT
  *   stream  : cudaStream_t

@@ -47,21 +47,16 @@ int fail(int code, const char *fmt, ...) {
       return fail(ACESO_ECUDA, "%s failed: %s", #expr, cudaGetErrorString(e_));            \
   } while (0)
 
-template <uint32_t M, int S, int B>
-void *kernel_ptr() {
-  return reinterpret_cast<void *>(&eval_kernel<M, S, B>);
-}
-
-template <int S, int B>
-void *eval_kernel_split(uint32_t mode) {
+template <int B>
+void *quad_kernel_for(uint32_t mode) {
   switch (mode) {
-    case 1: return kernel_ptr<1, S, B>();
-    case 2: return kernel_ptr<2, S, B>();
-    case 3: return kernel_ptr<3, S, B>();
-    case 4: return kernel_ptr<4, S, B>();
-    case 5: return kernel_ptr<5, S, B>();
-    case 6: return kernel_ptr<6, S, B>();
-    case 7: return kernel_ptr<7, S, B>();
+    case 1: return reinterpret_cast<void *>(&eval_kernel<1, B>);
+    case 2: return reinterpret_cast<void *>(&eval_kernel<2, B>);
+    case 3: return reinterpret_cast<void *>(&eval_kernel<3, B>);
+    case 4: return reinterpret_cast<void *>(&eval_kernel<4, B>);
+    case 5: return reinterpret_cast<void *>(&eval_kernel<5, B>);
+    case 6: return reinterpret_cast<void *>(&eval_kernel<6, B>);
+    case 7: return reinterpret_cast<void *>(&eval_kernel<7, B>);
     default: return nullptr;
   }
 }
@@ -136,7 +131,7 @@ void *scan_kernel_for(uint32_t mode) {
 // kernel 0: per-op/quad kernel (eval_kernel.cuh); kernel 1: event kernel (event_kernel.cuh);
 // kernel 2: dense kernel (dense_kernel.cuh, ACESO_HINT_DENSE); kernel 3: scan kernel
 // (scan_kernel.cuh, exact u64 tables; e64: wide transient-memory table)
-void *eval_kernel_for(uint32_t mode, int split, int minb, int kernel, int e64 = 0, int ev_warps = kWarps, int ev_sc = 4) {
+void *eval_kernel_for(uint32_t mode, int minb, int kernel, int e64 = 0, int ev_warps = kWarps, int ev_sc = 4) {
   if (kernel == 3) {
     // the scan kernel's default register target is 2 CTAs per SM (its ring and lists take
     // ~100 KB of shared memory per CTA); ACESO_MINB=3 selects the 80-register build
@@ -145,8 +140,7 @@ void *eval_kernel_for(uint32_t mode, int split, int minb, int kernel, int e64 = 
   }
   if (kernel == 1) return event_kernel_shape(mode, ev_warps, minb, ev_sc);
   if (kernel == 2) return minb == 2 ? dense_kernel_for<2>(mode) : dense_kernel_for<3>(mode);
-  if (minb == 2) return split == 2 ? eval_kernel_split<2, 2>(mode) : eval_kernel_split<1, 2>(mode);
-  return split == 2 ? eval_kernel_split<2, 3>(mode) : eval_kernel_split<1, 3>(mode);
+  return minb == 2 ? quad_kernel_for<2>(mode) : quad_kernel_for<3>(mode);
 }
 
 uint32_t bitlen(uint64_t v) {
@@ -172,7 +166,6 @@ struct aceso_ctx {
   const uint4 *px, *kx, *qr;
   const uint64_t *pd;
   const uint32_t *st;
-  int split;        // warps per tile (1 or 2)
   int minb;         // register target: 2 or 3 resident CTAs per SM
   int ev_warps;     // event kernel: warps per CTA (its kernels are templated on it; 8 is built)
   int ev_minb;      // event kernel: register target
@@ -781,11 +774,6 @@ int aceso_load_profile(const aceso_profile_desc *d, int cuda_device, aceso_ctx *
     cudaStreamDestroy(st);
     if (e != cudaSuccess) { rc = fail(e == cudaErrorMemoryAllocation ? ACESO_ENOMEM : ACESO_ECUDA, "upload: %s", cudaGetErrorString(e)); break; }
     const int nch = (L + 15) / 16;
-    ctx->split = 1;  // one warp per tile; ACESO_SPLIT=2 selects the forward/reverse warp pair
-    if (const char *env = getenv("ACESO_SPLIT")) {
-      int v = atoi(env);
-      if (v == 1 || (v == 2 && nch >= 2)) ctx->split = v;
-    }
     // register target: 3 resident CTAs per SM (80 registers) for models of up to 128 chunks;
     // the long models' event kernel runs faster at 2 (measured, 1K-layer GPT: 0.608 vs 0.571 of
     // the HBM roofline at 131,072 candidates, 0.641 vs 0.589 at 1M; GPT-3 1.3B / 13B, T5 and
@@ -838,10 +826,10 @@ int aceso_load_profile(const aceso_profile_desc *d, int cuda_device, aceso_ctx *
             kern == 3   ? (size_t)sc_smem_bytes((uint32_t)(nqs * 4 + 15) & ~15u)
             : kern == 1 ? (size_t)ev_smem_bytes((mode & ACESO_OUT_FULL) != 0, (uint32_t)ctx->ev_warps, ev_sc_for(ctx, mode), qo_bytes)
             : kern == 2 ? ((mode & ACESO_OUT_FULL) ? tab.dbytes_full : tab.dbytes) + kRingBytesPerCta
-                        : tabs + kRingBytesPerCta + (ctx->split == 2 ? (size_t)(kWarps / 2) * 32 * sizeof(Xchg) : 0);
+                        : tabs + kRingBytesPerCta;
         ctx->smem[kern][mode] = smem;
-        void *k = kern == 1 ? eval_kernel_for(mode, 1, ctx->ev_minb, 1, 0, ctx->ev_warps, ev_sc_for(ctx, mode))
-                            : eval_kernel_for(mode, ctx->split, ctx->minb, kern, ctx->e64);
+        void *k = kern == 1 ? eval_kernel_for(mode, ctx->ev_minb, 1, 0, ctx->ev_warps, ev_sc_for(ctx, mode))
+                            : eval_kernel_for(mode, ctx->minb, kern, ctx->e64);
         e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
         int occ = 0;
         if (e == cudaSuccess) e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k, kern == 1 ? 32 * ctx->ev_warps : kThreads, smem);
@@ -951,7 +939,7 @@ static int eval_impl(aceso_ctx *ctx, const uint8_t *d_codes, const uint64_t *d_h
   const int tpw_hint = P.nch <= 20 ? 3 : P.nch <= 24 ? 2 : 1;
   const int tpw = ((kern == 1 || kern == 3) && (flags & ACESO_HINT_OVERLAP) && tpw_hint > 1) ? std::max(tpw_hint, ctx->tiles_per_warp)
                                                                           : ctx->tiles_per_warp;
-  const int tiles_per_cta = (kern == 1 ? ctx->ev_warps : kern != 0 ? kWarps : kWarps / ctx->split) * tpw;
+  const int tiles_per_cta = (kern == 1 ? ctx->ev_warps : kWarps) * tpw;
   const int64_t need = (P.n_tiles + tiles_per_cta - 1) / tiles_per_cta;
   int grid = (int)std::max<int64_t>(1, std::min<int64_t>(need, ctx->max_ctas[kern][mode]));
   if (kern == 3) {
@@ -965,8 +953,8 @@ static int eval_impl(aceso_ctx *ctx, const uint8_t *d_codes, const uint64_t *d_h
   CUDA_TRY(cudaGetDevice(&prev));
   if (prev != ctx->device) CUDA_TRY(cudaSetDevice(ctx->device));
   void *args[] = {&P};
-  void *kfn = kern == 1 ? eval_kernel_for(mode, 1, ctx->ev_minb, 1, 0, ctx->ev_warps, ev_sc_for(ctx, mode))
-                        : eval_kernel_for(mode, ctx->split, ctx->minb, kern, ctx->e64);
+  void *kfn = kern == 1 ? eval_kernel_for(mode, ctx->ev_minb, 1, 0, ctx->ev_warps, ev_sc_for(ctx, mode))
+                        : eval_kernel_for(mode, ctx->minb, kern, ctx->e64);
   cudaError_t e = cudaLaunchKernel(kfn, dim3(grid), dim3(kern == 1 ? 32 * ctx->ev_warps : kThreads), args, ctx->smem[kern][mode],
                                    reinterpret_cast<cudaStream_t>(stream));
   if (prev != ctx->device) cudaSetDevice(prev);

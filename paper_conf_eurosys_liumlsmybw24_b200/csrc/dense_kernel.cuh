@@ -142,7 +142,7 @@ __global__ void __launch_bounds__(kThreads, MINB) dense_kernel(const __grid_cons
     if ((c & 1u) || j == 0) {
       if ((c & 1u) && j > 0) {
         s.S += tb.u32(pk + 4u);  // R5: p2p_fwd of the stage's last op (j-1)
-        stage_commit<MODE>(s, P, cand, active, false);
+        stage_commit<MODE>(s, P, cand, active);
         s.i += 1;
         s.S += tb.u32(kofs + 8u);  // R5: p2p_bwd of the stage's first op
       }
@@ -167,7 +167,7 @@ __global__ void __launch_bounds__(kThreads, MINB) dense_kernel(const __grid_cons
     if (g == 0) {
       cand = tile * 32 + lane;
       active = cand < P.n;
-      init_cand(s, sm, P, active ? __ldg(P.hdr + cand) : 0ull, false);
+      init_cand(s, sm, P, active ? __ldg(P.hdr + cand) : 0ull);
       max_tpl = max_dpl = 0;
       min_dpl = 7;
     }
@@ -213,7 +213,7 @@ __global__ void __launch_bounds__(kThreads, MINB) dense_kernel(const __grid_cons
       if (max_dpl > s.mbs) s.reasons |= ACESO_R_DPMBS;
       if (max_tpl >= n_tp || max_dpl >= n_dp || (min_dpl <= s.mbs && s.mbs - min_dpl >= n_b))
         s.reasons |= ACESO_R_TABLE;
-      stage_commit<MODE>(s, P, cand, active, false);  // last stage: no p2p_fwd
+      stage_commit<MODE>(s, P, cand, active);  // last stage: no p2p_fwd
       finish_cand<MODE>(s, P, cand, active, best_ck, best_idx);
       g = 0;
       tile += tile_stride;

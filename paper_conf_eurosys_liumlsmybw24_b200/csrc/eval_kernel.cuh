@@ -1,13 +1,9 @@
 // eval_kernel.cuh — batched evaluation of Aceso's performance/memory model (sm_100a).
 //
 // Work decomposition. A tile holds 32 candidates (tiled layout of include/aceso.h);
-// thread = candidate. With SPLIT = 2 a tile is processed by a PAIR of warps: part 0
-// walks ops [0, M) forward, part 1 walks ops [M, L) BACKWARD. Walking backward from
-// the last stage (index p-1), part 1 knows every stage's absolute index without a
-// pre-scan, so Eq. 1's in-flight factor min(p - i, N) is available when it closes a
-// stage. The stage that spans M is closed by part 0 after part 1 hands over its
-// partial sums through shared memory (named barrier per warp pair). SPLIT = 1 runs
-// one forward warp per tile (short models).
+// thread = candidate, one warp walks a tile's ops forward. (Round 1 also built a warp-pair
+// variant, one warp walking the second half of the ops backward; measured slower and
+// removed in round 2.)
 //
 // Data movement. The packed profile tables are staged into shared memory once per
 // CTA with one cp.async.bulk (TMA bulk copy, mbarrier completion); each warp streams
@@ -76,15 +72,6 @@ __device__ __forceinline__ void mbar_wait(uint32_t bar, uint32_t parity) {
       "r"(parity)
       : "memory");
 }
-// named barrier of a warp pair (immediate ids 1..4 so ptxas reserves only those)
-__device__ __forceinline__ void pair_bar_sync(int pair) {
-  switch (pair) {
-    case 0: asm volatile("bar.sync 1, 64;" ::: "memory"); break;
-    case 1: asm volatile("bar.sync 2, 64;" ::: "memory"); break;
-    case 2: asm volatile("bar.sync 3, 64;" ::: "memory"); break;
-    default: asm volatile("bar.sync 4, 64;" ::: "memory"); break;
-  }
-}
 __device__ __forceinline__ uint4 lds128(uint32_t a) {
   uint4 v;
   asm volatile("ld.shared.v4.u32 {%0, %1, %2, %3}, [%4];"
@@ -138,24 +125,16 @@ struct Cand {
   uint32_t mbs, p, N;
 };
 
-// hand-over record, part 1 -> part 0 (one per candidate of a tile)
-struct Xchg {
-  uint64_t S, A, W, D, comp, sumS, bestT, bestM;
-  uint32_t E, bt, bm, flags, gsum, reasons, nheads, pad;
-};
-
 // Closes the current stage i: Eq. 2 key, Eq. 1 memory, OOM, Heuristic-1 maxima.
 template <uint32_t MODE, class St>
-__device__ __forceinline__ void stage_commit(St &s, const EvalParams &P, int64_t c, bool active,
-                                             bool reverse) {
+__device__ __forceinline__ void stage_commit(St &s, const EvalParams &P, int64_t c, bool active) {
   s.sumS += s.S;
   const uint64_t tk = (uint64_t)(s.N - P.n_minus) * s.S + s.D;  // T_i - sum_k S_k (Eq. 2, R1, R6)
   const uint64_t infl = s.p > s.i ? (uint64_t)min(s.p - s.i, s.N) : 0ull;  // R2
   const uint64_t M = (s.W + infl * s.A + s.E) << P.mem_shift;              // Eq. 1 (R3, R4)
-  // argmax with the lowest stage index on ties (R11): forward visits ascending
-  // indices (strict >), the reverse part descending ones (>=, kNone = nothing yet)
-  if (reverse ? (tk >= s.bestT || s.bt == kNone) : (tk > s.bestT)) { s.bestT = tk; s.bt = s.i; }
-  if (reverse ? (M >= s.bestM || s.bm == kNone) : (M > s.bestM)) { s.bestM = M; s.bm = s.i; }
+  // argmax with the lowest stage index on ties (R11): ascending indices, strict >
+  if (tk > s.bestT) { s.bestT = tk; s.bt = s.i; }
+  if (M > s.bestM) { s.bestM = M; s.bm = s.i; }
   s.oom |= (M > P.C) ? 1u : 0u;  // R10
   if (MODE & kFull) {
     if (active && s.i < (uint32_t)P.p_max) {
@@ -226,7 +205,7 @@ __device__ __forceinline__ void fwd_event(Cand &s, const Smem &sm, const EvalPar
   const uint32_t head = c & 1u;
   if (head && j > 0) {
     s.S += ldk(sm, s.kbase + (toff_prev >> 1) + 4);  // R5: p2p_fwd of the stage's last op
-    stage_commit<MODE>(s, P, cand, active, false);
+    stage_commit<MODE>(s, P, cand, active);
     s.i += 1;
   }
   const uint32_t g = ((c >> 1) & 7u) + (c >> 5);
@@ -242,39 +221,7 @@ __device__ __forceinline__ void fwd_event(Cand &s, const Smem &sm, const EvalPar
   }
 }
 
-// reverse "pre" event at op j (before accumulating op j): op j+1 opened a run
-// (cn = code of op j+1, tn = its type offset), or j is the model's last op.
-template <uint32_t MODE>
-__device__ __forceinline__ void rev_pre(Cand &s, const Smem &sm, const EvalParams &P, uint32_t j,
-                                        uint32_t c, uint32_t cn, uint32_t toff, uint32_t tn) {
-  const uint32_t g = ((c >> 1) & 7u) + (c >> 5);
-  if (j + 1 == (uint32_t)P.L) {  // the last stage (p - 1), visited first
-    open_run<MODE>(s, sm, P, c);
-    s.gst = g;
-  } else if (cn & 1u) {  // op j+1 was a head: op j is the last op of the previous stage
-    open_run<MODE>(s, sm, P, c);
-    s.gst = g;
-    s.S += ldk(sm, s.kbase + (toff >> 1) + 4);  // R5: p2p_fwd of the last op
-  } else {               // tp/dp change at op j+1 inside a stage
-    s.S += ldk(sm, s.kbase + (tn >> 1));         // R13: reshard into op j+1 (its run)
-    if (g != s.gst) s.reasons |= ACESO_R_GSTAGE;
-    open_run<MODE>(s, sm, P, c);
-  }
-}
-
-// reverse "post" event at op j (after accumulating op j): op j is a stage head
-template <uint32_t MODE>
-__device__ __forceinline__ void rev_post(Cand &s, const Smem &sm, const EvalParams &P, uint32_t c,
-                                         uint32_t toff, int64_t cand, bool active) {
-  s.S += ldk(sm, s.kbase + (toff >> 1) + 8);  // R5: p2p_bwd of the first op (j >= M > 0)
-  s.gsum += 1u << (((c >> 1) & 7u) + (c >> 5));
-  s.nheads += 1;
-  stage_commit<MODE>(s, P, cand, active, true);
-  s.i -= 1;
-}
-
-__device__ __forceinline__ void init_cand(Cand &s, const Smem &sm, const EvalParams &P, uint64_t h,
-                                          bool reverse) {
+__device__ __forceinline__ void init_cand(Cand &s, const Smem &sm, const EvalParams &P, uint64_t h) {
   s.mbs = (uint32_t)(h & 0xff);
   s.p = (uint32_t)((h >> 8) & 0xff);
   s.reasons = (h >> 16) ? ACESO_R_HDR : 0u;
@@ -287,9 +234,9 @@ __device__ __forceinline__ void init_cand(Cand &s, const Smem &sm, const EvalPar
   s.S = s.A = s.W = s.D = s.comp = 0;
   s.E = 0;
   s.sumS = s.bestT = s.bestM = 0;
-  s.bt = s.bm = reverse ? kNone : 0u;
+  s.bt = s.bm = 0u;
   s.oom = s.gsum = s.nheads = s.head0 = 0;
-  s.i = reverse ? s.p - 1 : 0u;
+  s.i = 0u;
   s.rbase = sm.R;
   s.dbase = sm.D;
   s.kbase = 0;
@@ -301,8 +248,8 @@ __device__ __forceinline__ void init_cand(Cand &s, const Smem &sm, const EvalPar
 }
 
 // ---------------------------------------------------------------------------
-// 4-op groups ("quads"): the unit of the warp-uniform event test. One call site
-// per direction keeps the kernel small enough for the instruction cache.
+// 4-op groups ("quads"): the unit of the event test. One call site keeps the kernel
+// small enough for the instruction cache.
 // ---------------------------------------------------------------------------
 // forward quad qg (ops 4qg..4qg+3); w = the lane's 4 code bytes; pw = previous word
 template <uint32_t MODE>
@@ -340,57 +287,7 @@ __device__ __forceinline__ void quad_fwd(Cand &s, const Smem &sm, const EvalPara
   }
 }
 
-// reverse quad qg, ops visited from the highest down; nw = code word of the next quad
-// (visited before this one), tn = type offset of op 4qg+4. On return nw = w and
-// tn = type offset of op 4qg.
-template <uint32_t MODE>
-__device__ __forceinline__ void quad_rev(Cand &s, const Smem &sm, const EvalParams &P, uint32_t w,
-                                         uint32_t &nw, uint32_t &tn, uint32_t qg, int64_t cand,
-                                         bool active) {
-  const uint32_t nb = __funnelshift_r(w, nw, 8);  // next op's byte under each byte
-  // bits 1-3, 5-7: op j+1 opens a run (tp/dp change, or bit 1 = head of op j+1);
-  // bit 0: op j is a stage head
-  uint32_t x = ((w ^ nb) & 0xEEEEEEEEu) | ((nb & 0x01010101u) << 1) | (w & 0x01010101u);
-  const uint32_t j0 = qg * 4u;
-  const uint32_t nvalid = min(4u, (uint32_t)P.L - j0);
-  if (j0 + nvalid == (uint32_t)P.L) x |= 0x80u << (8 * (nvalid - 1));  // last op: last stage
-  const uint2 o = lds64(sm.QO + 8u * qg);
-  const uint32_t rcw = w & 0x10101010u;
-  const uint32_t mix = rcw ^ __byte_perm(rcw, 0, 0x0000);
-  if (o.x != kNone && !__any_sync(0xffffffffu, (x | mix) != 0u)) {
-    accumulate_quad<MODE>(s, o, rcw & 0x10u);
-    tn = toff_of(sm.T, j0);
-    nw = w;
-    return;
-  }
-  if (o.x != kNone && (x | mix) == 0u) {
-    accumulate_quad<MODE>(s, o, rcw & 0x10u);
-    tn = toff_of(sm.T, j0);
-    nw = w;
-    return;
-  }
-  const uint2 tt = lds64(sm.T + 2u * j0);
-  const uint32_t t4[4] = {(tt.x & 0xffffu) << 5, (tt.x >> 16) << 5, (tt.y & 0xffffu) << 5,
-                          (tt.y >> 16) << 5};
-  const uint32_t rc4 = w & 0x10101010u;
-#pragma unroll
-  for (int k = 3; k >= 0; --k) {
-    if ((uint32_t)k < nvalid) {
-      const uint32_t c = (w >> (8 * k)) & 0xffu;
-      const uint32_t e = (x >> (8 * k)) & 0xffu;
-      if (e & 0xfeu) {
-        const uint32_t cn = k < 3 ? (w >> (8 * k + 8)) & 0xffu : nw & 0xffu;
-        rev_pre<MODE>(s, sm, P, j0 + k, c, cn, t4[k], k < 3 ? t4[k + 1] : tn);
-      }
-      accumulate<MODE>(s, __byte_perm(rc4, 0, 0x4440 + k), t4[k]);
-      if (e & 1u) rev_post<MODE>(s, sm, P, c, t4[k], cand, active);
-    }
-  }
-  tn = t4[0];
-  nw = w;
-}
-
-// Candidate epilogue (forward part): validity, summary outputs, fused argmin.
+// Candidate epilogue: validity, summary outputs, fused argmin.
 template <uint32_t MODE, class St>
 __device__ __forceinline__ void finish_cand(St &s, const EvalParams &P, int64_t c, bool active,
                                             uint64_t &best_ck, int64_t &best_idx) {
@@ -430,7 +327,7 @@ __device__ __forceinline__ void finish_cand(St &s, const EvalParams &P, int64_t 
 // ---------------------------------------------------------------------------
 // MINB: resident CTAs per SM the register allocation targets (2: ~96 registers, lowest
 // latency per launch; 3: <= 80 registers, more warps when independent batches overlap)
-template <uint32_t MODE, int SPLIT, int MINB>
+template <uint32_t MODE, int MINB>
 __global__ void __launch_bounds__(kThreads, MINB) eval_kernel(const __grid_constant__ EvalParams P) {
   extern __shared__ __align__(128) unsigned char sm_raw[];
   __shared__ __align__(8) uint64_t s_tbar;
@@ -439,9 +336,6 @@ __global__ void __launch_bounds__(kThreads, MINB) eval_kernel(const __grid_const
   __shared__ int64_t s_idx[kWarps];
 
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-  const int npairs = kWarps / SPLIT;
-  const int pair = SPLIT == 2 ? (warp >> 1) : warp;
-  const int part = SPLIT == 2 ? (warp & 1) : 0;
   const uint32_t tab_bytes = (MODE & kFull) ? P.tab.bytes_full : P.tab.bytes;
   const uint32_t sb = smem_addr(sm_raw);
   Smem sm;
@@ -459,7 +353,6 @@ __global__ void __launch_bounds__(kThreads, MINB) eval_kernel(const __grid_const
   sm.TS = (uint32_t)P.T * kTypeStride;
   const uint32_t stage_bytes = tab_bytes + (P.tab.k_smem ? P.tab.bytesK : 0u);
   const uint32_t ring = sb + stage_bytes + (uint32_t)warp * kRingSlots * kSlotBytes;
-  Xchg *xch = reinterpret_cast<Xchg *>(sm_raw + stage_bytes + kRingBytesPerCta) + pair * 32;
 
   // ---- stage the packed tables (TMA bulk copies) ----
   if (threadIdx.x == 0) {
@@ -478,26 +371,19 @@ __global__ void __launch_bounds__(kThreads, MINB) eval_kernel(const __grid_const
     if (P.tab.k_smem) bulk_g2s(sb + tab_bytes, sm.Kg, P.tab.bytesK, bar);
   }
 
-  // ---- this warp's part of every tile it owns ----
+  // ---- every tile this warp owns ----
   const uint32_t nch = (uint32_t)P.nch;
-  const uint32_t nch0 = SPLIT == 2 ? (nch + 1) / 2 : nch;
-  const uint32_t c_lo = part ? nch0 : 0u, c_hi = part ? nch : nch0;
-  const uint32_t ngroups = (c_hi - c_lo + kSlotChunks - 1) / kSlotChunks;
-  const int64_t first_tile = (int64_t)blockIdx.x * npairs + pair;
-  const int64_t tile_stride = (int64_t)gridDim.x * npairs;
+  const uint32_t ngroups = (nch + kSlotChunks - 1) / kSlotChunks;
+  const int64_t first_tile = (int64_t)blockIdx.x * kWarps + warp;
+  const int64_t tile_stride = (int64_t)gridDim.x * kWarps;
   const int64_t my_tiles =
       first_tile < P.n_tiles ? (P.n_tiles - first_tile + tile_stride - 1) / tile_stride : 0;
   const int64_t units = my_tiles * ngroups;
   const unsigned char *codes = reinterpret_cast<const unsigned char *>(P.codes);
 
-  // chunk range of group g of this part (ascending addresses)
-  auto group_lo = [&](uint32_t g) {
-    return part ? (c_hi >= kSlotChunks * (g + 1) + c_lo ? c_hi - kSlotChunks * (g + 1) : c_lo)
-                : c_lo + kSlotChunks * g;
-  };
-  auto group_hi = [&](uint32_t g) {
-    return part ? c_hi - kSlotChunks * g : min(c_lo + kSlotChunks * (g + 1), c_hi);
-  };
+  // chunk range of group g
+  auto group_lo = [&](uint32_t g) { return kSlotChunks * g; };
+  auto group_hi = [&](uint32_t g) { return min(kSlotChunks * (g + 1), nch); };
   // issue cursor (lane 0)
   int64_t it_tile = first_tile;
   uint32_t it_g = 0;
@@ -522,8 +408,7 @@ __global__ void __launch_bounds__(kThreads, MINB) eval_kernel(const __grid_const
   uint64_t best_ck = ~0ull;
   int64_t best_idx = INT64_MAX;
   Cand s;
-  uint32_t cw = 0, ct = 0;  // forward: previous word; reverse: next word / next type offset
-  uint32_t cM = 0, tM = 0;  // reverse: code and type offset of op M (the part's first op)
+  uint32_t cw = 0;  // the previous code word
   int64_t tile = first_tile;
   uint32_t g = 0;
   int slot = 0;
@@ -534,57 +419,38 @@ __global__ void __launch_bounds__(kThreads, MINB) eval_kernel(const __grid_const
     if (g == 0) {
       cand = tile * 32 + lane;
       active = cand < P.n;
-      init_cand(s, sm, P, active ? __ldg(P.hdr + cand) : 0ull, part == 1);
+      init_cand(s, sm, P, active ? __ldg(P.hdr + cand) : 0ull);
       cw = 0;
-      ct = 0;
     }
     mbar_wait(smem_addr(&s_ring_bar[warp][slot]), phase);
     const uint32_t a = group_lo(g), b = group_hi(g);
     const uint32_t slot_a = ring + slot * kSlotBytes + lane * 16;
-    if (g == 0 && part == 0) {
+    if (g == 0) {
       // seed the previous word so that op 0 always opens the first run
       const uint32_t w0 = lds32(slot_a);
       cw = ((w0 & 0xffu) ^ 0x02u) << 24;
       s.head0 = w0 & 1u;
     }
-    if (part == 0) {
 #pragma unroll 1
-      for (uint32_t ch = a; ch < b; ++ch) {
-        const uint32_t nqc = min(4u, ((uint32_t)P.L - ch * 16u + 3u) >> 2);  // quads inside L
-        uint32_t wa = slot_a + (ch - a) * 512u;
-        uint32_t oa = sm.QO + 8u * (ch * 4u);
-        // software pipeline: the next quad's code word and signature offsets load while
-        // this quad is processed
-        uint32_t wn = lds32(wa);
-        uint2 on = lds64(oa);
+    for (uint32_t ch = a; ch < b; ++ch) {
+      const uint32_t nqc = min(4u, ((uint32_t)P.L - ch * 16u + 3u) >> 2);  // quads inside L
+      uint32_t wa = slot_a + (ch - a) * 512u;
+      uint32_t oa = sm.QO + 8u * (ch * 4u);
+      // software pipeline: the next quad's code word and signature offsets load while
+      // this quad is processed
+      uint32_t wn = lds32(wa);
+      uint2 on = lds64(oa);
 #pragma unroll 1
-        for (uint32_t q = 0; q < nqc; ++q) {
-          const uint32_t w = wn;
-          const uint2 o = on;
-          wa += 4u;
-          oa += 8u;
-          if (q + 1 < nqc) {
-            wn = lds32(wa);
-            on = lds64(oa);
-          }
-          quad_fwd<MODE>(s, sm, P, w, o, cw, ch * 4u + q, cand, active);
+      for (uint32_t q = 0; q < nqc; ++q) {
+        const uint32_t w = wn;
+        const uint2 o = on;
+        wa += 4u;
+        oa += 8u;
+        if (q + 1 < nqc) {
+          wn = lds32(wa);
+          on = lds64(oa);
         }
-      }
-    } else {
-#pragma unroll 1
-      for (uint32_t ch = b; ch-- > a;) {
-        const uint32_t nqc = min(4u, ((uint32_t)P.L - ch * 16u + 3u) >> 2);
-        uint32_t wa = slot_a + (ch - a) * 512u + 4u * nqc;
-#pragma unroll 1
-        for (uint32_t q = nqc; q-- > 0;) {
-          wa -= 4u;
-          const uint32_t w = lds32(wa);
-          quad_rev<MODE>(s, sm, P, w, cw, ct, ch * 4u + q, cand, active);
-        }
-        if (ch == c_lo) {
-          cM = lds32(slot_a + (ch - a) * 512u) & 0xffu;
-          tM = ct;
-        }
+        quad_fwd<MODE>(s, sm, P, w, o, cw, ch * 4u + q, cand, active);
       }
     }
     __syncwarp();
@@ -598,46 +464,8 @@ __global__ void __launch_bounds__(kThreads, MINB) eval_kernel(const __grid_const
     }
     if (++g == ngroups) {
       // ---- tile epilogue ----
-      if (SPLIT == 1) {
-        stage_commit<MODE>(s, P, cand, active, false);  // last stage: no p2p_fwd
-        finish_cand<MODE>(s, P, cand, active, best_ck, best_idx);
-      } else {
-        const uint32_t M = nch0 * 16u;
-        if (part == 1) {
-          // boundary pair (M-1, M): in-stage tp/dp change -> reshard of op M, symmetry
-          const uint32_t cb = codes[((size_t)tile * nch + (nch0 - 1)) * 512 + lane * 16 + 15];
-          if (!(cM & 1u) && ((cM ^ cb) & 0xEEu)) {
-            s.S += ldk(sm, s.kbase + (tM >> 1));
-            if ((((cb >> 1) & 7u) + (cb >> 5)) != s.gst) s.reasons |= ACESO_R_GSTAGE;
-          }
-          Xchg &xr = xch[lane];
-          xr.S = s.S; xr.A = s.A; xr.W = s.W; xr.D = s.D; xr.comp = s.comp; xr.E = s.E;
-          xr.sumS = s.sumS; xr.bestT = s.bestT; xr.bestM = s.bestM; xr.bt = s.bt; xr.bm = s.bm;
-          xr.flags = s.oom | ((cM & 1u) << 1);
-          xr.gsum = s.gsum; xr.reasons = s.reasons; xr.nheads = s.nheads;
-        }
-        pair_bar_sync(pair);
-        if (part == 0) {
-          const Xchg &xr = xch[lane];
-          if (xr.flags & 2u) {
-            // op M is a head: part 0's open stage ends at M-1 and is followed by a stage
-            s.S += ldk(sm, s.kbase + (toff_of(sm.T, M - 1) >> 1) + 4);  // R5 p2p_fwd
-          } else {
-            s.S += xr.S; s.A += xr.A; s.W += xr.W; s.D += xr.D; s.comp += xr.comp;
-            s.E = max(s.E, xr.E);
-          }
-          stage_commit<MODE>(s, P, cand, active, false);  // the stage spanning M
-          s.sumS += xr.sumS;
-          if (xr.bt != kNone && xr.bestT > s.bestT) { s.bestT = xr.bestT; s.bt = xr.bt; }
-          if (xr.bm != kNone && xr.bestM > s.bestM) { s.bestM = xr.bestM; s.bm = xr.bm; }
-          s.oom |= xr.flags & 1u;
-          s.gsum += xr.gsum;
-          s.reasons |= xr.reasons;
-          s.nheads += xr.nheads;
-          finish_cand<MODE>(s, P, cand, active, best_ck, best_idx);
-        }
-        pair_bar_sync(pair);  // hand-over record free for the next tile
-      }
+      stage_commit<MODE>(s, P, cand, active);  // last stage: no p2p_fwd
+      finish_cand<MODE>(s, P, cand, active, best_ck, best_idx);
       g = 0;
       tile += tile_stride;
     }

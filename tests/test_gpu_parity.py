@@ -391,15 +391,14 @@ def test_random_bytes_never_crash_and_match():
 
 
 # ---------------------------------------------------------------------------
-# every kernel variant: event kernel (default), quad kernel with one warp per tile or a
-# forward+reverse warp pair; 2 or 3 resident CTAs per SM
+# every kernel variant: event kernel (default), scan kernel, per-op (quad) kernel; 2 or 3
+# resident CTAs per SM
 # ---------------------------------------------------------------------------
 @pytest.mark.parametrize("minb", ["2", "3"])
-@pytest.mark.parametrize("kernel,split", [("scan", "1"), ("events", "1"), ("quad", "1"), ("quad", "2")])
+@pytest.mark.parametrize("kernel", ["scan", "events", "quad"])
 @pytest.mark.parametrize("name", ["gpt3-1.3b", "t5", "wrn", "gpt3-13b", "toy-a"])
-def test_kernel_variants_parity(kernel, split, minb, name, monkeypatch):
+def test_kernel_variants_parity(kernel, minb, name, monkeypatch):
     monkeypatch.setenv("ACESO_KERNEL", kernel)
-    monkeypatch.setenv("ACESO_SPLIT", split)
     monkeypatch.setenv("ACESO_MINB", minb)
     prof = P.WORKLOADS[name]()
     ctx = A.Context(prof, 0)  # the decomposition is fixed at load time
