@@ -202,8 +202,13 @@ template <uint32_t MODE>
 __device__ __forceinline__ void ev_rc_lookup(const EvalParams &P, uint32_t qsb, uint32_t rr, uint32_t pat,
                                              uint64_t &dS, uint64_t &dA, uint32_t &e1, uint64_t &dC) {
   const uint32_t idx = qsb + rr * 16u + pat;
+#ifdef ACESO_EXPERIMENT_RC_NOLOAD
+  const uint4 v0 = make_uint4(idx, idx >> 3, idx * 3u, idx >> 5);
+  const uint4 v1 = make_uint4(idx ^ 5u, 0u, idx, 0u);
+#else
   const uint4 v0 = __ldg(P.qr + 2u * idx);
   const uint4 v1 = __ldg(P.qr + 2u * idx + 1u);
+#endif
   dS += u64of(v0.x, v0.y);
   dA += u64of(v0.z, v0.w);
   e1 = max(e1, v1.x);
