@@ -413,17 +413,18 @@ class Primitives:
         if ("comp" in want) and mbs + 1 <= log2bg:
             one(mbs + 1, [])
 
+        # per-stage extrema of the tp / dp fields (one reduceat each)
+        st_tmin = np.minimum.reduceat(tpl_all, heads).tolist()
+        st_tmax = np.maximum.reduceat(tpl_all, heads).tolist()
+        st_dmin = np.minimum.reduceat(dpl_all, heads).tolist()
+        st_dmax = np.maximum.reduceat(dpl_all, heads).tolist()
+
         def stage_ok(sg, dt, dd):
-            x, y = int(heads[sg]), int(ends[sg])
-            t, d = tpl_all[x:y], dpl_all[x:y]
-            return t.min() + dt >= 0 and t.max() + dt <= 7 and d.min() + dd >= 0 and d.max() + dd <= 7
+            return (st_tmin[sg] + dt >= 0 and st_tmax[sg] + dt <= 7 and st_dmin[sg] + dd >= 0
+                    and st_dmax[sg] + dd <= 7)
 
         def dmax_after(changes):  # max dp field after per-stage shifts {stage: dd}
-            m = 0
-            for sg in range(p):
-                x, y = int(heads[sg]), int(ends[sg])
-                m = max(m, int(dpl_all[x:y].max()) + changes.get(sg, 0))
-            return m
+            return max(st_dmax[sg] + changes.get(sg, 0) for sg in range(p))
         for dt in (1, -1):
             if stage_ok(bn, dt, -dt):
                 one(max(mbs, dmax_after({bn: -dt})), [C.add(a, e, dt, -dt)])
@@ -502,6 +503,27 @@ class GPUEvaluator:
         self.ctx = ctx
         self.calls = 0
         self.evaluated = 0
+        self._tiled = None  # expand output, reused across batches (grown on demand)
+        self._flat = None   # FULL outputs of evaluate_cands, reused across batches
+
+    def _outputs(self, n):
+        """FULL output arrays for n candidates as views of one reused flat device buffer (the
+        search copies what it keeps before the next batch overwrites them)."""
+        from .api import Outputs
+        pm = self.ctx.n_devices
+        need = n * (3 + 4 * pm)  # int64 words: iter, max_mem, info (as int64 slot), 4 stage arrays
+        if self._flat is None or self._flat.numel() < need:
+            self._flat = torch.empty(max(need, 2 * (0 if self._flat is None else self._flat.numel())),
+                                     dtype=torch.int64, device=torch.device("cuda", self.ctx.device))
+        f = self._flat
+        o = Outputs(f[0:n], f[n:2 * n], f[2 * n:3 * n].view(torch.int32)[0:n])
+        o.p_max = pm
+        base = 3 * n
+        o.stage_T = f[base:base + pm * n].view(pm, n)
+        o.stage_mem = f[base + pm * n:base + 2 * pm * n].view(pm, n)
+        o.stage_comp = f[base + 2 * pm * n:base + 3 * pm * n].view(pm, n)
+        o.stage_comm = f[base + 3 * pm * n:base + 4 * pm * n].view(pm, n)
+        return o
 
     def evaluate(self, codes, hdr, dims=None, hashes=False):
         """Row-major codes [n][L] (+ optional dimension bytes [n][L]) -> FULL outputs
@@ -541,13 +563,21 @@ class GPUEvaluator:
         tb = torch.from_numpy(np.ascontiguousarray(bases)).to(dev)
         rk = torch.from_numpy(np.ascontiguousarray(ranks).view(np.int16)).to(dev)
         cd = torch.from_numpy(np.ascontiguousarray(cands).view(np.uint8)).to(dev)
-        tiled, hdr = self.ctx.expand(tb, cd, rk, n=n)
-        out, _ = self.ctx.eval(tiled, hdr, n=n, full=True, select=False)
+        from .api import tiled_bytes
+        need = int(tiled_bytes(max(n, 1), self.ctx.n_ops))
+        if self._tiled is None or self._tiled.numel() < need:
+            # aceso_expand writes every byte of the candidates' tiles; lanes past n in the
+            # last tile are never read into an output
+            self._tiled = torch.empty(max(need, 2 * (0 if self._tiled is None else self._tiled.numel())),
+                                      dtype=torch.uint8, device=dev)
+        tiled, hdr = self.ctx.expand(tb, cd, rk, n=n, tiled=self._tiled[:need])
+        out, _ = self.ctx.eval(tiled, hdr, n=n, full=True, select=False, out=self._outputs(n))
         hs = hash_candidates(tiled, hdr, self.ctx.n_ops, n=n)
         res = dict(iter=as_u64(out.iter_ns), max_mem=as_u64(out.max_mem), info=as_u32(out.info),
                    hash=hs.cpu().numpy().view(np.uint64), hash_dev=hs)
-        # per-stage rows stay on the device ([n][p_max] views): the search reads the few rows
-        # of the configurations it takes (Heuristic-2 needs them), not the whole batch
+        # per-stage rows stay on the device ([n][p_max] views of the reused buffer, valid until
+        # the next call): the search copies the rows of the configurations it may take
+        # (Heuristic-2 needs them), not the whole batch
         for k in ["stage_T", "stage_mem", "stage_comp", "stage_comm"]:
             res[k] = getattr(out, k).view(torch.int64).reshape(out.p_max, n).T
         return res
@@ -684,14 +714,33 @@ def _oom_excess(r, capacity):
     if len(rows) == 0:
         return ex
     sm = r["stage_mem"]
-    if isinstance(sm, torch.Tensor):
-        sm = sm[torch.from_numpy(rows).to(sm.device)].cpu().numpy()
-    else:
-        sm = np.asarray(sm)[rows].view(np.int64)
     p = ((info[rows] >> np.uint64(8)) & np.uint64(0xFF)).astype(np.int64)
+    if isinstance(sm, torch.Tensor):  # device FULL outputs: reduce there, copy 8 B per row
+        dev = sm.device
+        rt = torch.from_numpy(rows).to(dev)
+        pt = torch.from_numpy(p).to(dev)
+        live = torch.arange(sm.shape[1], device=dev)[None, :] < pt[:, None]
+        x = torch.clamp(sm[rt] - int(capacity), min=0)
+        ex[rows] = torch.where(live, x, torch.zeros_like(x)).sum(dim=1).cpu().numpy()
+        return ex
+    sm = np.asarray(sm)[rows].view(np.int64)
     live = np.arange(sm.shape[1])[None, :] < p[:, None]
     ex[rows] = np.where(live, np.maximum(sm.astype(np.int64) - int(capacity), 0), 0).sum(axis=1)
     return ex
+
+
+class _Take:
+    """arr[idx[t]] without copying arr (a chunk's view of its batch's arrays)."""
+    __slots__ = ("arr", "idx")
+
+    def __init__(self, arr, idx):
+        self.arr, self.idx = arr, idx
+
+    def __getitem__(self, t):
+        return self.arr[self.idx[t]]
+
+    def rows(self, a, b):
+        return self.arr[self.idx[a:b]]
 
 
 class _Chunk:
@@ -700,24 +749,49 @@ class _Chunk:
     materialised when the search takes them; they leave the set from the front (the
     improving node, the next frontier, GetBestOf)."""
 
-    def __init__(self, keys, idx, r, bases, ranks, cands, L, codes=None, mbs=None):
+    def __init__(self, keys, idx, r, bases, ranks, cands, L, codes=None, mbs=None, evaluator=None,
+                 keep_rows=64):
         self.keys = keys[idx]
         self.idx = idx
-        self.hash = r["hash"][idx]
-        self.info = r["info"][idx]
-        self.iter = r["iter"][idx]
-        self.mem = r["max_mem"][idx]
-        self.stage = (r["stage_comp"], r["stage_comm"], r["stage_T"], r["stage_mem"])  # [n][p_max]
-        self.cands = None if cands is None else cands[idx]
-        self.codes = None if codes is None else codes[idx]  # materialised rows (recompute attachment)
-        self.mbs = None if mbs is None else mbs[idx]
+        # the batch's arrays, read through idx (entry t = batch row idx[t]); nothing is copied
+        self.hash = _Take(r["hash"], idx)
+        self.info = _Take(r["info"], idx)
+        self.iter = _Take(r["iter"], idx)
+        self.mem = _Take(r["max_mem"], idx)
+        stage = (r["stage_comp"], r["stage_comm"], r["stage_T"], r["stage_mem"])  # [n][p_max]
+        self.cands = None if cands is None else _Take(cands, idx)
+        self.codes = None if codes is None else _Take(codes, idx)  # materialised rows (recompute attachment)
+        self.mbs = None if mbs is None else _Take(mbs, idx)
         self.bases, self.ranks, self.L = bases, ranks, L
         self.head = 0
+        self.evaluator = evaluator
+        if isinstance(stage[0], torch.Tensor):
+            # device rows (the evaluator's buffer, overwritten by its next batch): copy those of
+            # the best `keep_rows` entries, the ones the search takes first; later ones are
+            # re-evaluated on demand (node)
+            k = min(int(keep_rows), len(idx))
+            ti = torch.from_numpy(np.ascontiguousarray(idx[:k])).to(stage[0].device)
+            self.rows = torch.stack([x[ti] for x in stage], 1).cpu().numpy().view(np.uint64)  # [k][4][p_max]
+            self.stage = None
+        else:
+            self.rows = None
+            self.stage = stage
 
     def node(self, t):
         info = int(self.info[t])
         i = int(self.idx[t])
-        rows = [_row(x, i) for x in self.stage]
+        if self.stage is not None:
+            rows = [_row(x, i) for x in self.stage]
+        elif t < len(self.rows):
+            rows = list(self.rows[t])
+        else:
+            # beyond the copied rows: evaluate this one configuration again (same FULL outputs)
+            c1 = self.cands.rows(t, t + 1).copy()
+            b1 = int(c1[0]["base"])
+            c1["base"] = 0
+            r1 = self.evaluator.evaluate_cands(self.bases[b1:b1 + 1], self.ranks[b1:b1 + 1], c1)
+            rows = [np.asarray(r1[k][0].cpu().numpy()).view(np.uint64) if isinstance(r1[k], torch.Tensor)
+                    else r1[k][0] for k in ("stage_comp", "stage_comm", "stage_T", "stage_mem")]
         if self.codes is not None:
             return _Node(int(self.hash[t]), int(self.mbs[t]), perf_of(info, self.iter[t], self.mem[t]), info,
                          rows[0], rows[1], rows[2], int(self.iter[t]), int(self.mem[t]), None,
@@ -821,7 +895,7 @@ def _rc_variants(prof, codes, mbs, info, mem, stage_time, max_n=4096):
 
 def search(prof, evaluator, p_values=None, budget_s=10.0, max_hops=7, beam=4, heuristic2=True,
            max_batch=200000, max_k=None, patience=None, starts=None, attach_rc=8, root_modes=ROOT_MODES,
-           max_batches=None, init_first=("dp", "tp")):
+           max_batches=None, init_first=("dp", "tp"), chunk_rows=64):
     """Runs the batched Aceso search. Returns (best Result, stats dict).
 
     starts: optional extra initial configurations [(codes, mbs_log2)], each searched like the
@@ -841,7 +915,9 @@ def search(prof, evaluator, p_values=None, budget_s=10.0, max_hops=7, beam=4, he
     patience: a stage count's search stops after this many batches without improving its own
     best (None: only the clock budget, max_batches and exhausted searches stop).
     init_first: the initial configurations per stage count, devices to data parallelism first
-    and / or to tensor parallelism first (R28)."""
+    and / or to tensor parallelism first (R28).
+    chunk_rows: per hop and search, the per-stage rows of this many best new configurations
+    are copied from the device; configurations taken later are evaluated again."""
     from . import candidates as C
     t0 = time.perf_counter()
     L = prof.n_ops
@@ -943,7 +1019,8 @@ def search(prof, evaluator, p_values=None, budget_s=10.0, max_hops=7, beam=4, he
             idx = np.nonzero(keep & (owner == si))[0]
             # Heuristic-2: best estimated performance first (stable: generation order)
             idx = idx[np.lexsort((ex[idx], keys[idx]))]  # stable: generation order among equals
-            hop_chunks[si] = [_Chunk(keys, idx, r, bases, ranks, cands, L)] if len(idx) else []
+            hop_chunks[si] = [_Chunk(keys, idx, r, bases, ranks, cands, L, evaluator=evaluator,
+                                      keep_rows=chunk_rows)] if len(idx) else []
         # recomputation attached to the primitives' results: a second batch of the hop
         if attach_rc:
             rows, hdrs, mbss, rowner = [], [], [], []

@@ -501,6 +501,10 @@ def test_nccl_allreduce_min_single_rank():
     ("t5", dict(p_values=[4], max_hops=2, beam=2, max_k=4, patience=2)),
     ("wrn", dict(p_values=[2, 4], max_hops=2, beam=2, max_k=6, patience=2)),
     ("gpt-1k", dict(p_values=[8], max_hops=2, beam=1, max_k=2, patience=2, attach_rc=1, max_batches=8)),
+    # per-stage rows of only the best new configuration per hop copied from the device: every
+    # later take re-evaluates its configuration
+    ("gpt3-1.3b", dict(p_values=[2, 4], max_hops=3, beam=3, max_k=8, patience=3, chunk_rows=1)),
+    ("wrn", dict(p_values=[2, 4], max_hops=2, beam=2, max_k=6, patience=2, chunk_rows=1)),
 ])
 def test_search_driver_gpu_matches_oracle_trajectory(name, kw):
     """The batched search (Alg. 1/2 with Heuristic-2 over three resources, recomputation
