@@ -61,16 +61,16 @@ void *quad_kernel_for(uint32_t mode) {
   }
 }
 
-template <int B, int W, int SC>
+template <int B, int W, int SC, bool OCT>
 void *event_kernel_for(uint32_t mode) {
   switch (mode) {
-    case 1: return reinterpret_cast<void *>(&event_kernel<1, B, W, SC>);
-    case 2: return reinterpret_cast<void *>(&event_kernel<2, B, W, SC>);
-    case 3: return reinterpret_cast<void *>(&event_kernel<3, B, W, SC>);
-    case 4: return reinterpret_cast<void *>(&event_kernel<4, B, W, SC>);
-    case 5: return reinterpret_cast<void *>(&event_kernel<5, B, W, SC>);
-    case 6: return reinterpret_cast<void *>(&event_kernel<6, B, W, SC>);
-    case 7: return reinterpret_cast<void *>(&event_kernel<7, B, W, SC>);
+    case 1: return reinterpret_cast<void *>(&event_kernel<1, B, W, SC, OCT>);
+    case 2: return reinterpret_cast<void *>(&event_kernel<2, B, W, SC, OCT>);
+    case 3: return reinterpret_cast<void *>(&event_kernel<3, B, W, SC, OCT>);
+    case 4: return reinterpret_cast<void *>(&event_kernel<4, B, W, SC, OCT>);
+    case 5: return reinterpret_cast<void *>(&event_kernel<5, B, W, SC, OCT>);
+    case 6: return reinterpret_cast<void *>(&event_kernel<6, B, W, SC, OCT>);
+    case 7: return reinterpret_cast<void *>(&event_kernel<7, B, W, SC, OCT>);
     default: return nullptr;
   }
 }
@@ -79,11 +79,15 @@ void *event_kernel_for(uint32_t mode) {
 // Built: 8 warps at 2 or 3 CTAs per SM. Measured and dropped (round 2, every BASELINE
 // workload): 6 warps x 3 CTAs (18 warps per SM at 96 registers), 4 warps x 4 / 5 / 6 CTAs —
 // within 0.3% of the better 8-warp shape on the 1K-layer model and 1-10% slower elsewhere.
-// Ring slots: 8 chunks (4 KB) at 2 CTAs per SM, 4 chunks (2 KB) at 3.
-void *event_kernel_shape(uint32_t mode, int warps, int minb, int sc) {
+// Ring slots: 8 chunks (4 KB) at 2 CTAs per SM (needs the octet tables), 4 chunks (2 KB)
+// otherwise; octet recompute lookups whenever the octet tables exist.
+void *event_kernel_shape(uint32_t mode, int warps, int minb, int sc, int oct) {
   (void)warps;
-  if (minb == 2) return sc == 8 ? event_kernel_for<2, 8, 8>(mode) : event_kernel_for<2, 8, 4>(mode);
-  return event_kernel_for<3, 8, 4>(mode);
+  if (minb == 2) {
+    if (sc == 8) return event_kernel_for<2, 8, 8, true>(mode);
+    return oct ? event_kernel_for<2, 8, 4, true>(mode) : event_kernel_for<2, 8, 4, false>(mode);
+  }
+  return oct ? event_kernel_for<3, 8, 4, true>(mode) : event_kernel_for<3, 8, 4, false>(mode);
 }
 
 template <int B>
@@ -131,14 +135,15 @@ void *scan_kernel_for(uint32_t mode) {
 // kernel 0: per-op/quad kernel (eval_kernel.cuh); kernel 1: event kernel (event_kernel.cuh);
 // kernel 2: dense kernel (dense_kernel.cuh, ACESO_HINT_DENSE); kernel 3: scan kernel
 // (scan_kernel.cuh, exact u64 tables; e64: wide transient-memory table)
-void *eval_kernel_for(uint32_t mode, int minb, int kernel, int e64 = 0, int ev_warps = kWarps, int ev_sc = 4) {
+void *eval_kernel_for(uint32_t mode, int minb, int kernel, int e64 = 0, int ev_warps = kWarps, int ev_sc = 4,
+                      int ev_oct = 0) {
   if (kernel == 3) {
     // the scan kernel's default register target is 2 CTAs per SM (its ring and lists take
     // ~100 KB of shared memory per CTA); ACESO_MINB=3 selects the 80-register build
     if (minb == 3 && getenv("ACESO_MINB")) return e64 ? scan_kernel_for<true, 3>(mode) : scan_kernel_for<false, 3>(mode);
     return e64 ? scan_kernel_for<true, 2>(mode) : scan_kernel_for<false, 2>(mode);
   }
-  if (kernel == 1) return event_kernel_shape(mode, ev_warps, minb, ev_sc);
+  if (kernel == 1) return event_kernel_shape(mode, ev_warps, minb, ev_sc, ev_oct);
   if (kernel == 2) return minb == 2 ? dense_kernel_for<2>(mode) : dense_kernel_for<3>(mode);
   return minb == 2 ? quad_kernel_for<2>(mode) : quad_kernel_for<3>(mode);
 }
@@ -164,12 +169,16 @@ struct aceso_ctx {
   void *d_ev;       // event-kernel tables
   uint32_t qo_off, qo_bytes;
   const uint4 *px, *kx, *qr;
+  const uint4 *qr8;      // octet recompute records (8-chunk slots), null without them
+  const uint32_t *qo8;   // octet signature offsets
   const uint64_t *pd;
   const uint32_t *st;
   int minb;         // register target: 2 or 3 resident CTAs per SM
   int ev_warps;     // event kernel: warps per CTA (its kernels are templated on it; 8 is built)
   int ev_minb;      // event kernel: register target
   int ev_sc;        // event kernel: 16-op chunks per ring slot (8 at 2 CTAs per SM, else 4)
+  int has_oct;      // octet recompute tables built (the 8-chunk-slot kernel needs them)
+  int ev_oct;       // event kernel: octet recompute lookups (has_oct; ACESO_EV_OCT=0 turns them off)
   int tiles_per_warp;  // ACESO_TILES_PER_WARP (measurement knob): tiles each warp walks per launch (default 1)
   int max_ctas[4][8];  // per kernel and mode: resident CTAs (occupancy x SMs)
   int dense_kernel;    // schedule of ACESO_HINT_DENSE: 2 dense kernel (default), 0 per-op kernel (ACESO_DENSE_KERNEL=quad)
@@ -233,6 +242,8 @@ EvalParams make_params(const aceso_ctx *ctx, int64_t n, int64_t global_offset, i
   P.pd = ctx->pd;
   P.st = ctx->st;
   P.qr = ctx->qr;
+  P.qr8 = ctx->qr8;
+  P.qo8 = ctx->qo8;
   P.runs = (uint32_t)(ctx->n_b * ctx->n_tp);
   P.qo_bytes = ctx->qo_bytes;
   P.qo_off = ctx->qo_off;
@@ -530,6 +541,26 @@ int aceso_load_profile(const aceso_profile_desc *d, int cuda_device, aceso_ctx *
       eqo[q] = (uint32_t)it->second * RUNS * 16u;
     }
   }
+  // octet signatures (distinct type 8-tuples at ops 8o..8o+7): the 8-chunk-slot event kernel
+  // looks up a recompute-only chunk's deltas per octet (256 patterns) instead of per quad
+  const int no8 = 2 * ((L + 15) / 16);
+  std::vector<uint32_t> eo8(no8);
+  std::vector<std::array<int, 8>> osigs;
+  {
+    std::map<std::array<int, 8>, int> seen;
+    for (int o = 0; o < no8; ++o) {
+      std::array<int, 8> key;
+      for (int k = 0; k < 8; ++k) key[k] = 8 * o + k < L ? (int)d->op_type[8 * o + k] : -1;
+      auto it = seen.find(key);
+      if (it == seen.end()) {
+        it = seen.emplace(key, (int)osigs.size()).first;
+        osigs.push_back(key);
+      }
+      eo8[o] = (uint32_t)it->second * RUNS * 256u;
+    }
+  }
+  // octet table budget: at most 64 MB (else the quad tables serve every schedule)
+  const bool has_oct = osigs.size() * (size_t)RUNS * 256 * 32 <= ((size_t)64 << 20);
   auto al = [](size_t v) { return (v + 255) & ~(size_t)255; };
   const size_t ev_px = 0;
   const size_t ev_kx = al(ev_px + (size_t)RUNS * Lp1 * 32);
@@ -538,7 +569,9 @@ int aceso_load_profile(const aceso_profile_desc *d, int cuda_device, aceso_ctx *
   const size_t ev_qr = al(ev_st + (size_t)levels * RUNS * L * 4);
   const size_t ev_qo = al(ev_qr + esigs.size() * RUNS * 16 * 32);
   const uint32_t qo_bytes = a16((uint32_t)nq * 4u);
-  const size_t ev_bytes = al(ev_qo + qo_bytes);
+  const size_t ev_qo8 = al(ev_qo + qo_bytes);
+  const size_t ev_qr8 = al(ev_qo8 + (size_t)no8 * 4);
+  const size_t ev_bytes = has_oct ? al(ev_qr8 + osigs.size() * RUNS * 256 * 32) : al(ev_qo + qo_bytes);
   std::vector<unsigned char> ev(ev_bytes, 0);
   {
     auto put64 = [&](size_t off, uint64_t v) { memcpy(&ev[off], &v, 8); };
@@ -591,6 +624,30 @@ int aceso_load_profile(const aceso_profile_desc *d, int cuda_device, aceso_ctx *
             put64(o + 24, dC);
           }
       }
+    if (has_oct) {
+      for (int o = 0; o < no8; ++o) put32(ev_qo8 + (size_t)o * 4, eo8[o]);
+      for (int b = 0; b < NB; ++b)
+        for (int tp = 0; tp < NT; ++tp) {
+          const uint32_t rr = (uint32_t)(b * NT + tp);
+          for (size_t sg = 0; sg < osigs.size(); ++sg)
+            for (uint32_t m = 1; m < 256; ++m) {
+              uint64_t dS = 0, dA = 0, dC = 0, E1 = 0;
+              for (int k = 0; k < 8; ++k) {
+                const int t = osigs[sg][k];
+                if (t < 0 || !((m >> k) & 1u)) continue;
+                dS += (uint64_t)R(t, tp, b, ACESO_F_FWD_COMP) + R(t, tp, b, ACESO_F_FWD_COMM);
+                dA += (uint64_t)(R(t, tp, b, ACESO_F_ACT) - R(t, tp, b, ACESO_F_KEEP)) >> ms;
+                dC += (uint64_t)R(t, tp, b, ACESO_F_FWD_COMP);
+                E1 = std::max(E1, rec_e(t, tp, b, 1));
+              }
+              const size_t o = ev_qr8 + (((size_t)sg * RUNS + rr) * 256 + m) * 32;
+              put64(o, dS);
+              put64(o + 8, dA);
+              put32(o + 16, (uint32_t)E1);
+              put64(o + 24, dC);
+            }
+        }
+    }
     for (int tp = 0; tp < NT; ++tp)
       for (int dp = 0; dp < ND; ++dp) {
         uint64_t s = 0;
@@ -760,6 +817,7 @@ int aceso_load_profile(const aceso_profile_desc *d, int cuda_device, aceso_ctx *
   }
   ctx->qo_off = (uint32_t)ev_qo;
   ctx->qo_bytes = qo_bytes;
+  ctx->has_oct = has_oct ? 1 : 0;
   int rc = ACESO_OK;
   do {
     cudaStream_t st;
@@ -790,9 +848,12 @@ int aceso_load_profile(const aceso_profile_desc *d, int cuda_device, aceso_ctx *
     }
     ctx->ev_warps = kWarps;
     ctx->ev_minb = ctx->minb;
-    ctx->ev_sc = ctx->minb == 2 ? 8 : 4;
-    if (const char *env = getenv("ACESO_EV_SLOT"))  // measurement knob: 4 or 8 (8 needs 2 CTAs per SM)
-      if (atoi(env) == 4 || (atoi(env) == 8 && ctx->minb == 2)) ctx->ev_sc = atoi(env);
+    ctx->ev_oct = ctx->has_oct;
+    if (const char *env = getenv("ACESO_EV_OCT"))  // measurement knob: 0 = quad lookups
+      if (atoi(env) == 0) ctx->ev_oct = 0;
+    ctx->ev_sc = (ctx->minb == 2 && ctx->ev_oct) ? 8 : 4;
+    if (const char *env = getenv("ACESO_EV_SLOT"))  // measurement knob: 4 or 8 (8 needs 2 CTAs per SM and the octet tables)
+      if (atoi(env) == 4 || (atoi(env) == 8 && ctx->minb == 2 && ctx->ev_oct)) ctx->ev_sc = atoi(env);
     {
       const unsigned char *eb = reinterpret_cast<const unsigned char *>(ctx->d_ev);
       ctx->px = reinterpret_cast<const uint4 *>(eb + ev_px);
@@ -800,6 +861,8 @@ int aceso_load_profile(const aceso_profile_desc *d, int cuda_device, aceso_ctx *
       ctx->pd = reinterpret_cast<const uint64_t *>(eb + ev_pd);
       ctx->st = reinterpret_cast<const uint32_t *>(eb + ev_st);
       ctx->qr = reinterpret_cast<const uint4 *>(eb + ev_qr);
+      ctx->qr8 = has_oct ? reinterpret_cast<const uint4 *>(eb + ev_qr8) : nullptr;
+      ctx->qo8 = has_oct ? reinterpret_cast<const uint32_t *>(eb + ev_qo8) : nullptr;
       const unsigned char *cb = reinterpret_cast<const unsigned char *>(ctx->d_sc);
       ctx->sx = reinterpret_cast<const uint4 *>(cb + sc_sx);
       ctx->sk = reinterpret_cast<const uint4 *>(cb + sc_sk);
@@ -828,7 +891,7 @@ int aceso_load_profile(const aceso_profile_desc *d, int cuda_device, aceso_ctx *
             : kern == 2 ? ((mode & ACESO_OUT_FULL) ? tab.dbytes_full : tab.dbytes) + kRingBytesPerCta
                         : tabs + kRingBytesPerCta;
         ctx->smem[kern][mode] = smem;
-        void *k = kern == 1 ? eval_kernel_for(mode, ctx->ev_minb, 1, 0, ctx->ev_warps, ev_sc_for(ctx, mode))
+        void *k = kern == 1 ? eval_kernel_for(mode, ctx->ev_minb, 1, 0, ctx->ev_warps, ev_sc_for(ctx, mode), ctx->ev_oct)
                             : eval_kernel_for(mode, ctx->minb, kern, ctx->e64);
         e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
         int occ = 0;
@@ -953,7 +1016,7 @@ static int eval_impl(aceso_ctx *ctx, const uint8_t *d_codes, const uint64_t *d_h
   CUDA_TRY(cudaGetDevice(&prev));
   if (prev != ctx->device) CUDA_TRY(cudaSetDevice(ctx->device));
   void *args[] = {&P};
-  void *kfn = kern == 1 ? eval_kernel_for(mode, ctx->ev_minb, 1, 0, ctx->ev_warps, ev_sc_for(ctx, mode))
+  void *kfn = kern == 1 ? eval_kernel_for(mode, ctx->ev_minb, 1, 0, ctx->ev_warps, ev_sc_for(ctx, mode), ctx->ev_oct)
                         : eval_kernel_for(mode, ctx->minb, kern, ctx->e64);
   cudaError_t e = cudaLaunchKernel(kfn, dim3(grid), dim3(kern == 1 ? 32 * ctx->ev_warps : kThreads), args, ctx->smem[kern][mode],
                                    reinterpret_cast<cudaStream_t>(stream));

@@ -74,6 +74,8 @@ struct EvalParams {
   const uint64_t *pd;     // [n_tp * n_dp][L+1] DP all-reduce prefix sums
   const uint32_t *st;     // [levels][RUNS][L] sparse table of e0 = peak (range max)
   const uint4 *qr;        // [nsig][RUNS][16] x 2: {dS, dA} {E1, 0, dC} rc deltas of a quad pattern
+  const uint4 *qr8;       // [nsig8][RUNS][256] x 2: the same per octet pattern (8-chunk slots)
+  const uint32_t *qo8;    // [2 * nch] octet signature offsets (sig8 * RUNS * 256)
   uint32_t runs;          // RUNS = n_b * n_tp
   uint32_t qo_bytes;      // bytes of the per-quad signature table staged to shared memory
   uint32_t qo_off;        // its byte offset in the event blob

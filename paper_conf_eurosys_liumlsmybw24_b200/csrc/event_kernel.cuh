@@ -214,6 +214,18 @@ __device__ __forceinline__ void ev_rc_lookup(const EvalParams &P, uint32_t qsb, 
   e1 = max(e1, v1.x);
   if (MODE & kFull) dC += u64of(v1.z, v1.w);
 }
+// the same for an octet pattern (bit k = op 8o+k) from the octet records (8-chunk slots)
+template <uint32_t MODE>
+__device__ __forceinline__ void ev_rc_lookup8(const EvalParams &P, uint32_t osb, uint32_t rr, uint32_t pat,
+                                              uint64_t &dS, uint64_t &dA, uint32_t &e1, uint64_t &dC) {
+  const uint32_t idx = osb + rr * 256u + pat;
+  const uint4 v0 = __ldg(P.qr8 + 2u * idx);
+  const uint4 v1 = __ldg(P.qr8 + 2u * idx + 1u);
+  dS += u64of(v0.x, v0.y);
+  dA += u64of(v0.z, v0.w);
+  e1 = max(e1, v1.x);
+  if (MODE & kFull) dC += u64of(v1.z, v1.w);
+}
 // phase B: recompute deltas of a quad pattern under the open run, into the open stage
 template <uint32_t MODE>
 __device__ __forceinline__ void ev_rc_add(EvCand &s, const EvalParams &P, uint32_t qsb, uint32_t pat) {
@@ -419,10 +431,12 @@ __device__ __forceinline__ uint4 pad_tail(uint4 w4, uint32_t nvl) {
 }
 
 // W warps per CTA (the launch uses 32 W threads), SC chunks per ring slot
-template <uint32_t MODE, int MINB, int W, int SC>
+// OCT: recompute-only chunks are looked up per octet (P.qr8, 2 lookups per chunk) instead of
+// per quad (P.qr, 4 lookups); the quad tables still serve the drain's recompute items
+template <uint32_t MODE, int MINB, int W, int SC, bool OCT>
 __global__ void __launch_bounds__(32 * W, MINB) event_kernel(const __grid_constant__ EvalParams P) {
   constexpr uint32_t kEvSlotBytes = ev_slot_bytes(SC), kEvF = ev_f_off(SC), kEvC = ev_c_off(SC);
-  constexpr bool QG = SC == 8;  // signature table read through the L1
+  constexpr bool QG = SC == 8;  // quad signature table read through the L1 (not staged)
   extern __shared__ __align__(128) unsigned char sm_raw[];
   __shared__ __align__(8) uint64_t s_tbar;
   __shared__ __align__(8) uint64_t s_ring_bar[kEvRingSlots][W];
@@ -436,7 +450,6 @@ __global__ void __launch_bounds__(32 * W, MINB) event_kernel(const __grid_consta
   const uint32_t qo = sb + ev_qo_off(FULL, W, SC);
   const uint32_t lb = sb + warp * ev_warp_bytes(SC) + lane * 16u;  // see ev_warp_bytes
   const uint32_t lx = sb + ev_x_off(W, SC) + warp * kEvCap * 32u * XR + lane * XR;
-  const uint4 *qg = reinterpret_cast<const uint4 *>(P.evblob + P.qo_off);
 
   if (threadIdx.x == 0) {
     mbar_init(smem_addr(&s_tbar), 1);
@@ -497,11 +510,11 @@ __global__ void __launch_bounds__(32 * W, MINB) event_kernel(const __grid_consta
   // phase A, one 16-op chunk (ring address a, chunk index ci)
   auto chunk = [&](uint32_t a, uint32_t ci) {
     const uint4 w4 = lds128(a);
-    // QG: the chunk's quad signatures, requested ahead of the activity words (one broadcast
-    // L1 load; its latency is off the recompute lookups' critical path)
-    uint4 qsg = make_uint4(0u, 0u, 0u, 0u);
-    if (QG) asm volatile("ld.global.nc.v4.u32 {%0, %1, %2, %3}, [%4];"
-                         : "=r"(qsg.x), "=r"(qsg.y), "=r"(qsg.z), "=r"(qsg.w) : "l"(qg + ci));
+    // OCT: the chunk's two octet signatures, requested ahead of the activity words (one
+    // broadcast L1 load; its latency is off the recompute lookups' critical path)
+    uint2 qsg = make_uint2(0u, 0u);
+    if (OCT) asm volatile("ld.global.nc.v2.u32 {%0, %1}, [%2];"
+                          : "=r"(qsg.x), "=r"(qsg.y) : "l"(P.qo8 + 2u * ci));
     uint4 f;
     f.x = quad_activity(w4.x, pw);
     f.y = quad_activity(w4.y, w4.x);
@@ -532,12 +545,20 @@ __global__ void __launch_bounds__(32 * W, MINB) event_kernel(const __grid_consta
         // recompute flags in an event-free chunk: every op is in the open run, whose
         // (tp, dp) is that of op 0 of the chunk
         const uint32_t rr = ev_run(w4.x & 0xffu, s.mbs(), P);
-        const uint4 qs = QG ? qsg : lds128(qo + 16u * ci);
-        uint32_t pat;
-        if ((pat = quad_rc(f.x))) ev_rc_lookup<MODE>(P, qs.x, rr, pat, cS, cA, rE, cC);
-        if ((pat = quad_rc(f.y))) ev_rc_lookup<MODE>(P, qs.y, rr, pat, cS, cA, rE, cC);
-        if ((pat = quad_rc(f.z))) ev_rc_lookup<MODE>(P, qs.z, rr, pat, cS, cA, rE, cC);
-        if ((pat = quad_rc(f.w))) ev_rc_lookup<MODE>(P, qs.w, rr, pat, cS, cA, rE, cC);
+        if (OCT) {
+          // two octet lookups (256-pattern records) instead of four quad lookups
+          uint32_t pat;
+          if ((pat = quad_rc(f.x) | (quad_rc(f.y) << 4))) ev_rc_lookup8<MODE>(P, qsg.x, rr, pat, cS, cA, rE, cC);
+          if ((pat = quad_rc(f.z) | (quad_rc(f.w) << 4))) ev_rc_lookup8<MODE>(P, qsg.y, rr, pat, cS, cA, rE, cC);
+        } else {
+          const uint4 qs = QG ? __ldg(reinterpret_cast<const uint4 *>(P.evblob + P.qo_off) + ci)
+                              : lds128(qo + 16u * ci);
+          uint32_t pat;
+          if ((pat = quad_rc(f.x))) ev_rc_lookup<MODE>(P, qs.x, rr, pat, cS, cA, rE, cC);
+          if ((pat = quad_rc(f.y))) ev_rc_lookup<MODE>(P, qs.y, rr, pat, cS, cA, rE, cC);
+          if ((pat = quad_rc(f.z))) ev_rc_lookup<MODE>(P, qs.z, rr, pat, cS, cA, rE, cC);
+          if ((pat = quad_rc(f.w))) ev_rc_lookup<MODE>(P, qs.w, rr, pat, cS, cA, rE, cC);
+        }
       }
     }
   };

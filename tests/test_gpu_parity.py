@@ -417,16 +417,18 @@ def test_kernel_variants_parity(kernel, minb, name, monkeypatch):
         ctx.close()
 
 
-@pytest.mark.parametrize("minb,slot", [("2", "8"), ("2", "4"), ("3", "4")])
+@pytest.mark.parametrize("minb,slot,oct", [("2", "8", "1"), ("2", "4", "1"), ("3", "4", "1"), ("2", "4", "0"),
+                                           ("3", "4", "0")])
 @pytest.mark.parametrize("name", ["gpt3-1.3b", "wrn", "gpt-1k"])
-def test_event_kernel_two_tiles_per_warp_parity(minb, slot, name, monkeypatch):
-    """The event kernel at both register targets and both ring-slot sizes (ACESO_EV_SLOT;
-    FULL mode always runs 4-chunk slots) with every warp walking two tiles through its ring
-    (the persistent path of large batches): FULL and SUMMARY outputs, selection, a ragged
-    last tile."""
+def test_event_kernel_two_tiles_per_warp_parity(minb, slot, oct, name, monkeypatch):
+    """The event kernel at both register targets, both ring-slot sizes (ACESO_EV_SLOT; FULL
+    mode always runs 4-chunk slots) and both recompute lookup tables (octets, ACESO_EV_OCT=0:
+    quads) with every warp walking two tiles through its ring (the persistent path of large
+    batches): FULL and SUMMARY outputs, selection, a ragged last tile."""
     monkeypatch.setenv("ACESO_KERNEL", "events")
     monkeypatch.setenv("ACESO_MINB", minb)
     monkeypatch.setenv("ACESO_EV_SLOT", slot)
+    monkeypatch.setenv("ACESO_EV_OCT", oct)
     monkeypatch.setenv("ACESO_TILES_PER_WARP", "2")  # every warp walks two tiles through its ring
     prof = P.WORKLOADS[name]()
     ctx = A.Context(prof, 0)
