@@ -228,10 +228,14 @@ __device__ __forceinline__ void ev_rc_lookup8(const EvalParams &P, uint32_t osb,
 }
 // phase B: recompute deltas of a quad pattern under the open run, into the open stage
 template <uint32_t MODE>
-__device__ __forceinline__ void ev_rc_add(EvCand &s, const EvalParams &P, uint32_t qsb, uint32_t pat) {
+__device__ __forceinline__ void ev_rc_add(EvCand &s, const EvalParams &P, uint32_t qsb, uint32_t pat,
+                                          bool oct = false) {
   uint64_t dS = 0, dA = 0, dC = 0;
   uint32_t e1 = 0;
-  ev_rc_lookup<MODE>(P, qsb, s.rr(), pat, dS, dA, e1, dC);
+  if (oct)
+    ev_rc_lookup8<MODE>(P, qsb, s.rr(), pat, dS, dA, e1, dC);
+  else
+    ev_rc_lookup<MODE>(P, qsb, s.rr(), pat, dS, dA, e1, dC);
   s.S += dS;
   s.A -= dA;
   s.E = max(s.E, e1);
@@ -364,7 +368,7 @@ __device__ __forceinline__ uint32_t ev_rc_mask(uint4 f) {
 // lane with work left takes its next item in op order — an event (run close/open, stage
 // close) or a recompute segment (the recompute flags of one quad up to its next event:
 // one pattern lookup under the open run). lb, lx = this lane's bases (see ev_warp_bytes).
-template <uint32_t MODE, int SC>
+template <uint32_t MODE, int SC, bool OCT>
 __device__ __forceinline__ void ev_drain(EvCand &s, const EvalParams &P, uint32_t qo, uint32_t lb,
                                          uint32_t lx, int64_t cand, bool active) {
   constexpr uint32_t kEvF = ev_f_off(SC), kEvC = ev_c_off(SC);
@@ -397,15 +401,19 @@ __device__ __forceinline__ void ev_drain(EvCand &s, const EvalParams &P, uint32_
         ev_handle<MODE>(s, P, 4u * q0 + j, c, ent + kEvC, xe + 8u, cand, active);
         em &= em - 1u;
       } else {
-        // recompute flags of quad j/4 from op j up to the quad's next event (all bits of
-        // em and rm below j are consumed)
-        const uint32_t qb = j & ~3u;
-        const uint32_t nxt = em & (0xfu << qb);
-        const uint32_t lim = nxt ? __ffs(nxt) - 1u : qb + 4u;
+        // recompute flags of quad j/4 (OCT: octet j/8) from op j up to its next event (all
+        // bits of em and rm below j are consumed)
+        const uint32_t qb = OCT ? (j & ~7u) : (j & ~3u);
+        const uint32_t nxt = em & ((OCT ? 0xffu : 0xfu) << qb);
+        const uint32_t lim = nxt ? __ffs(nxt) - 1u : qb + (OCT ? 8u : 4u);
         const uint32_t seg = rm & ((1u << lim) - 1u);
-        const uint32_t qsb = SC == 8 ? __ldg(reinterpret_cast<const uint32_t *>(P.evblob + P.qo_off) + (q0 + (j >> 2)))
-                                     : lds32(qo + 4u * (q0 + (j >> 2)));
-        ev_rc_add<MODE>(s, P, qsb, seg >> qb);
+        uint32_t qsb;
+        if (OCT)
+          qsb = __ldg(P.qo8 + (q0 >> 1) + (j >> 3));  // q0 = 4 x chunk index
+        else
+          qsb = SC == 8 ? __ldg(reinterpret_cast<const uint32_t *>(P.evblob + P.qo_off) + (q0 + (j >> 2)))
+                        : lds32(qo + 4u * (q0 + (j >> 2)));
+        ev_rc_add<MODE>(s, P, qsb, seg >> qb, OCT);
         rm &= ~seg;
       }
     }
@@ -505,7 +513,7 @@ __global__ void __launch_bounds__(32 * W, MINB) event_kernel(const __grid_consta
   bool active = false;
   // the lists must hold what the next 2 chunks add
   auto drain_check = [&]() {
-    if (__any_sync(0xffffffffu, s.ec + 2u > (uint32_t)kEvCap)) ev_drain<MODE, SC>(s, P, qo, lb, lx, cand, active);
+    if (__any_sync(0xffffffffu, s.ec + 2u > (uint32_t)kEvCap)) ev_drain<MODE, SC, OCT>(s, P, qo, lb, lx, cand, active);
   };
   // phase A, one 16-op chunk (ring address a, chunk index ci)
   auto chunk = [&](uint32_t a, uint32_t ci) {
@@ -617,7 +625,7 @@ __global__ void __launch_bounds__(32 * W, MINB) event_kernel(const __grid_consta
       phase ^= slot ^ 1u;  // flips after slot 1
     }
     // ---- tile epilogue: drain, close the last run and stage (no p2p_fwd) ----
-    ev_drain<MODE, SC>(s, P, qo, lb, lx, cand, active);
+    ev_drain<MODE, SC, OCT>(s, P, qo, lb, lx, cand, active);
     s.S += cS;  // phase-A recompute deltas after the last event chunk (last stage)
     s.A -= cA;
     s.E = max(s.E, rE);
