@@ -253,6 +253,13 @@ __device__ __forceinline__ uint32_t quad_rc(uint32_t f) {
   return (((f & 0x10101010u) * 0x01020408u) >> 28);
 }
 
+// 8-bit pattern of the recompute flags of an octet (activity words a = ops 0-3, b = ops 4-7):
+// one multiply gathers a's flags to bits 24-27 and b's to bits 28-31 (checked exhaustively:
+// the cross terms fall below bit 24 or above bit 31)
+__device__ __forceinline__ uint32_t octet_rc(uint32_t a, uint32_t b) {
+  return ((((a & 0x10101010u) >> 4) | (b & 0x10101010u)) * 0x01020408u) >> 24;
+}
+
 // activity word of a quad: bit 4 of a byte = recompute flag, bit 0 = head, other bits =
 // tp/dp change against the previous op (p = the previous quad's word)
 __device__ __forceinline__ uint32_t quad_activity(uint32_t w, uint32_t p) {
@@ -556,8 +563,8 @@ __global__ void __launch_bounds__(32 * W, MINB) event_kernel(const __grid_consta
         if (OCT) {
           // two octet lookups (256-pattern records) instead of four quad lookups
           uint32_t pat;
-          if ((pat = quad_rc(f.x) | (quad_rc(f.y) << 4))) ev_rc_lookup8<MODE>(P, qsg.x, rr, pat, cS, cA, rE, cC);
-          if ((pat = quad_rc(f.z) | (quad_rc(f.w) << 4))) ev_rc_lookup8<MODE>(P, qsg.y, rr, pat, cS, cA, rE, cC);
+          if ((pat = octet_rc(f.x, f.y))) ev_rc_lookup8<MODE>(P, qsg.x, rr, pat, cS, cA, rE, cC);
+          if ((pat = octet_rc(f.z, f.w))) ev_rc_lookup8<MODE>(P, qsg.y, rr, pat, cS, cA, rE, cC);
         } else {
           const uint4 qs = QG ? __ldg(reinterpret_cast<const uint4 *>(P.evblob + P.qo_off) + ci)
                               : lds128(qo + 16u * ci);
@@ -577,19 +584,20 @@ __global__ void __launch_bounds__(32 * W, MINB) event_kernel(const __grid_consta
     ev_init(s, P, active ? __ldg(P.hdr + cand) : 0ull);
     cS = cA = cC = 0;
     rE = 0;
-    pw = 0;
+    {
+      // the tile's first slot: seed the previous word so that op 0 always shows a tp
+      // difference (an event); the group loop's wait on this slot then returns at once
+      mbar_wait(smem_addr(&s_ring_bar[0][warp]) + 8u * W * slot, phase);
+      const uint32_t w0 = lds32(lb + kEvSlotBytes * slot);
+      pw = ((w0 & 0xffu) ^ 0x02u) << 24;
+      s.run = ((w0 & 0xffu) ^ 0x02u) << 16;  // phase B rebuilds op 0's code against the same seed
+      s.fl = (w0 & 1u) << 17;                 // head0
+    }
 #pragma unroll 1
     for (uint32_t g = 0; g < ngroups; ++g) {
       const uint32_t ch0 = SC * g, nc = min((uint32_t)SC, nch - ch0);
       const uint32_t addr = lb + kEvSlotBytes * slot;
       mbar_wait(smem_addr(&s_ring_bar[0][warp]) + 8u * W * slot, phase);
-      if (g == 0) {
-        // seed the previous word so that op 0 always shows a tp difference (an event)
-        const uint32_t w0 = lds32(addr);
-        pw = ((w0 & 0xffu) ^ 0x02u) << 24;
-        s.run = ((w0 & 0xffu) ^ 0x02u) << 16;  // phase B rebuilds op 0's code against the same seed
-        s.fl = (w0 & 1u) << 17;                 // head0
-      }
       if (g == ngroups - 1u) {
         const uint32_t nvl = (uint32_t)P.L - 16u * (nch - 1u);  // valid ops of the last chunk
         if (nvl < 16u) {
