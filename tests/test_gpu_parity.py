@@ -768,3 +768,69 @@ def test_megatron_grid_gpu_matches_oracle(name):
     g = X.megatron_best(prof, S.GPUEvaluator(ctx))
     o = X.megatron_best(prof, OracleEvaluator(prof))
     assert g == o and g["best"] is not None
+
+
+# ---------------------------------------------------------------------------
+# greedy recompute levels: stages whose recompute flags are "every op of type rank < l by
+# activation size" (P:L255's greedy order), with the tie-prefix of the next rank, single
+# flipped flags, in-stage tp/dp changes and heads at chunk edges
+# ---------------------------------------------------------------------------
+def _level_candidates(prof, n, seed):
+    rng = np.random.default_rng(seed)
+    L, G = prof.n_ops, prof.n_devices
+    kmax = prof.n_tp - 1
+    rank = prof.rc_rank().astype(np.int64)
+    rows, hdrs = [], []
+    for _ in range(n):
+        p = int(rng.choice([q for q in (1, 2, 4, 8) if q <= G]))
+        cuts = set()
+        while len(cuts) < p - 1:
+            k = int(rng.integers(1, L // 16 + 1)) * 16 + int(rng.choice([-1, 0, 1, 7]))
+            if 0 < k < L:
+                cuts.add(k)
+        starts = [0] + sorted(cuts)
+        g = int(np.log2(G // p))
+        mbs = int(rng.integers(g, g + 3))
+        row = np.zeros(L, np.uint8)
+        for si, a in enumerate(starts):
+            b = starts[si + 1] if si + 1 < len(starts) else L
+            tpl = int(rng.integers(0, min(g, kmax) + 1))
+            lv = int(rng.choice([0, 1, 2, 3, 4, 6, 7, 255]))
+            rc = (rank < lv) if lv < 255 else np.ones(L, bool)
+            if lv < 255 and rng.random() < 0.4:  # greedy tie: the next rank's first ops too
+                x = int(rng.integers(a, b + 1))
+                rc = rc | ((rank == lv) & (np.arange(L) < x))
+            flips = rng.random(L) < (0.01 if rng.random() < 0.5 else 0.0)
+            trade = rng.random() < 0.3 and g > 0
+            for j in range(a, b):
+                t, d = tpl, g - tpl
+                if trade and (j // 16) % 7 == 3:  # in-stage trade (same device count)
+                    t = int(rng.integers(0, min(g, kmax) + 1))
+                    d = g - t
+                row[j] = ai.code(1 if j == a else 0, t, d, int(rc[j] ^ flips[j]))
+        rows.append(row)
+        hdrs.append(ai.header(mbs, p))
+    return np.array(rows, np.uint8), np.array(hdrs, np.uint64)
+
+
+@pytest.mark.parametrize("minb,slot,oct", [("2", "8", "1"), ("3", "4", "1"), ("2", "4", "0")])
+@pytest.mark.parametrize("name", ["gpt3-1.3b", "t5", "gpt-1k"])
+def test_event_kernel_recompute_levels_parity(minb, slot, oct, name, monkeypatch):
+    """Greedy recompute levels with ties, flipped flags and in-stage trades at both
+    register targets, ring-slot sizes and lookup tables: FULL and SUMMARY outputs, selection."""
+    monkeypatch.setenv("ACESO_KERNEL", "events")
+    monkeypatch.setenv("ACESO_MINB", minb)
+    monkeypatch.setenv("ACESO_EV_SLOT", slot)
+    monkeypatch.setenv("ACESO_EV_OCT", oct)
+    prof = P.WORKLOADS[name]()
+    ctx = A.Context(prof, 0)
+    _ctx_cache[id(prof)] = (prof, ctx)
+    try:
+        n = 200 if name == "gpt-1k" else 1100
+        codes, hdr = _level_candidates(prof, n, SEED + 41)
+        g, o, sel, _, _ = compare(prof, codes, hdr, full=True)
+        assert ((o["info"] & oracle.INFO_INVALID) == 0).mean() > 0.5
+        compare(prof, codes, hdr)
+    finally:
+        _ctx_cache.pop(id(prof), None)
+        ctx.close()
