@@ -522,9 +522,8 @@ __global__ void __launch_bounds__(32 * W, MINB) event_kernel(const __grid_consta
   auto drain_check = [&]() {
     if (__any_sync(0xffffffffu, s.ec + 2u > (uint32_t)kEvCap)) ev_drain<MODE, SC, OCT>(s, P, qo, lb, lx, cand, active);
   };
-  // phase A, one 16-op chunk (ring address a, chunk index ci)
-  auto chunk = [&](uint32_t a, uint32_t ci) {
-    const uint4 w4 = lds128(a);
+  // phase A, one 16-op chunk (its 16 code bytes w4, chunk index ci)
+  auto chunk = [&](const uint4 w4, uint32_t ci) {
     // OCT: the chunk's two octet signatures, requested ahead of the activity words (one
     // broadcast L1 load; its latency is off the recompute lookups' critical path)
     uint2 qsg = make_uint2(0u, 0u);
@@ -610,18 +609,26 @@ __global__ void __launch_bounds__(32 * W, MINB) event_kernel(const __grid_consta
       if (nc == (uint32_t)SC) {
 #pragma unroll 1
         for (uint32_t h = 0; h < (uint32_t)SC; h += 4u) {
+          // two chunks' code words requested back to back (the second chunk's shared-memory
+          // latency hides behind the first chunk's work)
           drain_check();
-          chunk(addr + 512u * h, ch0 + h);
-          chunk(addr + 512u * h + 512u, ch0 + h + 1u);
+          {
+            const uint4 wa = lds128(addr + 512u * h), wb = lds128(addr + 512u * h + 512u);
+            chunk(wa, ch0 + h);
+            chunk(wb, ch0 + h + 1u);
+          }
           drain_check();
-          chunk(addr + 512u * h + 1024u, ch0 + h + 2u);
-          chunk(addr + 512u * h + 1536u, ch0 + h + 3u);
+          {
+            const uint4 wc = lds128(addr + 512u * h + 1024u), wd = lds128(addr + 512u * h + 1536u);
+            chunk(wc, ch0 + h + 2u);
+            chunk(wd, ch0 + h + 3u);
+          }
         }
       } else {
 #pragma unroll 1
         for (uint32_t c = 0; c < nc; ++c) {
           if ((c & 1u) == 0u) drain_check();
-          chunk(addr + 512u * c, ch0 + c);
+          chunk(lds128(addr + 512u * c), ch0 + c);
         }
       }
       __syncwarp();
