@@ -27,9 +27,9 @@
  * fingerprints, brute-force enumeration of the toy spaces, and the inter-stage
  * sends (R5) against the 1F1B simulation with sender-side sends on pipelines
  * made uniform by compensating compute, and the DP sync of every stage (R6)
- * against the simulation with a zero-time backward (instant cascade). The
- * reshard term (R13) is "parity unpinned" beyond the worked example derived from
- * its reading.
+ * against the simulation with a zero-time backward (instant cascade), and the
+ * in-stage reshard (R13) against the simulation with the all-gather between the
+ * two halves of each microbatch on compensated uniform pipelines.
  */
 #include <stdint.h>
 #include <stdlib.h>

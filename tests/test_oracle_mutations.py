@@ -70,6 +70,17 @@ MUTATIONS = [
      "int t = P->op_type[last];\n      u64 v = rec_field(P, dim[last], t, tpl[last], (int)mbs_log2 - dpl[last], P2P_BWD);"),
     ("r13-drop-reshard", "R13, P:L261",
      "rs = rec_field(P, dim[j], t, tpl[j], b, RESHARD);", "rs = 0;"),
+    ("r13-reshard-at-stage-heads", "R13, P:L261 (a stage boundary is a p2p, not a reshard)",
+     "if (j > 0 && !head[j] && (tpl[j] != tpl[j - 1] || dpl[j] != dpl[j - 1]))",
+     "if (j > 0 && (tpl[j] != tpl[j - 1] || dpl[j] != dpl[j - 1]))"),
+    ("r13-reshard-on-every-op", "R13, P:L261 (only at a tp/dp change)",
+     "if (j > 0 && !head[j] && (tpl[j] != tpl[j - 1] || dpl[j] != dpl[j - 1]))",
+     "if (j > 0 && !head[j])"),
+    ("r13-sender-pays", "R13, P:L261 (the receiving op's record)",
+     "rs = rec_field(P, dim[j], t, tpl[j], b, RESHARD);",
+     "rs = rec_field(P, dim[j - 1], P->op_type[j - 1], tpl[j - 1], (int)mbs_log2 - dpl[j - 1], RESHARD);"),
+    ("r13-reshard-once-per-iteration", "R13 + Eq. 2 (per microbatch)",
+     "    S[i] += F + Bp + rs;", "    S[i] += F + Bp;\n    Dd[i] += rs;"),
     ("r9-no-gsum-check", "R9, P:L151", "if (gsum != (u64)P->G) reasons |= O_R_GSUM;", ";"),
     ("dim-ignored-for-compute", "TP dimension, P:L263-265",
      "u64 fc = rec_field(P, dim[j], t, tpl[j], b, FWD_COMP);", "u64 fc = rec_field(P, 0, t, tpl[j], b, FWD_COMP);"),

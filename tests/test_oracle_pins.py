@@ -331,6 +331,53 @@ def test_p2p_backward_sends_match_1f1b_simulation(p, mbs_log2):
 
 
 # --------------------------------------------------------------------------
+# R13 (in-stage tp/dp change: "an all-gather operation might be necessary between the
+# two halves") against the 1F1B simulation: the collective runs on the stage's devices between
+# the two halves of every microbatch, so the simulated stage takes F'_i = F_i + (changes in
+# stage i) x c per microbatch. Stages with fewer changes get the same amount of extra compute,
+# so the pipeline is uniform and Eq. 2 (R1) is exact -- but only if the oracle charges the
+# RECEIVING op's reshard once per change per microbatch, and nothing at a stage boundary (a
+# stage head whose tp/dp differs from the previous stage's last op pays a p2p, not a reshard)
+# or at the op before the change.
+# --------------------------------------------------------------------------
+@pytest.mark.parametrize("p", [1, 2, 3, 4])
+@pytest.mark.parametrize("mbs_log2", [1, 2, 3])
+@pytest.mark.parametrize("changes", [(1,), (2,), (0, 1), (2, 0, 1)])
+def test_reshard_matches_1f1b_simulation(p, mbs_log2, changes):
+    k, f, b, c = 6, 7, 13, 5
+    ch = [changes[i % len(changes)] for i in range(p)]  # tp/dp changes inside stage i
+    most = max(ch)
+    recs = {0: lambda tpl, bb: [f, 0, b, 0, 0, 0, 0, 1000, 0, 0],          # inner op: never charged
+            1: lambda tpl, bb: [f, 0, b, 0, 0, 0, 0, c, 0, 0],             # the op after a change
+            2: lambda tpl, bb: [f, 0, b, 0, 0, 0, 0, 3000, 0, 0],          # stage head: never charged
+            3: lambda tpl, bb: [f + c, 0, b, 0, 0, 0, 0, 1000, 0, 0],      # compensation, 1 change
+            4: lambda tpl, bb: [f + 2 * c, 0, b, 0, 0, 0, 0, 1000, 0, 0]}  # compensation, 2 changes
+    types, row = [], []
+    for i in range(p):
+        lay = [(1, 0)] * k  # (tpl, dpl): 2 devices per stage either way (in-stage symmetry)
+        recv = [2, 4][:ch[i]]  # ops that receive a new layout
+        for j in range(k):
+            flips = sum(1 for r in recv if j >= r)
+            lay[j] = (1, 0) if flips % 2 == 0 else (0, 1)
+        if i % 2 == 1:  # alternate the head's layout: a layout change across the stage boundary
+            lay = [(1 - t, 1 - d) for t, d in lay]
+        ty = [2] + [0] * (k - 1)
+        for r in recv:
+            ty[r] = 1
+        if most - ch[i] > 0:
+            ty[k - 1] = 3 if most - ch[i] == 1 else 4
+        types += ty
+        row += [ai.code(1 if j == 0 else 0, lay[j][0], lay[j][1], 0) for j in range(k)]
+    prof = mkprof(recs, types, n_tp=2, n_b=8, n_dp=2, G=2 * p, Bg=8)
+    N = 8 >> mbs_log2
+    out = ev(prof, [row], [ai.header(mbs_log2, p)])
+    assert out["info"][0] & oracle.INFO_INVALID == 0
+    mk, _ = simulate([k * f + most * c] * p, [k * b] * p, N)
+    assert int(out["iter"][0]) == mk == (N + p - 1) * (k * (f + b) + most * c)
+    assert len(set(int(x) for x in out["stage_T"][0, :p])) == 1
+
+
+# --------------------------------------------------------------------------
 # readings without an independent pin: worked examples (parity unpinned beyond these)
 # --------------------------------------------------------------------------
 def test_p2p_and_reshard_worked_example():
