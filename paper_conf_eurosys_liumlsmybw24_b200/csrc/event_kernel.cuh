@@ -62,7 +62,6 @@ __host__ __device__ constexpr uint32_t ev_qo_off(bool full, uint32_t w, int sc) 
 __host__ __device__ constexpr uint32_t ev_smem_bytes(bool full, uint32_t w, int sc, uint32_t qo_bytes) {
   return ev_qo_off(full, w, sc) + (sc == 8 ? 0u : qo_bytes);
 }
-__host__ __device__ constexpr uint32_t ev_snap_bytes(bool) { return 0u; }
 
 __device__ __forceinline__ uint64_t u64of(uint32_t lo, uint32_t hi) {
   return ((uint64_t)hi << 32) | lo;
@@ -202,13 +201,8 @@ template <uint32_t MODE>
 __device__ __forceinline__ void ev_rc_lookup(const EvalParams &P, uint32_t qsb, uint32_t rr, uint32_t pat,
                                              uint64_t &dS, uint64_t &dA, uint32_t &e1, uint64_t &dC) {
   const uint32_t idx = qsb + rr * 16u + pat;
-#ifdef ACESO_EXPERIMENT_RC_NOLOAD
-  const uint4 v0 = make_uint4(idx, idx >> 3, idx * 3u, idx >> 5);
-  const uint4 v1 = make_uint4(idx ^ 5u, 0u, idx, 0u);
-#else
   const uint4 v0 = __ldg(P.qr + 2u * idx);
   const uint4 v1 = __ldg(P.qr + 2u * idx + 1u);
-#endif
   dS += u64of(v0.x, v0.y);
   dA += u64of(v0.z, v0.w);
   e1 = max(e1, v1.x);
@@ -379,10 +373,6 @@ template <uint32_t MODE, int SC, bool OCT>
 __device__ __forceinline__ void ev_drain(EvCand &s, const EvalParams &P, uint32_t qo, uint32_t lb,
                                          uint32_t lx, int64_t cand, bool active) {
   constexpr uint32_t kEvF = ev_f_off(SC), kEvC = ev_c_off(SC);
-#ifdef ACESO_EXPERIMENT_NO_PHASEB
-  s.ec = 0;
-  return;
-#endif
   constexpr uint32_t XS = 32u * ev_xrec(MODE & kFull);  // X stride per entry
   uint32_t k = 0, em = 0, rm = 0, ent = 0, xe = 0, q0 = 0;
 #pragma unroll 1
@@ -550,11 +540,7 @@ __global__ void __launch_bounds__(32 * W, MINB) event_kernel(const __grid_consta
       rE = 0;
       s.ec = k + 1u;
     }
-#ifdef ACESO_EXPERIMENT_NO_RC
-    if (false) {
-#else
     if (__any_sync(0xffffffffu, rcc)) {
-#endif
       if (rcc) {
         // recompute flags in an event-free chunk: every op is in the open run, whose
         // (tp, dp) is that of op 0 of the chunk
