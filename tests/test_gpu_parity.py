@@ -834,3 +834,45 @@ def test_event_kernel_recompute_levels_parity(minb, slot, oct, name, monkeypatch
     finally:
         _ctx_cache.pop(id(prof), None)
         ctx.close()
+
+
+# ---------------------------------------------------------------------------
+# ring geometry of the event kernel: model lengths at chunk (16 ops) and ring-slot (4 or 8
+# chunks) boundaries, so that the paired chunk loads, partial last slots and the zero-padded
+# last chunk meet every case (one chunk, exactly one slot, one op past a slot, ...)
+# ---------------------------------------------------------------------------
+def _small_profile(L, seed):
+    rng = np.random.default_rng(seed)
+    T, NT, NB, ND, G = 7, 4, 6, 4, 8
+    rec = np.zeros((T, NT, NB, P.NF), np.int64)
+    rec[..., 0:4] = rng.integers(0, 1 << 16, size=(T, NT, NB, 4))
+    act = rng.integers(1, 1 << 12, size=(T, NT, NB))
+    rec[..., 4] = act
+    rec[..., 5] = (rng.random((T, NT, NB)) * act).astype(np.int64)
+    rec[..., 6] = rng.integers(0, 1 << 12, size=(T, NT, NB))
+    rec[..., 7:10] = rng.integers(0, 1 << 14, size=(T, NT, NB, 3))
+    wmem = rng.integers(0, 1 << 12, size=(T, NT, 2)).astype(np.int64)
+    dps = rng.integers(0, 1 << 16, size=(T, NT, ND)).astype(np.int64)
+    op_type = rng.integers(0, T, size=L).astype(np.uint16)
+    return P.Profile(f"ring{L}", op_type, [f"t{i}" for i in range(T)], rec, wmem, dps, G, 1 << 24, 64)
+
+
+@pytest.mark.parametrize("minb,slot", [("2", "8"), ("2", "4"), ("3", "4")])
+@pytest.mark.parametrize("L", [1, 15, 16, 17, 63, 64, 65, 127, 128, 129, 143, 144, 145, 255, 257])
+def test_event_kernel_ring_geometry_parity(L, minb, slot, monkeypatch):
+    monkeypatch.setenv("ACESO_KERNEL", "events")
+    monkeypatch.setenv("ACESO_MINB", minb)
+    monkeypatch.setenv("ACESO_EV_SLOT", slot)
+    prof = _small_profile(L, SEED + L)
+    ctx = A.Context(prof, 0)
+    _ctx_cache[id(prof)] = (prof, ctx)
+    try:
+        codes, hdr = ai.search_shaped(prof, SEED + 50 + L, 0, 333, group_size=16)
+        g, o, sel, _, _ = compare(prof, codes, hdr)
+        assert ((o["info"] & oracle.INFO_INVALID) == 0).mean() > 0.5
+        compare(prof, codes, hdr, full=True)
+        codes, hdr = ai.dense_random(prof, SEED + 51 + L, 0, 97)
+        compare(prof, codes, hdr)
+    finally:
+        _ctx_cache.pop(id(prof), None)
+        ctx.close()
