@@ -193,10 +193,11 @@ def cpu_baseline(prof, codes, hdr, target_core_s=15.0, what="candidates of the t
 class Batches:
     """Distinct device-resident batches (together larger than L2) of this rank's shard."""
 
-    def __init__(self, A, prof, dist, n, group, world, rank, dev, toy=False):
+    def __init__(self, A, prof, dist, n, group, world, rank, dev, toy=False, min_buf=0):
         self.n, self.L = n, prof.n_ops
         per_batch = A.tiled_bytes(n, self.L) + 8 * n
-        self.nbuf = max(2, int(np.ceil(1.3 * L2_BYTES / per_batch)))
+        # at least one distinct batch per stream in flight (min_buf), together larger than L2
+        self.nbuf = max(2, int(np.ceil(1.3 * L2_BYTES / per_batch)), min_buf)
         self.host, self.dev = [], []
         if toy:  # the whole space, replicated into distinct buffers
             import aceso_inputs as ai
@@ -682,7 +683,8 @@ def measure_workload(A, name, args, dev, hbm, src, world=1, rank=0, dist=None, s
         n = int(len(toy_space(prof)[1]))
     else:
         n = args.batch if (args.batch and name == args.config) else BATCH[name]
-    bt = Batches(A, prof, "search" if toy else args.dist, n, args.group, world, rank, dev, toy=toy)
+    bt = Batches(A, prof, "search" if toy else args.dist, n, args.group, world, rank, dev, toy=toy,
+                 min_buf=args.streams)
     per_batch = A.tiled_bytes(n, prof.n_ops) + 8 * n
     nstr = args.streams or (8 if per_batch < 64 * 2 ** 20 else 2)
     nstr = max(1, min(nstr, bt.nbuf))
