@@ -32,6 +32,26 @@ def _ptr(t):
     return None if t is None else ctypes.c_void_p(t.data_ptr())
 
 
+def _need(t, name, device, dtypes, numel):
+    """Argument check before a pointer crosses the C-ABI: a host tensor, another device, a
+    wrong element type or a short buffer would otherwise reach the kernel (a device fault)."""
+    if not isinstance(t, torch.Tensor):
+        raise TypeError(f"{name}: expected a torch.Tensor, got {type(t).__name__}")
+    if not t.is_cuda or t.device != device:
+        raise ValueError(f"{name}: must be on {device}, is on {t.device}")
+    if t.dtype not in dtypes:
+        raise ValueError(f"{name}: dtype {t.dtype} not in {dtypes}")
+    if not t.is_contiguous():
+        raise ValueError(f"{name}: must be contiguous")
+    if t.numel() < numel:
+        raise ValueError(f"{name}: {t.numel()} elements < {numel} needed")
+
+
+_I64 = (torch.int64,)
+_I32 = (torch.int32,)
+_U8 = (torch.uint8,)
+
+
 def _stream(stream):
     if stream is None:
         stream = torch.cuda.current_stream()
@@ -145,6 +165,16 @@ class Context:
             o.stage_comm = torch.zeros((pm, n), dtype=torch.int64, device=d)
         return o
 
+    def _check_outputs(self, out: Outputs, n: int, summary: bool, full: bool):
+        d = self._dev
+        if summary and n > 0:
+            _need(out.iter_ns, "out.iter_ns", d, _I64, n)
+            _need(out.max_mem, "out.max_mem", d, _I64, n)
+            _need(out.info, "out.info", d, _I32, n)
+        if full and n > 0:
+            for k in ("stage_T", "stage_mem", "stage_comp", "stage_comm"):
+                _need(getattr(out, k), f"out.{k}", d, _I64, int(out.p_max) * n)
+
     def alloc_select(self, n: int = 0) -> torch.Tensor:
         nb = int(L.load().aceso_select_buf_bytes(self._h, int(n)))
         return torch.zeros(nb, dtype=torch.uint8, device=self._dev)
@@ -160,6 +190,8 @@ class Context:
         if tiled is None:
             tiled = self.alloc_tiled(n)
         codes = codes.contiguous()
+        _need(codes, "codes", self._dev, _U8, n * self.n_ops)
+        _need(tiled, "tiled", self._dev, _U8, tiled_bytes(n, self.n_ops))
         _check(L.load().aceso_pack_rowmajor(_ptr(codes), n, int(codes.shape[1]), _ptr(tiled),
                                             _stream(stream)), "aceso_pack_rowmajor")
         return tiled
@@ -192,6 +224,16 @@ class Context:
             out = self.alloc_outputs(n, full=full)
         if select and sel is None:
             sel = self.alloc_select(n)
+        d = self._dev
+        if n > 0:
+            _need(codes, "codes", d, _U8, tiled_bytes(n, self.n_ops))
+            _need(hdr, "hdr", d, _I64, n)
+        if out is not None:
+            self._check_outputs(out, n, summary, full)
+        if select:
+            _need(sel, "sel", d, _U8, int(L.load().aceso_select_buf_bytes(self._h, n)))
+        if dims is not None and n > 0:
+            _need(dims, "dims", d, _U8, int(L.load().aceso_dims_bytes(n, self.n_ops)))
         cs = out.c_struct() if out is not None else None
         if global_key is not None:
             assert dims is None and select
@@ -248,6 +290,8 @@ class Context:
         n_total = global_offset + n if n_total is None else int(n_total)
         if sel is None:
             sel = self.alloc_select(n)
+        self._check_outputs(out, n, True, False)
+        _need(sel, "sel", self._dev, _U8, int(L.load().aceso_select_buf_bytes(self._h, n)))
         cs = out.c_struct()
         _check(L.load().aceso_select(self._h, ctypes.byref(cs), n, int(global_offset), n_total, _ptr(sel),
                                      _stream(stream)), "aceso_select")

@@ -876,3 +876,28 @@ def test_event_kernel_ring_geometry_parity(L, minb, slot, monkeypatch):
     finally:
         _ctx_cache.pop(id(prof), None)
         ctx.close()
+
+
+def test_binding_rejects_bad_tensors_before_the_call():
+    """Host tensors, wrong dtypes and short buffers raise in the binding (no pointer reaches the
+    kernel), and the context still evaluates correctly afterwards."""
+    prof = P.WORKLOADS["gpt3-1.3b"]()
+    ctx = ctx_for(prof)
+    codes, hdr = ai.search_shaped(prof, SEED + 60, 0, 100, group_size=16)
+    tiled = torch.from_numpy(ai.tile(codes))
+    hd = torch.from_numpy(np.ascontiguousarray(hdr, np.uint64).view(np.int64))
+    with pytest.raises(ValueError):
+        ctx.eval(tiled, hd.cuda(), n=100)  # host codes
+    with pytest.raises(ValueError):
+        ctx.eval(tiled.cuda(), hd, n=100)  # host headers
+    with pytest.raises(ValueError):
+        ctx.eval(tiled.cuda()[:-512], hd.cuda(), n=100)  # one chunk short
+    with pytest.raises(ValueError):
+        ctx.eval(tiled.cuda(), hd.cuda().to(torch.int32), n=100)  # wrong header type
+    with pytest.raises(ValueError):
+        ctx.eval(tiled.cuda(), hd.cuda(), n=100, out=ctx.alloc_outputs(99))  # short outputs
+    with pytest.raises(ValueError):
+        ctx.eval(tiled.cuda(), hd.cuda(), n=100, sel=torch.zeros(64, dtype=torch.uint8, device="cuda"))
+    with pytest.raises(ValueError):
+        ctx.eval(tiled.cuda(), hd.cuda(), n=100, full=True, out=ctx.alloc_outputs(50, full=True))
+    compare(prof, codes, hdr, full=True)  # the context is intact
