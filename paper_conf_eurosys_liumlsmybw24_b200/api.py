@@ -263,6 +263,7 @@ class Context:
             plane = torch.zeros(max(2, int(L.load().aceso_dims_bytes(n, self.n_ops))), dtype=torch.uint8,
                                 device=self._dev)
         dims = dims.contiguous()
+        _need(plane, "plane", self._dev, _U8, int(L.load().aceso_dims_bytes(n, self.n_ops)))
         _check(L.load().aceso_pack_dims(_ptr(dims), n, int(dims.shape[1]), _ptr(plane), _stream(stream)),
                "aceso_pack_dims")
         return plane
@@ -278,6 +279,14 @@ class Context:
         if hdr is None:
             hdr = torch.empty(max(n, 1), dtype=torch.int64, device=self._dev)
         nb = int(bases.shape[0])
+        d, stride = self._dev, 16 * ((self.n_ops + 15) // 16)
+        if n > 0:
+            _need(bases, "bases", d, _U8, nb * stride)
+            _need(cands, "cands", d, _U8, 56 * n)
+            if ranks is not None:
+                _need(ranks, "ranks", d, (torch.int16,), nb * 2 * stride)
+            _need(tiled, "tiled", d, _U8, tiled_bytes(n, self.n_ops))
+            _need(hdr, "hdr", d, _I64, n)
         _check(L.load().aceso_expand(_ptr(bases), _ptr(ranks) if ranks is not None else None, nb,
                                      self.n_ops, _ptr(cands), n, _ptr(tiled), _ptr(hdr), _stream(stream)),
                "aceso_expand")
@@ -304,6 +313,11 @@ def hash_candidates(codes: torch.Tensor, hdr: torch.Tensor, n_ops: int, n: int |
     n = int(hdr.shape[0]) if n is None else int(n)
     if out is None:
         out = torch.empty(n, dtype=torch.int64, device=hdr.device)
+    if n > 0:
+        d = hdr.device
+        _need(codes, "codes", d, _U8, tiled_bytes(n, n_ops))
+        _need(hdr, "hdr", d, _I64, n)
+        _need(out, "out", d, _I64, n)
     _check(L.load().aceso_hash(_ptr(codes), _ptr(hdr), n, int(n_ops), _ptr(out), _stream(stream)),
            "aceso_hash")
     return out
@@ -326,6 +340,10 @@ class VisitedSet:
         n = int(hashes.shape[0])
         if dup is None:
             dup = torch.empty(n, dtype=torch.uint8, device=hashes.device)
+        d = self.table.device
+        if n > 0:
+            _need(hashes, "hashes", d, _I64, n)
+            _need(dup, "dup", d, _U8, n)
         self.epoch += 1
         _check(L.load().aceso_dedup(_ptr(hashes), n, self.epoch, _ptr(self.table), self.slots, _ptr(dup),
                                     _ptr(self.status), _stream(stream)), "aceso_dedup")
@@ -355,6 +373,10 @@ def enum_cuts(n_ops: int, p: int, code: int, hdr: int, first: int, n: int, tiled
               hdr_out: torch.Tensor, stream=None):
     """aceso_enum_cuts: candidates [first, first + n) of the stage-partition family (p, code,
     hdr) written to device `tiled` (uint8, tiled layout) and `hdr_out` (int64)."""
+    if n > 0:
+        d = tiled.device
+        _need(tiled, "tiled", d, _U8, tiled_bytes(n, n_ops))
+        _need(hdr_out, "hdr_out", d, _I64, n)
     _check(L.load().aceso_enum_cuts(int(n_ops), int(p), int(code) & 0xFF, int(hdr), int(first), int(n),
                                     _ptr(tiled), _ptr(hdr_out), _stream(stream)), "aceso_enum_cuts")
 
