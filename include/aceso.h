@@ -33,7 +33,10 @@ extern "C" {
 /* Status codes (return values).                                             */
 /* ------------------------------------------------------------------------- */
 #define ACESO_OK       0
-#define ACESO_EINVAL  (-1) /* bad argument (null pointer, bad size, bad flags) */
+#define ACESO_EINVAL  (-1) /* bad argument (null pointer, bad size, bad flags;
+                              a device-pointer argument that is plain host memory
+                              or another device's memory: every call checks its
+                              device pointers with cudaPointerGetAttributes) */
 #define ACESO_ERANGE  (-2) /* a profile value does not fit the packed width,
                               keep > act, or a model-wide bound could overflow */
 #define ACESO_ECUDA   (-3) /* a CUDA runtime call failed (message in last_error) */

@@ -47,6 +47,29 @@ int fail(int code, const char *fmt, ...) {
       return fail(ACESO_ECUDA, "%s failed: %s", #expr, cudaGetErrorString(e_));            \
   } while (0)
 
+// A pointer the kernels dereference must be device-accessible from `device`: its device memory,
+// managed memory or mapped pinned host memory. Plain host memory (or another device's memory)
+// would fault inside the kernel, a sticky error that ends the CUDA context, so it is refused
+// here with ACESO_EINVAL naming the argument. Null is the caller's (size-dependent) check;
+// device -1: any device (the context-free calls).
+int check_dev_ptr(const void *p, const char *name, int device) {
+  if (!p) return ACESO_OK;
+  cudaPointerAttributes a;
+  if (cudaPointerGetAttributes(&a, p) != cudaSuccess) {
+    cudaGetLastError();  // clear the non-sticky lookup error
+    return fail(ACESO_EINVAL, "%s: not a CUDA-visible pointer", name);
+  }
+  if (a.type == cudaMemoryTypeUnregistered) return fail(ACESO_EINVAL, "%s: host memory, not device-accessible", name);
+  if (a.type == cudaMemoryTypeDevice && device >= 0 && a.device != device)
+    return fail(ACESO_EINVAL, "%s: memory of device %d, context on device %d", name, a.device, device);
+  return ACESO_OK;
+}
+#define PTR_TRY(p, dev)                                       \
+  do {                                                        \
+    const int r_ = check_dev_ptr((p), #p, (dev));             \
+    if (r_ != ACESO_OK) return r_;                            \
+  } while (0)
+
 template <int B>
 void *quad_kernel_for(uint32_t mode) {
   switch (mode) {
@@ -988,6 +1011,22 @@ static int eval_impl(aceso_ctx *ctx, const uint8_t *d_codes, const uint64_t *d_h
   }
   if ((mode & ACESO_FUSED_SELECT) && !d_sel) return fail(ACESO_EINVAL, "null select buffer");
   if (((uintptr_t)d_codes & 15) != 0) return fail(ACESO_EINVAL, "codes not 16-byte aligned");
+  if (n > 0) {
+    PTR_TRY(d_codes, ctx->device);
+    PTR_TRY(d_hdr, ctx->device);
+    if (mode & ACESO_OUT_SUMMARY) {
+      PTR_TRY(out->iter_ns, ctx->device);
+      PTR_TRY(out->max_mem, ctx->device);
+      PTR_TRY(out->info, ctx->device);
+    }
+    if (mode & ACESO_OUT_FULL) {
+      PTR_TRY(out->stage_T, ctx->device);
+      PTR_TRY(out->stage_mem, ctx->device);
+      PTR_TRY(out->stage_comp, ctx->device);
+      PTR_TRY(out->stage_comm, ctx->device);
+    }
+  }
+  if (mode & ACESO_FUSED_SELECT) PTR_TRY(d_sel, ctx->device);
 
   EvalParams P = make_params(ctx, n, global_offset, n_total, out, d_sel);
   P.codes = reinterpret_cast<const uint4 *>(d_codes);
@@ -1033,6 +1072,8 @@ size_t aceso_dims_bytes(int64_t n, int32_t n_ops) {
 int aceso_pack_dims(const uint8_t *d_rowmajor, int64_t n, int32_t n_ops, uint8_t *d_plane, void *stream) {
   if (n < 0 || n_ops < 1 || n_ops > kMaxOps || (n > 0 && (!d_rowmajor || !d_plane))) return fail(ACESO_EINVAL, "bad argument");
   if (((uintptr_t)d_plane & 1) != 0) return fail(ACESO_EINVAL, "dimension plane not 2-byte aligned");
+  PTR_TRY(d_rowmajor, -1);
+  PTR_TRY(d_plane, -1);
   if (n == 0) return ACESO_OK;
   const int64_t total = (int64_t)aceso_dims_bytes(n, n_ops) / 2;
   const int grid = (int)std::min<int64_t>((total + 255) / 256, 148 * 16);
@@ -1065,6 +1106,23 @@ int aceso_eval_dims(aceso_ctx *ctx, const uint8_t *d_codes, const uint8_t *d_dim
   }
   if ((mode & ACESO_FUSED_SELECT) && !d_sel) return fail(ACESO_EINVAL, "null select buffer");
   if (((uintptr_t)d_codes & 15) != 0) return fail(ACESO_EINVAL, "codes not 16-byte aligned");
+  if (n > 0) {
+    PTR_TRY(d_codes, ctx->device);
+    PTR_TRY(d_dims, ctx->device);
+    PTR_TRY(d_hdr, ctx->device);
+    if (mode & ACESO_OUT_SUMMARY) {
+      PTR_TRY(out->iter_ns, ctx->device);
+      PTR_TRY(out->max_mem, ctx->device);
+      PTR_TRY(out->info, ctx->device);
+    }
+    if (mode & ACESO_OUT_FULL) {
+      PTR_TRY(out->stage_T, ctx->device);
+      PTR_TRY(out->stage_mem, ctx->device);
+      PTR_TRY(out->stage_comp, ctx->device);
+      PTR_TRY(out->stage_comm, ctx->device);
+    }
+  }
+  if (mode & ACESO_FUSED_SELECT) PTR_TRY(d_sel, ctx->device);
   EvalParams P = make_params(ctx, n, global_offset, n_total, out, d_sel);
   P.codes = reinterpret_cast<const uint4 *>(d_codes);
   P.hdr = d_hdr;
@@ -1094,6 +1152,12 @@ int aceso_select(aceso_ctx *ctx, const aceso_eval_out *out, int64_t n, int64_t g
   if (!ctx || !d_sel) return fail(ACESO_EINVAL, "null argument");
   if (n < 0 || global_offset < 0 || n_total < global_offset + n) return fail(ACESO_EINVAL, "bad n / global_offset / n_total");
   if (n > 0 && (!out || !out->iter_ns || !out->max_mem || !out->info)) return fail(ACESO_EINVAL, "null summary");
+  if (n > 0) {
+    PTR_TRY(out->iter_ns, ctx->device);
+    PTR_TRY(out->max_mem, ctx->device);
+    PTR_TRY(out->info, ctx->device);
+  }
+  PTR_TRY(d_sel, ctx->device);
   const int64_t blocks = (n + 255) / 256;
   const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(blocks, 4 * ctx->sms));
   int prev = 0;
@@ -1129,6 +1193,10 @@ int aceso_pack_rowmajor(const uint8_t *d_rowmajor, int64_t n, int32_t n_ops, uin
                         void *stream) {
   if (n < 0 || n_ops < 1 || (n > 0 && (!d_rowmajor || !d_tiled))) return fail(ACESO_EINVAL, "bad argument");
   if (((uintptr_t)d_tiled & 15) != 0) return fail(ACESO_EINVAL, "tiled buffer not 16-byte aligned");
+  if (n > 0) {
+    PTR_TRY(d_rowmajor, -1);
+    PTR_TRY(d_tiled, -1);
+  }
   if (n == 0) return ACESO_OK;
   const int64_t total_vec = (int64_t)aceso_tiled_bytes(n, n_ops) / 16;
   const int grid = (int)std::min<int64_t>((total_vec + 255) / 256, 148 * 16);
@@ -1146,6 +1214,13 @@ int aceso_expand(const uint8_t *d_bases, const uint16_t *d_ranks, int32_t n_base
   if (n > 0 && (!d_bases || !d_cands || !d_tiled || !d_hdr)) return fail(ACESO_EINVAL, "null argument");
   if (((uintptr_t)d_tiled & 15) != 0 || ((uintptr_t)d_bases & 15) != 0)
     return fail(ACESO_EINVAL, "bases / tiled output not 16-byte aligned");
+  if (n > 0) {
+    PTR_TRY(d_bases, -1);
+    PTR_TRY(d_ranks, -1);
+    PTR_TRY(d_cands, -1);
+    PTR_TRY(d_tiled, -1);
+    PTR_TRY(d_hdr, -1);
+  }
   if (n == 0) return ACESO_OK;
   const int grid = (int)std::max<int64_t>(1, std::min<int64_t>((n + 255) / 256, 148 * 16));
   expand_kernel<<<grid, 256, 0, reinterpret_cast<cudaStream_t>(stream)>>>(
@@ -1168,6 +1243,10 @@ int aceso_enum_cuts(int32_t n_ops, int32_t p, uint8_t code, uint64_t hdr, int64_
   if (first < 0 || n < 0 || first + n > cnt) return fail(ACESO_EINVAL, "range [first, first + n) outside [0, %lld)", (long long)cnt);
   if (n > 0 && (!d_tiled || !d_hdr)) return fail(ACESO_EINVAL, "null argument");
   if (((uintptr_t)d_tiled & 15) != 0) return fail(ACESO_EINVAL, "tiled output not 16-byte aligned");
+  if (n > 0) {
+    PTR_TRY(d_tiled, -1);
+    PTR_TRY(d_hdr, -1);
+  }
   if (n == 0) return ACESO_OK;
   const int grid = (int)std::max<int64_t>(1, std::min<int64_t>((n + 255) / 256, 148 * 16));
   enum_cuts_kernel<<<grid, 256, 0, reinterpret_cast<cudaStream_t>(stream)>>>(
@@ -1182,6 +1261,11 @@ int aceso_hash(const uint8_t *d_codes, const uint64_t *d_hdr, int64_t n, int32_t
   if (n < 0 || n_ops < 1 || n_ops > kMaxOps || (n > 0 && (!d_codes || !d_hdr || !d_hash)))
     return fail(ACESO_EINVAL, "bad argument");
   if (((uintptr_t)d_codes & 15) != 0) return fail(ACESO_EINVAL, "codes not 16-byte aligned");
+  if (n > 0) {
+    PTR_TRY(d_codes, -1);
+    PTR_TRY(d_hdr, -1);
+    PTR_TRY(d_hash, -1);
+  }
   if (n == 0) return ACESO_OK;
   const int64_t tiles = (n + 31) / 32;
   const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(tiles, 148 * 32));
@@ -1205,6 +1289,12 @@ int aceso_dedup(const uint64_t *d_hash, int64_t n, uint32_t epoch, void *d_table
   if (!d_table || !d_status || (n > 0 && (!d_hash || !d_dup))) return fail(ACESO_EINVAL, "null argument");
   cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
   CUDA_TRY(cudaMemsetAsync(d_status, 0, sizeof(uint32_t), st));
+  PTR_TRY(d_table, -1);
+  PTR_TRY(d_status, -1);
+  if (n > 0) {
+    PTR_TRY(d_hash, -1);
+    PTR_TRY(d_dup, -1);
+  }
   if (n == 0) return ACESO_OK;
   const int grid = (int)std::max<int64_t>(1, std::min<int64_t>((n + 255) / 256, 148 * 16));
   VisitedEntry *t = reinterpret_cast<VisitedEntry *>(d_table);

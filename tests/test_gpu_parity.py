@@ -901,3 +901,35 @@ def test_binding_rejects_bad_tensors_before_the_call():
     with pytest.raises(ValueError):
         ctx.eval(tiled.cuda(), hd.cuda(), n=100, full=True, out=ctx.alloc_outputs(50, full=True))
     compare(prof, codes, hdr, full=True)  # the context is intact
+
+
+def test_capi_rejects_host_pointers():
+    """The C-ABI itself (below the binding's checks) refuses plain host memory with
+    ACESO_EINVAL instead of faulting in the kernel; the context stays usable."""
+    import ctypes
+    from paper_conf_eurosys_liumlsmybw24_b200 import _lib as L
+    prof = P.WORKLOADS["gpt3-1.3b"]()
+    ctx = ctx_for(prof)
+    codes, hdr = ai.search_shaped(prof, SEED + 61, 0, 64, group_size=16)
+    tiled_h = np.ascontiguousarray(ai.tile(codes))
+    hdr_h = np.ascontiguousarray(hdr, np.uint64)
+    tiled_d = torch.from_numpy(tiled_h).cuda()
+    hdr_d = torch.from_numpy(hdr_h.view(np.int64)).cuda()
+    out = ctx.alloc_outputs(64)
+    sel = ctx.alloc_select(64)
+    lib = L.load()
+    cs = out.c_struct()
+    st = ctypes.c_void_p(torch.cuda.current_stream().cuda_stream)
+    flags = L.OUT_SUMMARY | L.FUSED_SELECT
+    rc = lib.aceso_eval(ctx._h, ctypes.c_void_p(tiled_h.ctypes.data), ctypes.c_void_p(hdr_d.data_ptr()), 64, 0, 64,
+                        flags, ctypes.byref(cs), ctypes.c_void_p(sel.data_ptr()), st)
+    assert rc == L.ACESO_EINVAL and b"d_codes" in lib.aceso_last_error()
+    rc = lib.aceso_eval(ctx._h, ctypes.c_void_p(tiled_d.data_ptr()), ctypes.c_void_p(hdr_h.ctypes.data), 64, 0, 64,
+                        flags, ctypes.byref(cs), ctypes.c_void_p(sel.data_ptr()), st)
+    assert rc == L.ACESO_EINVAL and b"d_hdr" in lib.aceso_last_error()
+    hs = np.zeros(64, np.uint64)
+    rc = lib.aceso_hash(ctypes.c_void_p(tiled_d.data_ptr()), ctypes.c_void_p(hdr_d.data_ptr()), 64, prof.n_ops,
+                        ctypes.c_void_p(hs.ctypes.data), st)
+    assert rc == L.ACESO_EINVAL and b"d_hash" in lib.aceso_last_error()
+    torch.cuda.synchronize()
+    compare(prof, codes, hdr)  # nothing faulted: the context still evaluates
