@@ -52,8 +52,15 @@ int fail(int code, const char *fmt, ...) {
 // would fault inside the kernel, a sticky error that ends the CUDA context, so it is refused
 // here with ACESO_EINVAL naming the argument. Null is the caller's (size-dependent) check;
 // device -1: any device (the context-free calls).
+// The last 16 pointers that passed (exact addresses, with their device) are remembered per
+// thread: loops that reuse their buffers every step query the driver once per buffer.
 int check_dev_ptr(const void *p, const char *name, int device) {
   if (!p) return ACESO_OK;
+  static thread_local const void *ok_ptr[16];
+  static thread_local int ok_dev[16];
+  static thread_local unsigned ok_next;
+  for (int k = 0; k < 16; ++k)
+    if (ok_ptr[k] == p && (device < 0 || ok_dev[k] == device)) return ACESO_OK;
   cudaPointerAttributes a;
   if (cudaPointerGetAttributes(&a, p) != cudaSuccess) {
     cudaGetLastError();  // clear the non-sticky lookup error
@@ -62,6 +69,11 @@ int check_dev_ptr(const void *p, const char *name, int device) {
   if (a.type == cudaMemoryTypeUnregistered) return fail(ACESO_EINVAL, "%s: host memory, not device-accessible", name);
   if (a.type == cudaMemoryTypeDevice && device >= 0 && a.device != device)
     return fail(ACESO_EINVAL, "%s: memory of device %d, context on device %d", name, a.device, device);
+  if (device >= 0 || a.type == cudaMemoryTypeDevice) {  // remember it with the device it was checked for
+    const unsigned k = ok_next++ & 15u;
+    ok_ptr[k] = p;
+    ok_dev[k] = device >= 0 ? device : a.device;
+  }
   return ACESO_OK;
 }
 #define PTR_TRY(p, dev)                                       \
