@@ -37,7 +37,7 @@ def _need(t, name, device, dtypes, numel):
     wrong element type or a short buffer would otherwise reach the kernel (a device fault)."""
     if not isinstance(t, torch.Tensor):
         raise TypeError(f"{name}: expected a torch.Tensor, got {type(t).__name__}")
-    if not t.is_cuda or t.device != device:
+    if t.device != device:  # the context's device (always a CUDA device outside tests)
         raise ValueError(f"{name}: must be on {device}, is on {t.device}")
     if t.dtype not in dtypes:
         raise ValueError(f"{name}: dtype {t.dtype} not in {dtypes}")

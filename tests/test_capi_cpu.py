@@ -159,3 +159,24 @@ def test_enum_cuts_count_is_the_binomial():
             got = enum_cuts_count(L, p)
             assert got == (want if 0 <= want < (1 << 62) else -1), (L, p, got, want)
     assert enum_cuts_count(315, 9) == -1 and enum_cuts_count(0, 1) == -1 and enum_cuts_count(315, 0) == -1
+
+
+def test_binding_argument_checks_cpu():
+    """The binding's tensor check (api._need) refuses a wrong device, dtype, a non-contiguous
+    view and a short buffer before any pointer reaches the C-ABI (device = cpu stands in for
+    the context's CUDA device here)."""
+    import torch
+    from paper_conf_eurosys_liumlsmybw24_b200.api import _need
+    cpu = torch.device("cpu")
+    t = torch.zeros(64, dtype=torch.int64)
+    _need(t, "t", cpu, (torch.int64,), 64)  # passes
+    with pytest.raises(ValueError):
+        _need(t, "t", torch.device("cuda", 0), (torch.int64,), 64)
+    with pytest.raises(ValueError):
+        _need(t, "t", cpu, (torch.int32,), 64)
+    with pytest.raises(ValueError):
+        _need(t, "t", cpu, (torch.int64,), 65)
+    with pytest.raises(ValueError):
+        _need(t.view(8, 8).t(), "t", cpu, (torch.int64,), 8)
+    with pytest.raises(TypeError):
+        _need(t.numpy(), "t", cpu, (torch.int64,), 1)
