@@ -598,13 +598,19 @@ __global__ void __launch_bounds__(32 * W, MINB) event_kernel(const __grid_consta
           // two chunks' code words requested back to back (the second chunk's shared-memory
           // latency hides behind the first chunk's work)
           drain_check();
-          {
+          if (FULL) {  // (FULL modes: no paired loads; their extra live registers spill at 80)
+            chunk(lds128(addr + 512u * h), ch0 + h);
+            chunk(lds128(addr + 512u * h + 512u), ch0 + h + 1u);
+          } else {
             const uint4 wa = lds128(addr + 512u * h), wb = lds128(addr + 512u * h + 512u);
             chunk(wa, ch0 + h);
             chunk(wb, ch0 + h + 1u);
           }
           drain_check();
-          {
+          if (FULL) {
+            chunk(lds128(addr + 512u * h + 1024u), ch0 + h + 2u);
+            chunk(lds128(addr + 512u * h + 1536u), ch0 + h + 3u);
+          } else {
             const uint4 wc = lds128(addr + 512u * h + 1024u), wd = lds128(addr + 512u * h + 1536u);
             chunk(wc, ch0 + h + 2u);
             chunk(wd, ch0 + h + 3u);
