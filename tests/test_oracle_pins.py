@@ -4,6 +4,8 @@ the paper or mathematics fixes, not against a retyped copy of its formulas.
 P:Lnn = PAPER.md line; R# = reading in DESIGN.md §3.
 """
 import itertools
+import json
+import os
 
 import numpy as np
 import pytest
@@ -200,35 +202,45 @@ def test_zero_cost_op_move_changes_nothing():
 
 
 # --------------------------------------------------------------------------
-# Heuristic-1 on the Fig. 3 scenario, worked by hand
+# Heuristic-1 on the Fig. 3 scenario, worked by hand: tests/golden/fig3_scenario.json
 # --------------------------------------------------------------------------
-def fig3_profile():
-    # one op type; b index 0 = 1 sample/GPU, 1 = 2 samples/GPU; tpl 0/1
-    tab = {(0, 0): (100, 200, 10), (0, 1): (200, 400, 20), (1, 0): (60, 120, 5), (1, 1): (120, 240, 10)}
+GOLDEN = os.path.join(os.path.dirname(os.path.abspath(__file__)), "golden")
 
-    def r(tpl, b):
-        f, bw, a = tab[(tpl, b)]
-        return [f, 0, bw, 0, a, a, 0, 0, 0, 0]
-    return mkprof({0: r}, [0, 0, 0, 0], n_tp=2, n_b=2, n_dp=2, G=3, C=60, Bg=8)
+
+def _golden(name):
+    with open(os.path.join(GOLDEN, name)) as f:
+        return json.load(f)
+
+
+def fig3_profile():
+    g = _golden("fig3_scenario.json")
+    tab = {tuple(int(x) for x in k.split(",")): v for k, v in g["records"].items()}
+    pr = g["profile"]
+    return mkprof({0: lambda tpl, b: tab[(tpl, b)]}, [0] * pr["n_ops"], n_tp=pr["n_tp"], n_b=pr["n_b"],
+                  n_dp=pr["n_dp"], G=pr["n_devices"], C=pr["mem_capacity"], Bg=pr["global_batch"])
 
 
 def test_fig3_scenario():
+    g = _golden("fig3_scenario.json")
     prof = fig3_profile()
-    rows = [cand([2, 2], tpdp=[(0, 0), (0, 1)]),   # (a) even ops; 1 GPU + 2 GPUs (dp=2)
-            cand([2, 2], tpdp=[(1, 0), (0, 0)]),   # (b) stage 0 gets 2 GPUs (tp=2)
-            cand([3, 1], tpdp=[(1, 0), (0, 0)])]   # (c) migrate one op to stage 0
-    out = ev(prof, rows, [ai.header(1, 2)] * 3)
+    cs = g["candidates"]
+    rows = [cand(c["stage_sizes"], tpdp=[tuple(t) for t in c["tpdp"]]) for c in cs]
+    out = ev(prof, rows, [ai.header(c["mbs_log2"], c["p"]) for c in cs])
     info = out["info"]
-    # (a): Mem = (80, 20) > C=60 on stage 0 -> OOM, bottleneck stage 0 by memory
-    assert info[0] & oracle.INFO_OOM and info[0] & 0xFF == 0
-    assert list(out["stage_mem"][0, :2]) == [80, 20] and out["max_mem"][0] == 80
-    # (b): no OOM, stage 1 slowest -> bottleneck 1 by time; iter = 1920 + 3*1200
-    assert not info[1] & oracle.INFO_OOM and info[1] & 0xFF == 1
-    assert out["iter"][1] == 5520
-    # (c): balanced -> faster than (b): iter = 1680 + 3*1080
-    assert not info[2] & oracle.INFO_OOM and out["iter"][2] == 4920 < out["iter"][1]
+    for i, c in enumerate(cs):
+        e = g["expected"][c["name"]]
+        assert bool(info[i] & oracle.INFO_OOM) == e["oom"], c["name"]
+        if "bottleneck" in e:
+            assert info[i] & 0xFF == e["bottleneck"], c["name"]
+        if "stage_mem" in e:
+            assert list(out["stage_mem"][i, :len(e["stage_mem"])]) == e["stage_mem"]
+        if "max_mem" in e:
+            assert out["max_mem"][i] == e["max_mem"]
+        if "iter" in e:
+            assert out["iter"][i] == e["iter"], c["name"]
+    assert out["iter"][2] < out["iter"][1]  # the migration is faster
     # "better": feasible beats infeasible, then faster
-    assert oracle.select(out) == (0, 4920, 2)
+    assert oracle.select(out) == tuple(g["expected"]["select"])
 
 
 def test_bottleneck_ties_take_lowest_stage():
@@ -382,20 +394,20 @@ def test_reshard_matches_1f1b_simulation(p, mbs_log2, changes):
 # --------------------------------------------------------------------------
 def test_p2p_and_reshard_worked_example():
     """R5: stage i pays p2p_fwd of its last op (i < p-1) and p2p_bwd of its first op
-    (i > 0). R13: an in-stage tp/dp change charges the receiving op's reshard."""
+    (i > 0). R13: an in-stage tp/dp change charges the receiving op's reshard.
+    Fixture and derivation: tests/golden/p2p_reshard_example.json."""
+    g = _golden("p2p_reshard_example.json")
+
     def r(tpl, b):
-        return [10, 0, 20, 0, 0, 0, 0, 100 + tpl, 1000 + tpl, 2000 + tpl]
-    prof = mkprof({0: r}, [0] * 4, n_tp=2, n_b=2, n_dp=2, G=4, Bg=4)
-    # stage 0: ops 0,1 at (tp2,dp1) then (tp1,dp2) -> reshard on op 1 (tpl 0): 100
-    # stage 1: ops 2,3 at (tp2,dp1)
-    row = [ai.code(1, 1, 0, 0), ai.code(0, 0, 1, 0), ai.code(1, 1, 0, 0), ai.code(0, 1, 0, 0)]
-    out = ev(prof, [row], [ai.header(1, 2)])
-    S0 = 30 + 30 + 100 + 1000  # + p2p_fwd of op 1 (tpl 0)
-    S1 = 30 + 30 + 2001        # + p2p_bwd of op 2 (tpl 1)
-    N = 2
-    assert list(out["stage_T"][0, :2]) == [S0 + S1 + (N - 1) * S0, S0 + S1 + (N - 1) * S1]
-    assert list(out["stage_comp"][0, :2]) == [N * 60, N * 60]
-    assert list(out["stage_comm"][0, :2]) == [N * 1100, N * 2001]
+        return [v if isinstance(v, int) else int(v.split("+")[0]) + tpl for v in g["record"]]
+    pr = g["profile"]
+    prof = mkprof({0: r}, [0] * pr["n_ops"], n_tp=pr["n_tp"], n_b=pr["n_b"], n_dp=pr["n_dp"],
+                  G=pr["n_devices"], Bg=pr["global_batch"])
+    row = [ai.code(*op) for op in g["row"]]
+    out = ev(prof, [row], [ai.header(g["mbs_log2"], g["p"])])
+    p = g["p"]
+    for k in ("stage_T", "stage_comp", "stage_comm"):
+        assert list(out[k][0, :p]) == g["expected"][k], k
 
 
 # --------------------------------------------------------------------------
